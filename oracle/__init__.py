@@ -1,0 +1,227 @@
+"""CPU oracle for the OTIF proxy + windowing hot path — TEST INFRASTRUCTURE ONLY.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s ``cpu_baseline`` /
+``--impl reference`` legs may import this package.  The product package
+(``paper_conf_sigmod_bastanim22_b200``) never imports it and shares no code with it.
+
+This module is a thin ctypes binding over ``oracle/otif_ref.c`` (plain C99, fp64,
+single-threaded; every function cites the PAPER.md passage it follows).  Arguments
+are numpy arrays on the host.
+
+Parity status: resize, conv, threshold, components and pack are pinned by
+``tests/test_oracle_*.py``; grouping is pinned by invariants, brute force and
+special cases, while its exact greedy output beyond those pins is
+"parity unpinned" (PAPER.md's worked example, Fig. 3 at P:L122, is lost).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from typing import Sequence
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = os.path.join(_HERE, "otif_ref.c")
+
+QUANT_NONE = 0
+QUANT_BF16 = 1
+
+
+class WSize(ctypes.Structure):
+    _fields_ = [("w", ctypes.c_int32), ("h", ctypes.c_int32), ("cost", ctypes.c_int64)]
+
+
+class Window(ctypes.Structure):
+    _fields_ = [("frame", ctypes.c_int32), ("x", ctypes.c_int32), ("y", ctypes.c_int32),
+                ("w", ctypes.c_int32), ("h", ctypes.c_int32), ("size_idx", ctypes.c_int32)]
+
+
+WINDOW_DTYPE = np.dtype([("frame", "<i4"), ("x", "<i4"), ("y", "<i4"),
+                         ("w", "<i4"), ("h", "<i4"), ("size_idx", "<i4")])
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with gcc -O2 (no -ffast-math)."""
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < max(
+            os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "otif_ref.h"))):
+        subprocess.check_call(["gcc", "-std=c99", "-O2", "-fPIC", "-shared", "-Wall",
+                               "-o", _SO, _SRC, "-lm"])
+    return _SO
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    global _lib
+    if _lib is None:
+        _lib = ctypes.CDLL(build())
+        L = _lib
+        P = ctypes.c_void_p
+        i32, i64, sz = ctypes.c_int32, ctypes.c_int64, ctypes.c_size_t
+        L.otif_ref_round_bf16.argtypes = [ctypes.c_double]
+        L.otif_ref_round_bf16.restype = ctypes.c_double
+        L.otif_ref_resize.argtypes = [P, i32, i32, i32, P, i32, i32]
+        L.otif_ref_conv.argtypes = [P, i32, i32, i32, i32, P, P, i32, i32, i32, i32, i32, P]
+        L.otif_ref_proxy_n_weights.argtypes = [P, i32]
+        L.otif_ref_proxy_n_weights.restype = sz
+        L.otif_ref_proxy_grid.argtypes = [i32, i32, i32, P, P]
+        L.otif_ref_proxy_score.argtypes = [P, i32, i32, i32, i32, P, i32, P, sz, i32, P]
+        L.otif_ref_threshold.argtypes = [P, i64, ctypes.c_float, P]
+        L.otif_ref_components.argtypes = [P, i32, i32, i32, P]
+        L.otif_ref_group_frame.argtypes = [P, i32, i32, i32, i32, i32, i32, P, i32, i32, P, i32]
+        L.otif_ref_select_windows.argtypes = [P, i32, i32, i32, i32, i32, i32, i32, P, i32,
+                                              P, i32, P, P, P]
+        L.otif_ref_pack_windows.argtypes = [P, i32, i32, i32, i32, i32, P, i32, P, i32,
+                                            P, P, P, P]
+    return _lib
+
+
+def _p(a: np.ndarray) -> ctypes.c_void_p:
+    assert a.flags["C_CONTIGUOUS"]
+    return ctypes.c_void_p(a.ctypes.data)
+
+
+def _check(rc: int, what: str) -> int:
+    if rc < 0:
+        raise ValueError(f"{what}: oracle rejected the arguments (rc={rc})")
+    return rc
+
+
+def wsizes(sizes: Sequence[tuple]) -> ctypes.Array:
+    """[(w, h)] or [(w, h, cost)] -> ctypes array; default cost w*h (reading R8)."""
+    arr = (WSize * len(sizes))()
+    for i, s in enumerate(sizes):
+        w, h = int(s[0]), int(s[1])
+        arr[i].w, arr[i].h = w, h
+        arr[i].cost = int(s[2]) if len(s) > 2 else w * h
+    return arr
+
+
+def round_bf16(x: float) -> float:
+    return lib().otif_ref_round_bf16(float(x))
+
+
+def resize(src: np.ndarray, dh: int, dw: int) -> np.ndarray:
+    src = np.ascontiguousarray(src, dtype=np.uint8)
+    n, sh, sw, c = src.shape
+    assert c == 3
+    dst = np.empty((n, dh, dw, 3), np.uint8)
+    _check(lib().otif_ref_resize(_p(src), n, sh, sw, _p(dst), dh, dw), "resize")
+    return dst
+
+
+def conv(x: np.ndarray, weight: np.ndarray, bias: np.ndarray, stride: int, relu: bool = True,
+         round_bf16_out: bool = False) -> np.ndarray:
+    """x [n,h,w,cin] fp64, weight [cout,k,k,cin], bias [cout] -> [n,ceil(h/s),ceil(w/s),cout]."""
+    x = np.ascontiguousarray(x, np.float64)
+    weight = np.ascontiguousarray(weight, np.float64)
+    bias = np.ascontiguousarray(bias, np.float64)
+    n, h, w, cin = x.shape
+    cout, k, k2, cin2 = weight.shape
+    assert k == k2 and cin == cin2
+    ho, wo = -(-h // stride), -(-w // stride)
+    out = np.empty((n, ho, wo, cout), np.float64)
+    _check(lib().otif_ref_conv(_p(x), n, h, w, cin, _p(weight), _p(bias), cout, k, stride,
+                               int(relu), int(round_bf16_out), _p(out)), "conv")
+    return out
+
+
+def proxy_n_weights(enc: Sequence[int], dec: int) -> int:
+    e = np.ascontiguousarray(enc, np.int32)
+    return int(lib().otif_ref_proxy_n_weights(_p(e), dec))
+
+
+def proxy_grid(in_h: int, in_w: int, n_strided: int) -> tuple[int, int]:
+    gh, gw = np.zeros(1, np.int32), np.zeros(1, np.int32)
+    _check(lib().otif_ref_proxy_grid(in_h, in_w, n_strided, _p(gh), _p(gw)), "proxy_grid")
+    return int(gh[0]), int(gw[0])
+
+
+def proxy_score(img: np.ndarray, n_strided: int, enc: Sequence[int], dec: int,
+                weights: np.ndarray, quant: int = QUANT_BF16) -> np.ndarray:
+    img = np.ascontiguousarray(img, np.uint8)
+    n, h, w, c = img.shape
+    assert c == 3
+    weights = np.ascontiguousarray(weights, np.float32)
+    e = np.ascontiguousarray(enc, np.int32)
+    gh, gw = proxy_grid(h, w, n_strided)
+    out = np.empty((n, gh, gw), np.float64)
+    _check(lib().otif_ref_proxy_score(_p(img), n, h, w, n_strided, _p(e), dec, _p(weights),
+                                      weights.size, quant, _p(out)), "proxy_score")
+    return out
+
+
+def threshold(scores: np.ndarray, b: float) -> np.ndarray:
+    scores = np.ascontiguousarray(scores, np.float64)
+    mask = np.empty(scores.shape, np.uint8)
+    _check(lib().otif_ref_threshold(_p(scores), scores.size, ctypes.c_float(b), _p(mask)),
+           "threshold")
+    return mask
+
+
+def components(mask: np.ndarray, connectivity: int = 4) -> tuple[int, np.ndarray]:
+    mask = np.ascontiguousarray(mask, np.uint8)
+    gh, gw = mask.shape
+    labels = np.empty((gh, gw), np.int32)
+    n = _check(lib().otif_ref_components(_p(mask), gh, gw, connectivity, _p(labels)),
+               "components")
+    return n, labels
+
+
+def group_frame(mask: np.ndarray, cell: int, frame_w: int, frame_h: int, sizes, connectivity=4,
+                frame_index: int = 0) -> np.ndarray:
+    mask = np.ascontiguousarray(mask, np.uint8)
+    gh, gw = mask.shape
+    ws = wsizes(sizes)
+    cap = gh * gw + 1
+    out = np.zeros(cap, WINDOW_DTYPE)
+    m = _check(lib().otif_ref_group_frame(_p(mask), gh, gw, cell, frame_w, frame_h, connectivity,
+                                          ws, len(sizes), frame_index, _p(out), cap),
+               "group_frame")
+    return out[:m].copy()
+
+
+def select_windows(mask: np.ndarray, cell: int, frame_w: int, frame_h: int, sizes,
+                   connectivity: int = 4, capacity: int | None = None):
+    """mask [n,gh,gw] -> (windows[total], counts[n], offsets[n], total)."""
+    mask = np.ascontiguousarray(mask, np.uint8)
+    n, gh, gw = mask.shape
+    ws = wsizes(sizes)
+    if capacity is None:
+        capacity = n * ((gh * gw + 1) // 2) if connectivity == 4 else n * (((gh + 1) // 2) * ((gw + 1) // 2))
+        capacity = max(capacity, n)
+    win = np.zeros(max(capacity, 1), WINDOW_DTYPE)
+    counts = np.zeros(n, np.int32)
+    offs = np.zeros(n, np.int32)
+    total = np.zeros(1, np.int32)
+    _check(lib().otif_ref_select_windows(_p(mask), n, gh, gw, cell, frame_w, frame_h, connectivity,
+                                         ws, len(sizes), _p(win), capacity, _p(counts), _p(offs),
+                                         _p(total)), "select_windows")
+    t = int(total[0])
+    return win[:min(t, capacity)].copy(), counts, offs, t
+
+
+def pack_windows(src: np.ndarray, det_h: int, det_w: int, windows: np.ndarray, sizes,
+                 batch_cap: Sequence[int] | None = None):
+    """-> (batches list of [cap_s,h_s,w_s,3] u8, slot[total], size_count[k])."""
+    src = np.ascontiguousarray(src, np.uint8)
+    n, sh, sw, _ = src.shape
+    windows = np.ascontiguousarray(windows, WINDOW_DTYPE)
+    total = windows.shape[0]
+    k = len(sizes)
+    ws = wsizes(sizes)
+    if batch_cap is None:
+        batch_cap = [int((windows["size_idx"] == s).sum()) for s in range(k)]
+    batches = [np.zeros((max(int(batch_cap[s]), 0), int(sizes[s][1]), int(sizes[s][0]), 3), np.uint8)
+               for s in range(k)]
+    ptrs = (ctypes.c_void_p * k)(*[b.ctypes.data for b in batches])
+    caps = np.ascontiguousarray(batch_cap, np.int32)
+    slot = np.zeros(max(total, 1), np.int32)
+    counts = np.zeros(k, np.int32)
+    _check(lib().otif_ref_pack_windows(_p(src), n, sh, sw, det_h, det_w, _p(windows), total, ws, k,
+                                       ptrs, _p(caps), _p(slot), _p(counts)), "pack_windows")
+    return batches, slot[:total].copy(), counts

@@ -1,0 +1,100 @@
+/*
+ * otif_ref.h — CPU ORACLE for the OTIF proxy + windowing hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load this library.  The product path
+ * (paper_conf_sigmod_bastanim22_b200/) never links, imports or calls it, and this
+ * code shares nothing with the CUDA path (no headers, helpers or tables).
+ *
+ * Plain, slow, single-threaded C99 in fp64, following PAPER.md (OTIF, Bastani &
+ * Madden, SIGMOD'22) step by step; readings where the paper is silent are the
+ * ones listed in DESIGN.md §3 (SURVEY.md §8(c) R1–R17).  Citations "P:L<n>" are
+ * lines of /root/reference/PAPER.md.
+ *
+ * All pointers are HOST pointers.  Layouts: images u8 NHWC RGB (C = 3),
+ * activations fp64 NHWC, weights fp32 W[Cout][kh][kw][Cin] followed by b[Cout].
+ * Every function returns 0 on success and a negative value on bad arguments.
+ */
+#ifndef OTIF_REF_H
+#define OTIF_REF_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* quantisation modes of the proxy (reading R4) */
+#define OTIF_REF_QUANT_NONE 0 /* no rounding anywhere: pure fp64 */
+#define OTIF_REF_QUANT_BF16 1 /* weights and every inter-layer activation rounded to bf16 (RNE) */
+
+typedef struct { int32_t w, h; int64_t cost; } otif_ref_wsize;                /* (w,h) in W with T_{w,h} */
+typedef struct { int32_t frame, x, y, w, h, size_idx; } otif_ref_window;      /* r = (x,y,w,h) */
+
+/* Round an fp64 value to the nearest bf16 value, ties to even (reading R4). */
+double otif_ref_round_bf16(double x);
+
+/* Stage 1: bilinear resize, half-pixel centres, no antialias,
+ * round half up, u8 NHWC, C = 3.  src [n,sh,sw,3] -> dst [n,dh,dw,3]. */
+int otif_ref_resize(const uint8_t *src, int32_t n, int32_t sh, int32_t sw,
+                    uint8_t *dst, int32_t dh, int32_t dw);
+
+/* Stage 2, one layer: 3x3 conv (or 1x1 when k == 1), zero pad (k-1)/2,
+ * stride s in {1,2}, + bias, optional ReLU, optional bf16 rounding of the output.
+ * in [n,h,w,cin] fp64 -> out [n,ceil(h/s),ceil(w/s),cout] fp64.
+ * w/b are used exactly as given (caller pre-rounds weights for quant=bf16). */
+int otif_ref_conv(const double *in, int32_t n, int32_t h, int32_t w, int32_t cin,
+                  const double *weight, const double *bias, int32_t cout, int32_t k,
+                  int32_t stride, int32_t relu, int32_t round_bf16, double *out);
+
+/* Stage 2, whole proxy.  Encoder widths enc[5], decoder
+ * width dec; the first n_strided encoder layers have stride 2 (reading R1).
+ * weights: fp32 blob E1..E5, D1, D2.  img [n,in_h,in_w,3] u8 -> scores [n,gh,gw]
+ * fp64 with gh = ceil(in_h / 2^n_strided).  quant: OTIF_REF_QUANT_*. */
+size_t otif_ref_proxy_n_weights(const int32_t enc[5], int32_t dec);
+int otif_ref_proxy_grid(int32_t in_h, int32_t in_w, int32_t n_strided, int32_t *gh, int32_t *gw);
+int otif_ref_proxy_score(const uint8_t *img, int32_t n, int32_t in_h, int32_t in_w,
+                         int32_t n_strided, const int32_t enc[5], int32_t dec,
+                         const float *weights, size_t n_weights, int32_t quant,
+                         double *scores);
+
+/* Stage 3 ("exceeds"): mask = score > B, strict, compared in fp64. */
+int otif_ref_threshold(const double *scores, int64_t cells, float threshold, uint8_t *mask);
+
+/* Connected components: BFS seeded in row-major order; labels[gh*gw]
+ * = component index in seed order, -1 for negative cells.  Returns the count. */
+int otif_ref_components(const uint8_t *mask, int32_t gh, int32_t gw, int32_t connectivity,
+                        int32_t *labels);
+
+/* Stage 4 for one frame: windows covering the positive cells,
+ * greedy agglomerative merge, disjointness pass, full-frame fallback
+ * (P:L133).  Writes at most cap windows sorted by (y, x); returns the count
+ * (which may exceed cap) or a negative error. */
+int otif_ref_group_frame(const uint8_t *mask, int32_t gh, int32_t gw, int32_t cell,
+                         int32_t frame_w, int32_t frame_h, int32_t connectivity,
+                         const otif_ref_wsize *sizes, int32_t k, int32_t frame_index,
+                         otif_ref_window *out, int32_t cap);
+
+/* Stage 4 over a batch: compacted windows in (frame, y, x) order, counts,
+ * exclusive offsets, total.  Returns 0 (total is exact even if > capacity). */
+int otif_ref_select_windows(const uint8_t *mask, int32_t n, int32_t gh, int32_t gw,
+                            int32_t cell, int32_t frame_w, int32_t frame_h, int32_t connectivity,
+                            const otif_ref_wsize *sizes, int32_t k,
+                            otif_ref_window *windows, int32_t capacity,
+                            int32_t *frame_count, int32_t *frame_offset, int32_t *total);
+
+/* Stage 5: det = resize(src -> det_h x det_w) (a copy when
+ * equal); for windows in order, slot = running count of its size_idx;
+ * batches[s][slot] = det[frame][y:y+h, x:x+w, :].  Entries with slot >=
+ * batch_cap[s] are dropped; size_count[s] is exact. */
+int otif_ref_pack_windows(const uint8_t *src, int32_t n, int32_t sh, int32_t sw,
+                          int32_t det_h, int32_t det_w,
+                          const otif_ref_window *windows, int32_t total,
+                          const otif_ref_wsize *sizes, int32_t k,
+                          uint8_t *const *batches, const int32_t *batch_cap,
+                          int32_t *slot, int32_t *size_count);
+
+#ifdef __cplusplus
+}
+#endif
+#endif
