@@ -1,0 +1,192 @@
+/*
+ * otif.h — C ABI of the B200-native (sm_100a) OTIF proxy + windowing hot path.
+ *
+ * OTIF (Bastani & Madden, SIGMOD'22) runs, on every sampled frame, a segmentation
+ * proxy that scores each grid cell, thresholds the scores, groups the positive
+ * cells into rectangular windows of a few fixed sizes, and runs the detector on
+ * those windows in equal-size batches.  This library is that per-frame path.
+ * Citations "P:L<n>" are lines of the paper text; readings R<n> are
+ * listed in DESIGN.md §3.
+ *
+ * Conventions (all entry points):
+ *  - Pointers are CUDA DEVICE pointers unless marked [host].  All buffers are
+ *    allocated and owned by the caller; the library never allocates device memory
+ *    except in otif_proxy_create (packed weights) and otif_pipeline_create.
+ *  - Every call only enqueues work on `stream` and returns; it never synchronises.
+ *    The return value reports synchronous argument validation and launch errors;
+ *    asynchronous faults surface at the caller's next synchronisation.
+ *  - Images are u8 NHWC RGB (C = 3), rows densely packed (row stride 3*W bytes).
+ *  - No exception crosses the ABI and there is no CPU fallback: every stage runs in
+ *    this library's sm_100a kernels.  OTIF_EUNSUPPORTED is returned on a device
+ *    that is not sm_100 or for shapes the kernels do not cover.
+ */
+#ifndef OTIF_H
+#define OTIF_H
+
+#include <stddef.h>
+#include <stdint.h>
+#include <cuda_runtime_api.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    OTIF_OK = 0,
+    OTIF_EINVAL = 1,        /* bad argument (shape, NULL pointer, inconsistent sizes) */
+    OTIF_ENOMEM = 2,        /* allocation in *_create failed, or workspace too small */
+    OTIF_ECUDA = 3,         /* a CUDA runtime call or kernel launch failed */
+    OTIF_EUNSUPPORTED = 4   /* not an sm_100 device, or a shape beyond the kernels' limits */
+} otif_status;
+
+const char *otif_status_str(otif_status s);
+/* Thread-local human-readable detail for the last non-OK status of this thread. */
+const char *otif_last_error(void);
+/* Library version string, e.g. "otif-b200 0.1 sm_100a". */
+const char *otif_version(void);
+
+/* An element of the window-size set W with its detector time T_{w,h}.
+ * Costs are integers so that merge decisions and ties are exact (reading R8);
+ * the default is the window area w*h. */
+typedef struct { int32_t w, h; int64_t cost; } otif_wsize;
+
+/* A window r = (x, y, w, h) in detector pixels, half-open, (w, h) = sizes[size_idx]
+ * ("each r_i is a 4-tuple (r_i.x, r_i.y, r_i.w, r_i.h) ... (r_i.w, r_i.h) ∈ W"). */
+typedef struct { int32_t frame, x, y, w, h, size_idx; } otif_window;
+
+/* ---------------------------------------------------------------------------
+ * Stage 1 — resize (frames are decoded at the detector resolution and the
+ * proxy "inputs video at a lower resolution").  Bilinear with half-pixel
+ * centres, no antialias, fp32 blend, round half up (reading R13).
+ *   src [n, src_h, src_w, 3] u8  ->  dst [n, dst_h, dst_w, 3] u8.
+ * Any positive sizes (down- or up-scaling).  src and dst must not overlap.
+ * Errors: OTIF_EINVAL for non-positive sizes or NULL pointers. */
+otif_status otif_resize(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w,
+                        uint8_t *dst, int32_t dst_h, int32_t dst_w, cudaStream_t stream);
+
+/* ---------------------------------------------------------------------------
+ * Stage 2 — segmentation proxy CNN ("a five-layer encoder followed
+ * by a two-layer decoder ... a classification score at each ... cell").
+ * Shape (readings R1, R2): E1..E5 3x3 pad 1 + ReLU with widths enc[0..4]; the first
+ * n_strided (= log2 S, 1..5) encoder layers have stride 2; D1 3x3 pad 1 + ReLU
+ * (width dec); D2 1x1 -> 1 logit; score = sigmoid(logit).  Input (u - 128)/128.
+ * Precision (reading R4): bf16 weights and activations (RNE after bias + ReLU),
+ * fp32 accumulation on the tensor cores, fp32 logit and score.
+ * Supported widths: enc[0] == 32; enc[1..4] and dec in {64, 128, 256}; dec <= 256. */
+typedef struct {
+    int32_t in_h, in_w;     /* proxy input resolution */
+    int32_t n_strided;      /* log2 of the output stride S, 1..5 */
+    int32_t enc[5];         /* encoder widths */
+    int32_t dec;            /* decoder width (D1) */
+} otif_proxy_desc;
+
+typedef struct otif_proxy otif_proxy;
+
+/* weights: [host] fp32 blob, layers E1..E5, D1, D2 in order; per layer
+ * W[Cout][kh][kw][Cin] then b[Cout] (n_weights must match the descriptor).
+ * The handle owns the weights repacked (bf16, tap-major K blocks) in device memory;
+ * it is immutable after creation and may be shared by several streams.
+ * Uses the current CUDA device. */
+otif_status otif_proxy_create(const otif_proxy_desc *d, const float *weights, size_t n_weights,
+                              otif_proxy **out);
+void otif_proxy_destroy(otif_proxy *p);
+/* Output grid (gh, gw) = (ceil(in_h / S), ceil(in_w / S)). */
+otif_status otif_proxy_grid(const otif_proxy *p, int32_t *gh, int32_t *gw);
+/* Device workspace needed for a batch of n frames (activations between layers). */
+size_t otif_proxy_workspace_bytes(const otif_proxy *p, int32_t n);
+/* img [n, in_h, in_w, 3] u8 -> scores [n, gh, gw] fp32.
+ * workspace: >= otif_proxy_workspace_bytes(p, n) bytes, 256-B aligned.  It is
+ * initialised by the library on first use (a header tag records the layout) and
+ * must not be written by the caller between calls; a caller that reuses the memory
+ * for something else must zero its first 256 bytes before handing it back. */
+otif_status otif_proxy_score(const otif_proxy *p, const uint8_t *img, int32_t n, float *scores,
+                             void *workspace, size_t ws_bytes, cudaStream_t stream);
+
+/* ---------------------------------------------------------------------------
+ * Stages 3 + 4 — threshold and window selection ("After thresholding the
+ * scores by B_proxy, we derive a binary grid ... of positive cells"; P:L149–151:
+ * windows R_t with sizes in W covering every positive cell, found by greedy
+ * agglomerative merging of connected components while est(R) = Σ T decreases;
+ * fall back to the full frame when that is faster).  Exact algorithm:
+ * DESIGN.md §3 (readings R6–R11, R14, R15).  Integer arithmetic throughout.
+ *   exactly one of scores [n, gh, gw] fp32 / mask_in [n, gh, gw] u8 (0/1) is non-NULL;
+ *   mask_in is the "perfect proxy" mode of P:L153.  mask = scores > threshold.
+ *   sizes: [host] W, k entries (1 <= k <= 8); must contain (frame_w, frame_h)
+ *    and no size larger than the frame.
+ * Outputs: mask_out [n, gh, gw] u8 (optional, may be NULL); windows [capacity]
+ * compacted across the batch in (frame, y, x) order; frame_count[n], frame_offset[n]
+ * (exclusive prefix), total[1].  total and counts are exact even when windows beyond
+ * `capacity` are dropped; capacity = n*ceil(gh*gw/2) can never overflow.
+ * Limits: gh*gw <= 8192.  workspace: >= otif_select_workspace_bytes(n, gh, gw). */
+typedef struct { int32_t frame_w, frame_h, cell, connectivity; /* 4 or 8 */ } otif_grid_desc;
+size_t otif_select_workspace_bytes(int32_t n, int32_t gh, int32_t gw);
+otif_status otif_select_windows(const float *scores, const uint8_t *mask_in, float threshold,
+                                int32_t n, int32_t gh, int32_t gw, const otif_grid_desc *g,
+                                const otif_wsize *sizes, int32_t k,
+                                uint8_t *mask_out, otif_window *windows, int32_t capacity,
+                                int32_t *frame_count, int32_t *frame_offset, int32_t *total,
+                                void *workspace, size_t ws_bytes, cudaStream_t stream);
+
+/* ---------------------------------------------------------------------------
+ * Stage 5 — crop / resample / pack (the detector is initialised "at each of
+ * those sizes" and "high detection performance on GPUs relies heavily on batching
+ * many equal-dimension inputs together").
+ *   det = resize(src -> det_h x det_w) (bilinear as in stage 1; a plain copy when
+ *   equal); for the windows[0 .. min(*total, capacity)) in order, slot = running
+ *   count of its size_idx; batches[s][slot] = det[frame][y:y+h, x:x+w, :].
+ *   batches: [host] array of k device pointers, batches[s] is [batch_cap[s], h_s, w_s, 3].
+ *   batch_cap: [host] k capacities.  slot [capacity] int32 and size_count [k] are
+ *   device outputs; size_count is exact even when entries beyond batch_cap are dropped.
+ * `total` is read on the device (no host synchronisation). */
+otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w,
+                              int32_t det_h, int32_t det_w,
+                              const otif_window *windows, const int32_t *total, int32_t capacity,
+                              const otif_wsize *sizes, int32_t k,
+                              uint8_t *const *batches, const int32_t *batch_cap,
+                              int32_t *slot, int32_t *size_count, cudaStream_t stream);
+
+/* ---------------------------------------------------------------------------
+ * Whole path on HOST frames (the end-to-end call): for batches of up to max_batch
+ * frames, copy src (pinned or pageable host memory) to the device, run stages 1–5,
+ * and copy the windows and per-frame counts back.  Two CUDA streams overlap the
+ * host->device copy of batch b+1 with the compute of batch b.  The detector batches
+ * stay on the device (the detector runs there); their per-size fill counts
+ * are returned.
+ *   desc: proxy shape (in_h/in_w = proxy resolution); src frames are src_h x src_w,
+ *   the detector resolution is det_h x det_w; cell size, connectivity, W, threshold.
+ * Results: windows_out [host, cap_windows], frame_count_out [host, n],
+ * total_out [host], size_count_out [host, k] (all sizes accumulated over batches).
+ * The call returns after the last copy completes (it synchronises its own streams). */
+typedef struct {
+    otif_proxy_desc proxy;
+    int32_t src_h, src_w, det_h, det_w;
+    otif_grid_desc grid;
+    float threshold;
+    int32_t k;
+    otif_wsize sizes[8];
+    int32_t max_batch;          /* frames per device batch */
+    int32_t batch_cap[8];       /* detector batch capacity per size, per device batch */
+} otif_pipeline_desc;
+
+typedef struct otif_pipeline otif_pipeline;
+otif_status otif_pipeline_create(const otif_pipeline_desc *d, const float *weights, size_t n_weights,
+                                 otif_pipeline **out);
+void otif_pipeline_destroy(otif_pipeline *p);
+otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *src_host, int32_t n,
+                                   otif_window *windows_out, int32_t cap_windows,
+                                   int32_t *frame_count_out, int32_t *total_out,
+                                   int32_t *size_count_out);
+/* Same path on frames already resident in device memory; results stay on the
+ * device in the pipeline's buffers (otif_pipeline_last_* accessors) for the LAST
+ * batch; totals are accumulated on the device.  Enqueued on `stream`. */
+otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t *src_dev, int32_t n,
+                                     cudaStream_t stream);
+/* Device pointer to int64[4 + k] counters accumulated since create/reset:
+ * frames, positive cells, windows, window pixels, then windows per size. */
+const int64_t *otif_pipeline_counters(const otif_pipeline *p);
+otif_status otif_pipeline_reset_counters(otif_pipeline *p, cudaStream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* OTIF_H */

@@ -1,0 +1,192 @@
+// pack.cu — stage 5: crop (and, when the detector resolution differs
+// from the source, bilinearly resample) every window into its per-size dense
+// detector batch.  Slot = running count of the window's size in emission order.
+//
+// K7a slot_kernel: one CTA scans the window list in order; per size, a warp ballot
+//   gives each window its rank among same-size windows of its 32-window group, and
+//   running per-size carries make the slot.  size_count is written at the end.
+// K7b pack_kernel: persistent grid; one CTA per window (grid-stride).  Identity case:
+//   each thread produces 16 destination bytes (destination rows are 16-B aligned for
+//   every size in W with w*3 % 16 == 0) from two aligned 16-B source loads and a
+//   funnel shift, since a window's x offset makes the source row arbitrarily aligned.
+//   Resampling case: per output pixel bilinear blend (same arithmetic as resize.cu).
+#include <string.h>
+
+#include "common.cuh"
+
+namespace otif {
+
+constexpr int kMaxK = 8;
+
+struct PackParams {
+    const uint8_t *src;
+    int n, sh, sw, dh, dw;
+    size_t src_bytes;
+    const otif_window *win;
+    const int *total;
+    int capacity;
+    int k;
+    uint8_t *batch[kMaxK];
+    int cap[kMaxK];
+    int bw[kMaxK], bh[kMaxK];
+    int *slot;
+    int *size_count;
+};
+
+__global__ void __launch_bounds__(1024) slot_kernel(const __grid_constant__ PackParams p) {
+    __shared__ int s_warp_cnt[32][kMaxK];
+    __shared__ int s_carry[kMaxK];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    if (threadIdx.x < kMaxK) s_carry[threadIdx.x] = 0;
+    __syncthreads();
+    const int total = min(*p.total, p.capacity);
+    for (int base = 0; base < total; base += blockDim.x) {
+        const int g = base + threadIdx.x;
+        const int s = g < total ? p.win[g].size_idx : -1;
+        int rank = 0;
+        for (int z = 0; z < p.k; z++) {
+            unsigned m = __ballot_sync(0xffffffffu, s == z);
+            if (s == z) rank = __popc(m & ((1u << lane) - 1u));
+            if (lane == 0) s_warp_cnt[warp][z] = __popc(m);
+        }
+        __syncthreads();
+        if (g < total) {
+            int pre = s_carry[s];
+            for (int w = 0; w < warp; w++) pre += s_warp_cnt[w][s];
+            p.slot[g] = pre + rank;
+        }
+        __syncthreads();
+        if (threadIdx.x < p.k) {
+            int add = 0;
+            for (int w = 0; w < nw; w++) add += s_warp_cnt[w][threadIdx.x];
+            s_carry[threadIdx.x] += add;
+        }
+        __syncthreads();
+    }
+    // size_count counts every listed window, including those dropped for batch_cap
+    if (threadIdx.x < p.k) p.size_count[threadIdx.x] = s_carry[threadIdx.x];
+}
+
+__device__ __forceinline__ uint32_t fshift(uint32_t lo, uint32_t hi, uint32_t sh_bytes) {
+    return sh_bytes ? __funnelshift_r(lo, hi, sh_bytes * 8) : lo;
+}
+
+__global__ void __launch_bounds__(256) pack_kernel(const __grid_constant__ PackParams p) {
+    const int total = min(*p.total, p.capacity);
+    const bool identity = (p.dh == p.sh && p.dw == p.sw);
+    for (int g = blockIdx.x; g < total; g += gridDim.x) {
+        const otif_window w = p.win[g];
+        const int s = w.size_idx;
+        const int sl = p.slot[g];
+        if (sl >= p.cap[s]) continue;
+        uint8_t *dst = p.batch[s] + (size_t)sl * p.bh[s] * p.bw[s] * 3;
+        const int row_bytes = w.w * 3;
+        if (identity && (row_bytes & 15) == 0 && (((uintptr_t)p.batch[s]) & 15) == 0) {
+            const int per_row = row_bytes >> 4;
+            const uint8_t *fbase = p.src + (size_t)w.frame * p.sh * p.sw * 3;
+            const uintptr_t src_end = (uintptr_t)p.src + p.src_bytes;
+            for (int i = threadIdx.x; i < w.h * per_row; i += blockDim.x) {
+                const int r = i / per_row, c = i - r * per_row;
+                const uint8_t *s0 = fbase + ((size_t)(w.y + r) * p.sw + w.x) * 3 + c * 16;
+                const uintptr_t a = (uintptr_t)s0;
+                const uintptr_t al = a & ~(uintptr_t)15;
+                const uint32_t sh = (uint32_t)(a - al);
+                uint4 out;
+                if (al + 32 <= src_end) {
+                    const uint4 v0 = __ldg(reinterpret_cast<const uint4 *>(al));
+                    const uint4 v1 = sh ? __ldg(reinterpret_cast<const uint4 *>(al + 16)) : make_uint4(0, 0, 0, 0);
+                    uint32_t wv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
+                    const uint32_t q = sh >> 2, b = sh & 3;
+                    uint32_t o[4];
+#pragma unroll
+                    for (int j = 0; j < 4; j++) {
+                        uint32_t lo, hi;
+                        // wv[q + j], wv[q + j + 1] with q in 0..3 (unrolled select, no local memory)
+                        lo = q == 0 ? wv[j] : q == 1 ? wv[j + 1] : q == 2 ? wv[j + 2] : wv[j + 3];
+                        hi = q == 0 ? wv[j + 1] : q == 1 ? wv[j + 2] : q == 2 ? wv[j + 3] : wv[j + 4];
+                        o[j] = fshift(lo, hi, b);
+                    }
+                    out = make_uint4(o[0], o[1], o[2], o[3]);
+                } else {
+                    uint8_t bytes[16];
+#pragma unroll
+                    for (int j = 0; j < 16; j++) bytes[j] = s0[j];
+                    uint32_t o[4];
+#pragma unroll
+                    for (int j = 0; j < 4; j++)
+                        o[j] = (uint32_t)bytes[4 * j] | ((uint32_t)bytes[4 * j + 1] << 8) |
+                               ((uint32_t)bytes[4 * j + 2] << 16) | ((uint32_t)bytes[4 * j + 3] << 24);
+                    out = make_uint4(o[0], o[1], o[2], o[3]);
+                }
+                *reinterpret_cast<uint4 *>(dst + (size_t)r * row_bytes + c * 16) = out;
+            }
+        } else if (identity) {
+            const uint8_t *fbase = p.src + (size_t)w.frame * p.sh * p.sw * 3;
+            for (int i = threadIdx.x; i < w.h * row_bytes; i += blockDim.x) {
+                const int r = i / row_bytes, c = i - r * row_bytes;
+                dst[(size_t)r * row_bytes + c] = fbase[((size_t)(w.y + r) * p.sw + w.x) * 3 + c];
+            }
+        } else {
+            // resample: det pixel (w.y + r, w.x + x) of the det_h x det_w frame, bilinear from src
+            const uint8_t *fbase = p.src + (size_t)w.frame * p.sh * p.sw * 3;
+            for (int i = threadIdx.x; i < w.h * w.w; i += blockDim.x) {
+                const int r = i / w.w, x = i - r * w.w;
+                const int oy = w.y + r, ox = w.x + x;
+                float sy = fmaxf((float)((2 * oy + 1) * p.sh - p.dh) / (float)(2 * p.dh), 0.0f);
+                float sx = fmaxf((float)((2 * ox + 1) * p.sw - p.dw) / (float)(2 * p.dw), 0.0f);
+                int y0 = min((int)floorf(sy), p.sh - 1), x0 = min((int)floorf(sx), p.sw - 1);
+                int y1 = min(y0 + 1, p.sh - 1), x1 = min(x0 + 1, p.sw - 1);
+                float ly = sy - (float)y0, lx = sx - (float)x0;
+#pragma unroll
+                for (int c = 0; c < 3; c++) {
+                    float p00 = fbase[((size_t)y0 * p.sw + x0) * 3 + c], p01 = fbase[((size_t)y0 * p.sw + x1) * 3 + c];
+                    float p10 = fbase[((size_t)y1 * p.sw + x0) * 3 + c], p11 = fbase[((size_t)y1 * p.sw + x1) * 3 + c];
+                    float v = (1.0f - ly) * ((1.0f - lx) * p00 + lx * p01) + ly * ((1.0f - lx) * p10 + lx * p11);
+                    v = fminf(fmaxf(floorf(v + 0.5f), 0.0f), 255.0f);
+                    dst[(size_t)i * 3 + c] = (uint8_t)v;
+                }
+            }
+        }
+    }
+}
+
+}  // namespace otif
+
+using namespace otif;
+
+extern "C" otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w, int32_t det_h,
+                                         int32_t det_w, const otif_window *windows, const int32_t *total,
+                                         int32_t capacity, const otif_wsize *sizes, int32_t k,
+                                         uint8_t *const *batches, const int32_t *batch_cap, int32_t *slot,
+                                         int32_t *size_count, cudaStream_t stream) {
+    OTIF_REQUIRE(n >= 0 && src_h > 0 && src_w > 0 && det_h > 0 && det_w > 0, "otif_pack_windows: bad sizes");
+    OTIF_REQUIRE(k >= 1 && k <= kMaxK, "otif_pack_windows: k=%d not in [1,8]", k);
+    OTIF_REQUIRE(sizes && batches && batch_cap, "otif_pack_windows: NULL host arrays");
+    OTIF_REQUIRE(total && size_count && capacity >= 0, "otif_pack_windows: NULL total/size_count");
+    OTIF_REQUIRE(capacity == 0 || (windows && slot), "otif_pack_windows: NULL windows/slot");
+    OTIF_REQUIRE(src || n == 0, "otif_pack_windows: NULL src");
+    otif_status st = check_device(nullptr);
+    if (st != OTIF_OK) return st;
+    PackParams p;
+    memset(&p, 0, sizeof(p));
+    p.src = src; p.n = n; p.sh = src_h; p.sw = src_w; p.dh = det_h; p.dw = det_w;
+    p.src_bytes = (size_t)n * src_h * src_w * 3;
+    p.win = windows; p.total = total; p.capacity = capacity; p.k = k;
+    for (int s = 0; s < k; s++) {
+        OTIF_REQUIRE(sizes[s].w > 0 && sizes[s].h > 0 && sizes[s].w <= det_w && sizes[s].h <= det_h,
+                     "otif_pack_windows: size %d larger than the detector frame", s);
+        OTIF_REQUIRE(batch_cap[s] >= 0 && (batch_cap[s] == 0 || batches[s]), "otif_pack_windows: batch %d", s);
+        p.batch[s] = batches[s]; p.cap[s] = batch_cap[s]; p.bw[s] = sizes[s].w; p.bh[s] = sizes[s].h;
+    }
+    p.slot = slot; p.size_count = size_count;
+    int num_sms = 148;
+    check_device(&num_sms);
+    slot_kernel<<<1, 1024, 0, stream>>>(p);
+    OTIF_LAUNCH_CHECK();
+    if (capacity > 0) {
+        int grid = capacity < num_sms * 8 ? capacity : num_sms * 8;
+        pack_kernel<<<grid, 256, 0, stream>>>(p);
+        OTIF_LAUNCH_CHECK();
+    }
+    return OTIF_OK;
+}

@@ -1,0 +1,720 @@
+// proxy.cu — stage 2: the segmentation proxy CNN (readings R1, R2, R4).
+//
+//   E1 (3->32, 3x3, stride 2): CUDA-core direct conv from the u8 proxy image
+//       (K = 27 is too small for a tensor-core tile); bf16 output.
+//   E2..E5, D1 (3x3, pad 1): implicit-GEMM convolutions on the 5th-gen tensor cores
+//       (tcgen05.mma kind::f16, bf16 x bf16 -> fp32 in TMEM), one persistent,
+//       warp-specialised kernel per layer.
+//   D2 (1x1, 128->1) + sigmoid: fused into D1's epilogue (per-row GEMV over the
+//       bf16-rounded D1 activations read back from TMEM).
+//
+// Activation layout in HBM ("padded linear, chunk-planar").  A stride-1 3x3 conv over
+// an H x W map reads, for output pixel q, the input pixels q + kh*(W+2) + kw of the
+// zero-padded map flattened row-major with pitch W+2 — a pure linear shift per tap.
+// So every GEMM layer's input is stored zero-padded and flattened, frames stacked
+// (each frame owns H+1 rows of pitch W+2; the bottom pad of frame f is the top pad
+// of frame f+1), and channel-chunk planar: [plane][C/8][pixels][8 bf16].  Then the
+// A operand of one M tile (128 consecutive output positions) for ALL 9 taps is one
+// contiguous halo of 128 + 2(W+2) + 2 pixels per 8-channel chunk, loaded once with
+// 1-D bulk async copies and reused by 9 MMAs through shifted smem descriptors (the
+// no-swizzle K-major layout puts consecutive rows 16 B apart, so a shift of s pixels
+// is a +16*s start address).  Stride-2 layers read a parity-split input (4 planes:
+// even/odd rows x even/odd cols), on which each of the 9 taps is again a linear
+// shift (by 0, 1, pitch or pitch+1) within one plane.  Each layer's epilogue writes
+// its output directly into the next layer's layout; pad positions are never
+// written and stay zero (the workspace is zeroed once, see the tag kernels).
+// Output positions in the pad columns/rows are computed and discarded (≈6–12% of
+// MACs at the configs' sizes; the roofline counts only the algorithmic MACs).
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <vector>
+
+#include "common.cuh"
+
+namespace otif {
+
+constexpr int kConvThreads = 256;   // warp0 producer, warp1 MMA, warp2 TMEM alloc, warps4-7 epilogue
+constexpr int kTileM = 128;
+constexpr int kMaxStagesA = 4;
+constexpr int kMaxStagesB = 8;
+
+// ---------------------------------------------------------------------------
+// layouts
+// ---------------------------------------------------------------------------
+struct Layout {        // a GEMM layer's input buffer
+    int kind;          // 1: stride-1 padded (1 plane); 2: parity-split (4 planes)
+    int planes;
+    int pitch;         // pixels per padded row
+    int64_t fstride;   // pixels per frame slot
+    int64_t lcap;      // pixels per (plane, chunk) row of the buffer
+    int c8;            // channels / 8
+    size_t offset;     // byte offset inside the workspace
+    size_t bytes;
+};
+
+__host__ __device__ __forceinline__ int64_t layout_pixel(int kind, int pitch, int64_t fstride, int f, int y, int x,
+                                                         int &plane) {
+    if (kind == 1) {
+        plane = 0;
+        return (int64_t)f * fstride + (int64_t)(y + 1) * pitch + (x + 1);
+    }
+    plane = ((y & 1) << 1) | (x & 1);
+    return (int64_t)f * fstride + (int64_t)((y >> 1) + 1) * pitch + ((x >> 1) + 1);
+}
+
+struct ConvParams {
+    const uint8_t *act;         // input buffer (bytes)
+    int64_t lcap;
+    int c8_in;
+    int kb, ncb;                // channels per K block, number of K blocks
+    int P;                      // halo rows per A stage
+    int ngroups;
+    int group_plane[4];
+    int group_ntaps[4];
+    int group_shift[4][9];
+    const uint8_t *wpk;         // packed bf16 weights [cb][tap-in-loop-order][chunk][N][8]
+    const float *bias;          // [N]
+    int N;
+    int64_t mtot;
+    int ntiles;
+    int pitch;                  // q decode
+    int64_t fstride;
+    int out_h, out_w;
+    int stages_a, stages_b;
+    // destination
+    int out_kind;               // 1/2: next layout kind; 3: head scores
+    uint8_t *out;
+    int64_t out_lcap;
+    int out_c8;
+    int out_pitch;
+    int64_t out_fstride;
+    float *scores;
+    const float *w2;            // [N] bf16-rounded head weights (fp32 storage)
+    float b2;
+};
+
+// ---------------------------------------------------------------------------
+// workspace tag: zero the workspace once per layout (pads must be zero)
+// ---------------------------------------------------------------------------
+__global__ void ws_zero_kernel(uint8_t *ws, size_t bytes, uint64_t tag) {
+    if (*reinterpret_cast<volatile uint64_t *>(ws) == tag) return;
+    uint4 z = make_uint4(0, 0, 0, 0);
+    size_t n16 = bytes / 16;
+    for (size_t i = 16 + blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n16; i += (size_t)gridDim.x * blockDim.x)
+        reinterpret_cast<uint4 *>(ws)[i] = z;
+}
+__global__ void ws_tag_kernel(uint8_t *ws, uint64_t tag) { *reinterpret_cast<uint64_t *>(ws) = tag; }
+
+// ---------------------------------------------------------------------------
+// E1: 3x3 stride-2 conv 3 -> 32 on CUDA cores, u8 input, bf16 output in E2's layout
+// ---------------------------------------------------------------------------
+struct E1Params {
+    const uint8_t *img;
+    int n, h, w, oh, ow;
+    const float *wt;    // [27][32] (k = (kh*3+kw)*3+c), bf16-rounded
+    const float *bias;  // [32]
+    int out_kind, out_pitch;
+    int64_t out_fstride, out_lcap;
+    uint8_t *out;
+};
+
+__global__ void __launch_bounds__(256) e1_kernel(E1Params p) {
+    __shared__ float sw[27 * 32];
+    __shared__ float sb[32];
+    for (int i = threadIdx.x; i < 27 * 32; i += blockDim.x) sw[i] = p.wt[i];
+    if (threadIdx.x < 32) sb[threadIdx.x] = p.bias[threadIdx.x];
+    __syncthreads();
+    const int64_t total = (int64_t)p.n * p.oh * p.ow;
+    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        int ox = (int)(idx % p.ow);
+        int64_t t = idx / p.ow;
+        int oy = (int)(t % p.oh);
+        int f = (int)(t / p.oh);
+        float x[27];
+        const uint8_t *base = p.img + (size_t)f * p.h * p.w * 3;
+#pragma unroll
+        for (int kh = 0; kh < 3; kh++) {
+            int iy = 2 * oy - 1 + kh;
+#pragma unroll
+            for (int kw = 0; kw < 3; kw++) {
+                int ix = 2 * ox - 1 + kw;
+                bool ok = iy >= 0 && iy < p.h && ix >= 0 && ix < p.w;
+                const uint8_t *px = base + ((size_t)iy * p.w + ix) * 3;
+#pragma unroll
+                for (int c = 0; c < 3; c++)
+                    x[(kh * 3 + kw) * 3 + c] = ok ? ((float)((int)__ldg(px + c) - 128) * 0.0078125f) : 0.0f;
+            }
+        }
+        int plane;
+        int64_t L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, f, oy, ox, plane);
+#pragma unroll
+        for (int cc = 0; cc < 4; cc++) {
+            float acc[8];
+#pragma unroll
+            for (int j = 0; j < 8; j++) acc[j] = 0.0f;
+#pragma unroll
+            for (int k = 0; k < 27; k++) {
+#pragma unroll
+                for (int j = 0; j < 8; j++) acc[j] = fmaf(sw[k * 32 + cc * 8 + j], x[k], acc[j]);
+            }
+            uint32_t pk[4];
+#pragma unroll
+            for (int j = 0; j < 4; j++) {
+                float a = fmaxf(acc[2 * j] + sb[cc * 8 + 2 * j], 0.0f);
+                float b = fmaxf(acc[2 * j + 1] + sb[cc * 8 + 2 * j + 1], 0.0f);
+                pk[j] = pack_bf16x2(a, b);
+            }
+            uint8_t *dst = p.out + (((size_t)plane * 4 + cc) * p.out_lcap + L) * 16;
+            *reinterpret_cast<uint4 *>(dst) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// E2..E5, D1: persistent warp-specialised implicit-GEMM conv on tcgen05
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid_constant__ ConvParams p) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+
+    const uint32_t chunks = p.kb >> 3;
+    const uint32_t a_bytes = chunks * p.P * 16;
+    const uint32_t b_bytes = (uint32_t)p.N * p.kb * 2;
+    uint8_t *a_buf = smem;
+    uint8_t *b_buf = a_buf + (size_t)p.stages_a * a_bytes;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(b_buf + (size_t)p.stages_b * b_bytes);
+    uint64_t *a_full = bars;
+    uint64_t *a_empty = a_full + kMaxStagesA;
+    uint64_t *b_full = a_empty + kMaxStagesA;
+    uint64_t *b_empty = b_full + kMaxStagesB;
+    uint64_t *t_full = b_empty + kMaxStagesB;   // 2 accumulator stages
+    uint64_t *t_empty = t_full + 2;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(t_empty + 2);
+    float *s_bias = reinterpret_cast<float *>(tmem_slot + 4);
+    float *s_w2 = s_bias + 256;
+
+    const uint32_t tmem_cols = p.N * 2 <= 32 ? 32 : (p.N * 2 <= 64 ? 64 : (p.N * 2 <= 128 ? 128 : (p.N * 2 <= 256 ? 256 : 512)));
+
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < p.stages_a; i++) { mbar_init(&a_full[i], 1); mbar_init(&a_empty[i], 1); }
+        for (int i = 0; i < p.stages_b; i++) { mbar_init(&b_full[i], 1); mbar_init(&b_empty[i], 1); }
+        for (int i = 0; i < 2; i++) { mbar_init(&t_full[i], 1); mbar_init(&t_empty[i], 128); }
+        fence_barrier_init();
+    }
+    if (warp == 2) tmem_alloc(tmem_slot, tmem_cols);
+    for (int i = threadIdx.x; i < p.N; i += blockDim.x) {
+        s_bias[i] = p.bias[i];
+        if (p.out_kind == 3) s_w2[i] = p.w2[i];
+    }
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        // ===== producer: halo (A) and weight (B) bulk copies =====
+        if (lane == 0) {
+            uint32_t as = 0, ap = 0, bs = 0, bp = 0;
+            for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+                const int64_t q0 = (int64_t)tile * kTileM;
+                int tap_pos = 0;
+                for (int cb = 0; cb < p.ncb; cb++) {
+                    tap_pos = 0;
+                    for (int g = 0; g < p.ngroups; g++) {
+                        mbar_wait(&a_empty[as], ap ^ 1);
+                        mbar_arrive_expect_tx(&a_full[as], a_bytes);
+                        uint8_t *dst = a_buf + (size_t)as * a_bytes;
+                        const int plane = p.group_plane[g];
+                        for (uint32_t j = 0; j < chunks; j++) {
+                            const uint8_t *src =
+                                p.act + (((int64_t)plane * p.c8_in + cb * chunks + j) * p.lcap + q0) * 16;
+                            bulk_g2s(dst + j * p.P * 16, src, p.P * 16, &a_full[as]);
+                        }
+                        if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
+                        for (int t = 0; t < p.group_ntaps[g]; t++, tap_pos++) {
+                            mbar_wait(&b_empty[bs], bp ^ 1);
+                            mbar_arrive_expect_tx(&b_full[bs], b_bytes);
+                            bulk_g2s(b_buf + (size_t)bs * b_bytes, p.wpk + ((size_t)cb * 9 + tap_pos) * b_bytes, b_bytes,
+                                     &b_full[bs]);
+                            if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
+                        }
+                    }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ===== MMA issuer (single thread) =====
+        if (lane == 0) {
+            const uint32_t idesc = umma_idesc_bf16(kTileM, p.N);
+            uint32_t as = 0, ap = 0, bs = 0, bp = 0, acc = 0, accp = 0;
+            const uint32_t a_base = smem_u32(a_buf), b_base = smem_u32(b_buf);
+            const uint32_t lbo_a = p.P * 16, lbo_b = p.N * 16;
+            for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+                mbar_wait(&t_empty[acc], accp ^ 1);
+                tc_fence_after();
+                const uint32_t d = tmem_base + acc * p.N;
+                uint32_t accumulate = 0;
+                for (int cb = 0; cb < p.ncb; cb++) {
+                    for (int g = 0; g < p.ngroups; g++) {
+                        mbar_wait(&a_full[as], ap);
+                        tc_fence_after();
+                        const uint32_t a_stage = a_base + as * a_bytes;
+                        for (int t = 0; t < p.group_ntaps[g]; t++) {
+                            mbar_wait(&b_full[bs], bp);
+                            tc_fence_after();
+                            const uint32_t a_tap = a_stage + p.group_shift[g][t] * 16;
+                            const uint32_t b_stage = b_base + bs * b_bytes;
+                            for (uint32_t s = 0; s < chunks / 2; s++) {
+                                uint64_t ad = umma_desc(a_tap + 2 * s * lbo_a, lbo_a, 128);
+                                uint64_t bd = umma_desc(b_stage + 2 * s * lbo_b, lbo_b, 128);
+                                umma_bf16(d, ad, bd, idesc, accumulate);
+                                accumulate = 1;
+                            }
+                            umma_commit(&b_empty[bs]);
+                            if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
+                        }
+                        umma_commit(&a_empty[as]);
+                        if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
+                    }
+                }
+                umma_commit(&t_full[acc]);
+                if (++acc == 2) { acc = 0; accp ^= 1; }
+            }
+        }
+    } else if (warp >= 4) {
+        // ===== epilogue: TMEM -> regs -> bias, ReLU, bf16 -> next layer's layout =====
+        const int row = threadIdx.x - 128;          // TMEM lane == tile row
+        const int quarter = warp & 3;               // lanes 32*quarter .. +31
+        uint32_t acc = 0, accp = 0;
+        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+            mbar_wait(&t_full[acc], accp);
+            tc_fence_after();
+            const int64_t q = (int64_t)tile * kTileM + row;
+            const int f = (int)(q / p.fstride);
+            const int64_t r = q - (int64_t)f * p.fstride;
+            const int oy = (int)(r / p.pitch);
+            const int ox = (int)(r - (int64_t)oy * p.pitch);
+            const bool valid = q < p.mtot && oy < p.out_h && ox < p.out_w;
+            int plane = 0;
+            int64_t L = 0;
+            if (p.out_kind != 3) L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, f, oy, ox, plane);
+            const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * p.N;
+            float z = p.b2;
+            for (int cc = 0; cc < p.N / 32; cc++) {
+                uint32_t v[32];
+                tmem_ld32(taddr + cc * 32, v);
+                uint32_t pk[16];
+#pragma unroll
+                for (int j = 0; j < 16; j++) {
+                    float a = fmaxf(__uint_as_float(v[2 * j]) + s_bias[cc * 32 + 2 * j], 0.0f);
+                    float b = fmaxf(__uint_as_float(v[2 * j + 1]) + s_bias[cc * 32 + 2 * j + 1], 0.0f);
+                    pk[j] = pack_bf16x2(a, b);
+                }
+                if (p.out_kind == 3) {
+#pragma unroll
+                    for (int j = 0; j < 16; j++) {
+                        float a = __uint_as_float(pk[j] << 16);
+                        float b = __uint_as_float(pk[j] & 0xFFFF0000u);
+                        z = fmaf(s_w2[cc * 32 + 2 * j], a, z);
+                        z = fmaf(s_w2[cc * 32 + 2 * j + 1], b, z);
+                    }
+                } else if (valid) {
+#pragma unroll
+                    for (int c = 0; c < 4; c++) {
+                        uint8_t *dst = p.out + (((int64_t)plane * p.out_c8 + cc * 4 + c) * p.out_lcap + L) * 16;
+                        *reinterpret_cast<uint4 *>(dst) = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+                    }
+                }
+            }
+            if (p.out_kind == 3 && valid)
+                p.scores[((int64_t)f * p.out_h + oy) * p.out_w + ox] = 1.0f / (1.0f + expf(-z));
+            tc_fence_before();
+            mbar_arrive(&t_empty[acc]);
+            if (++acc == 2) { acc = 0; accp ^= 1; }
+        }
+    }
+    __syncwarp();
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        tmem_dealloc(tmem_base, tmem_cols);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// host side: plan, weight packing, launch
+// ---------------------------------------------------------------------------
+static uint16_t f32_to_bf16_rne(float f) {
+    uint32_t u;
+    memcpy(&u, &f, 4);
+    uint32_t lsb = (u >> 16) & 1u;
+    u += 0x7FFFu + lsb;
+    return (uint16_t)(u >> 16);
+}
+static float bf16_to_f32(uint16_t b) {
+    uint32_t u = (uint32_t)b << 16;
+    float f;
+    memcpy(&f, &u, 4);
+    return f;
+}
+
+struct GemmLayer {
+    int cin, cout, stride, in_h, in_w, out_h, out_w;
+    int kind;                     // input layout kind
+    int pitch;
+    int64_t fstride_unit;         // per-frame pixels of the input layout
+    int max_shift;
+    int ngroups, group_plane[4], group_ntaps[4], group_shift[4][9], group_tap[4][9];
+    int kb, ncb, P;
+    uint8_t *wpk_dev;
+    float *bias_dev;
+};
+
+}  // namespace otif
+
+struct otif_proxy {
+    otif_proxy_desc d;
+    int gh, gw;
+    int e1_oh, e1_ow;
+    otif::GemmLayer L[5];         // E2, E3, E4, E5, D1
+    float *e1_w_dev, *e1_b_dev;   // [27][32], [32]
+    float *w2_dev;                // [dec] bf16-rounded
+    float b2;
+    int num_sms;
+    uint64_t plan_hash;
+};
+
+namespace otif {
+
+static void build_layer(GemmLayer &g, int cin, int cout, int stride, int in_h, int in_w) {
+    g.cin = cin; g.cout = cout; g.stride = stride; g.in_h = in_h; g.in_w = in_w;
+    g.out_h = (in_h + stride - 1) / stride;
+    g.out_w = (in_w + stride - 1) / stride;
+    g.kb = cin < 64 ? cin : 64;
+    g.ncb = cin / g.kb;
+    for (int i = 0; i < 4; i++) g.group_ntaps[i] = 0;
+    if (stride == 1) {
+        g.kind = 1;
+        g.pitch = in_w + 2;
+        g.fstride_unit = (int64_t)(in_h + 1) * g.pitch;
+        g.max_shift = 2 * g.pitch + 2;
+        g.ngroups = 1;
+        g.group_plane[0] = 0;
+        for (int t = 0; t < 9; t++) {
+            g.group_tap[0][t] = t;
+            g.group_shift[0][t] = (t / 3) * g.pitch + (t % 3);
+        }
+        g.group_ntaps[0] = 9;
+    } else {
+        g.kind = 2;
+        g.pitch = g.out_w + 1;
+        g.fstride_unit = (int64_t)(g.out_h + 1) * g.pitch;
+        g.max_shift = g.pitch + 1;
+        // plane (rp, cp): rp = (kh != 1), cp = (kw != 1); shift = (kh != 0)*pitch + (kw != 0)
+        int ng = 0;
+        for (int plane = 0; plane < 4; plane++) {
+            int cnt = 0;
+            for (int t = 0; t < 9; t++) {
+                int kh = t / 3, kw = t % 3;
+                int pl = ((kh != 1) << 1) | (kw != 1);
+                if (pl != plane) continue;
+                g.group_tap[ng][cnt] = t;
+                g.group_shift[ng][cnt] = (kh != 0) * g.pitch + (kw != 0);
+                cnt++;
+            }
+            g.group_plane[ng] = plane;
+            g.group_ntaps[ng] = cnt;
+            ng++;
+        }
+        g.ngroups = ng;
+    }
+    g.P = (int)round_up(kTileM + g.max_shift, 8);
+}
+
+static Layout input_layout(const GemmLayer &g, int n) {
+    Layout l;
+    l.kind = g.kind;
+    l.planes = g.kind == 1 ? 1 : 4;
+    l.pitch = g.pitch;
+    l.fstride = g.fstride_unit;
+    int64_t mtot = (int64_t)n * g.fstride_unit;
+    l.lcap = round_up(round_up(mtot, kTileM) + g.max_shift + 8, 16);
+    l.c8 = g.cin / 8;
+    l.bytes = (size_t)l.planes * l.c8 * l.lcap * 16;
+    l.offset = 0;
+    return l;
+}
+
+static size_t plan_workspace(const otif_proxy *p, int n, Layout lay[5]) {
+    size_t off = 256;  // tag header
+    for (int i = 0; i < 5; i++) {
+        lay[i] = input_layout(p->L[i], n);
+        lay[i].offset = off;
+        off += round_up(lay[i].bytes, 256);
+    }
+    return off;
+}
+
+static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
+    size_t a = (size_t)(g.kb / 8) * g.P * 16;
+    size_t b = (size_t)g.cout * g.kb * 2;
+    size_t fixed = (2 * kMaxStagesA + 2 * kMaxStagesB + 4) * 8 + 16 + 2 * 256 * 4 + 1024;
+    size_t budget = 220 * 1024;
+    sa = 2; sb = 2;
+    // grow B (weights stream every tap) first, then A
+    while (sb < kMaxStagesB && sa * a + (sb + 1) * b + fixed <= budget && sb < 6) sb++;
+    while (sa < kMaxStagesA && (sa + 1) * a + sb * b + fixed <= budget && sa < 3) sa++;
+    bytes = sa * a + sb * b + fixed;
+}
+
+static otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws,
+                                size_t ws_bytes, cudaStream_t stream) {
+    Layout lay[5];
+    size_t need = plan_workspace(p, n, lay);
+    if (ws_bytes < need) {
+        set_error("otif_proxy_score: workspace %zu B < required %zu B", ws_bytes, need);
+        return OTIF_ENOMEM;
+    }
+    const uint64_t tag = p->plan_hash ^ ((uint64_t)n * 0x9E3779B97F4A7C15ull) ^ (uint64_t)need;
+    ws_zero_kernel<<<p->num_sms * 4, 256, 0, stream>>>(ws, need, tag);
+    OTIF_LAUNCH_CHECK();
+    ws_tag_kernel<<<1, 1, 0, stream>>>(ws, tag);
+    OTIF_LAUNCH_CHECK();
+
+    // E1
+    {
+        E1Params e;
+        e.img = img; e.n = n; e.h = p->d.in_h; e.w = p->d.in_w; e.oh = p->e1_oh; e.ow = p->e1_ow;
+        e.wt = p->e1_w_dev; e.bias = p->e1_b_dev;
+        e.out_kind = lay[0].kind; e.out_pitch = lay[0].pitch; e.out_fstride = lay[0].fstride;
+        e.out_lcap = lay[0].lcap; e.out = ws + lay[0].offset;
+        int64_t total = (int64_t)n * e.oh * e.ow;
+        int64_t blocks = cdiv(total, 256);
+        if (blocks > (int64_t)p->num_sms * 16) blocks = (int64_t)p->num_sms * 16;
+        if (blocks < 1) blocks = 1;
+        e1_kernel<<<(unsigned)blocks, 256, 0, stream>>>(e);
+        OTIF_LAUNCH_CHECK();
+    }
+    // E2..E5, D1
+    for (int li = 0; li < 5; li++) {
+        const GemmLayer &g = p->L[li];
+        ConvParams c;
+        memset(&c, 0, sizeof(c));
+        c.act = ws + lay[li].offset;
+        c.lcap = lay[li].lcap;
+        c.c8_in = g.cin / 8;
+        c.kb = g.kb; c.ncb = g.ncb; c.P = g.P; c.ngroups = g.ngroups;
+        for (int i = 0; i < 4; i++) {
+            c.group_plane[i] = g.group_plane[i];
+            c.group_ntaps[i] = g.group_ntaps[i];
+            for (int t = 0; t < 9; t++) c.group_shift[i][t] = g.group_shift[i][t];
+        }
+        c.wpk = g.wpk_dev; c.bias = g.bias_dev; c.N = g.cout;
+        c.mtot = (int64_t)n * g.fstride_unit;
+        c.ntiles = (int)cdiv(c.mtot, kTileM);
+        c.pitch = g.pitch; c.fstride = g.fstride_unit; c.out_h = g.out_h; c.out_w = g.out_w;
+        if (li < 4) {
+            c.out_kind = lay[li + 1].kind;
+            c.out = ws + lay[li + 1].offset;
+            c.out_lcap = lay[li + 1].lcap;
+            c.out_c8 = lay[li + 1].c8;
+            c.out_pitch = lay[li + 1].pitch;
+            c.out_fstride = lay[li + 1].fstride;
+        } else {
+            c.out_kind = 3;
+            c.scores = scores;
+            c.w2 = p->w2_dev;
+            c.b2 = p->b2;
+        }
+        size_t smem;
+        conv_smem(g, c.stages_a, c.stages_b, smem);
+        OTIF_CUDA(cudaFuncSetAttribute(conv_umma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
+        if (grid < 1) grid = 1;
+        conv_umma_kernel<<<grid, kConvThreads, smem, stream>>>(c);
+        OTIF_LAUNCH_CHECK();
+    }
+    return OTIF_OK;
+}
+
+}  // namespace otif
+
+// ---------------------------------------------------------------------------
+// C ABI
+// ---------------------------------------------------------------------------
+using namespace otif;
+
+static bool width_ok(int c) { return c == 64 || c == 128 || c == 256; }
+
+extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *weights, size_t n_weights,
+                                         otif_proxy **out) {
+    OTIF_REQUIRE(d && weights && out, "otif_proxy_create: NULL argument");
+    OTIF_REQUIRE(d->in_h > 0 && d->in_w > 0, "otif_proxy_create: bad input size %dx%d", d->in_w, d->in_h);
+    OTIF_REQUIRE(d->n_strided >= 1 && d->n_strided <= 5, "otif_proxy_create: n_strided %d not in [1,5]", d->n_strided);
+    if (d->enc[0] != 32 || !width_ok(d->enc[1]) || !width_ok(d->enc[2]) || !width_ok(d->enc[3]) ||
+        !width_ok(d->enc[4]) || !width_ok(d->dec)) {
+        set_error("otif_proxy_create: widths (%d,%d,%d,%d,%d|%d) unsupported (enc[0]=32, others in {64,128,256})",
+                  d->enc[0], d->enc[1], d->enc[2], d->enc[3], d->enc[4], d->dec);
+        return OTIF_EUNSUPPORTED;
+    }
+    int num_sms = 0;
+    otif_status st = check_device(&num_sms);
+    if (st != OTIF_OK) return st;
+
+    // expected blob size
+    int cin[7], cout[7], ks[7];
+    {
+        int c = 3;
+        for (int i = 0; i < 5; i++) { cin[i] = c; cout[i] = d->enc[i]; ks[i] = 3; c = d->enc[i]; }
+        cin[5] = c; cout[5] = d->dec; ks[5] = 3;
+        cin[6] = d->dec; cout[6] = 1; ks[6] = 1;
+    }
+    size_t offs[7], total = 0;
+    for (int i = 0; i < 7; i++) { offs[i] = total; total += (size_t)cout[i] * ks[i] * ks[i] * cin[i] + cout[i]; }
+    OTIF_REQUIRE(n_weights == total, "otif_proxy_create: n_weights %zu != %zu for this shape", n_weights, total);
+
+    otif_proxy *p = new (std::nothrow) otif_proxy();
+    if (!p) return OTIF_ENOMEM;
+    p->d = *d;
+    p->num_sms = num_sms;
+    // spatial chain
+    int h = d->in_h, w = d->in_w;
+    int hs[7], wss[7];
+    for (int i = 0; i < 6; i++) {
+        hs[i] = h; wss[i] = w;
+        int s = (i < 5 && i < d->n_strided) ? 2 : 1;
+        h = (h + s - 1) / s; w = (w + s - 1) / s;
+    }
+    p->gh = h; p->gw = w;
+    p->e1_oh = (d->in_h + 1) / 2;
+    p->e1_ow = (d->in_w + 1) / 2;
+
+    otif_status rc = OTIF_OK;
+    std::vector<float> host;
+    // E1 weights -> [27][32] with k = (kh*3+kw)*3 + c
+    {
+        std::vector<float> w1(27 * 32), b1(32);
+        for (int o = 0; o < 32; o++) {
+            for (int kh = 0; kh < 3; kh++)
+                for (int kw = 0; kw < 3; kw++)
+                    for (int c = 0; c < 3; c++) {
+                        float v = weights[offs[0] + ((size_t)(o * 3 + kh) * 3 + kw) * 3 + c];
+                        w1[((kh * 3 + kw) * 3 + c) * 32 + o] = bf16_to_f32(f32_to_bf16_rne(v));
+                    }
+            b1[o] = weights[offs[0] + (size_t)32 * 27 + o];
+        }
+        if (cudaMalloc(&p->e1_w_dev, w1.size() * 4) != cudaSuccess || cudaMalloc(&p->e1_b_dev, 32 * 4) != cudaSuccess) {
+            rc = OTIF_ENOMEM;
+        } else {
+            cudaMemcpy(p->e1_w_dev, w1.data(), w1.size() * 4, cudaMemcpyHostToDevice);
+            cudaMemcpy(p->e1_b_dev, b1.data(), 32 * 4, cudaMemcpyHostToDevice);
+        }
+    }
+    // GEMM layers E2..E5 (layer index 1..4) and D1 (5)
+    for (int li = 0; li < 5 && rc == OTIF_OK; li++) {
+        int layer = li + 1;
+        int s = (layer < 5 && layer < d->n_strided) ? 2 : 1;
+        GemmLayer &g = p->L[li];
+        build_layer(g, cin[layer], cout[layer], s, hs[layer], wss[layer]);
+        // pack: [cb][tap in loop order][chunk j][n][8]
+        const int chunks = g.kb / 8;
+        std::vector<uint16_t> pk((size_t)g.ncb * 9 * chunks * g.cout * 8);
+        const float *W = weights + offs[layer];
+        for (int cb = 0; cb < g.ncb; cb++) {
+            int pos = 0;
+            for (int gi = 0; gi < g.ngroups; gi++)
+                for (int t = 0; t < g.group_ntaps[gi]; t++, pos++) {
+                    int tap = g.group_tap[gi][t];
+                    int kh = tap / 3, kw = tap % 3;
+                    for (int j = 0; j < chunks; j++)
+                        for (int nn = 0; nn < g.cout; nn++)
+                            for (int e = 0; e < 8; e++) {
+                                int ci = cb * g.kb + j * 8 + e;
+                                float v = W[(((size_t)nn * 3 + kh) * 3 + kw) * g.cin + ci];
+                                pk[((((size_t)cb * 9 + pos) * chunks + j) * g.cout + nn) * 8 + e] = f32_to_bf16_rne(v);
+                            }
+                }
+        }
+        std::vector<float> bias(g.cout);
+        for (int nn = 0; nn < g.cout; nn++) bias[nn] = W[(size_t)g.cout * 9 * g.cin + nn];
+        if (cudaMalloc(&g.wpk_dev, pk.size() * 2) != cudaSuccess || cudaMalloc(&g.bias_dev, g.cout * 4) != cudaSuccess) {
+            rc = OTIF_ENOMEM;
+            break;
+        }
+        cudaMemcpy(g.wpk_dev, pk.data(), pk.size() * 2, cudaMemcpyHostToDevice);
+        cudaMemcpy(g.bias_dev, bias.data(), g.cout * 4, cudaMemcpyHostToDevice);
+    }
+    // D2 head
+    if (rc == OTIF_OK) {
+        std::vector<float> w2(d->dec);
+        for (int c = 0; c < d->dec; c++) w2[c] = bf16_to_f32(f32_to_bf16_rne(weights[offs[6] + c]));
+        p->b2 = weights[offs[6] + d->dec];
+        if (cudaMalloc(&p->w2_dev, d->dec * 4) != cudaSuccess) rc = OTIF_ENOMEM;
+        else cudaMemcpy(p->w2_dev, w2.data(), d->dec * 4, cudaMemcpyHostToDevice);
+    }
+    // smem feasibility
+    for (int li = 0; li < 5 && rc == OTIF_OK; li++) {
+        int sa, sb;
+        size_t bytes;
+        conv_smem(p->L[li], sa, sb, bytes);
+        if (bytes > 227 * 1024) {
+            set_error("otif_proxy_create: layer %d needs %zu B of shared memory (input too wide)", li + 2, bytes);
+            rc = OTIF_EUNSUPPORTED;
+        }
+    }
+    if (cudaGetLastError() != cudaSuccess && rc == OTIF_OK) rc = OTIF_ECUDA;
+    if (rc != OTIF_OK) {
+        otif_proxy_destroy(p);
+        return rc;
+    }
+    uint64_t hsh = 1469598103934665603ull;
+    auto mix = [&](uint64_t v) { hsh = (hsh ^ v) * 1099511628211ull; };
+    mix(d->in_h); mix(d->in_w); mix(d->n_strided);
+    for (int i = 0; i < 5; i++) mix(d->enc[i]);
+    mix(d->dec);
+    p->plan_hash = hsh | 1;
+    *out = p;
+    return OTIF_OK;
+}
+
+extern "C" void otif_proxy_destroy(otif_proxy *p) {
+    if (!p) return;
+    for (int i = 0; i < 5; i++) {
+        if (p->L[i].wpk_dev) cudaFree(p->L[i].wpk_dev);
+        if (p->L[i].bias_dev) cudaFree(p->L[i].bias_dev);
+    }
+    if (p->e1_w_dev) cudaFree(p->e1_w_dev);
+    if (p->e1_b_dev) cudaFree(p->e1_b_dev);
+    if (p->w2_dev) cudaFree(p->w2_dev);
+    delete p;
+}
+
+extern "C" otif_status otif_proxy_grid(const otif_proxy *p, int32_t *gh, int32_t *gw) {
+    OTIF_REQUIRE(p && gh && gw, "otif_proxy_grid: NULL argument");
+    *gh = p->gh;
+    *gw = p->gw;
+    return OTIF_OK;
+}
+
+extern "C" size_t otif_proxy_workspace_bytes(const otif_proxy *p, int32_t n) {
+    if (!p || n < 0) return 0;
+    Layout lay[5];
+    return plan_workspace(p, n, lay);
+}
+
+extern "C" otif_status otif_proxy_score(const otif_proxy *p, const uint8_t *img, int32_t n, float *scores,
+                                        void *workspace, size_t ws_bytes, cudaStream_t stream) {
+    OTIF_REQUIRE(p, "otif_proxy_score: NULL proxy");
+    OTIF_REQUIRE(n >= 0, "otif_proxy_score: n < 0");
+    if (n == 0) return OTIF_OK;
+    OTIF_REQUIRE(img && scores && workspace, "otif_proxy_score: NULL pointer");
+    OTIF_REQUIRE((((uintptr_t)workspace) & 255) == 0, "otif_proxy_score: workspace must be 256-B aligned");
+    otif_status st = check_device(nullptr);
+    if (st != OTIF_OK) return st;
+    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream);
+}

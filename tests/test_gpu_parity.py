@@ -1,0 +1,221 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, stage by stage on
+identical inputs, then end to end.  Criteria (north_star / SURVEY §8(c)):
+  resize & pack pixels within 1 LSB (identity crops byte-exact); proxy scores within
+  2e-2 of the quant=none oracle; masks bit-exact vs the quant=bf16 oracle except cells
+  within 1e-3 of the threshold; windows bit-exact given the same mask."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth import configs, video, weights
+from tests.helpers import BAND, as_tuples, oracle_scores, threshold, windows_np
+
+pytestmark = pytest.mark.gpu
+
+otif = pytest.importorskip("paper_conf_sigmod_bastanim22_b200")
+
+
+@pytest.fixture(scope="module")
+def blob():
+    return weights.proxy_weights()
+
+
+def _frames(wl, n, start=0):
+    return video.frames(wl, n, start=start)
+
+
+# ------------------------------------------------------------------ stage 1
+@pytest.mark.parametrize("wl,n,dh,dw", [
+    (configs.C1, 32, 64, 104), (configs.C2, 6, 135, 240), (configs.C3, 3, 270, 480),
+    (configs.C3, 2, 540, 960), (configs.C4_BASE, 3, 90, 160), (configs.C4_BASE, 2, 187, 333),
+    (configs.C1, 2, 300, 500)])
+def test_resize_parity(wl, n, dh, dw):
+    src = _frames(wl, n)
+    ref = oracle.resize(src.numpy(), dh, dw)
+    got = otif.otif_resize(src.cuda(), dh, dw).cpu().numpy()
+    d = np.abs(got.astype(np.int32) - ref)
+    assert d.max() <= 1
+    assert (d == 0).mean() > 0.95
+
+
+def test_resize_constant_and_identity():
+    src = torch.full((3, 135, 240, 3), 77, dtype=torch.uint8)
+    assert (otif.otif_resize(src.cuda(), 34, 60).cpu() == 77).all()
+    fr = _frames(configs.C1, 4)
+    assert torch.equal(otif.otif_resize(fr.cuda(), 256, 416).cpu(), fr)
+
+
+# ------------------------------------------------------------------ stage 2
+PROXY_CASES = [
+    (configs.C1, 32),        # S = 8, 8x13 grid, 32 frames (D1: 34 M-tiles, ragged tail)
+    (configs.C2, 4),         # S = 8, 17x30
+    (configs.C3, 2),         # S = 16 (c = 64, r = 1/4)
+    (configs.C4_SWEEP[2], 2),  # S = 4 (r = 1/8, c = 32): only E1, E2 strided
+    (configs.C4_SWEEP[3], 2),  # S = 32 (r = 1/2, c = 64): all five strided (the paper's case)
+]
+
+
+@pytest.mark.parametrize("wl,n", PROXY_CASES, ids=[c[0].name for c in PROXY_CASES])
+def test_proxy_parity(wl, n, blob):
+    src = _frames(wl, n)
+    img = oracle.resize(src.numpy(), wl.proxy_h, wl.proxy_w)
+    px = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, blob)
+    got = px.score(torch.from_numpy(img).cuda()).cpu().numpy().astype(np.float64)
+    ref_none = oracle_scores(img, wl, blob, oracle.QUANT_NONE)
+    ref_bf16 = oracle_scores(img, wl, blob, oracle.QUANT_BF16)
+    assert got.shape == ref_bf16.shape
+    assert np.abs(got - ref_none).max() <= 2e-2
+    # masks: bit-exact outside the 1e-3 band around each frozen threshold
+    for q in (0.5, 0.7, 0.9):
+        b = threshold(wl.name if wl.name in ("C1", "C2", "C3") else wl.name, q)
+        far = np.abs(ref_bf16 - b) > BAND
+        assert np.array_equal((got > np.float32(b))[far], (ref_bf16 > b)[far])
+
+
+def test_proxy_repeat_calls_reuse_workspace(blob):
+    wl = configs.C1
+    img = torch.from_numpy(oracle.resize(_frames(wl, 8).numpy(), wl.proxy_h, wl.proxy_w)).cuda()
+    px = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, blob)
+    a = px.score(img).clone()
+    b = px.score(img).clone()
+    c = px.score(img[:3]).clone()       # different n -> re-initialised workspace
+    d = px.score(img).clone()
+    assert torch.equal(a, b) and torch.equal(a[:3], c) and torch.equal(a, d)
+
+
+# ------------------------------------------------------------------ stages 3 + 4
+def _random_masks(rng, n, gh, gw):
+    out = np.zeros((n, gh, gw), np.uint8)
+    for f in range(n):
+        kind = f % 6
+        if kind == 0:
+            continue                                                    # empty
+        elif kind == 1:
+            out[f] = 1                                                  # full
+        elif kind == 2:
+            out[f] = (np.add.outer(np.arange(gh), np.arange(gw)) % 2 == 0)  # checkerboard
+        else:
+            out[f] = rng.random((gh, gw)) < rng.uniform(0.02, 0.5)
+    return out
+
+
+SELECT_CASES = [(configs.C1, 4), (configs.C2, 4), (configs.C3, 4), (configs.C4_SWEEP[0], 4),
+                (configs.C2, 8)]
+
+
+@pytest.mark.parametrize("wl,conn", SELECT_CASES, ids=[f"{c[0].name}-{c[1]}" for c in SELECT_CASES])
+def test_select_windows_mask_parity(wl, conn):
+    rng = np.random.default_rng(hash(wl.name) % 1000 + conn)
+    gh, gw = -(-wl.src_h // wl.cell), -(-wl.src_w // wl.cell)
+    masks = _random_masks(rng, 60, gh, gw)
+    # add ground-truth masks of the workload's own video (perfect proxy)
+    sc = video.make_scene(wl)
+    gt = np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell) for t in range(20)])
+    masks = np.concatenate([masks, gt])
+    ref_w, ref_c, ref_o, ref_t = oracle.select_windows(masks, wl.cell, wl.src_w, wl.src_h, wl.sizes, conn)
+    r = otif.otif_select_windows(None, torch.from_numpy(masks).cuda(), 0.0, wl.src_w, wl.src_h, wl.cell,
+                                 wl.sizes, connectivity=conn, want_mask=True)
+    total = int(r["total"].item())
+    assert total == ref_t
+    assert np.array_equal(r["counts"].cpu().numpy(), ref_c)
+    assert np.array_equal(r["offsets"].cpu().numpy(), ref_o)
+    assert as_tuples(windows_np(r["windows"], total)) == as_tuples(ref_w)
+    assert np.array_equal(r["mask"].cpu().numpy(), masks)
+
+
+def test_select_scores_input_and_capacity(blob):
+    wl = configs.C1
+    rng = np.random.default_rng(3)
+    scores = rng.random((40, 8, 13)).astype(np.float32)
+    b = 0.8
+    mask = oracle.threshold(scores.astype(np.float64), b)
+    ref_w, ref_c, ref_o, ref_t = oracle.select_windows(mask, 32, 416, 256, wl.sizes)
+    r = otif.otif_select_windows(torch.from_numpy(scores).cuda(), None, b, 416, 256, 32, wl.sizes, want_mask=True)
+    assert np.array_equal(r["mask"].cpu().numpy(), mask)
+    t = int(r["total"].item())
+    assert t == ref_t and as_tuples(windows_np(r["windows"], t)) == as_tuples(ref_w)
+    # capacity overflow: total and counts exact, first `capacity` windows kept
+    r2 = otif.otif_select_windows(torch.from_numpy(scores).cuda(), None, b, 416, 256, 32, wl.sizes, capacity=5)
+    assert int(r2["total"].item()) == ref_t
+    assert as_tuples(windows_np(r2["windows"], 5)) == as_tuples(ref_w[:5])
+
+
+def test_select_rejects_bad_arguments():
+    m = torch.zeros((1, 8, 13), dtype=torch.uint8, device="cuda")
+    with pytest.raises(Exception):
+        otif.otif_select_windows(None, m, 0.0, 416, 256, 32, [(64, 64)])              # no full frame
+    with pytest.raises(Exception):
+        otif.otif_select_windows(None, m, 0.0, 416, 256, 31, [(64, 64), (416, 256)])  # grid mismatch
+    with pytest.raises(Exception):
+        otif.otif_select_windows(None, m, 0.0, 416, 256, 32, [(64, 64), (416, 256)], connectivity=6)
+
+
+# ------------------------------------------------------------------ stage 5
+@pytest.mark.parametrize("wl", [configs.C1, configs.C2, configs.C3], ids=lambda w: w.name)
+def test_pack_identity_parity(wl):
+    n = 6
+    src = _frames(wl, n)
+    sc = video.make_scene(wl)
+    masks = np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell) for t in range(n)])
+    win, cnt, off, tot = oracle.select_windows(masks, wl.cell, wl.src_w, wl.src_h, wl.sizes)
+    caps = [int((win["size_idx"] == s).sum()) for s in range(len(wl.sizes))]
+    ref_b, ref_slot, ref_cnt = oracle.pack_windows(src.numpy(), wl.src_h, wl.src_w, win, wl.sizes, caps)
+    wt = torch.from_numpy(np.stack([win[f] for f in oracle.WINDOW_DTYPE.names], 1).astype(np.int32)).cuda()
+    total = torch.tensor([tot], dtype=torch.int32, device="cuda")
+    b, slot, scount = otif.otif_pack_windows(src.cuda(), wl.src_h, wl.src_w, wt, total, wl.sizes, caps)
+    assert np.array_equal(slot[:tot].cpu().numpy(), ref_slot)
+    assert np.array_equal(scount.cpu().numpy(), ref_cnt)
+    for s in range(len(wl.sizes)):
+        assert np.array_equal(b[s].cpu().numpy(), ref_b[s])
+
+
+def test_pack_resample_and_drops():
+    wl = configs.C4_BASE
+    src = _frames(wl, 2)
+    det_h, det_w = 360, 640
+    sizes = [(128, 128), (640, 360)]
+    rows = [(0, 5, 7, 128, 128, 0), (1, 0, 0, 640, 360, 1), (1, 512, 232, 128, 128, 0), (0, 3, 1, 128, 128, 0)]
+    win = np.zeros(len(rows), oracle.WINDOW_DTYPE)
+    for i, r in enumerate(rows):
+        win[i] = r
+    caps = [2, 1]
+    ref_b, ref_slot, ref_cnt = oracle.pack_windows(src.numpy(), det_h, det_w, win, sizes, caps)
+    wt = torch.tensor(rows, dtype=torch.int32, device="cuda")
+    total = torch.tensor([len(rows)], dtype=torch.int32, device="cuda")
+    b, slot, scount = otif.otif_pack_windows(src.cuda(), det_h, det_w, wt, total, sizes, caps)
+    assert np.array_equal(scount.cpu().numpy(), ref_cnt) and list(ref_cnt) == [3, 1]
+    assert np.array_equal(slot[:4].cpu().numpy(), ref_slot)
+    for s in range(2):
+        assert np.abs(b[s].cpu().numpy().astype(np.int32) - ref_b[s]).max() <= 1
+
+
+# ------------------------------------------------------------------ end to end
+def test_end_to_end_c1(blob):
+    """C1 (32 frames, oracle in seconds): GPU resize -> proxy -> select -> pack."""
+    wl = configs.C1
+    b = threshold("C1", 0.7)
+    src = _frames(wl, wl.n_frames)
+    src_d = src.cuda()
+    img_d = otif.otif_resize(src_d, wl.proxy_h, wl.proxy_w)
+    px = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, blob)
+    scores_d = px.score(img_d)
+    r = otif.otif_select_windows(scores_d, None, b, wl.src_w, wl.src_h, wl.cell, wl.sizes, want_mask=True)
+    total = int(r["total"].item())
+    gw_ = windows_np(r["windows"], total)
+    caps = [int((gw_["size_idx"] == s).sum()) for s in range(len(wl.sizes))]
+    batches, slot, scount = otif.otif_pack_windows(src_d, wl.src_h, wl.src_w, r["windows"], r["total"], wl.sizes, caps)
+    # oracle chain on the same frames
+    img = oracle.resize(src.numpy(), wl.proxy_h, wl.proxy_w)
+    ref_s = oracle_scores(img, wl, blob)
+    ref_mask = oracle.threshold(ref_s, b)
+    gmask = r["mask"].cpu().numpy()
+    far = np.abs(ref_s - b) > BAND
+    assert np.array_equal(gmask[far], ref_mask[far])
+    # windows are bit-exact given the same mask: feed the GPU mask to the oracle
+    ow, oc, oo, ot = oracle.select_windows(gmask, wl.cell, wl.src_w, wl.src_h, wl.sizes)
+    assert ot == total and as_tuples(ow) == as_tuples(gw_)
+    ob, oslot, ocnt = oracle.pack_windows(src.numpy(), wl.src_h, wl.src_w, ow, wl.sizes, caps)
+    assert np.array_equal(scount.cpu().numpy(), ocnt)
+    for s in range(len(wl.sizes)):
+        assert np.array_equal(batches[s].cpu().numpy(), ob[s])
