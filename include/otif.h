@@ -176,15 +176,27 @@ otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *src_host, in
                                    otif_window *windows_out, int32_t cap_windows,
                                    int32_t *frame_count_out, int32_t *total_out,
                                    int32_t *size_count_out);
-/* Same path on frames already resident in device memory; results stay on the
- * device in the pipeline's buffers (otif_pipeline_last_* accessors) for the LAST
- * batch; totals are accumulated on the device.  Enqueued on `stream`. */
+/* Same path on frames already resident in device memory, enqueued on `stream`
+ * without any host synchronisation.  Windows and detector batches of each device
+ * batch stay in the pipeline's device buffers (overwritten batch by batch); the
+ * counters below accumulate on the device across calls until reset. */
 otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t *src_dev, int32_t n,
                                      cudaStream_t stream);
-/* Device pointer to int64[4 + k] counters accumulated since create/reset:
- * frames, positive cells, windows, window pixels, then windows per size. */
+/* Device pointer to int64[5 + k] counters accumulated since create/reset (run_host
+ * resets them at its start): frames, positive cells, windows, window pixels, an
+ * order-independent hash of all windows (sum of 64-bit mixes of (frame,x,y,w,h,s)),
+ * then windows per size. */
 const int64_t *otif_pipeline_counters(const otif_pipeline *p);
 otif_status otif_pipeline_reset_counters(otif_pipeline *p, cudaStream_t stream);
+/* Per-stage device timing (CUDA events recorded between the stage launches on the
+ * compute stream).  enable != 0 starts recording (and clears previous records). */
+otif_status otif_pipeline_set_timing(otif_pipeline *p, int32_t enable);
+/* Synchronises on the recorded events and returns the accumulated milliseconds per
+ * stage since the last call: [0] resize, [1] proxy prep (workspace tag + E1),
+ * [2..6] E2, E3, E4, E5, D1+D2 (the tcgen05 GEMM layers), [7] select (K5 + K6),
+ * [8] pack (slots + copy), [9] append; n_ms >= 10.  *launches (optional) = kernels
+ * launched by the pipeline since the last call. */
+otif_status otif_pipeline_stage_ms(otif_pipeline *p, float *ms, int32_t n_ms, int64_t *launches);
 
 #ifdef __cplusplus
 }

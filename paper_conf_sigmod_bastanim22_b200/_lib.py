@@ -92,6 +92,10 @@ def lib() -> ctypes.CDLL:
         L.otif_pipeline_counters.restype = P
         L.otif_pipeline_reset_counters.argtypes = [P, P]
         L.otif_pipeline_reset_counters.restype = st
+        L.otif_pipeline_set_timing.argtypes = [P, i32]
+        L.otif_pipeline_set_timing.restype = st
+        L.otif_pipeline_stage_ms.argtypes = [P, P, i32, P]
+        L.otif_pipeline_stage_ms.restype = st
     _lib = L
     return L
 
@@ -106,4 +110,7 @@ EXPORTED = ("otif_status_str", "otif_last_error", "otif_version", "otif_resize",
             "otif_proxy_destroy", "otif_proxy_grid", "otif_proxy_workspace_bytes", "otif_proxy_score",
             "otif_select_workspace_bytes", "otif_select_windows", "otif_pack_windows",
             "otif_pipeline_create", "otif_pipeline_destroy", "otif_pipeline_run_host",
-            "otif_pipeline_run_device", "otif_pipeline_counters", "otif_pipeline_reset_counters")
+            "otif_pipeline_run_device", "otif_pipeline_counters", "otif_pipeline_reset_counters",
+            "otif_pipeline_set_timing", "otif_pipeline_stage_ms")
+STAGES = ("resize", "proxy_prep_e1", "conv_e2", "conv_e3", "conv_e4", "conv_e5", "conv_d1_head", "select",
+          "pack", "append")

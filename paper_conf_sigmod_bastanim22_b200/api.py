@@ -225,11 +225,22 @@ class Pipeline:
               "otif_pipeline_run_device")
 
     def counters(self) -> torch.Tensor:
-        """int64 [4 + k] device counters: frames, positive cells, windows, window pixels, per-size windows."""
+        """int64 [5 + k] device counters: frames, positive cells, windows, window pixels, hash, per-size."""
         ptr = lib().otif_pipeline_counters(self.handle)
-        n = 4 + self.k
+        n = 5 + self.k
         # wrap the device pointer without copying (read via a torch tensor view)
         return _device_view_i64(ptr, n)
+
+    def set_timing(self, enable: bool = True):
+        check(lib().otif_pipeline_set_timing(self.handle, int(enable)), "otif_pipeline_set_timing")
+
+    def stage_ms(self):
+        """-> (dict stage -> ms accumulated since the last call, kernel launches)."""
+        ms = (ctypes.c_float * len(_lib.STAGES))()
+        launches = ctypes.c_int64()
+        check(lib().otif_pipeline_stage_ms(self.handle, ms, len(_lib.STAGES), ctypes.byref(launches)),
+              "otif_pipeline_stage_ms")
+        return dict(zip(_lib.STAGES, list(ms))), launches.value
 
     def reset_counters(self, stream=None):
         check(lib().otif_pipeline_reset_counters(self.handle, _stream(stream)), "otif_pipeline_reset_counters")

@@ -1,0 +1,348 @@
+// pipeline.cu — the native runtime around the five stages: device buffers sized for
+// one batch, a compute stream and a copy stream, batch loop, and result accumulation
+// (otif_pipeline_*).  The detector batches stay on the device (the detector runs
+// there); windows, per-frame counts and counters are accumulated on the
+// device by append_kernel and copied back once per call.
+#include <string.h>
+
+#include <new>
+#include <vector>
+
+#include "common.cuh"
+
+namespace otif {
+
+otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws, size_t ws_bytes,
+                         cudaStream_t stream, cudaEvent_t *evs);
+
+// per-batch timing events: start, resize, proxy prep (tag + E1), E2, E3, E4, E5, D1+D2, select, pack, append
+constexpr int kStages = 10;
+
+// counters: [0] frames, [1] positive cells, [2] windows, [3] window pixels,
+//           [4] order-independent window hash (sum of 64-bit mixes), [5 + s] windows of size s
+constexpr int kCtrFixed = 5;
+
+__device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+// Append one batch's windows (frame index rebased to the global frame) and counts to the
+// run's output arrays; accumulate the counters.  One CTA.
+__global__ void __launch_bounds__(1024) append_kernel(const otif_window *__restrict__ win, const int *__restrict__ total,
+                                                      int capacity, const int *__restrict__ counts, int nb,
+                                                      const uint8_t *__restrict__ mask, int cells, int frame_base,
+                                                      otif_window *out_win, int out_cap, int *out_counts,
+                                                      int *out_total, unsigned long long *ctr, int k) {
+    __shared__ unsigned long long s_pix, s_hash, s_pos;
+    __shared__ unsigned long long s_size[8];
+    if (threadIdx.x == 0) { s_pix = 0; s_hash = 0; s_pos = 0; }
+    if (threadIdx.x < 8) s_size[threadIdx.x] = 0;
+    __syncthreads();
+    const int t = min(*total, capacity);
+    const int base = *out_total;
+    unsigned long long pix = 0, hsh = 0, pos = 0;
+    for (int i = threadIdx.x; i < t; i += blockDim.x) {
+        otif_window w = win[i];
+        w.frame += frame_base;
+        if (base + i < out_cap && out_win) out_win[base + i] = w;
+        pix += (unsigned long long)w.w * w.h;
+        unsigned long long key = ((unsigned long long)(unsigned)w.frame << 32) ^ ((unsigned long long)(unsigned)w.x << 16) ^
+                                 (unsigned)w.y;
+        hsh += mix64(key ^ mix64(((unsigned long long)w.w << 20) ^ ((unsigned long long)w.h << 4) ^ w.size_idx));
+        atomicAdd(&s_size[w.size_idx & 7], 1ull);
+    }
+    for (int i = threadIdx.x; i < nb; i += blockDim.x)
+        if (out_counts) out_counts[frame_base + i] = counts[i];
+    for (int i = threadIdx.x; i < nb * cells; i += blockDim.x) pos += mask[i];
+    atomicAdd(&s_pix, pix);
+    atomicAdd(&s_hash, hsh);
+    atomicAdd(&s_pos, pos);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        *out_total = base + *total;
+        ctr[0] += nb;
+        ctr[1] += s_pos;
+        ctr[2] += *total;
+        ctr[3] += s_pix;
+        ctr[4] += s_hash;
+        for (int s = 0; s < k; s++) ctr[kCtrFixed + s] += s_size[s];
+    }
+}
+
+}  // namespace otif
+
+using namespace otif;
+
+struct otif_pipeline {
+    otif_pipeline_desc d;
+    otif_proxy *proxy = nullptr;
+    int gh = 0, gw = 0, cells = 0, cap_w = 0;
+    uint8_t *src[2] = {nullptr, nullptr};
+    uint8_t *img = nullptr, *mask = nullptr, *proxy_ws = nullptr, *sel_ws = nullptr;
+    size_t proxy_ws_bytes = 0, sel_ws_bytes = 0;
+    float *scores = nullptr;
+    otif_window *windows = nullptr;
+    int *counts = nullptr, *offsets = nullptr, *total = nullptr, *slot = nullptr, *size_count = nullptr;
+    uint8_t *batches[8] = {};
+    unsigned long long *ctr = nullptr;
+    // run outputs (grown on demand)
+    otif_window *out_win = nullptr;
+    int out_win_cap = 0;
+    int *out_counts = nullptr;
+    int out_counts_cap = 0;
+    int *out_total = nullptr;
+    cudaStream_t s_compute = nullptr, s_copy = nullptr;
+    cudaEvent_t ev_h2d[2] = {}, ev_free[2] = {};
+    // optional per-stage timing (otif_pipeline_set_timing)
+    int timing = 0;
+    std::vector<cudaEvent_t> ev_pool;
+    size_t ev_used = 0;
+    int64_t launches = 0;
+};
+
+static cudaEvent_t *take_events(otif_pipeline *p, int k) {
+    while (p->ev_pool.size() < p->ev_used + k) {
+        cudaEvent_t e;
+        if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+        p->ev_pool.push_back(e);
+    }
+    cudaEvent_t *r = &p->ev_pool[p->ev_used];
+    p->ev_used += k;
+    return r;
+}
+
+static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int frame_base, cudaStream_t st) {
+    const otif_pipeline_desc &d = p->d;
+    otif_status rc;
+    cudaEvent_t *ev = p->timing ? take_events(p, kStages + 1) : nullptr;
+    if (ev) OTIF_CUDA(cudaEventRecord(ev[0], st));
+    rc = otif_resize(src, nb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w, st);
+    if (rc != OTIF_OK) return rc;
+    if (ev) OTIF_CUDA(cudaEventRecord(ev[1], st));
+    rc = launch_proxy(p->proxy, p->img, nb, p->scores, p->proxy_ws, p->proxy_ws_bytes, st, ev ? ev + 2 : nullptr);
+    if (rc != OTIF_OK) return rc;
+    rc = otif_select_windows(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask,
+                             p->windows, p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st);
+    if (rc != OTIF_OK) return rc;
+    if (ev) OTIF_CUDA(cudaEventRecord(ev[8], st));
+    rc = otif_pack_windows(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
+                           p->batches, d.batch_cap, p->slot, p->size_count, st);
+    if (rc != OTIF_OK) return rc;
+    if (ev) OTIF_CUDA(cudaEventRecord(ev[9], st));
+    append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts, nb, p->mask, p->cells, frame_base,
+                                      p->out_win, p->out_win_cap, p->out_counts, p->out_total, p->ctr, d.k);
+    OTIF_LAUNCH_CHECK();
+    if (ev) OTIF_CUDA(cudaEventRecord(ev[10], st));
+    // resize 1, proxy 8 (zero, tag, E1, 5 GEMM layers), select 2, pack 2, append 1
+    p->launches += 14;
+    return OTIF_OK;
+}
+
+#define PCUDA(call)                                                                    \
+    do {                                                                               \
+        cudaError_t e_ = (call);                                                       \
+        if (e_ != cudaSuccess) {                                                       \
+            set_error("%s: %s", #call, cudaGetErrorString(e_));                        \
+            otif_pipeline_destroy(p);                                                  \
+            return e_ == cudaErrorMemoryAllocation ? OTIF_ENOMEM : OTIF_ECUDA;         \
+        }                                                                              \
+    } while (0)
+
+extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const float *weights, size_t n_weights,
+                                            otif_pipeline **out) {
+    OTIF_REQUIRE(d && weights && out, "otif_pipeline_create: NULL argument");
+    OTIF_REQUIRE(d->max_batch > 0, "otif_pipeline_create: max_batch must be positive");
+    OTIF_REQUIRE(d->k >= 1 && d->k <= 8, "otif_pipeline_create: k=%d", d->k);
+    OTIF_REQUIRE(d->src_h > 0 && d->src_w > 0 && d->det_h > 0 && d->det_w > 0, "otif_pipeline_create: sizes");
+    OTIF_REQUIRE(d->grid.frame_w == d->det_w && d->grid.frame_h == d->det_h,
+                 "otif_pipeline_create: grid frame must be the detector resolution");
+    otif_pipeline *p = new (std::nothrow) otif_pipeline();
+    if (!p) return OTIF_ENOMEM;
+    p->d = *d;
+    otif_status rc = otif_proxy_create(&d->proxy, weights, n_weights, &p->proxy);
+    if (rc != OTIF_OK) { otif_pipeline_destroy(p); return rc; }
+    otif_proxy_grid(p->proxy, &p->gh, &p->gw);
+    OTIF_REQUIRE(p->gh == (d->grid.frame_h + d->grid.cell - 1) / d->grid.cell &&
+                     p->gw == (d->grid.frame_w + d->grid.cell - 1) / d->grid.cell,
+                 "otif_pipeline_create: proxy grid %dx%d does not match ceil(frame/cell)", p->gw, p->gh);
+    const int B = d->max_batch;
+    p->cells = p->gh * p->gw;
+    p->cap_w = B * ((p->cells + 1) / 2);
+    const size_t src_bytes = (size_t)B * d->src_h * d->src_w * 3;
+    PCUDA(cudaMalloc(&p->src[0], src_bytes));
+    PCUDA(cudaMalloc(&p->src[1], src_bytes));
+    PCUDA(cudaMalloc(&p->img, (size_t)B * d->proxy.in_h * d->proxy.in_w * 3));
+    p->proxy_ws_bytes = otif_proxy_workspace_bytes(p->proxy, B);
+    PCUDA(cudaMalloc(&p->proxy_ws, p->proxy_ws_bytes));
+    PCUDA(cudaMemset(p->proxy_ws, 0, p->proxy_ws_bytes));
+    p->sel_ws_bytes = otif_select_workspace_bytes(B, p->gh, p->gw);
+    PCUDA(cudaMalloc(&p->sel_ws, p->sel_ws_bytes));
+    PCUDA(cudaMalloc(&p->scores, (size_t)B * p->cells * 4));
+    PCUDA(cudaMalloc(&p->mask, (size_t)B * p->cells));
+    PCUDA(cudaMalloc(&p->windows, (size_t)p->cap_w * sizeof(otif_window)));
+    PCUDA(cudaMalloc(&p->counts, B * 4));
+    PCUDA(cudaMalloc(&p->offsets, B * 4));
+    PCUDA(cudaMalloc(&p->total, 4));
+    PCUDA(cudaMalloc(&p->slot, (size_t)p->cap_w * 4));
+    PCUDA(cudaMalloc(&p->size_count, 8 * 4));
+    for (int s = 0; s < d->k; s++)
+        if (d->batch_cap[s] > 0)
+            PCUDA(cudaMalloc(&p->batches[s], (size_t)d->batch_cap[s] * d->sizes[s].w * d->sizes[s].h * 3));
+    PCUDA(cudaMalloc(&p->ctr, (kCtrFixed + 8) * 8));
+    PCUDA(cudaMemset(p->ctr, 0, (kCtrFixed + 8) * 8));
+    PCUDA(cudaMalloc(&p->out_total, 4));
+    PCUDA(cudaStreamCreateWithFlags(&p->s_compute, cudaStreamNonBlocking));
+    PCUDA(cudaStreamCreateWithFlags(&p->s_copy, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; i++) {
+        PCUDA(cudaEventCreateWithFlags(&p->ev_h2d[i], cudaEventDisableTiming));
+        PCUDA(cudaEventCreateWithFlags(&p->ev_free[i], cudaEventDisableTiming));
+    }
+    PCUDA(cudaDeviceSynchronize());
+    *out = p;
+    return OTIF_OK;
+}
+
+extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
+    if (!p) return;
+    if (p->s_compute) cudaStreamSynchronize(p->s_compute);
+    if (p->s_copy) cudaStreamSynchronize(p->s_copy);
+    void *bufs[] = {p->src[0], p->src[1], p->img, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
+                    p->offsets, p->total, p->slot, p->size_count, p->ctr, p->out_win, p->out_counts, p->out_total};
+    for (void *b : bufs)
+        if (b) cudaFree(b);
+    for (int s = 0; s < 8; s++)
+        if (p->batches[s]) cudaFree(p->batches[s]);
+    for (cudaEvent_t e : p->ev_pool) cudaEventDestroy(e);
+    for (int i = 0; i < 2; i++) {
+        if (p->ev_h2d[i]) cudaEventDestroy(p->ev_h2d[i]);
+        if (p->ev_free[i]) cudaEventDestroy(p->ev_free[i]);
+    }
+    if (p->s_compute) cudaStreamDestroy(p->s_compute);
+    if (p->s_copy) cudaStreamDestroy(p->s_copy);
+    if (p->proxy) otif_proxy_destroy(p->proxy);
+    delete p;
+}
+
+static otif_status ensure_outputs(otif_pipeline *p, int n, int cap_windows) {
+    if (n > p->out_counts_cap) {
+        if (p->out_counts) cudaFree(p->out_counts);
+        p->out_counts = nullptr;
+        OTIF_CUDA(cudaMalloc(&p->out_counts, (size_t)n * 4));
+        p->out_counts_cap = n;
+    }
+    if (cap_windows > p->out_win_cap) {
+        if (p->out_win) cudaFree(p->out_win);
+        p->out_win = nullptr;
+        OTIF_CUDA(cudaMalloc(&p->out_win, (size_t)cap_windows * sizeof(otif_window)));
+        p->out_win_cap = cap_windows;
+    }
+    return OTIF_OK;
+}
+
+extern "C" otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *src_host, int32_t n,
+                                              otif_window *windows_out, int32_t cap_windows, int32_t *frame_count_out,
+                                              int32_t *total_out, int32_t *size_count_out) {
+    OTIF_REQUIRE(p && (src_host || n == 0) && n >= 0 && cap_windows >= 0, "otif_pipeline_run_host: bad arguments");
+    OTIF_REQUIRE(total_out, "otif_pipeline_run_host: NULL total_out");
+    otif_status rc = ensure_outputs(p, n > 0 ? n : 1, cap_windows > 0 ? cap_windows : 1);
+    if (rc != OTIF_OK) return rc;
+    const otif_pipeline_desc &d = p->d;
+    const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
+    const int out_cap = cap_windows;
+    OTIF_CUDA(cudaMemsetAsync(p->out_total, 0, 4, p->s_compute));
+    OTIF_CUDA(cudaMemsetAsync(p->ctr, 0, (kCtrFixed + 8) * 8, p->s_compute));
+    // the copy stream must not overwrite a src buffer before the compute stream is done with it
+    for (int i = 0; i < 2; i++) OTIF_CUDA(cudaEventRecord(p->ev_free[i], p->s_compute));
+    int b = 0;
+    for (int f0 = 0; f0 < n; f0 += d.max_batch, b++) {
+        const int nb = n - f0 < d.max_batch ? n - f0 : d.max_batch;
+        const int buf = b & 1;
+        OTIF_CUDA(cudaStreamWaitEvent(p->s_copy, p->ev_free[buf], 0));
+        OTIF_CUDA(cudaMemcpyAsync(p->src[buf], src_host + (size_t)f0 * frame_bytes, (size_t)nb * frame_bytes,
+                                  cudaMemcpyHostToDevice, p->s_copy));
+        OTIF_CUDA(cudaEventRecord(p->ev_h2d[buf], p->s_copy));
+        OTIF_CUDA(cudaStreamWaitEvent(p->s_compute, p->ev_h2d[buf], 0));
+        // out_win capacity is the caller's: windows beyond it are dropped (total stays exact)
+        int saved = p->out_win_cap;
+        p->out_win_cap = out_cap;
+        rc = run_batch(p, p->src[buf], nb, f0, p->s_compute);
+        p->out_win_cap = saved;
+        if (rc != OTIF_OK) return rc;
+        OTIF_CUDA(cudaEventRecord(p->ev_free[buf], p->s_compute));
+    }
+    int total = 0;
+    OTIF_CUDA(cudaMemcpyAsync(&total, p->out_total, 4, cudaMemcpyDeviceToHost, p->s_compute));
+    if (frame_count_out && n > 0)
+        OTIF_CUDA(cudaMemcpyAsync(frame_count_out, p->out_counts, (size_t)n * 4, cudaMemcpyDeviceToHost, p->s_compute));
+    unsigned long long ctr[kCtrFixed + 8];
+    OTIF_CUDA(cudaMemcpyAsync(ctr, p->ctr, sizeof(ctr), cudaMemcpyDeviceToHost, p->s_compute));
+    OTIF_CUDA(cudaStreamSynchronize(p->s_compute));
+    const int keep = total < cap_windows ? total : cap_windows;
+    if (windows_out && keep > 0)
+        OTIF_CUDA(cudaMemcpy(windows_out, p->out_win, (size_t)keep * sizeof(otif_window), cudaMemcpyDeviceToHost));
+    *total_out = total;
+    if (size_count_out)
+        for (int s = 0; s < d.k; s++) size_count_out[s] = (int32_t)ctr[kCtrFixed + s];
+    return OTIF_OK;
+}
+
+extern "C" otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t *src_dev, int32_t n,
+                                                cudaStream_t stream) {
+    OTIF_REQUIRE(p && (src_dev || n == 0) && n >= 0, "otif_pipeline_run_device: bad arguments");
+    const size_t frame_bytes = (size_t)p->d.src_h * p->d.src_w * 3;
+    // device runs keep no per-frame outputs beyond the last batch: counters only
+    otif_window *ow = p->out_win;
+    int *oc = p->out_counts;
+    int owc = p->out_win_cap;
+    p->out_win = nullptr;
+    p->out_counts = nullptr;
+    p->out_win_cap = 0;
+    OTIF_CUDA(cudaMemsetAsync(p->out_total, 0, 4, stream));
+    otif_status rc = OTIF_OK;
+    for (int f0 = 0; f0 < n && rc == OTIF_OK; f0 += p->d.max_batch) {
+        const int nb = n - f0 < p->d.max_batch ? n - f0 : p->d.max_batch;
+        rc = run_batch(p, src_dev + (size_t)f0 * frame_bytes, nb, f0, stream);
+    }
+    p->out_win = ow;
+    p->out_counts = oc;
+    p->out_win_cap = owc;
+    return rc;
+}
+
+extern "C" const int64_t *otif_pipeline_counters(const otif_pipeline *p) {
+    return p ? reinterpret_cast<const int64_t *>(p->ctr) : nullptr;
+}
+
+extern "C" otif_status otif_pipeline_reset_counters(otif_pipeline *p, cudaStream_t stream) {
+    OTIF_REQUIRE(p, "otif_pipeline_reset_counters: NULL");
+    OTIF_CUDA(cudaMemsetAsync(p->ctr, 0, (kCtrFixed + 8) * 8, stream));
+    return OTIF_OK;
+}
+
+extern "C" otif_status otif_pipeline_set_timing(otif_pipeline *p, int32_t enable) {
+    OTIF_REQUIRE(p, "otif_pipeline_set_timing: NULL");
+    p->timing = enable ? 1 : 0;
+    p->ev_used = 0;
+    p->launches = 0;
+    return OTIF_OK;
+}
+
+extern "C" otif_status otif_pipeline_stage_ms(otif_pipeline *p, float *ms, int32_t n_ms, int64_t *launches) {
+    OTIF_REQUIRE(p && ms && n_ms >= kStages, "otif_pipeline_stage_ms: need %d entries", kStages);
+    for (int s = 0; s < kStages; s++) ms[s] = 0.0f;
+    for (size_t b = 0; b + kStages + 1 <= p->ev_used; b += kStages + 1) {
+        OTIF_CUDA(cudaEventSynchronize(p->ev_pool[b + kStages]));
+        for (int s = 0; s < kStages; s++) {
+            float t = 0.0f;
+            OTIF_CUDA(cudaEventElapsedTime(&t, p->ev_pool[b + s], p->ev_pool[b + s + 1]));
+            ms[s] += t;
+        }
+    }
+    if (launches) *launches = p->launches;
+    p->ev_used = 0;
+    p->launches = 0;
+    return OTIF_OK;
+}

@@ -472,8 +472,9 @@ static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
     bytes = sa * a + sb * b + fixed;
 }
 
-static otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws,
-                                size_t ws_bytes, cudaStream_t stream) {
+// evs (optional): 6 events recorded after E1 (prep) and after each of the 5 GEMM layers
+otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws,
+                         size_t ws_bytes, cudaStream_t stream, cudaEvent_t *evs) {
     Layout lay[5];
     size_t need = plan_workspace(p, n, lay);
     if (ws_bytes < need) {
@@ -499,6 +500,7 @@ static otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, 
         if (blocks < 1) blocks = 1;
         e1_kernel<<<(unsigned)blocks, 256, 0, stream>>>(e);
         OTIF_LAUNCH_CHECK();
+        if (evs) OTIF_CUDA(cudaEventRecord(evs[0], stream));
     }
     // E2..E5, D1
     for (int li = 0; li < 5; li++) {
@@ -538,6 +540,7 @@ static otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, 
         if (grid < 1) grid = 1;
         conv_umma_kernel<<<grid, kConvThreads, smem, stream>>>(c);
         OTIF_LAUNCH_CHECK();
+        if (evs) OTIF_CUDA(cudaEventRecord(evs[1 + li], stream));
     }
     return OTIF_OK;
 }
@@ -716,5 +719,5 @@ extern "C" otif_status otif_proxy_score(const otif_proxy *p, const uint8_t *img,
     OTIF_REQUIRE((((uintptr_t)workspace) & 255) == 0, "otif_proxy_score: workspace must be 256-B aligned");
     otif_status st = check_device(nullptr);
     if (st != OTIF_OK) return st;
-    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream);
+    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream, nullptr);
 }

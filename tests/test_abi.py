@@ -1,0 +1,80 @@
+"""CPU checks of the boundary: libotif.so builds for sm_100a, loads without a GPU and
+exports every function include/otif.h declares; host-side validation paths."""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def libotif():
+    from paper_conf_sigmod_bastanim22_b200 import build
+    path = build.build()
+    return ctypes.CDLL(path)
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "otif.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(otif_[a-z_0-9]+)\s*\(", src)))
+
+
+def test_header_declares_the_path_calls():
+    names = header_functions()
+    for required in ("otif_resize", "otif_proxy_create", "otif_proxy_score", "otif_proxy_destroy",
+                     "otif_select_windows", "otif_pack_windows"):
+        assert required in names
+
+
+def test_library_exports_every_declared_symbol(libotif):
+    missing = [n for n in header_functions() if not hasattr(libotif, n)]
+    assert not missing, missing
+    from paper_conf_sigmod_bastanim22_b200 import _lib
+    assert set(_lib.EXPORTED) <= set(header_functions())
+
+
+def test_sass_is_sm100a_with_tcgen05(libotif):
+    import subprocess
+    from paper_conf_sigmod_bastanim22_b200 import build
+    out = subprocess.run(["cuobjdump", "-sass", build.LIB], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    assert "UTCHMMA" in out      # tcgen05.mma
+    assert "UBLKCP" in out       # cp.async.bulk (1-D TMA)
+    assert "LDTM" in out         # tcgen05.ld
+    assert "HMMA" not in out.replace("UTCHMMA", "")
+
+
+def test_status_strings_and_validation_without_gpu(libotif):
+    from paper_conf_sigmod_bastanim22_b200 import _lib
+    L = _lib.lib()
+    assert L.otif_status_str(0) == b"OTIF_OK"
+    assert L.otif_status_str(4) == b"OTIF_EUNSUPPORTED"
+    assert b"sm_100a" in L.otif_version()
+    # argument validation happens before any CUDA call
+    rc = L.otif_resize(None, 1, 0, 10, None, 5, 5, None)
+    assert rc == _lib.EINVAL and b"positive" in L.otif_last_error()
+    g = _lib.GridDesc(416, 256, 32, 4)
+    sizes = (_lib.WSize * 1)(_lib.WSize(64, 64, 4096))
+    rc = L.otif_select_windows(None, ctypes.c_void_p(1), ctypes.c_float(0.5), 1, 8, 13, ctypes.byref(g), sizes, 1,
+                               None, None, 0, None, None, None, None, 0, None)
+    assert rc == _lib.EINVAL and b"full frame" in L.otif_last_error()
+    rc = L.otif_select_windows(None, ctypes.c_void_p(1), ctypes.c_float(0.5), 1, 8, 12, ctypes.byref(g), sizes, 1,
+                               None, None, 0, None, None, None, None, 0, None)
+    assert rc == _lib.EINVAL and b"grid" in L.otif_last_error()
+    d = _lib.ProxyDesc()
+    d.in_h, d.in_w, d.n_strided, d.dec = 64, 104, 6, 128
+    h = ctypes.c_void_p()
+    rc = L.otif_proxy_create(ctypes.byref(d), ctypes.c_void_p(1), 10, ctypes.byref(h))
+    assert rc == _lib.EINVAL and b"n_strided" in L.otif_last_error()
+
+
+def test_product_package_does_not_import_the_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_sigmod_bastanim22_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".cpp", ".h")):
+                text = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in text and "from oracle" not in text and "otif_ref" not in text, f

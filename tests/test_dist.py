@@ -1,0 +1,73 @@
+"""Multi-process (gloo, world_size 2) checks of the N>1 host logic: clip sharding
+partitions the corpus, counters gather to every rank, totals and the window hash are
+independent of the sharding, the job time is the max over ranks."""
+import os
+import socket
+
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_sigmod_bastanim22_b200 import dist as odist
+
+
+def test_shard_clips_partition():
+    for n in (480, 7, 1, 0):
+        for world in (1, 2, 3, 4, 8):
+            got = [c for r in range(world) for c in odist.shard_clips(n, world, r)]
+            assert got == list(range(n))
+            sizes = [len(odist.shard_clips(n, world, r)) for r in range(world)]
+            assert max(sizes) - min(sizes) <= 1
+    with pytest.raises(ValueError):
+        odist.shard_clips(10, 2, 2)
+
+
+def _per_clip_counters(clip: int) -> torch.Tensor:
+    # deterministic fake per-clip counters (frames, pos, windows, pixels, hash, s0, s1, s2)
+    g = torch.Generator().manual_seed(clip)
+    v = torch.randint(0, 1000, (8,), generator=g, dtype=torch.int64)
+    v[0] = 450
+    v[4] = (clip * 0x9E3779B97F4A7C15) & 0x7FFFFFFFFFFFFFFF
+    return v
+
+
+def _worker(rank, world, port, n_clips, out):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    ctr = torch.zeros(8, dtype=torch.int64)
+    for c in odist.shard_clips(n_clips, world, rank):
+        ctr += _per_clip_counters(c)
+    g = odist.gather_counters(ctr)
+    t = odist.max_over_ranks(float(rank + 1))
+    out[rank] = (g.clone(), t, odist.combine(g))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+@pytest.mark.parametrize("world", [2])
+def test_gloo_gather_and_sharding_invariance(world):
+    n_clips = 10
+    mgr = mp.Manager()
+    out = mgr.dict()
+    mp.spawn(_worker, args=(world, _free_port(), n_clips, out), nprocs=world, join=True)
+    ref = sum(_per_clip_counters(c) for c in range(n_clips))
+    for r in range(world):
+        g, t, tot = out[r]
+        assert g.shape == (world, 8)
+        assert torch.equal(g.sum(0), ref)
+        assert t == float(world)              # max over ranks
+        assert tot["frames"] == 450 * n_clips
+        assert tot["window_hash"] == int(ref[4]) & ((1 << 64) - 1)
+    # same totals from a single process
+    single = odist.combine(ref.view(1, -1))
+    assert single == out[0][2]
