@@ -261,7 +261,7 @@ def _device_view_i64(ptr: int, n: int) -> torch.Tensor:
     out = torch.empty(n, dtype=torch.int64, device="cuda")
     # cudaMemcpy through torch: build a tensor from the raw pointer via __cuda_array_interface__
     class _CAI:
-        __cuda_array_interface__ = {"shape": (n,), "typestr": "<i8", "data": (ptr, True), "version": 3}
+        __cuda_array_interface__ = {"shape": (n,), "typestr": "<i8", "data": (ptr, False), "version": 3}
     src = torch.as_tensor(_CAI(), device="cuda")
     out.copy_(src)
     return out

@@ -481,7 +481,24 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         set_error("otif_proxy_score: workspace %zu B < required %zu B", ws_bytes, need);
         return OTIF_ENOMEM;
     }
-    const uint64_t tag = p->plan_hash ^ ((uint64_t)n * 0x9E3779B97F4A7C15ull) ^ (uint64_t)need;
+    // Lay the buffers out for the largest batch this workspace can hold, so that every
+    // batch size up to it shares one layout (and one zero-initialisation): a smaller
+    // final batch then does not re-zero the workspace.
+    int n_plan = n;
+    {
+        int64_t lo = n, hi = n;
+        while (hi < (1 << 24) && plan_workspace(p, (int)(hi * 2), lay) <= ws_bytes) hi *= 2;
+        int64_t top = hi * 2;
+        lo = hi;
+        while (top - lo > 1) {  // largest m in [hi, 2hi) with bytes(m) <= ws_bytes
+            int64_t mid = (lo + top) / 2;
+            if (plan_workspace(p, (int)mid, lay) <= ws_bytes) lo = mid;
+            else top = mid;
+        }
+        n_plan = (int)lo;
+        need = plan_workspace(p, n_plan, lay);
+    }
+    const uint64_t tag = p->plan_hash ^ ((uint64_t)n_plan * 0x9E3779B97F4A7C15ull) ^ (uint64_t)need;
     ws_zero_kernel<<<p->num_sms * 4, 256, 0, stream>>>(ws, need, tag);
     OTIF_LAUNCH_CHECK();
     ws_tag_kernel<<<1, 1, 0, stream>>>(ws, tag);

@@ -172,8 +172,20 @@ __global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_consta
         }
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < cells; i += blockDim.x)
-        if (par[i] >= 0) par[i] = uf_find(par, i);
+    // flatten: resolve every root with read-only walks into a scratch array first (a
+    // path-halving write racing with another thread's flatten store could leave a
+    // non-root parent behind), then publish.  px/py (2*cap >= cells ints) are free here.
+    {
+        int *lab = px;
+        for (int i = threadIdx.x; i < cells; i += blockDim.x) {
+            int x = par[i];
+            if (x >= 0)
+                while (par[x] != x) x = par[x];
+            lab[i] = x;
+        }
+        __syncthreads();
+        for (int i = threadIdx.x; i < cells; i += blockDim.x) par[i] = lab[i];
+    }
     __syncthreads();
 
     // raster-ordered component ids: exclusive scan of root flags over contiguous segments

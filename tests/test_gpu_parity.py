@@ -124,6 +124,22 @@ def test_select_windows_mask_parity(wl, conn):
     assert np.array_equal(r["mask"].cpu().numpy(), masks)
 
 
+@pytest.mark.parametrize("density", [0.3, 0.5, 0.7])
+def test_select_windows_stress_many_frames(density):
+    """Thousands of dense random frames: exercises concurrent union-find in every CTA."""
+    wl = configs.C2
+    rng = np.random.default_rng(int(density * 100))
+    masks = (rng.random((3000, 17, 30)) < density).astype(np.uint8)
+    for conn in (4, 8):
+        ref_w, ref_c, ref_o, ref_t = oracle.select_windows(masks, wl.cell, wl.src_w, wl.src_h, wl.sizes, conn)
+        r = otif.otif_select_windows(None, torch.from_numpy(masks).cuda(), 0.0, wl.src_w, wl.src_h, wl.cell,
+                                     wl.sizes, connectivity=conn)
+        t = int(r["total"].item())
+        assert t == ref_t
+        assert np.array_equal(r["counts"].cpu().numpy(), ref_c)
+        assert as_tuples(windows_np(r["windows"], t)) == as_tuples(ref_w)
+
+
 def test_select_scores_input_and_capacity(blob):
     wl = configs.C1
     rng = np.random.default_rng(3)
