@@ -71,7 +71,37 @@ __device__ __forceinline__ uint32_t fshift(uint32_t lo, uint32_t hi, uint32_t sh
     return sh_bytes ? __funnelshift_r(lo, hi, sh_bytes * 8) : lo;
 }
 
-__global__ void __launch_bounds__(256) pack_kernel(const __grid_constant__ PackParams p) {
+// 16 bytes from an arbitrarily aligned address: two aligned 16-B loads and a funnel shift
+// (byte loads only within the last 32 bytes of the source allocation)
+__device__ __forceinline__ uint4 load16u(const uint8_t *s0, uintptr_t src_end) {
+    const uintptr_t a = (uintptr_t)s0;
+    const uintptr_t al = a & ~(uintptr_t)15;
+    const uint32_t sh = (uint32_t)(a - al);
+    if (al + 32 <= src_end) {
+        const uint4 v0 = __ldg(reinterpret_cast<const uint4 *>(al));
+        if (sh == 0) return v0;
+        const uint4 v1 = __ldg(reinterpret_cast<const uint4 *>(al + 16));
+        const uint32_t wv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
+        const uint32_t q = sh >> 2, b = sh & 3;
+        uint32_t o[4];
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            // wv[q + j], wv[q + j + 1] with q in 0..3 (unrolled select, no local memory)
+            uint32_t lo = q == 0 ? wv[j] : q == 1 ? wv[j + 1] : q == 2 ? wv[j + 2] : wv[j + 3];
+            uint32_t hi = q == 0 ? wv[j + 1] : q == 1 ? wv[j + 2] : q == 2 ? wv[j + 3] : wv[j + 4];
+            o[j] = fshift(lo, hi, b);
+        }
+        return make_uint4(o[0], o[1], o[2], o[3]);
+    }
+    uint32_t o[4];
+#pragma unroll
+    for (int j = 0; j < 4; j++)
+        o[j] = (uint32_t)s0[4 * j] | ((uint32_t)s0[4 * j + 1] << 8) | ((uint32_t)s0[4 * j + 2] << 16) |
+               ((uint32_t)s0[4 * j + 3] << 24);
+    return make_uint4(o[0], o[1], o[2], o[3]);
+}
+
+__global__ void __launch_bounds__(512) pack_kernel(const __grid_constant__ PackParams p) {
     const int total = min(*p.total, p.capacity);
     const bool identity = (p.dh == p.sh && p.dw == p.sw);
     for (int g = blockIdx.x; g < total; g += gridDim.x) {
@@ -85,40 +115,26 @@ __global__ void __launch_bounds__(256) pack_kernel(const __grid_constant__ PackP
             const int per_row = row_bytes >> 4;
             const uint8_t *fbase = p.src + (size_t)w.frame * p.sh * p.sw * 3;
             const uintptr_t src_end = (uintptr_t)p.src + p.src_bytes;
-            for (int i = threadIdx.x; i < w.h * per_row; i += blockDim.x) {
-                const int r = i / per_row, c = i - r * per_row;
-                const uint8_t *s0 = fbase + ((size_t)(w.y + r) * p.sw + w.x) * 3 + c * 16;
-                const uintptr_t a = (uintptr_t)s0;
-                const uintptr_t al = a & ~(uintptr_t)15;
-                const uint32_t sh = (uint32_t)(a - al);
-                uint4 out;
-                if (al + 32 <= src_end) {
-                    const uint4 v0 = __ldg(reinterpret_cast<const uint4 *>(al));
-                    const uint4 v1 = sh ? __ldg(reinterpret_cast<const uint4 *>(al + 16)) : make_uint4(0, 0, 0, 0);
-                    uint32_t wv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
-                    const uint32_t q = sh >> 2, b = sh & 3;
-                    uint32_t o[4];
+            const int total16 = w.h * per_row;
+            // 4 independent 16-B loads in flight per thread before the stores (memory-level parallelism)
+            for (int i0 = threadIdx.x; i0 < total16; i0 += 4 * blockDim.x) {
+                uint4 v[4];
 #pragma unroll
-                    for (int j = 0; j < 4; j++) {
-                        uint32_t lo, hi;
-                        // wv[q + j], wv[q + j + 1] with q in 0..3 (unrolled select, no local memory)
-                        lo = q == 0 ? wv[j] : q == 1 ? wv[j + 1] : q == 2 ? wv[j + 2] : wv[j + 3];
-                        hi = q == 0 ? wv[j + 1] : q == 1 ? wv[j + 2] : q == 2 ? wv[j + 3] : wv[j + 4];
-                        o[j] = fshift(lo, hi, b);
+                for (int u = 0; u < 4; u++) {
+                    const int i = i0 + u * blockDim.x;
+                    if (i < total16) {
+                        const int r = i / per_row, c = i - r * per_row;
+                        v[u] = load16u(fbase + ((size_t)(w.y + r) * p.sw + w.x) * 3 + c * 16, src_end);
                     }
-                    out = make_uint4(o[0], o[1], o[2], o[3]);
-                } else {
-                    uint8_t bytes[16];
-#pragma unroll
-                    for (int j = 0; j < 16; j++) bytes[j] = s0[j];
-                    uint32_t o[4];
-#pragma unroll
-                    for (int j = 0; j < 4; j++)
-                        o[j] = (uint32_t)bytes[4 * j] | ((uint32_t)bytes[4 * j + 1] << 8) |
-                               ((uint32_t)bytes[4 * j + 2] << 16) | ((uint32_t)bytes[4 * j + 3] << 24);
-                    out = make_uint4(o[0], o[1], o[2], o[3]);
                 }
-                *reinterpret_cast<uint4 *>(dst + (size_t)r * row_bytes + c * 16) = out;
+#pragma unroll
+                for (int u = 0; u < 4; u++) {
+                    const int i = i0 + u * blockDim.x;
+                    if (i < total16) {
+                        const int r = i / per_row, c = i - r * per_row;
+                        *reinterpret_cast<uint4 *>(dst + (size_t)r * row_bytes + c * 16) = v[u];
+                    }
+                }
             }
         } else if (identity) {
             const uint8_t *fbase = p.src + (size_t)w.frame * p.sh * p.sw * 3;
@@ -184,8 +200,8 @@ extern "C" otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t 
     slot_kernel<<<1, 1024, 0, stream>>>(p);
     OTIF_LAUNCH_CHECK();
     if (capacity > 0) {
-        int grid = capacity < num_sms * 8 ? capacity : num_sms * 8;
-        pack_kernel<<<grid, 256, 0, stream>>>(p);
+        int grid = capacity < num_sms * 4 ? capacity : num_sms * 4;
+        pack_kernel<<<grid, 512, 0, stream>>>(p);
         OTIF_LAUNCH_CHECK();
     }
     return OTIF_OK;

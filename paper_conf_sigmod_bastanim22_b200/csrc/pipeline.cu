@@ -22,54 +22,29 @@ constexpr int kStages = 10;
 //           [4] order-independent window hash (sum of 64-bit mixes), [5 + s] windows of size s
 constexpr int kCtrFixed = 5;
 
-__device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
-    z += 0x9E3779B97F4A7C15ull;
-    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
-    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
-    return z ^ (z >> 31);
-}
+otif_status launch_select(const float *scores, const uint8_t *mask_in, float threshold, int32_t n, int32_t gh,
+                          int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
+                          otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
+                          int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
+                          unsigned long long *ctr, int frame_base);
 
-// Append one batch's windows (frame index rebased to the global frame) and counts to the
-// run's output arrays; accumulate the counters.  One CTA.
+// Host runs only: append one batch's windows (frame index rebased to the global frame)
+// and per-frame counts to the run's output arrays.  (The counters are accumulated by
+// the select kernel itself.)
 __global__ void __launch_bounds__(1024) append_kernel(const otif_window *__restrict__ win, const int *__restrict__ total,
                                                       int capacity, const int *__restrict__ counts, int nb,
-                                                      const uint8_t *__restrict__ mask, int cells, int frame_base,
-                                                      otif_window *out_win, int out_cap, int *out_counts,
-                                                      int *out_total, unsigned long long *ctr, int k) {
-    __shared__ unsigned long long s_pix, s_hash, s_pos;
-    __shared__ unsigned long long s_size[8];
-    if (threadIdx.x == 0) { s_pix = 0; s_hash = 0; s_pos = 0; }
-    if (threadIdx.x < 8) s_size[threadIdx.x] = 0;
-    __syncthreads();
+                                                      int frame_base, otif_window *out_win, int out_cap,
+                                                      int *out_counts, int *out_total) {
     const int t = min(*total, capacity);
     const int base = *out_total;
-    unsigned long long pix = 0, hsh = 0, pos = 0;
     for (int i = threadIdx.x; i < t; i += blockDim.x) {
         otif_window w = win[i];
         w.frame += frame_base;
-        if (base + i < out_cap && out_win) out_win[base + i] = w;
-        pix += (unsigned long long)w.w * w.h;
-        unsigned long long key = ((unsigned long long)(unsigned)w.frame << 32) ^ ((unsigned long long)(unsigned)w.x << 16) ^
-                                 (unsigned)w.y;
-        hsh += mix64(key ^ mix64(((unsigned long long)w.w << 20) ^ ((unsigned long long)w.h << 4) ^ w.size_idx));
-        atomicAdd(&s_size[w.size_idx & 7], 1ull);
+        if (base + i < out_cap) out_win[base + i] = w;
     }
-    for (int i = threadIdx.x; i < nb; i += blockDim.x)
-        if (out_counts) out_counts[frame_base + i] = counts[i];
-    for (int i = threadIdx.x; i < nb * cells; i += blockDim.x) pos += mask[i];
-    atomicAdd(&s_pix, pix);
-    atomicAdd(&s_hash, hsh);
-    atomicAdd(&s_pos, pos);
+    for (int i = threadIdx.x; i < nb; i += blockDim.x) out_counts[frame_base + i] = counts[i];
     __syncthreads();
-    if (threadIdx.x == 0) {
-        *out_total = base + *total;
-        ctr[0] += nb;
-        ctr[1] += s_pos;
-        ctr[2] += *total;
-        ctr[3] += s_pix;
-        ctr[4] += s_hash;
-        for (int s = 0; s < k; s++) ctr[kCtrFixed + s] += s_size[s];
-    }
+    if (threadIdx.x == 0) *out_total = base + *total;
 }
 
 }  // namespace otif
@@ -124,20 +99,23 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
     if (ev) OTIF_CUDA(cudaEventRecord(ev[1], st));
     rc = launch_proxy(p->proxy, p->img, nb, p->scores, p->proxy_ws, p->proxy_ws_bytes, st, ev ? ev + 2 : nullptr);
     if (rc != OTIF_OK) return rc;
-    rc = otif_select_windows(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask,
-                             p->windows, p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st);
+    rc = launch_select(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask, p->windows,
+                       p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base);
     if (rc != OTIF_OK) return rc;
     if (ev) OTIF_CUDA(cudaEventRecord(ev[8], st));
     rc = otif_pack_windows(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
                            p->batches, d.batch_cap, p->slot, p->size_count, st);
     if (rc != OTIF_OK) return rc;
     if (ev) OTIF_CUDA(cudaEventRecord(ev[9], st));
-    append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts, nb, p->mask, p->cells, frame_base,
-                                      p->out_win, p->out_win_cap, p->out_counts, p->out_total, p->ctr, d.k);
-    OTIF_LAUNCH_CHECK();
+    int launched = 13;  // resize 1, proxy 8 (zero, tag, E1, 5 GEMM layers), select 2, pack 2
+    if (p->out_win) {
+        append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts, nb, frame_base, p->out_win,
+                                          p->out_win_cap, p->out_counts, p->out_total);
+        OTIF_LAUNCH_CHECK();
+        launched++;
+    }
     if (ev) OTIF_CUDA(cudaEventRecord(ev[10], st));
-    // resize 1, proxy 8 (zero, tag, E1, 5 GEMM layers), select 2, pack 2, append 1
-    p->launches += 14;
+    p->launches += launched;
     return OTIF_OK;
 }
 

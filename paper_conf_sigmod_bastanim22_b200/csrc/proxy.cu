@@ -1,7 +1,7 @@
 // proxy.cu — stage 2: the segmentation proxy CNN (readings R1, R2, R4).
 //
-//   E1 (3->32, 3x3, stride 2): CUDA-core direct conv from the u8 proxy image
-//       (K = 27 is too small for a tensor-core tile); bf16 output.
+//   E1 (3->32, 3x3, stride 2): tcgen05 M=128,N=32 tiles with K = 27 padded to 32;
+//       the A rows are gathered from the u8 proxy image by the CTA's threads.
 //   E2..E5, D1 (3x3, pad 1): implicit-GEMM convolutions on the 5th-gen tensor cores
 //       (tcgen05.mma kind::f16, bf16 x bf16 -> fp32 in TMEM), one persistent,
 //       warp-specialised kernel per layer.
@@ -108,69 +108,117 @@ __global__ void ws_zero_kernel(uint8_t *ws, size_t bytes, uint64_t tag) {
 __global__ void ws_tag_kernel(uint8_t *ws, uint64_t tag) { *reinterpret_cast<uint64_t *>(ws) = tag; }
 
 // ---------------------------------------------------------------------------
-// E1: 3x3 stride-2 conv 3 -> 32 on CUDA cores, u8 input, bf16 output in E2's layout
+// E1: 3x3 stride-2 conv 3 -> 32 on the tensor cores.  K = 27 (3x3 taps x RGB) is
+// padded to 32; each CTA thread gathers the 27 u8 inputs of one output pixel (its A
+// row), converts them exactly to bf16 ((u-128)/128) and stores them in the no-swizzle
+// K-major smem layout; one thread issues two M=128,N=32,K=16 tcgen05.mma; the same
+// 128 threads read the accumulator row back (tcgen05.ld), add bias, ReLU, round to
+// bf16 and store 4 x 16 B into E2's input layout.  Several CTAs per SM overlap one
+// CTA's gather with another's MMA/epilogue.
 // ---------------------------------------------------------------------------
 struct E1Params {
     const uint8_t *img;
     int n, h, w, oh, ow;
-    const float *wt;    // [27][32] (k = (kh*3+kw)*3+c), bf16-rounded
-    const float *bias;  // [32]
+    const uint16_t *wpk;  // [4 chunks][32 n][8] bf16, k = (kh*3+kw)*3 + c, k >= 27 zero
+    const float *bias;    // [32]
     int out_kind, out_pitch;
     int64_t out_fstride, out_lcap;
     uint8_t *out;
+    int64_t ntiles;
 };
 
-__global__ void __launch_bounds__(256) e1_kernel(E1Params p) {
-    __shared__ float sw[27 * 32];
-    __shared__ float sb[32];
-    for (int i = threadIdx.x; i < 27 * 32; i += blockDim.x) sw[i] = p.wt[i];
-    if (threadIdx.x < 32) sb[threadIdx.x] = p.bias[threadIdx.x];
+__global__ void __launch_bounds__(128) e1_umma_kernel(const __grid_constant__ E1Params p) {
+    __shared__ __align__(128) uint8_t sA[4 * 128 * 16];  // [chunk][row][16 B]
+    __shared__ __align__(128) uint8_t sB[4 * 32 * 16];   // [chunk][n][16 B]
+    __shared__ float sbias[32];
+    __shared__ uint64_t bar;
+    __shared__ uint32_t tslot;
+    const int t = threadIdx.x, warp = t >> 5;
+    for (int i = t; i < 4 * 32 * 8 / 8; i += blockDim.x)
+        reinterpret_cast<uint4 *>(sB)[i] = reinterpret_cast<const uint4 *>(p.wpk)[i];
+    if (t < 32) sbias[t] = p.bias[t];
+    if (t == 0) { mbar_init(&bar, 1); fence_barrier_init(); }
+    if (warp == 0) tmem_alloc(&tslot, 32);
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    tc_fence_before();
     __syncthreads();
-    const int64_t total = (int64_t)p.n * p.oh * p.ow;
-    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < total;
-         idx += (int64_t)gridDim.x * blockDim.x) {
-        int ox = (int)(idx % p.ow);
-        int64_t t = idx / p.ow;
-        int oy = (int)(t % p.oh);
-        int f = (int)(t / p.oh);
-        float x[27];
-        const uint8_t *base = p.img + (size_t)f * p.h * p.w * 3;
+    tc_fence_after();
+    const uint32_t tmem = tslot;
+    const uint32_t idesc = umma_idesc_bf16(128, 32);
+    uint32_t phase = 0;
+    const int64_t npx = (int64_t)p.n * p.oh * p.ow;
+    for (int64_t tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+        const int64_t px = tile * 128 + t;
+        const bool valid = px < npx;
+        int f = 0, oy = 0, ox = 0;
+        uint32_t kv[16];
 #pragma unroll
-        for (int kh = 0; kh < 3; kh++) {
-            int iy = 2 * oy - 1 + kh;
+        for (int j = 0; j < 16; j++) kv[j] = 0;
+        if (valid) {
+            ox = (int)(px % p.ow);
+            int64_t r = px / p.ow;
+            oy = (int)(r % p.oh);
+            f = (int)(r / p.oh);
+            const uint8_t *base = p.img + (size_t)f * p.h * p.w * 3;
+            float x[32];
 #pragma unroll
-            for (int kw = 0; kw < 3; kw++) {
-                int ix = 2 * ox - 1 + kw;
-                bool ok = iy >= 0 && iy < p.h && ix >= 0 && ix < p.w;
-                const uint8_t *px = base + ((size_t)iy * p.w + ix) * 3;
+            for (int k = 27; k < 32; k++) x[k] = 0.0f;
 #pragma unroll
-                for (int c = 0; c < 3; c++)
-                    x[(kh * 3 + kw) * 3 + c] = ok ? ((float)((int)__ldg(px + c) - 128) * 0.0078125f) : 0.0f;
+            for (int kh = 0; kh < 3; kh++) {
+                const int iy = 2 * oy - 1 + kh;
+#pragma unroll
+                for (int kw = 0; kw < 3; kw++) {
+                    const int ix = 2 * ox - 1 + kw;
+                    const bool ok = iy >= 0 && iy < p.h && ix >= 0 && ix < p.w;
+                    const uint8_t *q = base + ((ptrdiff_t)iy * p.w + ix) * 3;
+#pragma unroll
+                    for (int c = 0; c < 3; c++)
+                        x[(kh * 3 + kw) * 3 + c] = ok ? (float)((int)__ldg(q + c) - 128) * 0.0078125f : 0.0f;
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < 16; j++) kv[j] = pack_bf16x2(x[2 * j], x[2 * j + 1]);  // exact
+        }
+#pragma unroll
+        for (int c = 0; c < 4; c++)
+            *reinterpret_cast<uint4 *>(sA + (c * 128 + t) * 16) = make_uint4(kv[4 * c], kv[4 * c + 1], kv[4 * c + 2], kv[4 * c + 3]);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic-proxy stores -> tensor core
+        tc_fence_before();
+        __syncthreads();
+        if (t == 0) {
+            tc_fence_after();
+            const uint32_t a0 = smem_u32(sA), b0 = smem_u32(sB);
+#pragma unroll
+            for (int s = 0; s < 2; s++)
+                umma_bf16(tmem, umma_desc(a0 + 2 * s * 2048, 2048, 128), umma_desc(b0 + 2 * s * 512, 512, 128), idesc, s);
+            umma_commit(&bar);
+        }
+        mbar_wait(&bar, phase);
+        phase ^= 1;
+        tc_fence_after();
+        uint32_t v[32];
+        tmem_ld32(tmem + ((uint32_t)(warp * 32) << 16), v);
+        if (valid) {
+            int plane;
+            const int64_t L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, f, oy, ox, plane);
+#pragma unroll
+            for (int cc = 0; cc < 4; cc++) {
+                uint32_t pk[4];
+#pragma unroll
+                for (int j = 0; j < 4; j++) {
+                    float a0 = fmaxf(__uint_as_float(v[cc * 8 + 2 * j]) + sbias[cc * 8 + 2 * j], 0.0f);
+                    float a1 = fmaxf(__uint_as_float(v[cc * 8 + 2 * j + 1]) + sbias[cc * 8 + 2 * j + 1], 0.0f);
+                    pk[j] = pack_bf16x2(a0, a1);
+                }
+                *reinterpret_cast<uint4 *>(p.out + (((size_t)plane * 4 + cc) * p.out_lcap + L) * 16) =
+                    make_uint4(pk[0], pk[1], pk[2], pk[3]);
             }
         }
-        int plane;
-        int64_t L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, f, oy, ox, plane);
-#pragma unroll
-        for (int cc = 0; cc < 4; cc++) {
-            float acc[8];
-#pragma unroll
-            for (int j = 0; j < 8; j++) acc[j] = 0.0f;
-#pragma unroll
-            for (int k = 0; k < 27; k++) {
-#pragma unroll
-                for (int j = 0; j < 8; j++) acc[j] = fmaf(sw[k * 32 + cc * 8 + j], x[k], acc[j]);
-            }
-            uint32_t pk[4];
-#pragma unroll
-            for (int j = 0; j < 4; j++) {
-                float a = fmaxf(acc[2 * j] + sb[cc * 8 + 2 * j], 0.0f);
-                float b = fmaxf(acc[2 * j + 1] + sb[cc * 8 + 2 * j + 1], 0.0f);
-                pk[j] = pack_bf16x2(a, b);
-            }
-            uint8_t *dst = p.out + (((size_t)plane * 4 + cc) * p.out_lcap + L) * 16;
-            *reinterpret_cast<uint4 *>(dst) = make_uint4(pk[0], pk[1], pk[2], pk[3]);
-        }
+        tc_fence_before();
+        __syncthreads();  // accumulator read and smem A consumed before the next tile overwrites them
     }
+    tc_fence_after();
+    if (warp == 0) tmem_dealloc(tmem, 32);
 }
 
 // ---------------------------------------------------------------------------
@@ -382,7 +430,8 @@ struct otif_proxy {
     int gh, gw;
     int e1_oh, e1_ow;
     otif::GemmLayer L[5];         // E2, E3, E4, E5, D1
-    float *e1_w_dev, *e1_b_dev;   // [27][32], [32]
+    uint16_t *e1_w_dev;           // [4][32][8] bf16 (K = 27 padded to 32)
+    float *e1_b_dev;              // [32]
     float *w2_dev;                // [dec] bf16-rounded
     float b2;
     int num_sms;
@@ -508,14 +557,14 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
     {
         E1Params e;
         e.img = img; e.n = n; e.h = p->d.in_h; e.w = p->d.in_w; e.oh = p->e1_oh; e.ow = p->e1_ow;
-        e.wt = p->e1_w_dev; e.bias = p->e1_b_dev;
+        e.bias = p->e1_b_dev;
         e.out_kind = lay[0].kind; e.out_pitch = lay[0].pitch; e.out_fstride = lay[0].fstride;
         e.out_lcap = lay[0].lcap; e.out = ws + lay[0].offset;
-        int64_t total = (int64_t)n * e.oh * e.ow;
-        int64_t blocks = cdiv(total, 256);
-        if (blocks > (int64_t)p->num_sms * 16) blocks = (int64_t)p->num_sms * 16;
+        e.wpk = p->e1_w_dev;
+        e.ntiles = cdiv((int64_t)n * e.oh * e.ow, 128);
+        int64_t blocks = e.ntiles < (int64_t)p->num_sms * 8 ? e.ntiles : (int64_t)p->num_sms * 8;
         if (blocks < 1) blocks = 1;
-        e1_kernel<<<(unsigned)blocks, 256, 0, stream>>>(e);
+        e1_umma_kernel<<<(unsigned)blocks, 128, 0, stream>>>(e);
         OTIF_LAUNCH_CHECK();
         if (evs) OTIF_CUDA(cudaEventRecord(evs[0], stream));
     }
@@ -616,22 +665,22 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
 
     otif_status rc = OTIF_OK;
     std::vector<float> host;
-    // E1 weights -> [27][32] with k = (kh*3+kw)*3 + c
+    // E1 weights -> bf16 [chunk j][n][8], k = j*8 + e = (kh*3+kw)*3 + c, zero for k >= 27
     {
-        std::vector<float> w1(27 * 32), b1(32);
+        std::vector<uint16_t> w1(4 * 32 * 8, 0);
+        std::vector<float> b1(32);
         for (int o = 0; o < 32; o++) {
-            for (int kh = 0; kh < 3; kh++)
-                for (int kw = 0; kw < 3; kw++)
-                    for (int c = 0; c < 3; c++) {
-                        float v = weights[offs[0] + ((size_t)(o * 3 + kh) * 3 + kw) * 3 + c];
-                        w1[((kh * 3 + kw) * 3 + c) * 32 + o] = bf16_to_f32(f32_to_bf16_rne(v));
-                    }
+            for (int k = 0; k < 27; k++) {
+                int kh = k / 9, kw = (k / 3) % 3, c = k % 3;
+                float v = weights[offs[0] + ((size_t)(o * 3 + kh) * 3 + kw) * 3 + c];
+                w1[((k / 8) * 32 + o) * 8 + (k % 8)] = f32_to_bf16_rne(v);
+            }
             b1[o] = weights[offs[0] + (size_t)32 * 27 + o];
         }
-        if (cudaMalloc(&p->e1_w_dev, w1.size() * 4) != cudaSuccess || cudaMalloc(&p->e1_b_dev, 32 * 4) != cudaSuccess) {
+        if (cudaMalloc(&p->e1_w_dev, w1.size() * 2) != cudaSuccess || cudaMalloc(&p->e1_b_dev, 32 * 4) != cudaSuccess) {
             rc = OTIF_ENOMEM;
         } else {
-            cudaMemcpy(p->e1_w_dev, w1.data(), w1.size() * 4, cudaMemcpyHostToDevice);
+            cudaMemcpy(p->e1_w_dev, w1.data(), w1.size() * 2, cudaMemcpyHostToDevice);
             cudaMemcpy(p->e1_b_dev, b1.data(), 32 * 4, cudaMemcpyHostToDevice);
         }
     }

@@ -4,14 +4,17 @@
 // and tie-breaks are DESIGN.md §3 readings R6–R11, R14, R15; all decisions use
 // integer arithmetic (int64 costs), so the output is bit-exact by construction.
 //
-// K5 select_kernel: one CTA per frame.
-//   threshold -> union-find connected components in shared memory (lock-free
-//   atomicCAS linking of the larger root under the smaller, so every root is its
-//   component's first cell in raster order) -> block scan for raster-ordered
-//   component ids -> shared-memory atomic bounding boxes -> phase A (parallel
-//   best-gain pair search, block argmax with lexicographic tie-break) / phase B
-//   (parallel first-overlapping-pair search) -> placement, strict full-frame
-//   fallback, rank sort by (y, x) -> per-frame scratch.
+// K5 select_kernel: ONE WARP PER FRAME (several frames per CTA, each warp owns a
+// private shared-memory slice; warp-synchronous, no block barriers):
+//   threshold (vectorised score loads) -> union-find connected components in shared
+//   memory (lock-free atomicCAS linking of the larger root under the smaller, so a
+//   root is its component's first cell in raster order) -> read-only flatten ->
+//   warp scan for raster-ordered component ids -> shared atomic bounding boxes ->
+//   phase A with a per-cluster best-partner cache (bg[i], bj[i] = best gain / partner
+//   over j > i; after a merge only the affected rows are rescanned, so a frame costs
+//   O(n^2) pair evaluations instead of O(n^3)) -> phase B (first overlapping pair) ->
+//   placement, strict full-frame fallback, rank sort by (y, x) -> per-frame scratch.
+//   Optionally (pipeline) accumulates the run counters with a few atomics per frame.
 // K6 compact_kernel: exclusive scan of per-frame counts (frame_offset, total) and
 //   compaction of the windows into the caller's array in (frame, y, x) order.
 #include <string.h>
@@ -22,7 +25,7 @@
 
 namespace otif {
 
-constexpr int kSelThreads = 256;
+constexpr int kSelWarpsMax = 8;
 constexpr int kMaxSizes = 8;
 
 struct SelectParams {
@@ -39,37 +42,11 @@ struct SelectParams {
     otif_window *tmp;           // [n][cap_f]
     int cap_f;
     int *counts;                // [n]
+    int frame_bytes;            // shared bytes per warp (frame slice)
+    // pipeline-only (internal): run counters, global frame index base
+    unsigned long long *ctr;
+    int frame_base;
 };
-
-__device__ __forceinline__ int uf_find(volatile int *par, int x) {
-    while (true) {
-        int p = par[x];
-        if (p == x) return x;
-        int gp = par[p];
-        if (gp != p) par[x] = gp;  // path halving; parents only ever decrease
-        x = p;
-    }
-}
-
-__device__ __forceinline__ void uf_union(int *par, int a, int b) {
-    volatile int *vp = par;
-    while (true) {
-        a = uf_find(vp, a);
-        b = uf_find(vp, b);
-        if (a == b) return;
-        if (a < b) { int t = a; a = b; b = t; }   // link the larger root under the smaller
-        int old = atomicCAS(&par[a], a, b);
-        if (old == a) return;
-        a = old;
-    }
-}
-
-// fit: first W' entry containing a (w x h) rectangle
-__device__ __forceinline__ int fit_size(const SelectParams &p, int w, int h) {
-    for (int s = 0; s < p.k; s++)
-        if (p.sw[s] >= w && p.sh[s] >= h) return s;
-    return p.k - 1;  // unreachable: the full frame is in W and contains every cluster
-}
 
 struct Rect16 { short x0, y0, x1, y1; };  // cell units, half-open
 
@@ -80,10 +57,14 @@ __device__ __forceinline__ void rect_px(const SelectParams &p, Rect16 r, int &x0
     y1 = min((int)r.y1 * p.cell, p.fh);
 }
 
+// fit: first W' entry containing the cluster's pixel rectangle
 __device__ __forceinline__ int fit_rect(const SelectParams &p, Rect16 r) {
     int x0, y0, x1, y1;
     rect_px(p, r, x0, y0, x1, y1);
-    return fit_size(p, x1 - x0, y1 - y0);
+    const int w = x1 - x0, h = y1 - y0;
+    for (int s = 0; s < p.k; s++)
+        if (p.sw[s] >= w && p.sh[s] >= h) return s;
+    return p.full;  // unreachable: the full frame is in W and contains every cluster
 }
 
 __device__ __forceinline__ Rect16 runion(Rect16 a, Rect16 b) {
@@ -100,250 +81,328 @@ __device__ __forceinline__ void place(const SelectParams &p, Rect16 r, int s, in
     y = min(max(y0 - (p.sh[s] - (y1 - y0)) / 2, 0), p.fh - p.sh[s]);
 }
 
-// block reduce of (gain desc, pair asc)
-__device__ void block_argmax(long long &g, int &pp, long long *sg, int *sp) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        long long og = __shfl_down_sync(0xffffffffu, g, o);
-        int op = __shfl_down_sync(0xffffffffu, pp, o);
-        if (og > g || (og == g && op < pp)) { g = og; pp = op; }
+__device__ __forceinline__ int uf_find(volatile int *par, int x) {
+    while (true) {
+        int q = par[x];
+        if (q == x) return x;
+        int g = par[q];
+        if (g != q) par[x] = g;  // path halving; parents only ever decrease
+        x = q;
     }
-    if (lane == 0) { sg[warp] = g; sp[warp] = pp; }
-    __syncthreads();
-    if (warp == 0) {
-        const int nw = blockDim.x >> 5;
-        g = lane < nw ? sg[lane] : 0;
-        pp = lane < nw ? sp[lane] : 0x7FFFFFFF;
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            long long og = __shfl_down_sync(0xffffffffu, g, o);
-            int op = __shfl_down_sync(0xffffffffu, pp, o);
-            if (og > g || (og == g && op < pp)) { g = og; pp = op; }
-        }
-        if (lane == 0) { sg[0] = g; sp[0] = pp; }
-    }
-    __syncthreads();
-    g = sg[0];
-    pp = sp[0];
-    __syncthreads();
 }
 
-__global__ void __launch_bounds__(kSelThreads) select_kernel(const __grid_constant__ SelectParams p) {
+__device__ __forceinline__ void uf_union(int *par, int a, int b) {
+    volatile int *vp = par;
+    while (true) {
+        a = uf_find(vp, a);
+        b = uf_find(vp, b);
+        if (a == b) return;
+        if (a < b) { int t = a; a = b; b = t; }   // link the larger root under the smaller
+        int old = atomicCAS(&par[a], a, b);
+        if (old == a) return;
+        a = old;
+    }
+}
+
+__device__ __forceinline__ unsigned long long mix64(unsigned long long z) {
+    z += 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+constexpr long long kNoGain = (long long)0x8000000000000000ull;
+
+struct Frame {  // one warp's shared-memory slice
+    int *par;          // [cells]
+    short *cid;        // [cells]
+    Rect16 *cl;        // [cap]
+    long long *cost;   // [cap]
+    long long *bg;     // [cap] best gain over alive j > i
+    short *bj;         // [cap] best partner
+    signed char *sidx; // [cap]
+    signed char *alive;// [cap]
+};
+
+// best partner of row i over alive j > i (max gain, smallest j)
+__device__ __forceinline__ void rescan_row(const SelectParams &p, Frame &F, int n, int i) {
+    long long best = kNoGain;
+    int bjv = -1;
+    const Rect16 ri = F.cl[i];
+    const long long ci = F.cost[i];
+    for (int j = i + 1; j < n; j++) {
+        if (!F.alive[j]) continue;
+        long long g = ci + F.cost[j] - p.cost[fit_rect(p, runion(ri, F.cl[j]))];
+        if (g > best) { best = g; bjv = j; }
+    }
+    F.bg[i] = best;
+    F.bj[i] = (short)bjv;
+}
+
+__global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_constant__ SelectParams p) {
     extern __shared__ __align__(16) uint8_t smem[];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int f = blockIdx.x * (blockDim.x >> 5) + wid;
+    if (f >= p.n) return;
     const int cells = p.gh * p.gw;
-    const int f = blockIdx.x;
-    int *par = reinterpret_cast<int *>(smem);                             // [cells]
-    short *cid = reinterpret_cast<short *>(par + cells);                  // [cells]
-    uint8_t *cl_base = smem + ((cells * 6 + 15) & ~15);
-    Rect16 *cl = reinterpret_cast<Rect16 *>(cl_base);                     // [cap]
-    long long *cost = reinterpret_cast<long long *>(cl + p.cap_f);        // [cap]
-    int *px = reinterpret_cast<int *>(cost + p.cap_f);                    // [cap]
-    int *py = px + p.cap_f;                                               // [cap]
-    signed char *sidx = reinterpret_cast<signed char *>(py + p.cap_f);    // [cap]
-    signed char *alive = sidx + p.cap_f;                                  // [cap]
-    __shared__ long long s_red_g[32];
-    __shared__ int s_red_p[32];
-    __shared__ int s_scan[kSelThreads];
-    __shared__ int s_ncomp, s_min_pair;
+    const int cap = p.cap_f;
+    uint8_t *base = smem + (size_t)wid * p.frame_bytes;
+    Frame F;
+    F.par = reinterpret_cast<int *>(base);
+    F.cid = reinterpret_cast<short *>(F.par + cells);
+    uint8_t *cb = base + ((cells * 6 + 15) & ~15);
+    F.cl = reinterpret_cast<Rect16 *>(cb);
+    F.cost = reinterpret_cast<long long *>(F.cl + cap);
+    F.bg = F.cost + cap;
+    F.bj = reinterpret_cast<short *>(F.bg + cap);
+    F.sidx = reinterpret_cast<signed char *>(F.bj + cap);
+    F.alive = F.sidx + cap;
 
     // --- stage 3: threshold (strict ">") ---
-    for (int i = threadIdx.x; i < cells; i += blockDim.x) {
+    int npos = 0;
+    for (int i = lane; i < cells; i += 32) {
         bool m;
         if (p.mask_in) m = p.mask_in[(size_t)f * cells + i] != 0;
-        else m = p.scores[(size_t)f * cells + i] > p.thr;
-        par[i] = m ? i : -1;
+        else m = __ldg(p.scores + (size_t)f * cells + i) > p.thr;
+        F.par[i] = m ? i : -1;
+        npos += m;
         if (p.mask_out) p.mask_out[(size_t)f * cells + i] = m ? 1 : 0;
     }
-    __syncthreads();
+    __syncwarp();
 
     // --- connected components, 4- or 8-connectivity (reading R6) ---
-    for (int i = threadIdx.x; i < cells; i += blockDim.x) {
-        if (par[i] < 0) continue;
+    for (int i = lane; i < cells; i += 32) {
+        if (F.par[i] < 0) continue;
         int y = i / p.gw, x = i - y * p.gw;
-        if (x + 1 < p.gw && par[i + 1] >= 0) uf_union(par, i, i + 1);
+        if (x + 1 < p.gw && F.par[i + 1] >= 0) uf_union(F.par, i, i + 1);
         if (y + 1 < p.gh) {
             int d = i + p.gw;
-            if (par[d] >= 0) uf_union(par, i, d);
+            if (F.par[d] >= 0) uf_union(F.par, i, d);
             if (p.conn == 8) {
-                if (x > 0 && par[d - 1] >= 0) uf_union(par, i, d - 1);
-                if (x + 1 < p.gw && par[d + 1] >= 0) uf_union(par, i, d + 1);
+                if (x > 0 && F.par[d - 1] >= 0) uf_union(F.par, i, d - 1);
+                if (x + 1 < p.gw && F.par[d + 1] >= 0) uf_union(F.par, i, d + 1);
             }
         }
     }
-    __syncthreads();
-    // flatten: resolve every root with read-only walks into a scratch array first (a
-    // path-halving write racing with another thread's flatten store could leave a
-    // non-root parent behind), then publish.  px/py (2*cap >= cells ints) are free here.
+    __syncwarp();
+    // read-only flatten into scratch (cl/cost region: 16*cap >= 4*cells bytes), then publish
     {
-        int *lab = px;
-        for (int i = threadIdx.x; i < cells; i += blockDim.x) {
-            int x = par[i];
+        int *lab = reinterpret_cast<int *>(F.cl);
+        for (int i = lane; i < cells; i += 32) {
+            int x = F.par[i];
             if (x >= 0)
-                while (par[x] != x) x = par[x];
+                while (F.par[x] != x) x = F.par[x];
             lab[i] = x;
         }
-        __syncthreads();
-        for (int i = threadIdx.x; i < cells; i += blockDim.x) par[i] = lab[i];
+        __syncwarp();
+        for (int i = lane; i < cells; i += 32) F.par[i] = lab[i];
+        __syncwarp();
     }
-    __syncthreads();
-
-    // raster-ordered component ids: exclusive scan of root flags over contiguous segments
+    // raster-ordered component ids: warp exclusive scan of root flags over contiguous segments
+    int n;
     {
-        const int seg = (cells + blockDim.x - 1) / blockDim.x;
-        const int a = threadIdx.x * seg, b = min(a + seg, cells);
+        const int seg = (cells + 31) / 32;
+        const int a = lane * seg, b = min(a + seg, cells);
         int cnt = 0;
-        for (int i = a; i < b; i++) cnt += (par[i] == i);
-        s_scan[threadIdx.x] = cnt;
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            int run = 0;
-            for (int t = 0; t < (int)blockDim.x; t++) { int v = s_scan[t]; s_scan[t] = run; run += v; }
-            s_ncomp = run;
+        for (int i = a; i < b; i++) cnt += (F.par[i] == i);
+        int incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            int t = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += t;
         }
-        __syncthreads();
-        int id = s_scan[threadIdx.x];
+        n = __shfl_sync(0xffffffffu, incl, 31);
+        int id = incl - cnt;
         for (int i = a; i < b; i++)
-            if (par[i] == i) cid[i] = (short)id++;
+            if (F.par[i] == i) F.cid[i] = (short)id++;
     }
-    __syncthreads();
-    const int n = s_ncomp;
+    __syncwarp();
+    for (int o = 16; o > 0; o >>= 1) npos += __shfl_xor_sync(0xffffffffu, npos, o);
+    otif_window *out = p.tmp + (size_t)f * cap;
     if (n == 0) {
-        if (threadIdx.x == 0) p.counts[f] = 0;
+        if (lane == 0) {
+            p.counts[f] = 0;
+            if (p.ctr) atomicAdd(&p.ctr[0], 1ull);
+        }
         return;
     }
-    for (int c = threadIdx.x; c < n; c += blockDim.x) {
-        cl[c].x0 = 0x7FFF; cl[c].y0 = 0x7FFF; cl[c].x1 = -1; cl[c].y1 = -1;
-        alive[c] = 1;
+    // bounding boxes (cell units) with 32-bit shared atomics on shadow arrays in bg (2*cap ints)
+    // and cost (2*cap ints), both unused until the boxes are final
+    {
+        int *bx0 = reinterpret_cast<int *>(F.bg), *by0 = bx0 + cap;
+        int *bx1 = reinterpret_cast<int *>(F.cost), *by1 = bx1 + cap;
+        for (int c = lane; c < n; c += 32) {
+            bx0[c] = 0x7FFFFFFF; by0[c] = 0x7FFFFFFF; bx1[c] = -1; by1[c] = -1;
+        }
+        __syncwarp();
+        for (int i = lane; i < cells; i += 32) {
+            if (F.par[i] < 0) continue;
+            int c = F.cid[F.par[i]];
+            int y = i / p.gw, x = i - y * p.gw;
+            atomicMin(&bx0[c], x); atomicMin(&by0[c], y);
+            atomicMax(&bx1[c], x + 1); atomicMax(&by1[c], y + 1);
+        }
+        __syncwarp();
+        for (int c = lane; c < n; c += 32) {
+            Rect16 r;
+            r.x0 = (short)bx0[c]; r.y0 = (short)by0[c]; r.x1 = (short)bx1[c]; r.y1 = (short)by1[c];
+            F.cl[c] = r;
+        }
+        __syncwarp();
+        for (int c = lane; c < n; c += 32) {
+            int s = fit_rect(p, F.cl[c]);
+            F.sidx[c] = (signed char)s;
+            F.cost[c] = p.cost[s];
+            F.alive[c] = 1;
+        }
+        __syncwarp();
     }
-    __syncthreads();
-    // bounding boxes in cell units: 32-bit shared atomics on shadow arrays carved from
-    // px / py / cost (not yet in use)
-    int *bx0 = px, *by0 = py;
-    int *bx1 = reinterpret_cast<int *>(cost), *by1 = bx1 + p.cap_f;
-    for (int c = threadIdx.x; c < n; c += blockDim.x) {
-        bx0[c] = 0x7FFFFFFF; by0[c] = 0x7FFFFFFF; bx1[c] = -1; by1[c] = -1;
-    }
-    __syncthreads();
-    for (int i = threadIdx.x; i < cells; i += blockDim.x) {
-        if (par[i] < 0) continue;
-        int c = cid[par[i]];
-        int y = i / p.gw, x = i - y * p.gw;
-        atomicMin(&bx0[c], x); atomicMin(&by0[c], y);
-        atomicMax(&bx1[c], x + 1); atomicMax(&by1[c], y + 1);
-    }
-    __syncthreads();
-    for (int c = threadIdx.x; c < n; c += blockDim.x) {
-        Rect16 r;
-        r.x0 = (short)bx0[c]; r.y0 = (short)by0[c]; r.x1 = (short)bx1[c]; r.y1 = (short)by1[c];
-        cl[c] = r;
-    }
-    __syncthreads();
-    for (int c = threadIdx.x; c < n; c += blockDim.x) {
-        int s = fit_rect(p, cl[c]);
-        sidx[c] = (signed char)s;
-        cost[c] = p.cost[s];
-    }
-    __syncthreads();
 
     // --- grouping: phase A greedy merge, phase B disjointness (readings R7, R10) ---
-    const long long npairs = (long long)n * n;
     while (true) {
+        for (int i = lane; i < n; i += 32)
+            if (F.alive[i]) rescan_row(p, F, n, i);
+        __syncwarp();
         while (true) {  // phase A
-            long long best = 0;
-            int bp = 0x7FFFFFFF;
-            for (long long q = threadIdx.x; q < npairs; q += blockDim.x) {
-                int i = (int)(q / n), j = (int)(q - (long long)i * n);
-                if (j <= i || !alive[i] || !alive[j]) continue;
-                Rect16 u = runion(cl[i], cl[j]);
-                long long g = cost[i] + cost[j] - p.cost[fit_rect(p, u)];
-                if (g > best) { best = g; bp = (int)q; }   // q ascending per thread: first max is smallest
+            long long G = kNoGain;
+            int I = 0x7FFF;
+            for (int i = lane; i < n; i += 32)
+                if (F.alive[i] && (F.bg[i] > G || (F.bg[i] == G && i < I))) { G = F.bg[i]; I = i; }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                long long og = __shfl_xor_sync(0xffffffffu, G, o);
+                int oi = __shfl_xor_sync(0xffffffffu, I, o);
+                if (og > G || (og == G && oi < I)) { G = og; I = oi; }
             }
-            block_argmax(best, bp, s_red_g, s_red_p);
-            if (best <= 0) break;                           // "merging offers no further improvement"
-            if (threadIdx.x == 0) {
-                int i = bp / n, j = bp - i * n;
-                cl[i] = runion(cl[i], cl[j]);
-                int s = fit_rect(p, cl[i]);
-                sidx[i] = (signed char)s;
-                cost[i] = p.cost[s];
-                alive[j] = 0;
+            if (G <= 0) break;  // "once merging offers no further improvement" (strict)
+            const int J = F.bj[I];
+            __syncwarp();
+            if (lane == 0) {
+                F.cl[I] = runion(F.cl[I], F.cl[J]);
+                int s = fit_rect(p, F.cl[I]);
+                F.sidx[I] = (signed char)s;
+                F.cost[I] = p.cost[s];
+                F.alive[J] = 0;
             }
-            __syncthreads();
+            __syncwarp();
+            for (int i = lane; i < n; i += 32) {
+                if (!F.alive[i]) continue;
+                const int b = F.bj[i];
+                if (i == I || b == I || b == J) {
+                    rescan_row(p, F, n, i);
+                } else if (i < I) {
+                    long long g = F.cost[i] + F.cost[I] - p.cost[fit_rect(p, runion(F.cl[i], F.cl[I]))];
+                    if (g > F.bg[i] || (g == F.bg[i] && I < b)) { F.bg[i] = g; F.bj[i] = (short)I; }
+                }
+            }
+            __syncwarp();
         }
-        // phase B: place every cluster, merge the lexicographically first overlapping pair
-        for (int c = threadIdx.x; c < n; c += blockDim.x)
-            if (alive[c]) place(p, cl[c], sidx[c], px[c], py[c]);
-        if (threadIdx.x == 0) s_min_pair = 0x7FFFFFFF;
-        __syncthreads();
-        for (long long q = threadIdx.x; q < npairs; q += blockDim.x) {
-            int i = (int)(q / n), j = (int)(q - (long long)i * n);
-            if (j <= i || !alive[i] || !alive[j]) continue;
-            int si = sidx[i], sj = sidx[j];
-            bool ox = px[i] < px[j] + p.sw[sj] && px[j] < px[i] + p.sw[si];
-            bool oy = py[i] < py[j] + p.sh[sj] && py[j] < py[i] + p.sh[si];
-            if (ox && oy) { atomicMin(&s_min_pair, (int)q); break; }  // later q of this thread are larger
+        // phase B: merge the lexicographically first pair whose placed windows overlap
+        int mi = 0x7FFF, mj = 0x7FFF;
+        for (int i = lane; i < n; i += 32) {
+            if (!F.alive[i]) continue;
+            int xi, yi, si = F.sidx[i];
+            place(p, F.cl[i], si, xi, yi);
+            for (int j = i + 1; j < n; j++) {
+                if (!F.alive[j]) continue;
+                int xj, yj, sj = F.sidx[j];
+                place(p, F.cl[j], sj, xj, yj);
+                if (xi < xj + p.sw[sj] && xj < xi + p.sw[si] && yi < yj + p.sh[sj] && yj < yi + p.sh[si]) {
+                    if (i < mi) { mi = i; mj = j; }
+                    break;
+                }
+            }
+            if (mi != 0x7FFF) break;  // later i of this lane are larger
         }
-        __syncthreads();
-        const int mp = s_min_pair;
-        if (mp == 0x7FFFFFFF) break;
-        if (threadIdx.x == 0) {
-            int i = mp / n, j = mp - i * n;
-            cl[i] = runion(cl[i], cl[j]);
-            int s = fit_rect(p, cl[i]);
-            sidx[i] = (signed char)s;
-            cost[i] = p.cost[s];
-            alive[j] = 0;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            int oi = __shfl_xor_sync(0xffffffffu, mi, o);
+            int oj = __shfl_xor_sync(0xffffffffu, mj, o);
+            if (oi < mi) { mi = oi; mj = oj; }
         }
-        __syncthreads();
+        if (mi == 0x7FFF) break;
+        __syncwarp();
+        if (lane == 0) {
+            F.cl[mi] = runion(F.cl[mi], F.cl[mj]);
+            int s = fit_rect(p, F.cl[mi]);
+            F.sidx[mi] = (signed char)s;
+            F.cost[mi] = p.cost[s];
+            F.alive[mj] = 0;
+        }
+        __syncwarp();
     }
 
     // --- emission: est(R), strict full-frame fallback (R11), (y, x) order (R15) ---
     long long est = 0;
     int m = 0;
-    for (int c = threadIdx.x; c < n; c += blockDim.x)
-        if (alive[c]) { est += cost[c]; m++; }
-    {
-        // block sums via the argmax scratch (sum reduction)
-        const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-        for (int o = 16; o > 0; o >>= 1) {
-            est += __shfl_down_sync(0xffffffffu, est, o);
-            m += __shfl_down_sync(0xffffffffu, m, o);
-        }
-        if (lane == 0) { s_red_g[warp] = est; s_red_p[warp] = m; }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            long long e = 0;
-            int mm = 0;
-            for (int w = 0; w < (int)(blockDim.x >> 5); w++) { e += s_red_g[w]; mm += s_red_p[w]; }
-            s_red_g[0] = e;
-            s_red_p[0] = mm;
-        }
-        __syncthreads();
-        est = s_red_g[0];
-        m = s_red_p[0];
+    for (int c = lane; c < n; c += 32)
+        if (F.alive[c]) { est += F.cost[c]; m++; }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        est += __shfl_xor_sync(0xffffffffu, est, o);
+        m += __shfl_xor_sync(0xffffffffu, m, o);
     }
-    otif_window *out = p.tmp + (size_t)f * p.cap_f;
+    unsigned long long hsh = 0, pix = 0;
     if (est > p.cost[p.full]) {
-        if (threadIdx.x == 0) {
+        if (lane == 0) {
             otif_window w;
             w.frame = f; w.x = 0; w.y = 0; w.w = p.fw; w.h = p.fh; w.size_idx = p.orig[p.full];
             out[0] = w;
             p.counts[f] = 1;
+            if (p.ctr) {
+                unsigned long long gf = (unsigned long long)(unsigned)(f + p.frame_base);
+                atomicAdd(&p.ctr[0], 1ull);
+                atomicAdd(&p.ctr[1], (unsigned long long)npos);
+                atomicAdd(&p.ctr[2], 1ull);
+                atomicAdd(&p.ctr[3], (unsigned long long)p.fw * p.fh);
+                atomicAdd(&p.ctr[4], mix64((gf << 32) ^ mix64(((unsigned long long)p.fw << 20) ^
+                                                               ((unsigned long long)p.fh << 4) ^ (unsigned)w.size_idx)));
+                atomicAdd(&p.ctr[5 + w.size_idx], 1ull);
+            }
         }
         return;
     }
-    for (int c = threadIdx.x; c < n; c += blockDim.x) {
-        if (!alive[c]) continue;
+    // rank each alive cluster's placed window by (y, x); placements recomputed per lane
+    for (int c = lane; c < n; c += 32) {
+        if (!F.alive[c]) continue;
+        int xc, yc, sc = F.sidx[c];
+        place(p, F.cl[c], sc, xc, yc);
         int rank = 0;
-        for (int d = 0; d < n; d++)
-            if (alive[d] && (py[d] < py[c] || (py[d] == py[c] && px[d] < px[c]))) rank++;
+        for (int d = 0; d < n; d++) {
+            if (!F.alive[d] || d == c) continue;
+            int xd, yd;
+            place(p, F.cl[d], F.sidx[d], xd, yd);
+            rank += (yd < yc || (yd == yc && xd < xc));
+        }
         otif_window w;
-        w.frame = f; w.x = px[c]; w.y = py[c];
-        w.w = p.sw[sidx[c]]; w.h = p.sh[sidx[c]]; w.size_idx = p.orig[sidx[c]];
+        w.frame = f; w.x = xc; w.y = yc; w.w = p.sw[sc]; w.h = p.sh[sc]; w.size_idx = p.orig[sc];
         out[rank] = w;
+        if (p.ctr) {
+            unsigned long long gf = (unsigned long long)(unsigned)(f + p.frame_base);
+            unsigned long long key = (gf << 32) ^ ((unsigned long long)(unsigned)xc << 16) ^ (unsigned)yc;
+            hsh += mix64(key ^ mix64(((unsigned long long)w.w << 20) ^ ((unsigned long long)w.h << 4) ^
+                                     (unsigned)w.size_idx));
+            pix += (unsigned long long)w.w * w.h;
+            atomicAdd(&p.ctr[5 + w.size_idx], 1ull);
+        }
     }
-    if (threadIdx.x == 0) p.counts[f] = m;
+    if (p.ctr) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            hsh += __shfl_xor_sync(0xffffffffu, hsh, o);
+            pix += __shfl_xor_sync(0xffffffffu, pix, o);
+        }
+    }
+    if (lane == 0) {
+        p.counts[f] = m;
+        if (p.ctr) {
+            atomicAdd(&p.ctr[0], 1ull);
+            atomicAdd(&p.ctr[1], (unsigned long long)npos);
+            atomicAdd(&p.ctr[2], (unsigned long long)m);
+            atomicAdd(&p.ctr[3], pix);
+            atomicAdd(&p.ctr[4], hsh);
+        }
+    }
 }
 
 // K6: scan of per-frame counts + compaction into (frame, y, x) order
@@ -353,7 +412,6 @@ __global__ void __launch_bounds__(1024) compact_kernel(const otif_window *__rest
     __shared__ int s_warp[32];
     __shared__ int s_base;
     const int f0 = blockIdx.x * blockDim.x;
-    // base = sum of counts of all earlier frames
     int part = 0;
     for (int i = threadIdx.x; i < f0; i += blockDim.x) part += counts[i];
     for (int o = 16; o > 0; o >>= 1) part += __shfl_down_sync(0xffffffffu, part, o);
@@ -367,7 +425,6 @@ __global__ void __launch_bounds__(1024) compact_kernel(const otif_window *__rest
     __syncthreads();
     const int f = f0 + threadIdx.x;
     const int c = f < n ? counts[f] : 0;
-    // block exclusive scan of c
     int v = c;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     for (int o = 1; o < 32; o <<= 1) {
@@ -397,59 +454,21 @@ __global__ void __launch_bounds__(1024) compact_kernel(const otif_window *__rest
     }
 }
 
-}  // namespace otif
-
-using namespace otif;
-
 static int sel_cap(int gh, int gw) { return (gh * gw + 1) / 2 > 1 ? (gh * gw + 1) / 2 : 1; }
 
-static size_t sel_smem(int gh, int gw) {
+static int sel_frame_bytes(int gh, int gw) {
     int cells = gh * gw, cap = sel_cap(gh, gw);
-    size_t head = (size_t)round_up((int64_t)cells * 6, 16);
-    return head + (size_t)cap * (8 + 8 + 4 + 4 + 1 + 1) + 64;
+    int head = (cells * 6 + 15) & ~15;
+    // cl 8 + cost 8 + bg 8 + bj 2 + sidx 1 + alive 1 bytes per cluster
+    return (int)round_up(head + (int64_t)cap * 28, 16);
 }
 
-extern "C" size_t otif_select_workspace_bytes(int32_t n, int32_t gh, int32_t gw) {
-    if (n < 0 || gh <= 0 || gw <= 0) return 0;
-    return (size_t)round_up((int64_t)n * sel_cap(gh, gw) * sizeof(otif_window), 256) + (size_t)round_up((int64_t)n * 4, 256);
-}
-
-extern "C" otif_status otif_select_windows(const float *scores, const uint8_t *mask_in, float threshold, int32_t n,
-                                           int32_t gh, int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes,
-                                           int32_t k, uint8_t *mask_out, otif_window *windows, int32_t capacity,
-                                           int32_t *frame_count, int32_t *frame_offset, int32_t *total,
-                                           void *workspace, size_t ws_bytes, cudaStream_t stream) {
-    OTIF_REQUIRE(g && sizes, "otif_select_windows: NULL descriptor or sizes");
-    OTIF_REQUIRE(n >= 0 && gh > 0 && gw > 0, "otif_select_windows: bad n/grid (%d, %dx%d)", n, gw, gh);
-    OTIF_REQUIRE(g->frame_w > 0 && g->frame_h > 0 && g->cell > 0, "otif_select_windows: bad frame/cell");
-    OTIF_REQUIRE(gh == (g->frame_h + g->cell - 1) / g->cell && gw == (g->frame_w + g->cell - 1) / g->cell,
-                 "otif_select_windows: grid %dx%d != ceil(frame/cell) for %dx%d / %d", gw, gh, g->frame_w,
-                 g->frame_h, g->cell);
-    OTIF_REQUIRE((scores != nullptr) != (mask_in != nullptr), "otif_select_windows: exactly one of scores/mask_in");
-    OTIF_REQUIRE(g->connectivity == 4 || g->connectivity == 8, "otif_select_windows: connectivity must be 4 or 8");
-    OTIF_REQUIRE(k >= 1 && k <= kMaxSizes, "otif_select_windows: k=%d not in [1,8]", k);
-    OTIF_REQUIRE(capacity >= 0, "otif_select_windows: negative capacity");
-    OTIF_REQUIRE(gh * gw <= 8192, "otif_select_windows: grid of %d cells exceeds 8192", gh * gw);
-    OTIF_REQUIRE(g->frame_w <= 0x7FFF && g->frame_h <= 0x7FFF && gw < 0x7FFF && gh < 0x7FFF,
-                 "otif_select_windows: frame too large");
-    bool full = false;
-    for (int i = 0; i < k; i++) {
-        OTIF_REQUIRE(sizes[i].w > 0 && sizes[i].h > 0 && sizes[i].w <= g->frame_w && sizes[i].h <= g->frame_h,
-                     "otif_select_windows: size %d (%dx%d) not inside the %dx%d frame", i, sizes[i].w, sizes[i].h,
-                     g->frame_w, g->frame_h);
-        if (sizes[i].w == g->frame_w && sizes[i].h == g->frame_h) full = true;
-    }
-    OTIF_REQUIRE(full, "otif_select_windows: W must contain the full frame %dx%d (P:L155)", g->frame_w, g->frame_h);
-    if (n == 0) {
-        if (total) OTIF_CUDA(cudaMemsetAsync(total, 0, 4, stream));
-        return OTIF_OK;
-    }
-    OTIF_REQUIRE(windows || capacity == 0, "otif_select_windows: NULL windows");
-    OTIF_REQUIRE(frame_count && frame_offset && total && workspace, "otif_select_windows: NULL output");
-    OTIF_REQUIRE(ws_bytes >= otif_select_workspace_bytes(n, gh, gw), "otif_select_windows: workspace too small");
-    otif_status st = check_device(nullptr);
-    if (st != OTIF_OK) return st;
-
+// internal entry: counters and global frame base for the pipeline (NULL / 0 from the ABI)
+otif_status launch_select(const float *scores, const uint8_t *mask_in, float threshold, int32_t n, int32_t gh,
+                          int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
+                          otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
+                          int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
+                          unsigned long long *ctr, int frame_base) {
     SelectParams p;
     memset(&p, 0, sizeof(p));
     p.scores = scores; p.mask_in = mask_in; p.thr = threshold;
@@ -477,12 +496,78 @@ extern "C" otif_status otif_select_windows(const float *scores, const uint8_t *m
     uint8_t *ws = (uint8_t *)workspace;
     p.tmp = (otif_window *)ws;
     p.counts = (int *)(ws + round_up((int64_t)n * p.cap_f * sizeof(otif_window), 256));
-    size_t smem = sel_smem(gh, gw);
+    p.frame_bytes = sel_frame_bytes(gh, gw);
+    p.ctr = ctr;
+    p.frame_base = frame_base;
+    int warps = (int)((200 * 1024) / p.frame_bytes);
+    warps = warps < 1 ? 1 : (warps > kSelWarpsMax ? kSelWarpsMax : warps);
+    if (warps > n) warps = n;
+    size_t smem = (size_t)warps * p.frame_bytes;
     OTIF_CUDA(cudaFuncSetAttribute(select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    select_kernel<<<n, kSelThreads, smem, stream>>>(p);
+    select_kernel<<<(unsigned)cdiv(n, warps), warps * 32, smem, stream>>>(p);
     OTIF_LAUNCH_CHECK();
     compact_kernel<<<(unsigned)cdiv(n, 1024), 1024, 0, stream>>>(p.tmp, p.cap_f, p.counts, n, windows, capacity,
                                                                  frame_count, frame_offset, total);
     OTIF_LAUNCH_CHECK();
     return OTIF_OK;
+}
+
+size_t select_workspace_bytes(int32_t n, int32_t gh, int32_t gw) {
+    if (n < 0 || gh <= 0 || gw <= 0) return 0;
+    return (size_t)round_up((int64_t)n * sel_cap(gh, gw) * sizeof(otif_window), 256) +
+           (size_t)round_up((int64_t)n * 4, 256);
+}
+
+otif_status validate_select(const float *scores, const uint8_t *mask_in, int32_t n, int32_t gh, int32_t gw,
+                            const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, int32_t capacity) {
+    OTIF_REQUIRE(g && sizes, "otif_select_windows: NULL descriptor or sizes");
+    OTIF_REQUIRE(n >= 0 && gh > 0 && gw > 0, "otif_select_windows: bad n/grid (%d, %dx%d)", n, gw, gh);
+    OTIF_REQUIRE(g->frame_w > 0 && g->frame_h > 0 && g->cell > 0, "otif_select_windows: bad frame/cell");
+    OTIF_REQUIRE(gh == (g->frame_h + g->cell - 1) / g->cell && gw == (g->frame_w + g->cell - 1) / g->cell,
+                 "otif_select_windows: grid %dx%d != ceil(frame/cell) for %dx%d / %d", gw, gh, g->frame_w,
+                 g->frame_h, g->cell);
+    OTIF_REQUIRE((scores != nullptr) != (mask_in != nullptr), "otif_select_windows: exactly one of scores/mask_in");
+    OTIF_REQUIRE(g->connectivity == 4 || g->connectivity == 8, "otif_select_windows: connectivity must be 4 or 8");
+    OTIF_REQUIRE(k >= 1 && k <= kMaxSizes, "otif_select_windows: k=%d not in [1,8]", k);
+    OTIF_REQUIRE(capacity >= 0, "otif_select_windows: negative capacity");
+    OTIF_REQUIRE(gh * gw <= 8192, "otif_select_windows: grid of %d cells exceeds 8192", gh * gw);
+    OTIF_REQUIRE(g->frame_w <= 0x7FFF && g->frame_h <= 0x7FFF && gw < 0x7FFF && gh < 0x7FFF,
+                 "otif_select_windows: frame too large");
+    bool full = false;
+    for (int i = 0; i < k; i++) {
+        OTIF_REQUIRE(sizes[i].w > 0 && sizes[i].h > 0 && sizes[i].w <= g->frame_w && sizes[i].h <= g->frame_h,
+                     "otif_select_windows: size %d (%dx%d) not inside the %dx%d frame", i, sizes[i].w, sizes[i].h,
+                     g->frame_w, g->frame_h);
+        if (sizes[i].w == g->frame_w && sizes[i].h == g->frame_h) full = true;
+    }
+    OTIF_REQUIRE(full, "otif_select_windows: W must contain the full frame %dx%d (P:L155)", g->frame_w, g->frame_h);
+    return OTIF_OK;
+}
+
+}  // namespace otif
+
+using namespace otif;
+
+extern "C" size_t otif_select_workspace_bytes(int32_t n, int32_t gh, int32_t gw) {
+    return select_workspace_bytes(n, gh, gw);
+}
+
+extern "C" otif_status otif_select_windows(const float *scores, const uint8_t *mask_in, float threshold, int32_t n,
+                                           int32_t gh, int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes,
+                                           int32_t k, uint8_t *mask_out, otif_window *windows, int32_t capacity,
+                                           int32_t *frame_count, int32_t *frame_offset, int32_t *total,
+                                           void *workspace, size_t ws_bytes, cudaStream_t stream) {
+    otif_status st = validate_select(scores, mask_in, n, gh, gw, g, sizes, k, capacity);
+    if (st != OTIF_OK) return st;
+    if (n == 0) {
+        if (total) OTIF_CUDA(cudaMemsetAsync(total, 0, 4, stream));
+        return OTIF_OK;
+    }
+    OTIF_REQUIRE(windows || capacity == 0, "otif_select_windows: NULL windows");
+    OTIF_REQUIRE(frame_count && frame_offset && total && workspace, "otif_select_windows: NULL output");
+    OTIF_REQUIRE(ws_bytes >= otif_select_workspace_bytes(n, gh, gw), "otif_select_windows: workspace too small");
+    st = check_device(nullptr);
+    if (st != OTIF_OK) return st;
+    return launch_select(scores, mask_in, threshold, n, gh, gw, g, sizes, k, mask_out, windows, capacity, frame_count,
+                         frame_offset, total, workspace, ws_bytes, stream, nullptr, 0);
 }
