@@ -189,7 +189,12 @@ class Pipeline:
             d.sizes[i].w, d.sizes[i].h = int(s[0]), int(s[1])
             d.sizes[i].cost = int(s[2]) if len(s) > 2 else int(s[0]) * int(s[1])
         d.max_batch = int(max_batch)
-        caps = batch_cap or [max_batch * 4] * d.k
+        if batch_cap is None:
+            # a full-frame window is the only window of its frame; smaller sizes get headroom
+            caps = [max_batch if (int(w[0]), int(w[1])) == (workload.src_w, workload.src_h) else max_batch * 4
+                    for w in workload.sizes]
+        else:
+            caps = batch_cap
         for i in range(d.k):
             d.batch_cap[i] = int(caps[i])
         self.k = d.k

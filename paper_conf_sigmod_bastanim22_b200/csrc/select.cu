@@ -26,6 +26,7 @@
 namespace otif {
 
 constexpr int kSelWarpsMax = 8;
+constexpr int kMatMax = 128;  // fit-matrix capacity (components per frame); larger n -> rescan path
 constexpr int kMaxSizes = 8;
 
 struct SelectParams {
@@ -43,6 +44,8 @@ struct SelectParams {
     int cap_f;
     int *counts;                // [n]
     int frame_bytes;            // shared bytes per warp (frame slice)
+    int nmat;                   // gain-matrix capacity (components); 0 = rescan path only
+    int gmat_offset;            // byte offset of the gain matrix in a frame slice
     // pipeline-only (internal): run counters, global frame index base
     unsigned long long *ctr;
     int frame_base;
@@ -137,6 +140,150 @@ __device__ __forceinline__ void rescan_row(const SelectParams &p, Frame &F, int 
     }
     F.bg[i] = best;
     F.bj[i] = (short)bjv;
+}
+
+// Greedy grouping with a pairwise fit matrix (n <= nmat).  U[i][j] (i < j, one byte)
+// caches the W' index of fit(union(c_i, c_j)) — the gain is then cost_i + cost_j -
+// cost[U[i][j]] (integer, exact) — and 0xFF marks a dead column.  Row bests (bg[i],
+// bj[i]) = max gain over alive j > i, smallest j.  A merge of (I, J) refreshes the n
+// entries of row/column I, kills column J, and recomputes only the affected row bests
+// (row I and rows whose best was I or J, each by the whole warp over the cached row;
+// rows i < I compare against their new U[i][I]) — O(n) work per merge on a warp.
+// Same decisions as the oracle: max gain, ties to the lexicographically smallest (i, j).
+constexpr uint8_t kDead = 0xFF;
+
+__device__ __forceinline__ long long gain_u(const SelectParams &p, const Frame &F, int i, int j, uint8_t u) {
+    return F.cost[i] + F.cost[j] - p.cost[u];
+}
+
+// warp-cooperative recompute of row i's best partner (all lanes call with the same i)
+__device__ __forceinline__ void row_best_warp(const SelectParams &p, Frame &F, const uint8_t *U, int S, int n, int i,
+                                              int lane) {
+    long long best = kNoGain;
+    int arg = 0x7FFF;
+    const uint8_t *row = U + (size_t)i * S;
+    for (int j = i + 1 + lane; j < n; j += 32) {
+        const uint8_t u = row[j];
+        if (u == kDead) continue;
+        const long long g = gain_u(p, F, i, j, u);
+        if (g > best) { best = g; arg = j; }   // j ascending per lane: first max is smallest
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        long long ob = __shfl_xor_sync(0xffffffffu, best, o);
+        int oa = __shfl_xor_sync(0xffffffffu, arg, o);
+        if (ob > best || (ob == best && oa < arg)) { best = ob; arg = oa; }
+    }
+    if (lane == 0) {
+        F.bg[i] = arg == 0x7FFF ? kNoGain : best;
+        F.bj[i] = (short)(arg == 0x7FFF ? -1 : arg);
+    }
+}
+
+__device__ void merge_update_mat(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U, int I, int J) {
+    const int S = p.nmat;
+    __syncwarp();
+    if (lane == 0) {
+        F.cl[I] = runion(F.cl[I], F.cl[J]);
+        int s = fit_rect(p, F.cl[I]);
+        F.sidx[I] = (signed char)s;
+        F.cost[I] = p.cost[s];
+        F.alive[J] = 0;
+    }
+    __syncwarp();
+    const Rect16 rI = F.cl[I];
+    for (int j = lane; j < n; j += 32) {
+        if (j < J) U[(size_t)j * S + J] = kDead;  // column J dies
+        if (j == I || !F.alive[j]) continue;
+        const uint8_t u = (uint8_t)fit_rect(p, runion(rI, F.cl[j]));
+        if (j < I) U[(size_t)j * S + I] = u;
+        else U[(size_t)I * S + j] = u;
+    }
+    __syncwarp();
+    // lane-owned rows: cheap updates in place, full recomputes flagged for the warp
+    for (int t = 0; t * 32 < n; t++) {
+        const int i = t * 32 + lane;
+        bool redo = false;
+        if (i < n && F.alive[i]) {
+            const int b = F.bj[i];
+            if (i == I) {
+                redo = true;                       // row I's entries all changed
+            } else if (b == I) {                   // (i < I) best partner grew
+                const long long g = gain_u(p, F, i, I, U[(size_t)i * S + I]);
+                if (g >= F.bg[i]) F.bg[i] = g;     // still the max, same (smallest) partner
+                else redo = true;                  // decreased: another partner may win
+            } else if (b == J) {                   // best partner died
+                // if I (< J) now reaches the old best gain it is the new best: any other
+                // partner with that gain has an index > J (J was the smallest such)
+                const long long g = i < I ? gain_u(p, F, i, I, U[(size_t)i * S + I]) : kNoGain;
+                if (i < I && g >= F.bg[i]) { F.bg[i] = g; F.bj[i] = (short)I; }
+                else redo = true;
+            } else if (i < I) {
+                const uint8_t u = U[(size_t)i * S + I];
+                const long long g = gain_u(p, F, i, I, u);
+                if (g > F.bg[i] || (g == F.bg[i] && I < b)) { F.bg[i] = g; F.bj[i] = (short)I; }
+            }
+        }
+        unsigned m = __ballot_sync(0xffffffffu, redo);
+        while (m) {
+            const int l = __ffs(m) - 1;
+            m &= m - 1;
+            row_best_warp(p, F, U, S, n, t * 32 + l, lane);
+        }
+    }
+    __syncwarp();
+}
+
+__device__ void greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U) {
+    const int S = p.nmat;
+    for (int q = lane; q < n * n; q += 32) {
+        const int i = q / n, j = q - i * n;
+        if (j > i) U[(size_t)i * S + j] = (uint8_t)fit_rect(p, runion(F.cl[i], F.cl[j]));
+    }
+    __syncwarp();
+    for (int i = 0; i < n; i++) row_best_warp(p, F, U, S, n, i, lane);
+    __syncwarp();
+    while (true) {
+        while (true) {  // phase A
+            long long Gv = kNoGain;
+            int I = 0x7FFF;
+            for (int i = lane; i < n; i += 32)
+                if (F.alive[i] && (F.bg[i] > Gv || (F.bg[i] == Gv && i < I))) { Gv = F.bg[i]; I = i; }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                long long og = __shfl_xor_sync(0xffffffffu, Gv, o);
+                int oi = __shfl_xor_sync(0xffffffffu, I, o);
+                if (og > Gv || (og == Gv && oi < I)) { Gv = og; I = oi; }
+            }
+            if (Gv <= 0) break;
+            merge_update_mat(p, F, n, lane, U, I, F.bj[I]);
+        }
+        // phase B: lexicographically first pair of alive clusters whose placed windows overlap
+        int mi = 0x7FFF, mj = 0x7FFF;
+        for (int i = lane; i < n; i += 32) {
+            if (!F.alive[i]) continue;
+            int xi, yi, si = F.sidx[i];
+            place(p, F.cl[i], si, xi, yi);
+            for (int j = i + 1; j < n; j++) {
+                if (!F.alive[j]) continue;
+                int xj, yj, sj = F.sidx[j];
+                place(p, F.cl[j], sj, xj, yj);
+                if (xi < xj + p.sw[sj] && xj < xi + p.sw[si] && yi < yj + p.sh[sj] && yj < yi + p.sh[si]) {
+                    if (i < mi) { mi = i; mj = j; }
+                    break;
+                }
+            }
+            if (mi != 0x7FFF) break;
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            int oi = __shfl_xor_sync(0xffffffffu, mi, o);
+            int oj = __shfl_xor_sync(0xffffffffu, mj, o);
+            if (oi < mi) { mi = oi; mj = oj; }
+        }
+        if (mi == 0x7FFF) break;
+        merge_update_mat(p, F, n, lane, U, mi, mj);
+    }
 }
 
 __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_constant__ SelectParams p) {
@@ -259,6 +406,9 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
     }
 
     // --- grouping: phase A greedy merge, phase B disjointness (readings R7, R10) ---
+    if (p.nmat > 0 && n <= p.nmat) {
+        greedy_matrix(p, F, n, lane, base + p.gmat_offset);
+    } else
     while (true) {
         for (int i = lane; i < n; i += 32)
             if (F.alive[i]) rescan_row(p, F, n, i);
@@ -497,10 +647,26 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
     p.tmp = (otif_window *)ws;
     p.counts = (int *)(ws + round_up((int64_t)n * p.cap_f * sizeof(otif_window), 256));
     p.frame_bytes = sel_frame_bytes(gh, gw);
+    // gain matrix for frames with up to nmat components, when int32 gains are exact
+    long long max_cost = 0;
+    for (int s = 0; s < k; s++) max_cost = sizes[s].cost > max_cost ? sizes[s].cost : max_cost;
+    bool small_costs = max_cost < (1ll << 30);
+    for (int s = 0; s < k; s++) small_costs = small_costs && sizes[s].cost >= 0;
+    p.nmat = 0;
+    p.gmat_offset = p.frame_bytes;
+    if (small_costs) {
+        int nm = p.cap_f < kMatMax ? p.cap_f : kMatMax;
+        p.nmat = (int)round_up(nm, 8);
+        p.frame_bytes += (int)round_up(p.nmat * p.nmat, 16);
+    }
     p.ctr = ctr;
     p.frame_base = frame_base;
     int warps = (int)((200 * 1024) / p.frame_bytes);
     warps = warps < 1 ? 1 : (warps > kSelWarpsMax ? kSelWarpsMax : warps);
+    // spread small batches over the SMs rather than packing frames into few CTAs
+    int num_sms = 148;
+    check_device(&num_sms);
+    while (warps > 1 && cdiv(n, warps) < 2 * num_sms) warps--;
     if (warps > n) warps = n;
     size_t smem = (size_t)warps * p.frame_bytes;
     OTIF_CUDA(cudaFuncSetAttribute(select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
