@@ -84,7 +84,7 @@ class ClockSampler:
              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
         try:
             self.p = subprocess.Popen(["nvidia-smi", "-i", str(gpu_index), f"--query-gpu={q}", "--format=csv,noheader,nounits",
-                                       "-lms", "200"], stdout=self.f, stderr=subprocess.DEVNULL)
+                                       "-lms", "50"], stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
             self.p = None
 
@@ -207,7 +207,7 @@ def run_otif(args):
     # device path: the whole clip is one device batch by default (every stage is one launch
     # over all frames, so latency-bound stages see enough frames to fill the SMs)
     batch = args.batch if args.batch > 0 else n
-    pipe = otif.Pipeline(wl, blob, b, max_batch=batch)
+    pipe = otif.Pipeline(wl, blob, b, max_batch=batch, proxy_batch=args.proxy_batch)
     stream = torch.cuda.current_stream()
     for _ in range(args.warmup):
         pipe.run_device(src)
@@ -337,11 +337,12 @@ def run_otif(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["otif", "reference"], default="otif")
     ap.add_argument("--batch", type=int, default=0, help="device batch (0 = whole clip)")
     ap.add_argument("--host-batch", type=int, default=512, help="device batch of the host (e2e) path")
+    ap.add_argument("--proxy-batch", type=int, default=0, help="frames per resize+proxy launch (0 = batch)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--oracle-frames", type=int, default=32)
     ap.add_argument("--no-e2e", action="store_true")

@@ -164,8 +164,10 @@ typedef struct {
     float threshold;
     int32_t k;
     otif_wsize sizes[8];
-    int32_t max_batch;          /* frames per device batch */
+    int32_t max_batch;          /* frames per device batch (one select / pack launch each) */
     int32_t batch_cap[8];       /* detector batch capacity per size, per device batch */
+    int32_t proxy_batch;        /* frames per resize + proxy launch within a batch (0 = max_batch);
+                                   small enough keeps each layer's activations L2-resident */
 } otif_pipeline_desc;
 
 typedef struct otif_pipeline otif_pipeline;

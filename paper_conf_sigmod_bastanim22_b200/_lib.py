@@ -7,7 +7,7 @@ import ctypes
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libotif.so")
+LIB_PATH = os.environ.get("OTIF_LIB_OVERRIDE") or os.path.join(HERE, "libotif.so")
 
 OK, EINVAL, ENOMEM, ECUDA, EUNSUPPORTED = 0, 1, 2, 3, 4
 
@@ -41,7 +41,7 @@ class PipelineDesc(ctypes.Structure):
     _fields_ = [("proxy", ProxyDesc), ("src_h", ctypes.c_int32), ("src_w", ctypes.c_int32),
                 ("det_h", ctypes.c_int32), ("det_w", ctypes.c_int32), ("grid", GridDesc),
                 ("threshold", ctypes.c_float), ("k", ctypes.c_int32), ("sizes", WSize * 8),
-                ("max_batch", ctypes.c_int32), ("batch_cap", ctypes.c_int32 * 8)]
+                ("max_batch", ctypes.c_int32), ("batch_cap", ctypes.c_int32 * 8), ("proxy_batch", ctypes.c_int32)]
 
 
 _lib = None

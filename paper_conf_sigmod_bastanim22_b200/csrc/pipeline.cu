@@ -1,8 +1,13 @@
-// pipeline.cu — the native runtime around the five stages: device buffers sized for
-// one batch, a compute stream and a copy stream, batch loop, and result accumulation
-// (otif_pipeline_*).  The detector batches stay on the device (the detector runs
-// there); windows, per-frame counts and counters are accumulated on the
-// device by append_kernel and copied back once per call.
+// pipeline.cu — the native runtime around the five stages (otif_pipeline_*): device
+// buffers, a compute stream and a copy stream, the batch loop, and result accumulation.
+//
+// A device batch (max_batch frames) runs resize + proxy in mini-batches of proxy_batch
+// frames — small enough that each layer's activations stay resident in the 126 MB L2
+// for the next layer — writing the scores of the whole batch; then one select launch and
+// one pack launch cover the whole batch (the latency-bound grouping needs thousands of
+// frames in flight to fill 148 SMs).  The detector batches stay on the device (the
+// detector runs there); windows, per-frame counts and counters are accumulated
+// on the device and copied back once per host call.
 #include <string.h>
 
 #include <new>
@@ -14,19 +19,19 @@ namespace otif {
 
 otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws, size_t ws_bytes,
                          cudaStream_t stream, cudaEvent_t *evs);
-
-// per-batch timing events: start, resize, proxy prep (tag + E1), E2, E3, E4, E5, D1+D2, select, pack, append
-constexpr int kStages = 10;
-
-// counters: [0] frames, [1] positive cells, [2] windows, [3] window pixels,
-//           [4] order-independent window hash (sum of 64-bit mixes), [5 + s] windows of size s
-constexpr int kCtrFixed = 5;
-
 otif_status launch_select(const float *scores, const uint8_t *mask_in, float threshold, int32_t n, int32_t gh,
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
                           unsigned long long *ctr, int frame_base);
+
+// timing stages: resize, proxy prep (tag + E1), E2, E3, E4, E5, D1+D2, select, pack, append
+constexpr int kStages = 10;
+enum { ST_START = -1, ST_RESIZE = 0, ST_PREP = 1, ST_SELECT = 7, ST_PACK = 8, ST_APPEND = 9 };
+
+// counters: [0] frames, [1] positive cells, [2] windows, [3] window pixels,
+//           [4] order-independent window hash (sum of 64-bit mixes), [5 + s] windows of size s
+constexpr int kCtrFixed = 5;
 
 // Host runs only: append one batch's windows (frame index rebased to the global frame)
 // and per-frame counts to the run's output arrays.  (The counters are accumulated by
@@ -54,7 +59,7 @@ using namespace otif;
 struct otif_pipeline {
     otif_pipeline_desc d;
     otif_proxy *proxy = nullptr;
-    int gh = 0, gw = 0, cells = 0, cap_w = 0;
+    int gh = 0, gw = 0, cells = 0, cap_w = 0, pb = 0;
     uint8_t *src[2] = {nullptr, nullptr};
     uint8_t *img = nullptr, *mask = nullptr, *proxy_ws = nullptr, *sel_ws = nullptr;
     size_t proxy_ws_bytes = 0, sel_ws_bytes = 0;
@@ -63,7 +68,7 @@ struct otif_pipeline {
     int *counts = nullptr, *offsets = nullptr, *total = nullptr, *slot = nullptr, *size_count = nullptr;
     uint8_t *batches[8] = {};
     unsigned long long *ctr = nullptr;
-    // run outputs (grown on demand)
+    // run outputs of host calls (grown on demand)
     otif_window *out_win = nullptr;
     int out_win_cap = 0;
     int *out_counts = nullptr;
@@ -71,51 +76,66 @@ struct otif_pipeline {
     int *out_total = nullptr;
     cudaStream_t s_compute = nullptr, s_copy = nullptr;
     cudaEvent_t ev_h2d[2] = {}, ev_free[2] = {};
-    // optional per-stage timing (otif_pipeline_set_timing)
+    // optional per-stage timing: an ordered log of (stage, event); the time between an
+    // event and its predecessor is charged to the event's stage (ST_START opens a span)
     int timing = 0;
     std::vector<cudaEvent_t> ev_pool;
+    std::vector<int> ev_stage;
     size_t ev_used = 0;
     int64_t launches = 0;
 };
 
-static cudaEvent_t *take_events(otif_pipeline *p, int k) {
-    while (p->ev_pool.size() < p->ev_used + k) {
+static otif_status mark(otif_pipeline *p, int stage, cudaStream_t st, cudaEvent_t *out = nullptr) {
+    if (!p->timing) return OTIF_OK;
+    if (p->ev_pool.size() <= p->ev_used) {
         cudaEvent_t e;
-        if (cudaEventCreate(&e) != cudaSuccess) return nullptr;
+        OTIF_CUDA(cudaEventCreate(&e));
         p->ev_pool.push_back(e);
+        p->ev_stage.push_back(0);
     }
-    cudaEvent_t *r = &p->ev_pool[p->ev_used];
-    p->ev_used += k;
-    return r;
+    p->ev_stage[p->ev_used] = stage;
+    if (out) *out = p->ev_pool[p->ev_used];
+    OTIF_CUDA(cudaEventRecord(p->ev_pool[p->ev_used++], st));
+    return OTIF_OK;
 }
+
+#define RC(x)                           \
+    do {                                \
+        otif_status rc_ = (x);          \
+        if (rc_ != OTIF_OK) return rc_; \
+    } while (0)
 
 static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int frame_base, cudaStream_t st) {
     const otif_pipeline_desc &d = p->d;
-    otif_status rc;
-    cudaEvent_t *ev = p->timing ? take_events(p, kStages + 1) : nullptr;
-    if (ev) OTIF_CUDA(cudaEventRecord(ev[0], st));
-    rc = otif_resize(src, nb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w, st);
-    if (rc != OTIF_OK) return rc;
-    if (ev) OTIF_CUDA(cudaEventRecord(ev[1], st));
-    rc = launch_proxy(p->proxy, p->img, nb, p->scores, p->proxy_ws, p->proxy_ws_bytes, st, ev ? ev + 2 : nullptr);
-    if (rc != OTIF_OK) return rc;
-    rc = launch_select(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask, p->windows,
-                       p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base);
-    if (rc != OTIF_OK) return rc;
-    if (ev) OTIF_CUDA(cudaEventRecord(ev[8], st));
-    rc = otif_pack_windows(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
-                           p->batches, d.batch_cap, p->slot, p->size_count, st);
-    if (rc != OTIF_OK) return rc;
-    if (ev) OTIF_CUDA(cudaEventRecord(ev[9], st));
-    int launched = 13;  // resize 1, proxy 8 (zero, tag, E1, 5 GEMM layers), select 2, pack 2
+    const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
+    cudaEvent_t evs[6];
+    for (int m0 = 0; m0 < nb; m0 += p->pb) {
+        const int mb = nb - m0 < p->pb ? nb - m0 : p->pb;
+        RC(mark(p, ST_START, st));
+        RC(otif_resize(src + (size_t)m0 * frame_bytes, mb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w, st));
+        RC(mark(p, ST_RESIZE, st));
+        // six log entries for the proxy (after E1, after each GEMM layer); launch_proxy
+        // re-records these events at their actual points in the stream
+        for (int i = 0; i < 6 && p->timing; i++) RC(mark(p, ST_PREP + i, st, &evs[i]));
+        RC(launch_proxy(p->proxy, p->img, mb, p->scores + (size_t)m0 * p->cells, p->proxy_ws, p->proxy_ws_bytes, st,
+                        p->timing ? evs : nullptr));
+        p->launches += 9;  // resize 1, proxy 8 (zero, tag, E1, 5 GEMM layers)
+    }
+    RC(mark(p, ST_START, st));
+    RC(launch_select(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask, p->windows,
+                     p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base));
+    RC(mark(p, ST_SELECT, st));
+    RC(otif_pack_windows(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
+                         p->batches, d.batch_cap, p->slot, p->size_count, st));
+    RC(mark(p, ST_PACK, st));
+    p->launches += 4;  // select 2, pack 2
     if (p->out_win) {
         append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts, nb, frame_base, p->out_win,
                                           p->out_win_cap, p->out_counts, p->out_total);
         OTIF_LAUNCH_CHECK();
-        launched++;
+        p->launches += 1;
+        RC(mark(p, ST_APPEND, st));
     }
-    if (ev) OTIF_CUDA(cudaEventRecord(ev[10], st));
-    p->launches += launched;
     return OTIF_OK;
 }
 
@@ -133,6 +153,7 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
                                             otif_pipeline **out) {
     OTIF_REQUIRE(d && weights && out, "otif_pipeline_create: NULL argument");
     OTIF_REQUIRE(d->max_batch > 0, "otif_pipeline_create: max_batch must be positive");
+    OTIF_REQUIRE(d->proxy_batch >= 0, "otif_pipeline_create: proxy_batch must be >= 0");
     OTIF_REQUIRE(d->k >= 1 && d->k <= 8, "otif_pipeline_create: k=%d", d->k);
     OTIF_REQUIRE(d->src_h > 0 && d->src_w > 0 && d->det_h > 0 && d->det_w > 0, "otif_pipeline_create: sizes");
     OTIF_REQUIRE(d->grid.frame_w == d->det_w && d->grid.frame_h == d->det_h,
@@ -143,17 +164,21 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     otif_status rc = otif_proxy_create(&d->proxy, weights, n_weights, &p->proxy);
     if (rc != OTIF_OK) { otif_pipeline_destroy(p); return rc; }
     otif_proxy_grid(p->proxy, &p->gh, &p->gw);
-    OTIF_REQUIRE(p->gh == (d->grid.frame_h + d->grid.cell - 1) / d->grid.cell &&
-                     p->gw == (d->grid.frame_w + d->grid.cell - 1) / d->grid.cell,
-                 "otif_pipeline_create: proxy grid %dx%d does not match ceil(frame/cell)", p->gw, p->gh);
+    if (p->gh != (d->grid.frame_h + d->grid.cell - 1) / d->grid.cell ||
+        p->gw != (d->grid.frame_w + d->grid.cell - 1) / d->grid.cell) {
+        set_error("otif_pipeline_create: proxy grid %dx%d does not match ceil(frame/cell)", p->gw, p->gh);
+        otif_pipeline_destroy(p);
+        return OTIF_EINVAL;
+    }
     const int B = d->max_batch;
+    p->pb = (d->proxy_batch > 0 && d->proxy_batch < B) ? d->proxy_batch : B;
     p->cells = p->gh * p->gw;
     p->cap_w = B * ((p->cells + 1) / 2);
     const size_t src_bytes = (size_t)B * d->src_h * d->src_w * 3;
     PCUDA(cudaMalloc(&p->src[0], src_bytes));
     PCUDA(cudaMalloc(&p->src[1], src_bytes));
-    PCUDA(cudaMalloc(&p->img, (size_t)B * d->proxy.in_h * d->proxy.in_w * 3));
-    p->proxy_ws_bytes = otif_proxy_workspace_bytes(p->proxy, B);
+    PCUDA(cudaMalloc(&p->img, (size_t)p->pb * d->proxy.in_h * d->proxy.in_w * 3));
+    p->proxy_ws_bytes = otif_proxy_workspace_bytes(p->proxy, p->pb);
     PCUDA(cudaMalloc(&p->proxy_ws, p->proxy_ws_bytes));
     PCUDA(cudaMemset(p->proxy_ws, 0, p->proxy_ws_bytes));
     p->sel_ws_bytes = otif_select_workspace_bytes(B, p->gh, p->gw);
@@ -225,17 +250,18 @@ extern "C" otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *s
                                               int32_t *total_out, int32_t *size_count_out) {
     OTIF_REQUIRE(p && (src_host || n == 0) && n >= 0 && cap_windows >= 0, "otif_pipeline_run_host: bad arguments");
     OTIF_REQUIRE(total_out, "otif_pipeline_run_host: NULL total_out");
-    otif_status rc = ensure_outputs(p, n > 0 ? n : 1, cap_windows > 0 ? cap_windows : 1);
-    if (rc != OTIF_OK) return rc;
+    RC(ensure_outputs(p, n > 0 ? n : 1, cap_windows > 0 ? cap_windows : 1));
     const otif_pipeline_desc &d = p->d;
     const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
-    const int out_cap = cap_windows;
     OTIF_CUDA(cudaMemsetAsync(p->out_total, 0, 4, p->s_compute));
     OTIF_CUDA(cudaMemsetAsync(p->ctr, 0, (kCtrFixed + 8) * 8, p->s_compute));
     // the copy stream must not overwrite a src buffer before the compute stream is done with it
     for (int i = 0; i < 2; i++) OTIF_CUDA(cudaEventRecord(p->ev_free[i], p->s_compute));
+    const int cap_saved = p->out_win_cap;
+    p->out_win_cap = cap_windows;  // windows beyond the caller's capacity are dropped (total stays exact)
+    otif_status rc = OTIF_OK;
     int b = 0;
-    for (int f0 = 0; f0 < n; f0 += d.max_batch, b++) {
+    for (int f0 = 0; f0 < n && rc == OTIF_OK; f0 += d.max_batch, b++) {
         const int nb = n - f0 < d.max_batch ? n - f0 : d.max_batch;
         const int buf = b & 1;
         OTIF_CUDA(cudaStreamWaitEvent(p->s_copy, p->ev_free[buf], 0));
@@ -243,14 +269,11 @@ extern "C" otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *s
                                   cudaMemcpyHostToDevice, p->s_copy));
         OTIF_CUDA(cudaEventRecord(p->ev_h2d[buf], p->s_copy));
         OTIF_CUDA(cudaStreamWaitEvent(p->s_compute, p->ev_h2d[buf], 0));
-        // out_win capacity is the caller's: windows beyond it are dropped (total stays exact)
-        int saved = p->out_win_cap;
-        p->out_win_cap = out_cap;
         rc = run_batch(p, p->src[buf], nb, f0, p->s_compute);
-        p->out_win_cap = saved;
-        if (rc != OTIF_OK) return rc;
-        OTIF_CUDA(cudaEventRecord(p->ev_free[buf], p->s_compute));
+        if (rc == OTIF_OK) OTIF_CUDA(cudaEventRecord(p->ev_free[buf], p->s_compute));
     }
+    p->out_win_cap = cap_saved;
+    if (rc != OTIF_OK) return rc;
     int total = 0;
     OTIF_CUDA(cudaMemcpyAsync(&total, p->out_total, 4, cudaMemcpyDeviceToHost, p->s_compute));
     if (frame_count_out && n > 0)
@@ -271,14 +294,11 @@ extern "C" otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t 
                                                 cudaStream_t stream) {
     OTIF_REQUIRE(p && (src_dev || n == 0) && n >= 0, "otif_pipeline_run_device: bad arguments");
     const size_t frame_bytes = (size_t)p->d.src_h * p->d.src_w * 3;
-    // device runs keep no per-frame outputs beyond the last batch: counters only
+    // device runs keep no per-frame outputs beyond the current batch: counters only
     otif_window *ow = p->out_win;
     int *oc = p->out_counts;
-    int owc = p->out_win_cap;
     p->out_win = nullptr;
     p->out_counts = nullptr;
-    p->out_win_cap = 0;
-    OTIF_CUDA(cudaMemsetAsync(p->out_total, 0, 4, stream));
     otif_status rc = OTIF_OK;
     for (int f0 = 0; f0 < n && rc == OTIF_OK; f0 += p->d.max_batch) {
         const int nb = n - f0 < p->d.max_batch ? n - f0 : p->d.max_batch;
@@ -286,7 +306,6 @@ extern "C" otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t 
     }
     p->out_win = ow;
     p->out_counts = oc;
-    p->out_win_cap = owc;
     return rc;
 }
 
@@ -311,13 +330,13 @@ extern "C" otif_status otif_pipeline_set_timing(otif_pipeline *p, int32_t enable
 extern "C" otif_status otif_pipeline_stage_ms(otif_pipeline *p, float *ms, int32_t n_ms, int64_t *launches) {
     OTIF_REQUIRE(p && ms && n_ms >= kStages, "otif_pipeline_stage_ms: need %d entries", kStages);
     for (int s = 0; s < kStages; s++) ms[s] = 0.0f;
-    for (size_t b = 0; b + kStages + 1 <= p->ev_used; b += kStages + 1) {
-        OTIF_CUDA(cudaEventSynchronize(p->ev_pool[b + kStages]));
-        for (int s = 0; s < kStages; s++) {
-            float t = 0.0f;
-            OTIF_CUDA(cudaEventElapsedTime(&t, p->ev_pool[b + s], p->ev_pool[b + s + 1]));
-            ms[s] += t;
-        }
+    if (p->ev_used > 0) OTIF_CUDA(cudaEventSynchronize(p->ev_pool[p->ev_used - 1]));
+    for (size_t i = 1; i < p->ev_used; i++) {
+        const int s = p->ev_stage[i];
+        if (s < 0) continue;  // a span start: no time charged
+        float t = 0.0f;
+        OTIF_CUDA(cudaEventElapsedTime(&t, p->ev_pool[i - 1], p->ev_pool[i]));
+        ms[s] += t;
     }
     if (launches) *launches = p->launches;
     p->ev_used = 0;

@@ -83,6 +83,7 @@ struct ConvParams {
     int64_t fstride;
     int out_h, out_w;
     int stages_a, stages_b;
+    int mt;                     // 128-row sub-tiles per CTA tile (share each A halo and B stage)
     // destination
     int out_kind;               // 1/2: next layout kind; 3: head scores
     uint8_t *out;
@@ -224,6 +225,7 @@ __global__ void __launch_bounds__(128) e1_umma_kernel(const __grid_constant__ E1
 // ---------------------------------------------------------------------------
 // E2..E5, D1: persistent warp-specialised implicit-GEMM conv on tcgen05
 // ---------------------------------------------------------------------------
+template <int MT>
 __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     const int warp = threadIdx.x >> 5;
@@ -245,7 +247,8 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
     float *s_bias = reinterpret_cast<float *>(tmem_slot + 4);
     float *s_w2 = s_bias + 256;
 
-    const uint32_t tmem_cols = p.N * 2 <= 32 ? 32 : (p.N * 2 <= 64 ? 64 : (p.N * 2 <= 128 ? 128 : (p.N * 2 <= 256 ? 256 : 512)));
+    const uint32_t acc_cols = 2 * MT * p.N;  // two accumulator stages of MT sub-tiles x N columns
+    const uint32_t tmem_cols = acc_cols <= 32 ? 32 : (acc_cols <= 64 ? 64 : (acc_cols <= 128 ? 128 : (acc_cols <= 256 ? 256 : 512)));
 
     if (threadIdx.x == 0) {
         for (int i = 0; i < p.stages_a; i++) { mbar_init(&a_full[i], 1); mbar_init(&a_empty[i], 1); }
@@ -268,7 +271,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
         if (lane == 0) {
             uint32_t as = 0, ap = 0, bs = 0, bp = 0;
             for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
-                const int64_t q0 = (int64_t)tile * kTileM;
+                const int64_t q0 = (int64_t)tile * kTileM * MT;
                 int tap_pos = 0;
                 for (int cb = 0; cb < p.ncb; cb++) {
                     tap_pos = 0;
@@ -304,7 +307,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
             for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
                 mbar_wait(&t_empty[acc], accp ^ 1);
                 tc_fence_after();
-                const uint32_t d = tmem_base + acc * p.N;
+                const uint32_t d = tmem_base + acc * MT * p.N;
                 uint32_t accumulate = 0;
                 for (int cb = 0; cb < p.ncb; cb++) {
                     for (int g = 0; g < p.ngroups; g++) {
@@ -317,9 +320,13 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                             const uint32_t a_tap = a_stage + p.group_shift[g][t] * 16;
                             const uint32_t b_stage = b_base + bs * b_bytes;
                             for (uint32_t s = 0; s < chunks / 2; s++) {
-                                uint64_t ad = umma_desc(a_tap + 2 * s * lbo_a, lbo_a, 128);
-                                uint64_t bd = umma_desc(b_stage + 2 * s * lbo_b, lbo_b, 128);
-                                umma_bf16(d, ad, bd, idesc, accumulate);
+                                const uint64_t bd = umma_desc(b_stage + 2 * s * lbo_b, lbo_b, 128);
+                                // the mt sub-tiles share this B stage: rows 128*m.. of the halo
+#pragma unroll
+                                for (int m = 0; m < MT; m++) {
+                                    uint64_t ad = umma_desc(a_tap + 2 * s * lbo_a + m * (kTileM * 16), lbo_a, 128);
+                                    umma_bf16(d + m * p.N, ad, bd, idesc, accumulate);
+                                }
                                 accumulate = 1;
                             }
                             umma_commit(&b_empty[bs]);
@@ -341,7 +348,8 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
         for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
             mbar_wait(&t_full[acc], accp);
             tc_fence_after();
-            const int64_t q = (int64_t)tile * kTileM + row;
+          for (int m = 0; m < MT; m++) {
+            const int64_t q = (int64_t)tile * kTileM * MT + m * kTileM + row;
             const int f = (int)(q / p.fstride);
             const int64_t r = q - (int64_t)f * p.fstride;
             const int oy = (int)(r / p.pitch);
@@ -350,7 +358,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
             int plane = 0;
             int64_t L = 0;
             if (p.out_kind != 3) L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, f, oy, ox, plane);
-            const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * p.N;
+            const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + (acc * MT + m) * p.N;
             float z = p.b2;
             for (int cc = 0; cc < p.N / 32; cc++) {
                 uint32_t v[32];
@@ -380,6 +388,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
             }
             if (p.out_kind == 3 && valid)
                 p.scores[((int64_t)f * p.out_h + oy) * p.out_w + ox] = 1.0f / (1.0f + expf(-z));
+          }
             tc_fence_before();
             mbar_arrive(&t_empty[acc]);
             if (++acc == 2) { acc = 0; accp ^= 1; }
@@ -418,7 +427,7 @@ struct GemmLayer {
     int64_t fstride_unit;         // per-frame pixels of the input layout
     int max_shift;
     int ngroups, group_plane[4], group_ntaps[4], group_shift[4][9], group_tap[4][9];
-    int kb, ncb, P;
+    int kb, ncb, P, mt;
     uint8_t *wpk_dev;
     float *bias_dev;
 };
@@ -482,7 +491,14 @@ static void build_layer(GemmLayer &g, int cin, int cout, int stride, int in_h, i
         }
         g.ngroups = ng;
     }
-    g.P = (int)round_up(kTileM + g.max_shift, 8);
+    // mt sub-tiles of 128 rows per CTA tile so that every tap issues >= 256 columns of MMA
+    // work (mt * N = 256): amortises the per-stage barrier and copy overheads of small N
+    g.mt = cout >= 256 ? 1 : (cout >= 128 ? 2 : 4);
+    if (const char *e = getenv("OTIF_CONV_MT_MAX")) {  // tuning experiments only
+        int cap = atoi(e);
+        if (cap >= 1 && g.mt > cap) g.mt = cap;
+    }
+    g.P = (int)round_up(kTileM * g.mt + g.max_shift, 8);
 }
 
 static Layout input_layout(const GemmLayer &g, int n) {
@@ -492,7 +508,7 @@ static Layout input_layout(const GemmLayer &g, int n) {
     l.pitch = g.pitch;
     l.fstride = g.fstride_unit;
     int64_t mtot = (int64_t)n * g.fstride_unit;
-    l.lcap = round_up(round_up(mtot, kTileM) + g.max_shift + 8, 16);
+    l.lcap = round_up(round_up(mtot, (int64_t)kTileM * g.mt) + g.max_shift + 8, 16);
     l.c8 = g.cin / 8;
     l.bytes = (size_t)l.planes * l.c8 * l.lcap * 16;
     l.offset = 0;
@@ -576,7 +592,7 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         c.act = ws + lay[li].offset;
         c.lcap = lay[li].lcap;
         c.c8_in = g.cin / 8;
-        c.kb = g.kb; c.ncb = g.ncb; c.P = g.P; c.ngroups = g.ngroups;
+        c.kb = g.kb; c.ncb = g.ncb; c.P = g.P; c.ngroups = g.ngroups; c.mt = g.mt;
         for (int i = 0; i < 4; i++) {
             c.group_plane[i] = g.group_plane[i];
             c.group_ntaps[i] = g.group_ntaps[i];
@@ -584,7 +600,7 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         }
         c.wpk = g.wpk_dev; c.bias = g.bias_dev; c.N = g.cout;
         c.mtot = (int64_t)n * g.fstride_unit;
-        c.ntiles = (int)cdiv(c.mtot, kTileM);
+        c.ntiles = (int)cdiv(c.mtot, (int64_t)kTileM * g.mt);
         c.pitch = g.pitch; c.fstride = g.fstride_unit; c.out_h = g.out_h; c.out_w = g.out_w;
         if (li < 4) {
             c.out_kind = lay[li + 1].kind;
@@ -601,10 +617,11 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         }
         size_t smem;
         conv_smem(g, c.stages_a, c.stages_b, smem);
-        OTIF_CUDA(cudaFuncSetAttribute(conv_umma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
         int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
         if (grid < 1) grid = 1;
-        conv_umma_kernel<<<grid, kConvThreads, smem, stream>>>(c);
+        auto kern = g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>);
+        OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        kern<<<grid, kConvThreads, smem, stream>>>(c);
         OTIF_LAUNCH_CHECK();
         if (evs) OTIF_CUDA(cudaEventRecord(evs[1 + li], stream));
     }
