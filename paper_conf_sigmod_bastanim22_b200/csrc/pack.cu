@@ -101,7 +101,80 @@ __device__ __forceinline__ uint4 load16u(const uint8_t *s0, uintptr_t src_end) {
     return make_uint4(o[0], o[1], o[2], o[3]);
 }
 
-__global__ void __launch_bounds__(512) pack_kernel(const __grid_constant__ PackParams p) {
+// TMA bulk path for windows whose source rows are 16-B aligned (all windows placed on
+// 16-px multiples, which the cell grid produces for most of them): one thread streams
+// the window through a ring of shared-memory chunks with 1-D bulk async copies —
+// global->shared (the window's rows of a chunk; a single copy when the window spans
+// full frame rows, so its bytes are contiguous) then shared->global into the packed
+// detector batch (contiguous).  Loads run kBulkLead chunks ahead of the stores.
+constexpr int kBulkStages = 3;
+constexpr int kBulkLead = 1;                 // <= kBulkStages - 1
+constexpr int kBulkStage = 16384;            // bytes per ring stage
+
+__device__ __forceinline__ void bulk_s2g(void *dst_gmem, const void *src_smem, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst_gmem), "r"(smem_u32(src_smem)),
+                 "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// One thread streams one window through the ring.  A window spanning full frame rows is
+// one contiguous byte range in the source: it moves in 16 KB chunks regardless of rows;
+// otherwise a chunk is as many whole rows as fit in a stage (one g2s per row).
+__device__ void pack_window_bulk(uint8_t *ring, uint64_t *bars, uint32_t &chunk_seq, const uint8_t *fbase, int sw,
+                                 const otif_window &w, uint8_t *dst) {
+    const uint32_t row_bytes = (uint32_t)w.w * 3;
+    const bool contiguous = (w.x == 0 && w.w == sw);
+    const uint32_t total = (uint32_t)w.h * row_bytes;
+    const int rpc = (int)(kBulkStage / row_bytes);  // >= 1 (checked by the caller)
+    const uint32_t chunk_bytes = contiguous ? (uint32_t)kBulkStage : rpc * row_bytes;
+    const int nchunks = (int)((total + chunk_bytes - 1) / chunk_bytes);
+    const uint8_t *wsrc = fbase + ((size_t)w.y * sw + w.x) * 3;
+    const uint32_t base = chunk_seq;
+    for (int i = 0; i < nchunks + kBulkLead; i++) {
+        if (i < nchunks) {
+            const uint32_t c = base + i, s = c % kBulkStages;
+            // stage s is reused by chunk i: the store of chunk i - kBulkStages must have read it
+            bulk_wait_read<kBulkStages - kBulkLead - 1>();
+            const uint32_t off = (uint32_t)i * chunk_bytes;
+            const uint32_t bytes = min(chunk_bytes, total - off);
+            uint8_t *buf = ring + (size_t)s * kBulkStage;
+            mbar_arrive_expect_tx(&bars[s], bytes);
+            if (contiguous) {
+                bulk_g2s(buf, wsrc + off, bytes, &bars[s]);
+            } else {
+                const int r0 = i * rpc, nr = (int)(bytes / row_bytes);
+                for (int r = 0; r < nr; r++)
+                    bulk_g2s(buf + r * row_bytes, wsrc + (size_t)(r0 + r) * sw * 3, row_bytes, &bars[s]);
+            }
+        }
+        const int j = i - kBulkLead;
+        if (j >= 0 && j < nchunks) {
+            const uint32_t c = base + j, s = c % kBulkStages;
+            mbar_wait(&bars[s], (c / kBulkStages) & 1);
+            const uint32_t off = (uint32_t)j * chunk_bytes;
+            bulk_s2g(dst + off, ring + (size_t)s * kBulkStage, min(chunk_bytes, total - off));
+            bulk_commit();
+        }
+    }
+    chunk_seq = base + nchunks;
+    bulk_wait_all();
+}
+
+__global__ void __launch_bounds__(128) pack_kernel(const __grid_constant__ PackParams p) {
+    extern __shared__ __align__(128) uint8_t ring[];  // kBulkStages x kBulkStage bytes
+    __shared__ uint64_t bars[kBulkStages];
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < kBulkStages; i++) mbar_init(&bars[i], 1);
+        fence_barrier_init();
+    }
+    __syncthreads();
+    uint32_t chunk_seq = 0;
     const int total = min(*p.total, p.capacity);
     const bool identity = (p.dh == p.sh && p.dw == p.sw);
     for (int g = blockIdx.x; g < total; g += gridDim.x) {
@@ -111,7 +184,11 @@ __global__ void __launch_bounds__(512) pack_kernel(const __grid_constant__ PackP
         if (sl >= p.cap[s]) continue;
         uint8_t *dst = p.batch[s] + (size_t)sl * p.bh[s] * p.bw[s] * 3;
         const int row_bytes = w.w * 3;
-        if (identity && (row_bytes & 15) == 0 && (((uintptr_t)p.batch[s]) & 15) == 0) {
+        if (identity && (row_bytes & 15) == 0 && row_bytes <= kBulkStage && (((uintptr_t)p.batch[s]) & 15) == 0 &&
+            ((w.x * 3) & 15) == 0 && ((p.sw * 3) & 15) == 0 && (((uintptr_t)p.src) & 15) == 0) {
+            if (threadIdx.x == 0)
+                pack_window_bulk(ring, bars, chunk_seq, p.src + (size_t)w.frame * p.sh * p.sw * 3, p.sw, w, dst);
+        } else if (identity && (row_bytes & 15) == 0 && (((uintptr_t)p.batch[s]) & 15) == 0) {
             const int per_row = row_bytes >> 4;
             const uint8_t *fbase = p.src + (size_t)w.frame * p.sh * p.sw * 3;
             const uintptr_t src_end = (uintptr_t)p.src + p.src_bytes;
@@ -200,8 +277,10 @@ extern "C" otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t 
     slot_kernel<<<1, 1024, 0, stream>>>(p);
     OTIF_LAUNCH_CHECK();
     if (capacity > 0) {
-        int grid = capacity < num_sms * 4 ? capacity : num_sms * 4;
-        pack_kernel<<<grid, 512, 0, stream>>>(p);
+        int grid = capacity < num_sms * 6 ? capacity : num_sms * 6;
+        const int smem = kBulkStages * kBulkStage;
+        OTIF_CUDA(cudaFuncSetAttribute(pack_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        pack_kernel<<<grid, 128, smem, stream>>>(p);
         OTIF_LAUNCH_CHECK();
     }
     return OTIF_OK;

@@ -39,6 +39,16 @@ def test_resize_parity(wl, n, dh, dw):
     assert (d == 0).mean() > 0.95
 
 
+@pytest.mark.parametrize("wl,f", [(configs.C2, 4), (configs.C1, 4), (configs.C4_BASE, 2), (configs.C4_BASE, 8),
+                                  (configs.C3, 4)])
+def test_resize_even_factor_bit_exact(wl, f):
+    """Even integer factors: the output is exactly the rounded 2x2 mean — bit-exact."""
+    src = _frames(wl, 3)
+    ref = oracle.resize(src.numpy(), wl.src_h // f, wl.src_w // f)
+    got = otif.otif_resize(src.cuda(), wl.src_h // f, wl.src_w // f).cpu().numpy()
+    assert np.array_equal(got, ref)
+
+
 def test_resize_constant_and_identity():
     src = torch.full((3, 135, 240, 3), 77, dtype=torch.uint8)
     assert (otif.otif_resize(src.cuda(), 34, 60).cpu() == 77).all()
