@@ -92,7 +92,7 @@ def full(path, tag, names):
     for d in res:
         t = d.get("gpu__time_duration.sum", 0)
         tu = d.get("gpu__time_duration.sum.unit", "")
-        t_us = t / 1000 if tu == "nsecond" else (t * 1000 if tu == "msecond" else t)
+        t_us = t / 1000 if tu in ("nsecond", "ns") else (t * 1000 if tu in ("msecond", "ms") else t)
         lines.append(f"| {d['layer']} | {t_us:.1f} | {d.get('dram__bytes_read.sum', 0) / 1e6:.1f} | "
                      f"{d.get('dram__bytes_write.sum', 0) / 1e6:.1f} | {d.get('lts__t_bytes.sum', 0) / 1e6:.1f} | "
                      f"{d.get('sm__mem_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed', 0):.1f} | "
