@@ -11,8 +11,10 @@
 //   root is its component's first cell in raster order) -> read-only flatten ->
 //   warp scan for raster-ordered component ids -> shared atomic bounding boxes ->
 //   phase A with a per-cluster best-partner cache (bg[i], bj[i] = best gain / partner
-//   over j > i; after a merge only the affected rows are rescanned, so a frame costs
-//   O(n^2) pair evaluations instead of O(n^3)) -> phase B (first overlapping pair) ->
+//   over j > i) over a one-byte fit-index matrix U[i][j] (n <= 128; a merge refreshes
+//   row/column I and recomputes only the rows whose cached best can have changed —
+//   larger n falls back to row rescans without the matrix) -> phase B (first
+//   overlapping pair) ->
 //   placement, strict full-frame fallback, rank sort by (y, x) -> per-frame scratch.
 //   Optionally (pipeline) accumulates the run counters with a few atomics per frame.
 // K6 compact_kernel: exclusive scan of per-frame counts (frame_offset, total) and
@@ -89,7 +91,10 @@ __device__ __forceinline__ int uf_find(volatile int *par, int x) {
         int q = par[x];
         if (q == x) return x;
         int g = par[q];
-        if (g != q) par[x] = g;  // path halving; parents only ever decrease
+        // path halving; parents only ever decrease and always stay ancestors, so the
+        // unsynchronised halving writes racing with other lanes' reads are benign
+        // (compute-sanitizer racecheck reports them as warnings by design)
+        if (g != q) par[x] = g;
         x = q;
     }
 }
@@ -225,6 +230,7 @@ __device__ void merge_update_mat(const SelectParams &p, Frame &F, int n, int lan
             }
         }
         unsigned m = __ballot_sync(0xffffffffu, redo);
+        __syncwarp();  // this group's bj/bg reads happen-before lane 0's rewrites below
         while (m) {
             const int l = __ffs(m) - 1;
             m &= m - 1;
@@ -692,7 +698,8 @@ otif_status validate_select(const float *scores, const uint8_t *mask_in, int32_t
     OTIF_REQUIRE(gh == (g->frame_h + g->cell - 1) / g->cell && gw == (g->frame_w + g->cell - 1) / g->cell,
                  "otif_select_windows: grid %dx%d != ceil(frame/cell) for %dx%d / %d", gw, gh, g->frame_w,
                  g->frame_h, g->cell);
-    OTIF_REQUIRE((scores != nullptr) != (mask_in != nullptr), "otif_select_windows: exactly one of scores/mask_in");
+    OTIF_REQUIRE(n == 0 || (scores != nullptr) != (mask_in != nullptr),
+                 "otif_select_windows: exactly one of scores/mask_in");
     OTIF_REQUIRE(g->connectivity == 4 || g->connectivity == 8, "otif_select_windows: connectivity must be 4 or 8");
     OTIF_REQUIRE(k >= 1 && k <= kMaxSizes, "otif_select_windows: k=%d not in [1,8]", k);
     OTIF_REQUIRE(capacity >= 0, "otif_select_windows: negative capacity");

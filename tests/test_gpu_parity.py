@@ -245,3 +245,97 @@ def test_end_to_end_c1(blob):
     assert np.array_equal(scount.cpu().numpy(), ocnt)
     for s in range(len(wl.sizes)):
         assert np.array_equal(batches[s].cpu().numpy(), ob[s])
+
+
+# ------------------------------------------------------------------ full size (bench launch configuration)
+def test_full_size_c2_sampled(blob):
+    """C2 at its full size (4500 frames, one launch per stage as bench.py times it);
+    sampled frames are recomputed one by one on the oracle."""
+    wl = configs.C2
+    b = threshold("C2", 0.7)
+    n = wl.n_frames
+    src = torch.empty((n, wl.src_h, wl.src_w, 3), dtype=torch.uint8, device="cuda")
+    video.make_scene(wl).render(range(n), out=src)
+    img = otif.otif_resize(src, wl.proxy_h, wl.proxy_w)
+    px = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, blob)
+    scores = px.score(img)
+    r = otif.otif_select_windows(scores, None, b, wl.src_w, wl.src_h, wl.cell, wl.sizes, want_mask=True)
+    total = int(r["total"].item())
+    counts = r["counts"].cpu().numpy()
+    offs = r["offsets"].cpu().numpy()
+    assert counts.sum() == total and offs[-1] + counts[-1] == total
+    allw = windows_np(r["windows"], total)
+    caps = [int((allw["size_idx"] == s).sum()) for s in range(len(wl.sizes))]
+    batches, slot, scount = otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], wl.sizes, caps)
+    assert list(scount.cpu().numpy()) == caps
+    rng = np.random.default_rng(11)
+    sample = sorted(set([0, 1, n - 1] + list(rng.integers(0, n, 9))))
+    src_s = src[sample].cpu().numpy()
+    img_ref = oracle.resize(src_s, wl.proxy_h, wl.proxy_w)
+    assert np.array_equal(img[sample].cpu().numpy(), img_ref)       # even factor: bit-exact
+    ref_s = oracle_scores(img_ref, wl, blob)
+    ref_none = oracle_scores(img_ref, wl, blob, oracle.QUANT_NONE)
+    got_s = scores[sample].cpu().numpy().astype(np.float64)
+    assert np.abs(got_s - ref_none).max() <= 2e-2
+    gmask = r["mask"][sample].cpu().numpy()
+    far = np.abs(ref_s - b) > BAND
+    assert np.array_equal(gmask[far], (ref_s > b)[far])
+    slot_np = slot[:total].cpu().numpy()
+    for i, f in enumerate(sample):
+        ow = oracle.group_frame(gmask[i], wl.cell, wl.src_w, wl.src_h, wl.sizes, frame_index=f)
+        mine = allw[offs[f]:offs[f] + counts[f]]
+        assert as_tuples(ow) == as_tuples(mine)
+        for gi in range(offs[f], offs[f] + counts[f]):
+            w = allw[gi]
+            crop = src_s[i, w["y"]:w["y"] + w["h"], w["x"]:w["x"] + w["w"]]
+            assert np.array_equal(batches[w["size_idx"]][slot_np[gi]].cpu().numpy(), crop)
+
+
+@pytest.mark.parametrize("wl", [configs.C3, configs.C4_SWEEP[3], configs.C1], ids=lambda w: w.name)
+def test_pipeline_host_vs_stages(wl, blob):
+    """The native runtime (otif_pipeline_run_host, several device batches) returns exactly
+    the windows of the stage-by-stage path (whose parity with the oracle is tested above)."""
+    b = threshold(wl.name, 0.7)
+    n = 70
+    src = video.frames(wl, n)
+    pipe = otif.Pipeline(wl, blob, b, max_batch=32)
+    win, counts, sc, tot = pipe.run_host(src.contiguous())
+    src_d = src.cuda()
+    img = otif.otif_resize(src_d, wl.proxy_h, wl.proxy_w)
+    px = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, blob)
+    r = otif.otif_select_windows(px.score(img), None, b, wl.src_w, wl.src_h, wl.cell, wl.sizes)
+    t = int(r["total"].item())
+    assert tot == t
+    assert np.array_equal(counts, r["counts"].cpu().numpy())
+    assert np.array_equal(win, r["windows"][:t].cpu().numpy())
+    ref = windows_np(r["windows"], t)
+    assert list(sc) == [int((ref["size_idx"] == s).sum()) for s in range(len(wl.sizes))]
+
+
+def test_edge_cases():
+    wl = configs.C1
+    # n = 0 everywhere
+    empty = torch.empty((0, wl.src_h, wl.src_w, 3), dtype=torch.uint8, device="cuda")
+    assert otif.otif_resize(empty, 64, 104).shape == (0, 64, 104, 3)
+    r = otif.otif_select_windows(None, torch.zeros((0, 8, 13), dtype=torch.uint8, device="cuda"), 0.0,
+                                 416, 256, 32, wl.sizes)
+    assert int(r["total"].item()) == 0
+    # k = 1 (only the full frame): any positive frame -> exactly one full-frame window
+    m = torch.zeros((3, 8, 13), dtype=torch.uint8)
+    m[1, 2, 3] = 1
+    m[2] = 1
+    r = otif.otif_select_windows(None, m.cuda(), 0.0, 416, 256, 32, [(416, 256)])
+    assert int(r["total"].item()) == 2
+    assert windows_np(r["windows"], 2).tolist() == [(1, 0, 0, 416, 256, 0), (2, 0, 0, 416, 256, 0)]
+    # single-cell grid (frame smaller than a cell)
+    r = otif.otif_select_windows(None, torch.ones((2, 1, 1), dtype=torch.uint8, device="cuda"), 0.0, 20, 10, 32,
+                                 [(20, 10)])
+    assert windows_np(r["windows"], 2).tolist() == [(0, 0, 0, 20, 10, 0), (1, 0, 0, 20, 10, 0)]
+    # largest grid the kernel accepts (8192 cells), random mask, vs oracle
+    rng = np.random.default_rng(2)
+    big = (rng.random((4, 64, 128)) < 0.02).astype(np.uint8)
+    sizes = [(64, 64), (256, 256), (4096, 2048)]
+    ref_w, ref_c, _, ref_t = oracle.select_windows(big, 32, 4096, 2048, sizes)
+    r = otif.otif_select_windows(None, torch.from_numpy(big).cuda(), 0.0, 4096, 2048, 32, sizes)
+    t = int(r["total"].item())
+    assert t == ref_t and as_tuples(windows_np(r["windows"], t)) == as_tuples(ref_w)
