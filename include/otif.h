@@ -146,6 +146,33 @@ otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t src_h, int3
                               int32_t *slot, int32_t *size_count, cudaStream_t stream);
 
 /* ---------------------------------------------------------------------------
+ * §8(f) NEXT-1 — choosing the fixed window sizes W: "we first initialize W
+ * to only contain the size corresponding to the entire video frame ... We then
+ * repeatedly greedily add the window size to W that provides the greatest decrease to
+ * Σ_t est(R(I_t; W)), until |W| = k", assuming a perfect proxy (masks = ground-truth
+ * cells).  masks [n, gh, gw] u8 (device); candidates [host] m sizes (the full
+ * frame is implicit, cost full_cost); ties go to the earliest candidate; the loop stops
+ * early when no candidate decreases the sum (reading R19).  Outputs [host]:
+ * chosen_idx[k] (-1 = full frame at [0], candidate index after, -2 = not filled) and
+ * est[k] (Σ_t est after each addition).  Synchronises `stream` once per round.
+ * workspace: >= otif_choose_workspace_bytes(n, gh, gw, m). */
+size_t otif_choose_workspace_bytes(int32_t n, int32_t gh, int32_t gw, int32_t m);
+otif_status otif_choose_window_sizes(const uint8_t *masks, int32_t n, int32_t gh, int32_t gw,
+                                     const otif_grid_desc *g, const otif_wsize *candidates, int32_t m,
+                                     int64_t full_cost, int32_t k, int32_t *chosen_idx, int64_t *est,
+                                     void *workspace, size_t ws_bytes, cudaStream_t stream);
+
+/* §8(f) NEXT-2 — proxy tuning: the recall of windows R_ij is "the fraction
+ * of detections computed by θ_best that are covered by rectangles in R_ij".  A detection
+ * box counts as covered when it lies inside one window of its frame (reading R18).
+ *   boxes [nb][5] int32 (frame, x0, y0, x1, y1), half-open, clipped to the frame;
+ *   windows / frame_offset / frame_count as produced by otif_select_windows for n frames.
+ * covered: device uint64, set to the number of covered boxes (enqueued; no sync). */
+otif_status otif_window_recall(const int32_t *boxes, int64_t nb, const otif_window *windows,
+                               const int32_t *frame_offset, const int32_t *frame_count, int32_t n,
+                               unsigned long long *covered, cudaStream_t stream);
+
+/* ---------------------------------------------------------------------------
  * Whole path on HOST frames (the end-to-end call): for batches of up to max_batch
  * frames, copy src (pinned or pageable host memory) to the device, run stages 1–5,
  * and copy the windows and per-frame counts back.  Two CUDA streams overlap the

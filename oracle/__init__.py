@@ -225,3 +225,45 @@ def pack_windows(src: np.ndarray, det_h: int, det_w: int, windows: np.ndarray, s
     _check(lib().otif_ref_pack_windows(_p(src), n, sh, sw, det_h, det_w, _p(windows), total, ws, k,
                                        ptrs, _p(caps), _p(slot), _p(counts)), "pack_windows")
     return batches, slot[:total].copy(), counts
+
+
+def _lib2():
+    L = lib()
+    if not getattr(L, "_next_bound", False):
+        P, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+        L.otif_ref_frame_est.argtypes = [P, i32, i32, i32, i32, i32, i32, P, i32]
+        L.otif_ref_frame_est.restype = i64
+        L.otif_ref_choose_window_sizes.argtypes = [P, i32, i32, i32, i32, i32, i32, i32, P, i32, i64, i32, P, P]
+        L.otif_ref_covered.argtypes = [P, i64, P, i32]
+        L.otif_ref_covered.restype = i64
+        L._next_bound = True
+    return L
+
+
+def frame_est(mask: np.ndarray, cell: int, frame_w: int, frame_h: int, sizes, connectivity: int = 4) -> int:
+    mask = np.ascontiguousarray(mask, np.uint8)
+    gh, gw = mask.shape
+    return int(_lib2().otif_ref_frame_est(_p(mask), gh, gw, cell, frame_w, frame_h, connectivity, wsizes(sizes),
+                                          len(sizes)))
+
+
+def choose_window_sizes(masks: np.ndarray, cell: int, frame_w: int, frame_h: int, candidates, k: int,
+                        full_cost: int | None = None, connectivity: int = 4):
+    """NEXT-1 -> (chosen candidate indices with -1 for the full frame, est after each)."""
+    masks = np.ascontiguousarray(masks, np.uint8)
+    n, gh, gw = masks.shape
+    full_cost = frame_w * frame_h if full_cost is None else full_cost
+    idx = np.zeros(k, np.int32)
+    est = np.zeros(k, np.int64)
+    cands = wsizes(candidates)
+    nw = _check(_lib2().otif_ref_choose_window_sizes(_p(masks), n, gh, gw, cell, frame_w, frame_h, connectivity,
+                                                     cands, len(candidates), full_cost, k, _p(idx), _p(est)),
+                "choose_window_sizes")
+    return idx[:nw].tolist(), est[:nw].tolist()
+
+
+def covered(boxes: np.ndarray, windows: np.ndarray) -> int:
+    """NEXT-2 recall numerator: boxes int32 [nb, 5] (frame, x0, y0, x1, y1)."""
+    boxes = np.ascontiguousarray(boxes, np.int32).reshape(-1, 5)
+    windows = np.ascontiguousarray(windows, WINDOW_DTYPE)
+    return int(_lib2().otif_ref_covered(_p(boxes), boxes.shape[0], _p(windows), windows.shape[0]))

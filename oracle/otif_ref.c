@@ -458,3 +458,73 @@ int otif_ref_pack_windows(const uint8_t *src, int32_t n, int32_t sh, int32_t sw,
     free(owned);
     return 0;
 }
+
+/* ------------------------------------------------------------------------- */
+/* est(R_t) = Σ_{r in R_t} T_{r.w, r.h} of the windows stage 4 emits. */
+int64_t otif_ref_frame_est(const uint8_t *mask, int32_t gh, int32_t gw, int32_t cell, int32_t frame_w,
+                           int32_t frame_h, int32_t connectivity, const otif_ref_wsize *sizes, int32_t k) {
+    int32_t cap = gh * gw + 1;
+    otif_ref_window *R = (otif_ref_window *)malloc(sizeof(otif_ref_window) * cap);
+    int m = otif_ref_group_frame(mask, gh, gw, cell, frame_w, frame_h, connectivity, sizes, k, 0, R, cap);
+    int64_t est = 0;
+    for (int i = 0; i < m; i++) est += sizes[R[i].size_idx].cost;
+    free(R);
+    return m < 0 ? -1 : est;
+}
+
+/* NEXT-1 — P:L155: "we first initialize W to only contain the size corresponding to the
+ * entire video frame ... We then repeatedly greedily add the window size to W that
+ * provides the greatest decrease to Σ_t est(R(I_t; W)), until |W| = k." */
+int otif_ref_choose_window_sizes(const uint8_t *masks, int32_t n, int32_t gh, int32_t gw, int32_t cell,
+                                 int32_t frame_w, int32_t frame_h, int32_t connectivity,
+                                 const otif_ref_wsize *candidates, int32_t m, int64_t full_cost, int32_t k,
+                                 int32_t *chosen_idx, int64_t *est) {
+    if (n < 0 || m < 0 || k < 1) return -1;
+    otif_ref_wsize *W = (otif_ref_wsize *)malloc(sizeof(otif_ref_wsize) * (k + 1));
+    int32_t *used = (int32_t *)calloc(m > 0 ? m : 1, sizeof(int32_t));
+    W[0].w = frame_w; W[0].h = frame_h; W[0].cost = full_cost;
+    int32_t nw = 1;
+    int64_t cur = 0;
+    for (int32_t f = 0; f < n; f++)
+        cur += otif_ref_frame_est(masks + (size_t)f * gh * gw, gh, gw, cell, frame_w, frame_h, connectivity, W, nw);
+    chosen_idx[0] = -1;
+    est[0] = cur;
+    while (nw < k) {
+        int32_t best = -1;
+        int64_t best_sum = cur;
+        for (int32_t c = 0; c < m; c++) {
+            if (used[c]) continue;
+            W[nw] = candidates[c];
+            int64_t sum = 0;
+            for (int32_t f = 0; f < n; f++)
+                sum += otif_ref_frame_est(masks + (size_t)f * gh * gw, gh, gw, cell, frame_w, frame_h, connectivity,
+                                          W, nw + 1);
+            if (sum < best_sum) { best_sum = sum; best = c; }  /* greatest decrease; ties: earliest */
+        }
+        if (best < 0) break;  /* no candidate decreases the sum (reading R19) */
+        used[best] = 1;
+        W[nw] = candidates[best];
+        chosen_idx[nw] = best;
+        est[nw] = best_sum;
+        cur = best_sum;
+        nw++;
+    }
+    free(W);
+    free(used);
+    return nw;
+}
+
+/* NEXT-2 — P:L232: "The recall is the fraction of detections computed by θ_best that are
+ * covered by rectangles in R_ij"; reading R18: contained in one window of its frame. */
+int64_t otif_ref_covered(const int32_t *boxes, int64_t nb, const otif_ref_window *windows, int32_t total) {
+    int64_t covered = 0;
+    for (int64_t i = 0; i < nb; i++) {
+        const int32_t *b = boxes + i * 5;
+        for (int32_t g = 0; g < total; g++) {
+            const otif_ref_window *r = &windows[g];
+            if (r->frame != b[0]) continue;
+            if (r->x <= b[1] && b[3] <= r->x + r->w && r->y <= b[2] && b[4] <= r->y + r->h) { covered++; break; }
+        }
+    }
+    return covered;
+}

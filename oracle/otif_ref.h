@@ -94,6 +94,29 @@ int otif_ref_pack_windows(const uint8_t *src, int32_t n, int32_t sh, int32_t sw,
                           uint8_t *const *batches, const int32_t *batch_cap,
                           int32_t *slot, int32_t *size_count);
 
+/* est(R_t) of one frame's windows: Σ T over the windows stage 4 emits. */
+int64_t otif_ref_frame_est(const uint8_t *mask, int32_t gh, int32_t gw, int32_t cell, int32_t frame_w,
+                           int32_t frame_h, int32_t connectivity, const otif_ref_wsize *sizes, int32_t k);
+
+/* NEXT-1: choose the fixed window-size set.  "we first initialize W to only
+ * contain the size corresponding to the entire video frame ... We then repeatedly greedily
+ * add the window size to W that provides the greatest decrease to Σ_t est(R(I_t; W)),
+ * until |W| = k", over perfect-proxy masks.  candidates: m sizes (the full frame
+ * excluded); ties go to the earliest candidate; stops early when no candidate decreases
+ * the sum (reading R19).  chosen_idx[k]: candidate index of each added size (-1 = the
+ * full frame, always chosen_idx[0]); est[k]: Σ_t est after each addition.  Returns the
+ * number of sizes chosen (<= k). */
+int otif_ref_choose_window_sizes(const uint8_t *masks, int32_t n, int32_t gh, int32_t gw, int32_t cell,
+                                 int32_t frame_w, int32_t frame_h, int32_t connectivity,
+                                 const otif_ref_wsize *candidates, int32_t m, int64_t full_cost, int32_t k,
+                                 int32_t *chosen_idx, int64_t *est);
+
+/* NEXT-2: recall = fraction of detections "covered by rectangles" — a
+ * detection [x0,x1) x [y0,y1) (clipped to the frame) counts as covered when it lies
+ * inside one window of its frame (reading R18).  boxes: int32 [nb][5] = (frame, x0, y0,
+ * x1, y1); windows/total as from otif_ref_select_windows.  Returns the covered count. */
+int64_t otif_ref_covered(const int32_t *boxes, int64_t nb, const otif_ref_window *windows, int32_t total);
+
 #ifdef __cplusplus
 }
 #endif

@@ -79,6 +79,13 @@ def lib() -> ctypes.CDLL:
     L.otif_select_windows.restype = st
     L.otif_pack_windows.argtypes = [P, i32, i32, i32, i32, i32, P, P, i32, P, i32, P, P, P, P, P]
     L.otif_pack_windows.restype = st
+    L.otif_choose_workspace_bytes.argtypes = [i32, i32, i32, i32]
+    L.otif_choose_workspace_bytes.restype = sz
+    L.otif_choose_window_sizes.argtypes = [P, i32, i32, i32, ctypes.POINTER(GridDesc), P, i32, ctypes.c_int64, i32,
+                                           P, P, P, sz, P]
+    L.otif_choose_window_sizes.restype = st
+    L.otif_window_recall.argtypes = [P, ctypes.c_int64, P, P, P, i32, P, P]
+    L.otif_window_recall.restype = st
     if hasattr(L, "otif_pipeline_create"):
         L.otif_pipeline_create.argtypes = [ctypes.POINTER(PipelineDesc), P, sz, ctypes.POINTER(P)]
         L.otif_pipeline_create.restype = st
@@ -111,6 +118,7 @@ EXPORTED = ("otif_status_str", "otif_last_error", "otif_version", "otif_resize",
             "otif_select_workspace_bytes", "otif_select_windows", "otif_pack_windows",
             "otif_pipeline_create", "otif_pipeline_destroy", "otif_pipeline_run_host",
             "otif_pipeline_run_device", "otif_pipeline_counters", "otif_pipeline_reset_counters",
-            "otif_pipeline_set_timing", "otif_pipeline_stage_ms")
+            "otif_pipeline_set_timing", "otif_pipeline_stage_ms", "otif_choose_workspace_bytes",
+            "otif_choose_window_sizes", "otif_window_recall")
 STAGES = ("resize", "proxy_prep_e1", "conv_e2", "conv_e3", "conv_e4", "conv_e5", "conv_d1_head", "select",
           "pack", "append")

@@ -23,7 +23,7 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base);
+                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum);
 
 // timing stages: resize, proxy prep (tag + E1), E2, E3, E4, E5, D1+D2, select, pack, append
 constexpr int kStages = 10;
@@ -123,7 +123,8 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
     }
     RC(mark(p, ST_START, st));
     RC(launch_select(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask, p->windows,
-                     p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base));
+                     p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base,
+                     nullptr));
     RC(mark(p, ST_SELECT, st));
     RC(otif_pack_windows(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
                          p->batches, d.batch_cap, p->slot, p->size_count, st));

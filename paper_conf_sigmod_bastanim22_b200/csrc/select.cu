@@ -51,6 +51,7 @@ struct SelectParams {
     // pipeline-only (internal): run counters, global frame index base
     unsigned long long *ctr;
     int frame_base;
+    unsigned long long *est_sum;  // internal: Σ est(R_t) over frames (window-size selection)
 };
 
 struct Rect16 { short x0, y0, x1, y1; };  // cell units, half-open
@@ -505,6 +506,7 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
             w.frame = f; w.x = 0; w.y = 0; w.w = p.fw; w.h = p.fh; w.size_idx = p.orig[p.full];
             out[0] = w;
             p.counts[f] = 1;
+            if (p.est_sum) atomicAdd(p.est_sum, (unsigned long long)p.cost[p.full]);
             if (p.ctr) {
                 unsigned long long gf = (unsigned long long)(unsigned)(f + p.frame_base);
                 atomicAdd(&p.ctr[0], 1ull);
@@ -551,6 +553,7 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
     }
     if (lane == 0) {
         p.counts[f] = m;
+        if (p.est_sum) atomicAdd(p.est_sum, (unsigned long long)est);
         if (p.ctr) {
             atomicAdd(&p.ctr[0], 1ull);
             atomicAdd(&p.ctr[1], (unsigned long long)npos);
@@ -624,7 +627,7 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base) {
+                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum) {
     SelectParams p;
     memset(&p, 0, sizeof(p));
     p.scores = scores; p.mask_in = mask_in; p.thr = threshold;
@@ -667,6 +670,7 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
     }
     p.ctr = ctr;
     p.frame_base = frame_base;
+    p.est_sum = est_sum;
     int warps = (int)((200 * 1024) / p.frame_bytes);
     warps = warps < 1 ? 1 : (warps > kSelWarpsMax ? kSelWarpsMax : warps);
     // spread small batches over the SMs rather than packing frames into few CTAs
@@ -742,5 +746,5 @@ extern "C" otif_status otif_select_windows(const float *scores, const uint8_t *m
     st = check_device(nullptr);
     if (st != OTIF_OK) return st;
     return launch_select(scores, mask_in, threshold, n, gh, gw, g, sizes, k, mask_out, windows, capacity, frame_count,
-                         frame_offset, total, workspace, ws_bytes, stream, nullptr, 0);
+                         frame_offset, total, workspace, ws_bytes, stream, nullptr, 0, nullptr);
 }
