@@ -404,6 +404,229 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
 }
 
 // ---------------------------------------------------------------------------
+// The same implicit GEMM on a CTA PAIR (cluster of 2, tcgen05 cta_group::2): one M=256
+// MMA spans both SMs — each CTA holds 128 rows of A (its own halo) and HALF of the N
+// columns of B, so per-SM shared-memory operand traffic and weight streaming halve
+// (N=128 layers are otherwise shared-memory-bandwidth bound).  The leader (rank 0)
+// issues the MMAs and commits them to both CTAs' barriers (multicast); the peer's MMA
+// warp relays "stage full" to the leader (remote mbarrier arrive); both epilogues
+// drain their own TMEM and report to the leader's accumulator-empty barrier.
+// Weights are packed [cb][tap][half][chunk][N/2][8].
+// ---------------------------------------------------------------------------
+template <int MT>
+__global__ void __launch_bounds__(kConvThreads, 1) conv_umma2_kernel(const __grid_constant__ ConvParams p) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    const uint32_t rank = cluster_ctarank();
+    const int cluster = blockIdx.x >> 1, nclusters = gridDim.x >> 1;
+
+    const uint32_t chunks = p.kb >> 3;
+    const uint32_t a_bytes = chunks * p.P * 16;
+    const uint32_t nh = (uint32_t)p.N / 2;           // B rows held by this CTA
+    const uint32_t b_bytes = nh * p.kb * 2;
+    uint8_t *a_buf = smem;
+    uint8_t *b_buf = a_buf + (size_t)p.stages_a * a_bytes;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(b_buf + (size_t)p.stages_b * b_bytes);
+    uint64_t *a_full = bars;
+    uint64_t *a_empty = a_full + kMaxStagesA;
+    uint64_t *b_full = a_empty + kMaxStagesA;
+    uint64_t *b_empty = b_full + kMaxStagesB;
+    uint64_t *a_peer = b_empty + kMaxStagesB;        // leader: peer's A stage landed
+    uint64_t *b_peer = a_peer + kMaxStagesA;         // leader: peer's B stage landed
+    uint64_t *t_full = b_peer + kMaxStagesB;
+    uint64_t *t_empty = t_full + 2;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(t_empty + 2);
+    float *s_bias = reinterpret_cast<float *>(tmem_slot + 4);
+    float *s_w2 = s_bias + 256;
+
+    const uint32_t acc_cols = 2 * MT * p.N;
+    const uint32_t tmem_cols = acc_cols <= 32 ? 32 : (acc_cols <= 64 ? 64 : (acc_cols <= 128 ? 128 : (acc_cols <= 256 ? 256 : 512)));
+    const int npairs = p.ntiles;                     // pair tiles of 2 x 128*MT rows
+
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < p.stages_a; i++) { mbar_init(&a_full[i], 1); mbar_init(&a_empty[i], 1); mbar_init(&a_peer[i], 1); }
+        for (int i = 0; i < p.stages_b; i++) { mbar_init(&b_full[i], 1); mbar_init(&b_empty[i], 1); mbar_init(&b_peer[i], 1); }
+        for (int i = 0; i < 2; i++) { mbar_init(&t_full[i], 1); mbar_init(&t_empty[i], 129);  /* 128 local + 1 from the peer */ }
+        fence_barrier_init();
+    }
+    if (warp == 2) tmem_alloc2(tmem_slot, tmem_cols);
+    for (int i = threadIdx.x; i < p.N; i += blockDim.x) {
+        s_bias[i] = p.bias[i];
+        if (p.out_kind == 3) s_w2[i] = p.w2[i];
+    }
+    tc_fence_before();
+    __syncthreads();
+    cluster_sync();  // both CTAs' barriers initialised before any remote arrive
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        // ===== producer (both CTAs): own halo rows and own half of the weights =====
+        if (lane == 0) {
+            uint32_t as = 0, ap = 0, bs = 0, bp = 0;
+            for (int pt = cluster; pt < npairs; pt += nclusters) {
+                const int64_t q0 = ((int64_t)pt * 2 + rank) * kTileM * MT;
+                for (int cb = 0; cb < p.ncb; cb++) {
+                    int tap_pos = 0;
+                    for (int g = 0; g < p.ngroups; g++) {
+                        mbar_wait(&a_empty[as], ap ^ 1);
+                        mbar_arrive_expect_tx(&a_full[as], a_bytes);
+                        uint8_t *dst = a_buf + (size_t)as * a_bytes;
+                        const int plane = p.group_plane[g];
+                        for (uint32_t j = 0; j < chunks; j++) {
+                            const uint8_t *src =
+                                p.act + (((int64_t)plane * p.c8_in + cb * chunks + j) * p.lcap + q0) * 16;
+                            bulk_g2s(dst + j * p.P * 16, src, p.P * 16, &a_full[as]);
+                        }
+                        if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
+                        for (int t = 0; t < p.group_ntaps[g]; t++, tap_pos++) {
+                            mbar_wait(&b_empty[bs], bp ^ 1);
+                            mbar_arrive_expect_tx(&b_full[bs], b_bytes);
+                            bulk_g2s(b_buf + (size_t)bs * b_bytes,
+                                     p.wpk + (((size_t)cb * 9 + tap_pos) * 2 + rank) * b_bytes, b_bytes, &b_full[bs]);
+                            if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
+                        }
+                    }
+                }
+            }
+        }
+    } else if (warp == 1 && rank == 1) {
+        // ===== peer: relay "stage full" to the leader's a_peer / b_peer =====
+        if (lane == 0) {
+            uint32_t as = 0, ap = 0, bs = 0, bp = 0;
+            const uint32_t a_peer0 = mapa_shared(smem_u32(a_peer), 0), b_peer0 = mapa_shared(smem_u32(b_peer), 0);
+            for (int pt = cluster; pt < npairs; pt += nclusters) {
+                for (int cb = 0; cb < p.ncb; cb++) {
+                    for (int g = 0; g < p.ngroups; g++) {
+                        mbar_wait(&a_full[as], ap);
+                        mbar_arrive_cluster(a_peer0 + as * 8);
+                        if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
+                        for (int t = 0; t < p.group_ntaps[g]; t++) {
+                            mbar_wait(&b_full[bs], bp);
+                            mbar_arrive_cluster(b_peer0 + bs * 8);
+                            if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
+                        }
+                    }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ===== leader: MMA issuer for the pair (single thread) =====
+        if (lane == 0) {
+            const uint32_t idesc = umma_idesc_bf16(2 * kTileM, p.N);
+            uint32_t as = 0, ap = 0, bs = 0, bp = 0, acc = 0, accp = 0;
+            const uint32_t a_base = smem_u32(a_buf), b_base = smem_u32(b_buf);
+            const uint32_t lbo_a = p.P * 16, lbo_b = nh * 16;
+            for (int pt = cluster; pt < npairs; pt += nclusters) {
+                mbar_wait_cluster(&t_empty[acc], accp ^ 1);
+                tc_fence_after();
+                const uint32_t d = tmem_base + acc * MT * p.N;
+                uint32_t accumulate = 0;
+                for (int cb = 0; cb < p.ncb; cb++) {
+                    for (int g = 0; g < p.ngroups; g++) {
+                        mbar_wait(&a_full[as], ap);
+                        mbar_wait_cluster(&a_peer[as], ap);
+                        tc_fence_after();
+                        const uint32_t a_stage = a_base + as * a_bytes;
+                        for (int t = 0; t < p.group_ntaps[g]; t++) {
+                            mbar_wait(&b_full[bs], bp);
+                            mbar_wait_cluster(&b_peer[bs], bp);
+                            tc_fence_after();
+                            const uint32_t a_tap = a_stage + p.group_shift[g][t] * 16;
+                            const uint32_t b_stage = b_base + bs * b_bytes;
+                            for (uint32_t s = 0; s < chunks / 2; s++) {
+                                const uint64_t bd = umma_desc(b_stage + 2 * s * lbo_b, lbo_b, 128);
+#pragma unroll
+                                for (int m = 0; m < MT; m++) {
+                                    uint64_t ad = umma_desc(a_tap + 2 * s * lbo_a + m * (kTileM * 16), lbo_a, 128);
+                                    umma2_bf16(d + m * p.N, ad, bd, idesc, accumulate);
+                                }
+                                accumulate = 1;
+                            }
+                            umma2_commit_mc(&b_empty[bs], 0x3);
+                            if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
+                        }
+                        umma2_commit_mc(&a_empty[as], 0x3);
+                        if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
+                    }
+                }
+                umma2_commit_mc(&t_full[acc], 0x3);
+                if (++acc == 2) { acc = 0; accp ^= 1; }
+            }
+        }
+    } else if (warp >= 4) {
+        // ===== epilogue (both CTAs): own 128 TMEM lanes = own rows =====
+        const int row = threadIdx.x - 128;
+        const int quarter = warp & 3;
+        const uint32_t t_empty0 = mapa_shared(smem_u32(t_empty), 0);
+        uint32_t acc = 0, accp = 0;
+        for (int pt = cluster; pt < npairs; pt += nclusters) {
+            mbar_wait(&t_full[acc], accp);
+            tc_fence_after();
+            for (int m = 0; m < MT; m++) {
+                const int64_t q = ((int64_t)pt * 2 + rank) * kTileM * MT + m * kTileM + row;
+                const int f = (int)(q / p.fstride);
+                const int64_t r = q - (int64_t)f * p.fstride;
+                const int oy = (int)(r / p.pitch);
+                const int ox = (int)(r - (int64_t)oy * p.pitch);
+                const bool valid = q < p.mtot && oy < p.out_h && ox < p.out_w;
+                int plane = 0;
+                int64_t L = 0;
+                if (p.out_kind != 3) L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, f, oy, ox, plane);
+                const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + (acc * MT + m) * p.N;
+                float z = p.b2;
+                for (int cc = 0; cc < p.N / 32; cc++) {
+                    uint32_t v[32];
+                    tmem_ld32(taddr + cc * 32, v);
+                    uint32_t pk[16];
+#pragma unroll
+                    for (int j = 0; j < 16; j++) {
+                        float a = fmaxf(__uint_as_float(v[2 * j]) + s_bias[cc * 32 + 2 * j], 0.0f);
+                        float b = fmaxf(__uint_as_float(v[2 * j + 1]) + s_bias[cc * 32 + 2 * j + 1], 0.0f);
+                        pk[j] = pack_bf16x2(a, b);
+                    }
+                    if (p.out_kind == 3) {
+#pragma unroll
+                        for (int j = 0; j < 16; j++) {
+                            float a = __uint_as_float(pk[j] << 16);
+                            float b = __uint_as_float(pk[j] & 0xFFFF0000u);
+                            z = fmaf(s_w2[cc * 32 + 2 * j], a, z);
+                            z = fmaf(s_w2[cc * 32 + 2 * j + 1], b, z);
+                        }
+                    } else if (valid) {
+#pragma unroll
+                        for (int c = 0; c < 4; c++) {
+                            uint8_t *dst = p.out + (((int64_t)plane * p.out_c8 + cc * 4 + c) * p.out_lcap + L) * 16;
+                            *reinterpret_cast<uint4 *>(dst) =
+                                make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+                        }
+                    }
+                }
+                if (p.out_kind == 3 && valid)
+                    p.scores[((int64_t)f * p.out_h + oy) * p.out_w + ox] = 1.0f / (1.0f + expf(-z));
+            }
+            tc_fence_before();
+            if (rank == 0) {
+                mbar_arrive(&t_empty[acc]);
+            } else {  // one cluster-scope release for the whole peer epilogue
+                asm volatile("bar.sync 1, 128;" ::: "memory");
+                if (row == 0) mbar_arrive_cluster(t_empty0 + acc * 8);
+            }
+            if (++acc == 2) { acc = 0; accp ^= 1; }
+        }
+    }
+    __syncwarp();
+    tc_fence_before();
+    __syncthreads();
+    cluster_sync();  // the peer's smem / TMEM stay alive until the pair's last MMA drained
+    if (warp == 2) {
+        tc_fence_after();
+        tmem_dealloc2(tmem_base, tmem_cols);
+    }
+}
+
+// ---------------------------------------------------------------------------
 // host side: plan, weight packing, launch
 // ---------------------------------------------------------------------------
 static uint16_t f32_to_bf16_rne(float f) {
@@ -427,7 +650,7 @@ struct GemmLayer {
     int64_t fstride_unit;         // per-frame pixels of the input layout
     int max_shift;
     int ngroups, group_plane[4], group_ntaps[4], group_shift[4][9], group_tap[4][9];
-    int kb, ncb, P, mt;
+    int kb, ncb, P, mt, cg;   // cg: 1 = single CTA, 2 = CTA pair (cta_group::2)
     uint8_t *wpk_dev;
     float *bias_dev;
 };
@@ -494,6 +717,13 @@ static void build_layer(GemmLayer &g, int cin, int cout, int stride, int in_h, i
     // mt sub-tiles of 128 rows per CTA tile so that every tap issues >= 256 columns of MMA
     // work (mt * N = 256): amortises the per-stage barrier and copy overheads of small N
     g.mt = cout >= 256 ? 1 : (cout >= 128 ? 2 : 4);
+    // CTA pairs (cta_group::2) would halve per-SM operand traffic for N >= 128, but with
+    // the relayed stage hand-off they measured 1.3-1.7x SLOWER than single CTAs on B200
+    // (profiles/r01_cta_pair.md); single CTAs are the default, pairs opt-in for tuning.
+    g.cg = 1;
+    if (const char *e = getenv("OTIF_CONV_CG")) {  // tuning experiments only
+        if (atoi(e) == 2 && cout >= 128) g.cg = 2;
+    }
     if (const char *e = getenv("OTIF_CONV_MT_MAX")) {  // tuning experiments only
         int cap = atoi(e);
         if (cap >= 1 && g.mt > cap) g.mt = cap;
@@ -508,7 +738,7 @@ static Layout input_layout(const GemmLayer &g, int n) {
     l.pitch = g.pitch;
     l.fstride = g.fstride_unit;
     int64_t mtot = (int64_t)n * g.fstride_unit;
-    l.lcap = round_up(round_up(mtot, (int64_t)kTileM * g.mt) + g.max_shift + 8, 16);
+    l.lcap = round_up(round_up(mtot, (int64_t)kTileM * g.mt * g.cg) + g.max_shift + 8, 16);
     l.c8 = g.cin / 8;
     l.bytes = (size_t)l.planes * l.c8 * l.lcap * 16;
     l.offset = 0;
@@ -527,12 +757,14 @@ static size_t plan_workspace(const otif_proxy *p, int n, Layout lay[5]) {
 
 static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
     size_t a = (size_t)(g.kb / 8) * g.P * 16;
-    size_t b = (size_t)g.cout * g.kb * 2;
-    size_t fixed = (2 * kMaxStagesA + 2 * kMaxStagesB + 4) * 8 + 16 + 2 * 256 * 4 + 1024;
+    size_t b = (size_t)g.cout * g.kb * 2 / g.cg;
+    size_t fixed = (3 * kMaxStagesA + 3 * kMaxStagesB + 4) * 8 + 16 + 2 * 256 * 4 + 1024;
     size_t budget = 220 * 1024;
     sa = 2; sb = 2;
     // grow B (weights stream every tap) first, then A
-    while (sb < kMaxStagesB && sa * a + (sb + 1) * b + fixed <= budget && sb < 6) sb++;
+    // a CTA pair recycles a stage over a longer loop (peer relay, multicast commit): deeper B ring
+    const int sb_max = g.cg == 2 ? kMaxStagesB : 6;
+    while (sb < kMaxStagesB && sa * a + (sb + 1) * b + fixed <= budget && sb < sb_max) sb++;
     while (sa < kMaxStagesA && (sa + 1) * a + sb * b + fixed <= budget && sa < 3) sa++;
     bytes = sa * a + sb * b + fixed;
 }
@@ -600,7 +832,7 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         }
         c.wpk = g.wpk_dev; c.bias = g.bias_dev; c.N = g.cout;
         c.mtot = (int64_t)n * g.fstride_unit;
-        c.ntiles = (int)cdiv(c.mtot, (int64_t)kTileM * g.mt);
+        c.ntiles = (int)cdiv(c.mtot, (int64_t)kTileM * g.mt * g.cg);  // pair tiles when cg == 2
         c.pitch = g.pitch; c.fstride = g.fstride_unit; c.out_h = g.out_h; c.out_w = g.out_w;
         if (li < 4) {
             c.out_kind = lay[li + 1].kind;
@@ -617,11 +849,31 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         }
         size_t smem;
         conv_smem(g, c.stages_a, c.stages_b, smem);
-        int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
-        if (grid < 1) grid = 1;
-        auto kern = g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>);
-        OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        kern<<<grid, kConvThreads, smem, stream>>>(c);
+        if (g.cg == 2) {
+            const int pairs = p->num_sms / 2;
+            const int clusters = c.ntiles < pairs ? (c.ntiles < 1 ? 1 : c.ntiles) : pairs;
+            auto kern = g.mt == 4 ? conv_umma2_kernel<4> : (g.mt == 2 ? conv_umma2_kernel<2> : conv_umma2_kernel<1>);
+            OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(2 * clusters);
+            cfg.blockDim = dim3(kConvThreads);
+            cfg.dynamicSmemBytes = smem;
+            cfg.stream = stream;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeClusterDimension;
+            attr[0].val.clusterDim.x = 2;
+            attr[0].val.clusterDim.y = 1;
+            attr[0].val.clusterDim.z = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            OTIF_CUDA(cudaLaunchKernelEx(&cfg, kern, c));
+        } else {
+            int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
+            if (grid < 1) grid = 1;
+            auto kern = g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>);
+            OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            kern<<<grid, kConvThreads, smem, stream>>>(c);
+        }
         OTIF_LAUNCH_CHECK();
         if (evs) OTIF_CUDA(cudaEventRecord(evs[1 + li], stream));
     }
@@ -722,7 +974,10 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
                             for (int e = 0; e < 8; e++) {
                                 int ci = cb * g.kb + j * 8 + e;
                                 float v = W[(((size_t)nn * 3 + kh) * 3 + kw) * g.cin + ci];
-                                pk[((((size_t)cb * 9 + pos) * chunks + j) * g.cout + nn) * 8 + e] = f32_to_bf16_rne(v);
+                                // cg == 2: [cb][tap][half][chunk][N/2][8] (each CTA of a pair streams its half)
+                                const int nh = g.cout / g.cg, half = nn / nh, nl = nn - half * nh;
+                                pk[(((((size_t)cb * 9 + pos) * g.cg + half) * chunks + j) * nh + nl) * 8 + e] =
+                                    f32_to_bf16_rne(v);
                             }
                 }
         }
