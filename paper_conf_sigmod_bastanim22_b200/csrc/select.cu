@@ -27,8 +27,9 @@
 
 namespace otif {
 
-constexpr int kSelWarpsMax = 8;
+constexpr int kSelWarpsMax = 16;
 constexpr int kMatMax = 128;  // fit-matrix capacity (components per frame); larger n -> rescan path
+constexpr int kSmallClusters = 64;  // components per frame in the first (high-occupancy) pass
 constexpr int kMaxSizes = 8;
 
 struct SelectParams {
@@ -52,6 +53,12 @@ struct SelectParams {
     unsigned long long *ctr;
     int frame_base;
     unsigned long long *est_sum;  // internal: Σ est(R_t) over frames (window-size selection)
+    // two-pass scheduling: pass 1 gives every frame a small slice (ccap clusters) and
+    // defers frames with more components to pass 2 (full-size slices, frames from the list)
+    int ccap;                   // cluster capacity of a slice
+    int *defer_list;
+    int *defer_count;
+    int from_list;
 };
 
 struct Rect16 { short x0, y0, x1, y1; };  // cell units, half-open
@@ -296,10 +303,15 @@ __device__ void greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, 
 __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_constant__ SelectParams p) {
     extern __shared__ __align__(16) uint8_t smem[];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    const int f = blockIdx.x * (blockDim.x >> 5) + wid;
-    if (f >= p.n) return;
+    int f = blockIdx.x * (blockDim.x >> 5) + wid;
+    if (p.from_list) {
+        if (f >= *p.defer_count) return;
+        f = p.defer_list[f];
+    } else if (f >= p.n) {
+        return;
+    }
     const int cells = p.gh * p.gw;
-    const int cap = p.cap_f;
+    const int cap = p.ccap;
     uint8_t *base = smem + (size_t)wid * p.frame_bytes;
     Frame F;
     F.par = reinterpret_cast<int *>(base);
@@ -339,14 +351,14 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
         }
     }
     __syncwarp();
-    // read-only flatten into scratch (cl/cost region: 16*cap >= 4*cells bytes), then publish
+    // read-only flatten into scratch (the cid array, free until the id scan), then publish
     {
-        int *lab = reinterpret_cast<int *>(F.cl);
+        short *lab = F.cid;
         for (int i = lane; i < cells; i += 32) {
             int x = F.par[i];
             if (x >= 0)
                 while (F.par[x] != x) x = F.par[x];
-            lab[i] = x;
+            lab[i] = (short)x;
         }
         __syncwarp();
         for (int i = lane; i < cells; i += 32) F.par[i] = lab[i];
@@ -372,7 +384,11 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
     }
     __syncwarp();
     for (int o = 16; o > 0; o >>= 1) npos += __shfl_xor_sync(0xffffffffu, npos, o);
-    otif_window *out = p.tmp + (size_t)f * cap;
+    otif_window *out = p.tmp + (size_t)f * p.cap_f;
+    if (n > cap) {  // more components than this slice holds: defer to the full-size pass
+        if (lane == 0) p.defer_list[atomicAdd(p.defer_count, 1)] = f;
+        return;
+    }
     if (n == 0) {
         if (lane == 0) {
             p.counts[f] = 0;
@@ -615,11 +631,14 @@ __global__ void __launch_bounds__(1024) compact_kernel(const otif_window *__rest
 
 static int sel_cap(int gh, int gw) { return (gh * gw + 1) / 2 > 1 ? (gh * gw + 1) / 2 : 1; }
 
-static int sel_frame_bytes(int gh, int gw) {
-    int cells = gh * gw, cap = sel_cap(gh, gw);
+// shared bytes of one frame slice holding ccap clusters and an nmat x nmat fit matrix
+static int sel_frame_bytes(int gh, int gw, int ccap, int nmat, int *gmat_offset) {
+    int cells = gh * gw;
     int head = (cells * 6 + 15) & ~15;
     // cl 8 + cost 8 + bg 8 + bj 2 + sidx 1 + alive 1 bytes per cluster
-    return (int)round_up(head + (int64_t)cap * 28, 16);
+    int body = (int)round_up(head + (int64_t)ccap * 28, 16);
+    *gmat_offset = body;
+    return body + (int)round_up((int64_t)nmat * nmat, 16);
 }
 
 // internal entry: counters and global frame base for the pipeline (NULL / 0 from the ABI)
@@ -655,33 +674,39 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
     uint8_t *ws = (uint8_t *)workspace;
     p.tmp = (otif_window *)ws;
     p.counts = (int *)(ws + round_up((int64_t)n * p.cap_f * sizeof(otif_window), 256));
-    p.frame_bytes = sel_frame_bytes(gh, gw);
-    // gain matrix for frames with up to nmat components, when int32 gains are exact
+    // fit matrix only when int32 gains are exact
     long long max_cost = 0;
     for (int s = 0; s < k; s++) max_cost = sizes[s].cost > max_cost ? sizes[s].cost : max_cost;
     bool small_costs = max_cost < (1ll << 30);
     for (int s = 0; s < k; s++) small_costs = small_costs && sizes[s].cost >= 0;
-    p.nmat = 0;
-    p.gmat_offset = p.frame_bytes;
-    if (small_costs) {
-        int nm = p.cap_f < kMatMax ? p.cap_f : kMatMax;
-        p.nmat = (int)round_up(nm, 8);
-        p.frame_bytes += (int)round_up(p.nmat * p.nmat, 16);
-    }
     p.ctr = ctr;
     p.frame_base = frame_base;
     p.est_sum = est_sum;
-    int warps = (int)((200 * 1024) / p.frame_bytes);
-    warps = warps < 1 ? 1 : (warps > kSelWarpsMax ? kSelWarpsMax : warps);
-    // spread small batches over the SMs rather than packing frames into few CTAs
+    p.defer_list = p.counts + round_up(n, 64);
+    p.defer_count = p.defer_list + round_up(n, 64);
+    OTIF_CUDA(cudaMemsetAsync(p.defer_count, 0, 4, stream));
     int num_sms = 148;
     check_device(&num_sms);
-    while (warps > 1 && cdiv(n, warps) < 2 * num_sms) warps--;
-    if (warps > n) warps = n;
-    size_t smem = (size_t)warps * p.frame_bytes;
-    OTIF_CUDA(cudaFuncSetAttribute(select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    select_kernel<<<(unsigned)cdiv(n, warps), warps * 32, smem, stream>>>(p);
-    OTIF_LAUNCH_CHECK();
+    for (int pass = 0; pass < 2; pass++) {
+        // pass 0: small slices (<= kSmallClusters components, many frames per SM);
+        // pass 1: the deferred frames with full-size slices
+        const int ccap = pass == 0 ? (p.cap_f < kSmallClusters ? p.cap_f : kSmallClusters) : p.cap_f;
+        if (pass == 1 && ccap == (p.cap_f < kSmallClusters ? p.cap_f : kSmallClusters)) break;  // nothing deferred
+        p.ccap = ccap;
+        p.from_list = pass;
+        p.nmat = small_costs ? (int)round_up(ccap < kMatMax ? ccap : kMatMax, 8) : 0;
+        p.frame_bytes = sel_frame_bytes(gh, gw, ccap, p.nmat, &p.gmat_offset);
+        int warps = (int)((200 * 1024) / p.frame_bytes);
+        warps = warps < 1 ? 1 : (warps > kSelWarpsMax ? kSelWarpsMax : warps);
+        if (pass == 0) {  // spread small batches over the SMs rather than packing frames into few CTAs
+            while (warps > 1 && cdiv(n, warps) < 2 * num_sms) warps--;
+        }
+        if (warps > n) warps = n;
+        const size_t smem = (size_t)warps * p.frame_bytes;
+        OTIF_CUDA(cudaFuncSetAttribute(select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        select_kernel<<<(unsigned)cdiv(n, warps), warps * 32, smem, stream>>>(p);
+        OTIF_LAUNCH_CHECK();
+    }
     compact_kernel<<<(unsigned)cdiv(n, 1024), 1024, 0, stream>>>(p.tmp, p.cap_f, p.counts, n, windows, capacity,
                                                                  frame_count, frame_offset, total);
     OTIF_LAUNCH_CHECK();
@@ -690,8 +715,9 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
 
 size_t select_workspace_bytes(int32_t n, int32_t gh, int32_t gw) {
     if (n < 0 || gh <= 0 || gw <= 0) return 0;
+    // per-frame window scratch; counts, the deferred-frame list and its counter
     return (size_t)round_up((int64_t)n * sel_cap(gh, gw) * sizeof(otif_window), 256) +
-           (size_t)round_up((int64_t)n * 4, 256);
+           (size_t)round_up((round_up(n, 64) * 2 + 64) * 4, 256);
 }
 
 otif_status validate_select(const float *scores, const uint8_t *mask_in, int32_t n, int32_t gh, int32_t gw,
