@@ -270,6 +270,39 @@ def run_otif(args):
     step_sum = sum(stage_ms.values())
     stages["conv_share_of_step"] = conv_ms / step_sum if step_sum else None
 
+    # perfect-proxy line: stages 3-5 on ground-truth cell masks (mask_in), which
+    # gives object-aligned windows instead of the random-init proxy's full-frame fallback
+    perfect = None
+    if not args.no_perfect:
+        sc = video.make_scene(wl, clip=rank)
+        masks = torch.from_numpy(np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell)
+                                           for t in range(n)])).to(dev)
+        caps = [n if (s[0], s[1]) == (wl.src_w, wl.src_h) else 8 * n for s in wl.sizes]
+
+        def perfect_step():
+            r = otif.otif_select_windows(None, masks, 0.0, wl.src_w, wl.src_h, wl.cell, wl.sizes)
+            otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], wl.sizes, caps)
+            return r
+
+        for _ in range(2):
+            perfect_step()
+        torch.cuda.synchronize()
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        p0.record()
+        for _ in range(args.steps):
+            r = perfect_step()
+        p1.record()
+        torch.cuda.synchronize()
+        pms = p0.elapsed_time(p1) / args.steps
+        tot = int(r["total"].item())
+        wins = r["windows"][:tot].cpu().numpy()
+        px = int((wins[:, 3].astype(np.int64) * wins[:, 4]).sum()) if tot else 0
+        perfect = {"what": "select (mask_in = ground-truth cells) + pack per step; allocations inside",
+                   "frames_per_s": n / (pms / 1000.0), "ms_per_step": pms, "windows_per_frame": tot / n,
+                   "window_area_fraction": px / (n * wl.src_w * wl.src_h),
+                   "pack_bytes_per_step": 2 * 3 * px}
+        del masks
+
     # end to end through the C ABI with HOST frames: pinned H2D + D2H inside the timed region
     e2e = None
     if not args.no_e2e:
@@ -321,6 +354,7 @@ def run_otif(args):
                          f"{batch} frames; achieved = algorithmic FLOPs / event-timed duration",
                          "layers": per_layer},
             "stages": stages,
+            "perfect_proxy": perfect,
             "cpu_baseline": cpu_baseline,
             "e2e": e2e,
             "gpu_launches": int(launches),
@@ -347,6 +381,7 @@ def main():
     ap.add_argument("--oracle-frames", type=int, default=32)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-perfect", action="store_true", help="skip the perfect-proxy (ground-truth mask) line")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
