@@ -25,6 +25,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "otif_ref.c")
+_SRCS = [_SRC, os.path.join(_HERE, "otif_ref_tracks.c")]
 
 QUANT_NONE = 0
 QUANT_BF16 = 1
@@ -44,11 +45,12 @@ WINDOW_DTYPE = np.dtype([("frame", "<i4"), ("x", "<i4"), ("y", "<i4"),
 
 
 def build(force: bool = False) -> str:
-    """Compile liboracle.so with gcc -O2 (no -ffast-math)."""
+    """Compile liboracle.so with gcc -O2 (no -ffast-math; -ffp-contract=off so every
+    arithmetic operation is one IEEE rounding in the written order)."""
     if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < max(
-            os.path.getmtime(_SRC), os.path.getmtime(os.path.join(_HERE, "otif_ref.h"))):
-        subprocess.check_call(["gcc", "-std=c99", "-O2", "-fPIC", "-shared", "-Wall",
-                               "-o", _SO, _SRC, "-lm"])
+            [os.path.getmtime(f) for f in _SRCS] + [os.path.getmtime(os.path.join(_HERE, "otif_ref.h"))]):
+        subprocess.check_call(["gcc", "-std=c99", "-O2", "-ffp-contract=off", "-fPIC", "-shared", "-Wall",
+                               "-o", _SO] + _SRCS + ["-lm"])
     return _SO
 
 
@@ -267,3 +269,76 @@ def covered(boxes: np.ndarray, windows: np.ndarray) -> int:
     boxes = np.ascontiguousarray(boxes, np.int32).reshape(-1, 5)
     windows = np.ascontiguousarray(windows, WINDOW_DTYPE)
     return int(_lib2().otif_ref_covered(_p(boxes), boxes.shape[0], _p(windows), windows.shape[0]))
+
+
+# --------------------------------------------------------------------------- NEXT-4
+def _lib3():
+    L = lib()
+    if not getattr(L, "_tracks_bound", False):
+        P, i32, i64, f32 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_float
+        L.otif_ref_track_resample.argtypes = [P, P, i64, i32, P]
+        L.otif_ref_track_distance.argtypes = [P, P, i32]
+        L.otif_ref_track_distance.restype = f32
+        L.otif_ref_dbscan.argtypes = [P, i64, i32, f32, i32, P, P]
+        L.otif_ref_dbscan.restype = i32
+        L.otif_ref_track_centers.argtypes = [P, P, i64, i32, i32, P, P]
+        L.otif_ref_track_refine.argtypes = [P, P, i64, i32, P, P, i32, i32, f32, P, P]
+        L._tracks_bound = True
+    return L
+
+
+def _tracks_in(pts, offsets):
+    pts = np.ascontiguousarray(pts, np.float32).reshape(-1, 2)
+    offsets = np.ascontiguousarray(offsets, np.int64)
+    return pts, offsets, offsets.shape[0] - 1
+
+
+def track_resample(pts: np.ndarray, offsets: np.ndarray, npts: int = 20) -> np.ndarray:
+    """P:L196 arc-length resampling (reading R21) -> float32 [n, npts, 2]."""
+    pts, offsets, n = _tracks_in(pts, offsets)
+    out = np.zeros((n, npts, 2), np.float32)
+    _check(_lib3().otif_ref_track_resample(_p(pts), _p(offsets), n, npts, _p(out)), "track_resample")
+    return out
+
+
+def track_distance(a: np.ndarray, b: np.ndarray) -> float:
+    """P:L196 mean point distance of two resampled tracks [npts, 2] (fp32, reading R22)."""
+    a = np.ascontiguousarray(a, np.float32)
+    b = np.ascontiguousarray(b, np.float32)
+    assert a.shape == b.shape and a.shape[-1] == 2
+    return float(_lib3().otif_ref_track_distance(_p(a), _p(b), a.shape[0]))
+
+
+def dbscan(P: np.ndarray, eps: float, min_pts: int):
+    """P:L198 DBSCAN over resampled tracks [n, npts, 2] (reading R23) -> (nc, labels, core)."""
+    P = np.ascontiguousarray(P, np.float32)
+    n, npts = P.shape[0], P.shape[1]
+    labels = np.zeros(n, np.int32)
+    core = np.zeros(n, np.uint8)
+    nc = _check(_lib3().otif_ref_dbscan(_p(P), n, npts, eps, min_pts, _p(labels), _p(core)), "dbscan")
+    return nc, labels, core.astype(bool)
+
+
+def track_centers(P: np.ndarray, labels: np.ndarray, nc: int):
+    """P:L198 cluster centres -> (centers float32 [nc, npts, 2], sizes int32 [nc])."""
+    P = np.ascontiguousarray(P, np.float32)
+    labels = np.ascontiguousarray(labels, np.int32)
+    n, npts = P.shape[0], P.shape[1]
+    centers = np.zeros((nc, npts, 2), np.float32)
+    sizes = np.zeros(nc, np.int32)
+    _check(_lib3().otif_ref_track_centers(_p(P), _p(labels), n, npts, nc, _p(centers), _p(sizes)), "track_centers")
+    return centers, sizes
+
+
+def track_refine(pts: np.ndarray, offsets: np.ndarray, centers: np.ndarray, sizes: np.ndarray, k: int = 10,
+                 rho: float = 0.0):
+    """P:L200 refinement of query tracks -> (out float32 [m, 4] = start x, y, end x, y; used int32 [m])."""
+    pts, offsets, m = _tracks_in(pts, offsets)
+    centers = np.ascontiguousarray(centers, np.float32)
+    sizes = np.ascontiguousarray(sizes, np.int32)
+    nc, npts = centers.shape[0], (centers.shape[1] if centers.ndim == 3 else 20)
+    out = np.zeros((m, 4), np.float32)
+    used = np.zeros(m, np.int32)
+    _check(_lib3().otif_ref_track_refine(_p(pts), _p(offsets), m, npts, _p(centers), _p(sizes), nc, k, rho, _p(out),
+                                         _p(used)), "track_refine")
+    return out, used

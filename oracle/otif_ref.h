@@ -117,6 +117,43 @@ int otif_ref_choose_window_sizes(const uint8_t *masks, int32_t n, int32_t gh, in
  * x1, y1); windows/total as from otif_ref_select_windows.  Returns the covered count. */
 int64_t otif_ref_covered(const int32_t *boxes, int64_t nb, const otif_ref_window *windows, int32_t total);
 
+/* ------------------------------------------------------------------------- */
+/* NEXT-4: track refinement, otif_ref_tracks.c.  A track is a sequence of
+ * detection centres (x, y) (reading R20): pts float32 [total][2], offsets int64 [n+1].
+ * These functions take the integer decisions (neighbour, core, nearest) in fp32, the
+ * kernel's precision (R21–R25), and compute resampled points and centres in
+ * fp64 with a fixed operation order, so that the GPU can match them bit for bit.      */
+
+/* P:L196 "we compute N points evenly spaced along each track": arc-length resampling
+ * (reading R21).  out float32 [n][npts][2]. */
+int otif_ref_track_resample(const float *pts, const int64_t *offsets, int64_t n, int32_t npts, float *out);
+
+/* P:L196 d(s1, s2) = (1/N) Σ_i eucl(P(s1)[i], P(s2)[i]), fp32 (reading R22). */
+float otif_ref_track_distance(const float *a, const float *b, int32_t npts);
+
+/* P:L198 DBSCAN over resampled tracks P [n][npts][2] (reading R23): neighbours d <= eps
+ * (a track is its own neighbour), core iff |neighbours| >= min_pts, clusters = connected
+ * components of core tracks numbered by their smallest index, a border track joins the
+ * smallest-numbered cluster among its core neighbours, noise = -1.  labels int32 [n];
+ * core u8 [n] (may be NULL).  Returns the number of clusters. */
+int32_t otif_ref_dbscan(const float *P, int64_t n, int32_t npts, float eps, int32_t min_pts, int32_t *labels,
+                        uint8_t *core);
+
+/* P:L198 "the center of a cluster ... p_i is the average of points in {P(s)[i] | s ∈ c}":
+ * fp64 sum over members in index order, divided by the count, rounded to fp32.
+ * centers float32 [nc][npts][2], sizes int32 [nc]. */
+int otif_ref_track_centers(const float *P, const int32_t *labels, int64_t n, int32_t npts, int32_t nc,
+                           float *centers, int32_t *sizes);
+
+/* P:L200 refinement of query tracks (raw pts/offsets, m tracks): candidates = cluster
+ * centres passing within rho of the first AND the last detection (rho <= 0: all centres;
+ * reading R24); keep the k closest by (d, cluster index); start/end = per-coordinate lower
+ * weighted median of the kept centres' first/last points, weights = cluster sizes (reading
+ * R25).  out float32 [m][4] = (start x, start y, end x, end y); a track with no candidate
+ * keeps its own first/last detection.  used int32 [m] = number of clusters kept. */
+int otif_ref_track_refine(const float *pts, const int64_t *offsets, int64_t m, int32_t npts, const float *centers,
+                          const int32_t *sizes, int32_t nc, int32_t k, float rho, float *out, int32_t *used);
+
 #ifdef __cplusplus
 }
 #endif
