@@ -173,6 +173,58 @@ otif_status otif_window_recall(const int32_t *boxes, int64_t nb, const otif_wind
                                unsigned long long *covered, cudaStream_t stream);
 
 /* ---------------------------------------------------------------------------
+ * §8(f) NEXT-4 — track refinement.  "we cluster tracks in S* prior to
+ * inference, and construct a spatial index over cluster centers ... During inference,
+ * we approximate the k-nearest neighbor lookup for a computed track s".
+ * A track is a sequence of detection centres (reading R20):
+ *   pts [total][2] float32 (x, y) in pixels, device; offsets [n+1] int64, device,
+ *   track t = pts[offsets[t] .. offsets[t+1]), every track non-empty.
+ * Resampled tracks P [n][npts][2] float32 (npts = N, 2 <= N <= 32; the paper uses
+ * N = 20).  Coordinates must be finite.  Decisions (d <= eps, the k nearest)
+ * are taken in fp32 with one IEEE rounding per operation in a fixed order (readings
+ * R21–R25), so results are reproducible bit for bit.  All calls enqueue on `stream` and
+ * do not synchronise; argument errors are reported synchronously (OTIF_EINVAL). */
+
+/* P:L196 "we compute N points evenly spaced along each track": arc-length resampling,
+ * endpoints included (reading R21).  P: caller-owned device [n][npts][2]. */
+otif_status otif_track_resample(const float *pts, const int64_t *offsets, int64_t n, int32_t npts, float *P,
+                                cudaStream_t stream);
+
+/* P:L198 DBSCAN over S* with d(s1, s2) = (1/N) Σ_i eucl(P(s1)[i], P(s2)[i]):
+ * neighbours d <= eps (a track neighbours itself), core iff >= min_pts neighbours,
+ * clusters = connected components of core tracks numbered by their smallest index, a
+ * border track joins the smallest-numbered cluster among its core neighbours, noise = -1
+ * (reading R23: the classic algorithm run in index order).
+ *   labels [n] int32, core [n] u8 (may be NULL), n_clusters: device int32 — all
+ *   caller-owned device memory.  workspace >= otif_dbscan_workspace_bytes(n) (holds the
+ *   n x n neighbour bitmap, n^2/8 bytes).  n <= 2^20. */
+size_t otif_dbscan_workspace_bytes(int64_t n);
+otif_status otif_track_dbscan(const float *P, int64_t n, int32_t npts, float eps, int32_t min_pts, int32_t *labels,
+                              uint8_t *core, int32_t *n_clusters, void *workspace, size_t ws_bytes,
+                              cudaStream_t stream);
+
+/* P:L198 cluster centres: p_i = mean of {P(s)[i] | s in c}, summed in fp64 over the
+ * members in index order, divided by the count, rounded to fp32.  nc = the host value of
+ * n_clusters; labels outside [0, nc) are ignored.  centers [nc][npts][2] float32, sizes
+ * [nc] int32: caller-owned device.  workspace >= otif_centers_workspace_bytes(n, nc). */
+size_t otif_centers_workspace_bytes(int64_t n, int32_t nc);
+otif_status otif_track_centers(const float *P, const int32_t *labels, int64_t n, int32_t npts, int32_t nc,
+                               float *centers, int32_t *sizes, void *workspace, size_t ws_bytes,
+                               cudaStream_t stream);
+
+/* P:L200 refinement of m query tracks (raw pts/offsets as above): the candidate centres
+ * pass within rho pixels of the first AND of the last detection (rho <= 0: all centres;
+ * reading R24); the k closest candidates by (d, cluster index) are kept; start / end =
+ * per-coordinate lower weighted median of the kept centres' first / last points with the
+ * cluster sizes as weights (reading R25).  A track with no candidate keeps its own first
+ * and last detection.  out [m][4] float32 (start x, start y, end x, end y), used [m]
+ * int32 (clusters kept): caller-owned device.  1 <= k <= 16; the centres must fit in
+ * shared memory next to the query buffers (nc <= 1000 at N = 20, else OTIF_EUNSUPPORTED). */
+otif_status otif_track_refine(const float *pts, const int64_t *offsets, int64_t m, int32_t npts,
+                              const float *centers, const int32_t *sizes, int32_t nc, int32_t k, float rho,
+                              float *out, int32_t *used, cudaStream_t stream);
+
+/* ---------------------------------------------------------------------------
  * Whole path on HOST frames (the end-to-end call): for batches of up to max_batch
  * frames, copy src (pinned or pageable host memory) to the device, run stages 1–5,
  * and copy the windows and per-frame counts back.  Two CUDA streams overlap the

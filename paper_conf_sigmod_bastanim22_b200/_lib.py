@@ -86,6 +86,19 @@ def lib() -> ctypes.CDLL:
     L.otif_choose_window_sizes.restype = st
     L.otif_window_recall.argtypes = [P, ctypes.c_int64, P, P, P, i32, P, P]
     L.otif_window_recall.restype = st
+    i64, f32 = ctypes.c_int64, ctypes.c_float
+    L.otif_track_resample.argtypes = [P, P, i64, i32, P, P]
+    L.otif_track_resample.restype = st
+    L.otif_dbscan_workspace_bytes.argtypes = [i64]
+    L.otif_dbscan_workspace_bytes.restype = sz
+    L.otif_track_dbscan.argtypes = [P, i64, i32, f32, i32, P, P, P, P, sz, P]
+    L.otif_track_dbscan.restype = st
+    L.otif_centers_workspace_bytes.argtypes = [i64, i32]
+    L.otif_centers_workspace_bytes.restype = sz
+    L.otif_track_centers.argtypes = [P, P, i64, i32, i32, P, P, P, sz, P]
+    L.otif_track_centers.restype = st
+    L.otif_track_refine.argtypes = [P, P, i64, i32, P, P, i32, i32, f32, P, P, P]
+    L.otif_track_refine.restype = st
     if hasattr(L, "otif_pipeline_create"):
         L.otif_pipeline_create.argtypes = [ctypes.POINTER(PipelineDesc), P, sz, ctypes.POINTER(P)]
         L.otif_pipeline_create.restype = st
@@ -119,6 +132,7 @@ EXPORTED = ("otif_status_str", "otif_last_error", "otif_version", "otif_resize",
             "otif_pipeline_create", "otif_pipeline_destroy", "otif_pipeline_run_host",
             "otif_pipeline_run_device", "otif_pipeline_counters", "otif_pipeline_reset_counters",
             "otif_pipeline_set_timing", "otif_pipeline_stage_ms", "otif_choose_workspace_bytes",
-            "otif_choose_window_sizes", "otif_window_recall")
+            "otif_choose_window_sizes", "otif_window_recall", "otif_track_resample", "otif_dbscan_workspace_bytes",
+            "otif_track_dbscan", "otif_centers_workspace_bytes", "otif_track_centers", "otif_track_refine")
 STAGES = ("resize", "proxy_prep_e1", "conv_e2", "conv_e3", "conv_e4", "conv_e5", "conv_d1_head", "select",
           "pack", "append")

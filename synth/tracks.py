@@ -34,9 +34,9 @@ class TrackWorkload:
     seed: int
     n_points: int = 20    # N ("In our implementation, N = 20")
     k: int = 10           # k nearest clusters ("k = 10")
-    eps: float = 24.0     # DBSCAN radius in pixels (reading R23)
+    eps: float = 12.0     # DBSCAN radius in pixels (reading R23)
     min_pts: int = 8      # DBSCAN core threshold (reading R23)
-    rho: float = 64.0     # "pass close to d1 and dn" radius in pixels (reading R24)
+    rho: float = 32.0     # "pass close to d1 and dn" radius in pixels (reading R24)
 
 
 def _bezier(p0, p1, p2, m: int):
