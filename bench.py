@@ -303,6 +303,12 @@ def run_otif(args):
                    "pack_bytes_per_step": 2 * 3 * px}
         del masks
 
+    # §8(f) NEXT-4: track index over S* + refinement of gap-16 query tracks (C6)
+    next4 = None
+    if not args.no_next4:
+        from scripts import tracks_bench
+        next4 = tracks_bench.run(tracks_bench.tracks.C6, reps=5)
+
     # end to end through the C ABI with HOST frames: pinned H2D + D2H inside the timed region
     e2e = None
     if not args.no_e2e:
@@ -355,6 +361,7 @@ def run_otif(args):
                          "layers": per_layer},
             "stages": stages,
             "perfect_proxy": perfect,
+            "track_refinement": next4,
             "cpu_baseline": cpu_baseline,
             "e2e": e2e,
             "gpu_launches": int(launches),
@@ -382,6 +389,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-perfect", action="store_true", help="skip the perfect-proxy (ground-truth mask) line")
+    ap.add_argument("--no-next4", action="store_true", help="skip the NEXT-4 track-refinement line")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
