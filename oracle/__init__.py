@@ -25,7 +25,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "otif_ref.c")
-_SRCS = [_SRC, os.path.join(_HERE, "otif_ref_tracks.c")]
+_SRCS = [_SRC, os.path.join(_HERE, "otif_ref_tracks.c"), os.path.join(_HERE, "otif_ref_train.c")]
 
 QUANT_NONE = 0
 QUANT_BF16 = 1
@@ -342,3 +342,63 @@ def track_refine(pts: np.ndarray, offsets: np.ndarray, centers: np.ndarray, size
     _check(_lib3().otif_ref_track_refine(_p(pts), _p(offsets), m, npts, _p(centers), _p(sizes), nc, k, rho, _p(out),
                                          _p(used)), "track_refine")
     return out, used
+
+
+# --------------------------------------------------------------------------- NEXT-3
+def _lib4():
+    L = lib()
+    if not getattr(L, "_train_bound", False):
+        P, i32, i64, f64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_double
+        L.otif_ref_cell_labels.argtypes = [P, i64, i32, i32, i32, i32, i32, i32, P]
+        L.otif_ref_conv_backward.argtypes = [P, i32, i32, i32, i32, P, i32, i32, i32, P, P, P, P]
+        L.otif_ref_proxy_grad.argtypes = [P, i32, i32, i32, i32, P, i32, P, P, P, P]
+        L.otif_ref_adam.argtypes = [P, P, P, P, i64, i32, f64, f64, f64, f64]
+        L._train_bound = True
+    return L
+
+
+def cell_labels(boxes: np.ndarray, n: int, gh: int, gw: int, cell: int, frame_w: int, frame_h: int) -> np.ndarray:
+    """P:L139 training labels -> u8 [n, gh, gw]."""
+    boxes = np.ascontiguousarray(boxes, np.int32).reshape(-1, 5)
+    out = np.zeros((n, gh, gw), np.uint8)
+    _check(_lib4().otif_ref_cell_labels(_p(boxes), boxes.shape[0], n, gh, gw, cell, frame_w, frame_h, _p(out)),
+           "cell_labels")
+    return out
+
+
+def conv_backward(x: np.ndarray, weight: np.ndarray, dy: np.ndarray, stride: int, need_dx: bool = True):
+    """fp64 conv backward: x [n,h,w,cin], weight [cout,k,k,cin], dy [n,ho,wo,cout] -> (dx, dW, db)."""
+    x = np.ascontiguousarray(x, np.float64)
+    weight = np.ascontiguousarray(weight, np.float64)
+    dy = np.ascontiguousarray(dy, np.float64)
+    n, h, w, cin = x.shape
+    cout, k = weight.shape[0], weight.shape[1]
+    dx = np.zeros_like(x) if need_dx else None
+    dW = np.zeros_like(weight)
+    db = np.zeros(cout)
+    _check(_lib4().otif_ref_conv_backward(_p(x), n, h, w, cin, _p(weight), cout, k, stride, _p(dy),
+                                          _p(dx) if need_dx else None, _p(dW), _p(db)), "conv_backward")
+    return dx, dW, db
+
+
+def proxy_grad(img: np.ndarray, n_strided: int, enc, dec: int, weights: np.ndarray, labels: np.ndarray):
+    """NEXT-3 one batch -> (mean BCE loss, fp64 gradient blob)."""
+    img = np.ascontiguousarray(img, np.uint8)
+    n, h, w, _ = img.shape
+    weights = np.ascontiguousarray(weights, np.float64)
+    labels = np.ascontiguousarray(labels, np.uint8)
+    e = np.ascontiguousarray(enc, np.int32)
+    grad = np.zeros_like(weights)
+    loss = np.zeros(1)
+    _check(_lib4().otif_ref_proxy_grad(_p(img), n, h, w, n_strided, _p(e), dec, _p(weights), _p(labels), _p(loss),
+                                       _p(grad)), "proxy_grad")
+    return float(loss[0]), grad
+
+
+def adam(w: np.ndarray, m: np.ndarray, v: np.ndarray, g: np.ndarray, t: int, lr: float, b1: float = 0.9,
+         b2: float = 0.999, eps: float = 1e-8):
+    """Reading R27 Adam step, in place on fp64 arrays."""
+    for a in (w, m, v):
+        assert a.dtype == np.float64 and a.flags["C_CONTIGUOUS"]
+    g = np.ascontiguousarray(g, np.float64)
+    _check(_lib4().otif_ref_adam(_p(w), _p(m), _p(v), _p(g), w.size, t, lr, b1, b2, eps), "adam")

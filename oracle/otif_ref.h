@@ -154,6 +154,30 @@ int otif_ref_track_centers(const float *P, const int32_t *labels, int64_t n, int
 int otif_ref_track_refine(const float *pts, const int64_t *offsets, int64_t m, int32_t npts, const float *centers,
                           const int32_t *sizes, int32_t nc, int32_t k, float rho, float *out, int32_t *used);
 
+/* ------------------------------------------------------------------------- */
+/* NEXT-3: proxy training labels and training, otif_ref_train.c, fp64. */
+
+/* label 1 at a cell some detection intersects.  boxes int32 [nb][5] = (frame,
+ * x0, y0, x1, y1), half-open pixels; labels u8 [n][gh][gw]. */
+int otif_ref_cell_labels(const int32_t *boxes, int64_t nb, int32_t n, int32_t gh, int32_t gw, int32_t cell,
+                         int32_t frame_w, int32_t frame_h, uint8_t *labels);
+
+/* Backward of one convolution (pad (k−1)/2, stride 1 or 2) given dy = ∂L/∂(conv output):
+ * dx [n,h,w,cin] (may be NULL), dW [cout][k][k][cin], db [cout] — overwritten. */
+int otif_ref_conv_backward(const double *x, int32_t n, int32_t h, int32_t w, int32_t cin, const double *weight,
+                           int32_t cout, int32_t k, int32_t stride, const double *dy, double *dx, double *dW,
+                           double *db);
+
+/* One batch: forward (quant none), mean BCE-with-logits loss vs labels (reading R26),
+ * gradient of every weight and bias (fp64 blob in the proxy weight layout). */
+int otif_ref_proxy_grad(const uint8_t *img, int32_t n, int32_t in_h, int32_t in_w, int32_t n_strided,
+                        const int32_t enc[5], int32_t dec, const double *weights, const uint8_t *labels,
+                        double *loss, double *grad);
+
+/* Adam step t >= 1 (reading R27), in place on w, m, v. */
+int otif_ref_adam(double *w, double *m, double *v, const double *g, int64_t count, int32_t t, double lr, double b1,
+                  double b2, double eps);
+
 #ifdef __cplusplus
 }
 #endif
