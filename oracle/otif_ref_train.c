@@ -36,6 +36,7 @@ int otif_ref_cell_labels(const int32_t *boxes, int64_t nb, int32_t n, int32_t gh
                 for (int64_t b = 0; b < nb; b++) {
                     const int32_t *d = boxes + 5 * b;
                     if (d[0] != f) continue;
+                    if (d[1] >= d[3] || d[2] >= d[4]) continue;   /* an empty box intersects nothing */
                     if (d[1] < ax1 && ax0 < d[3] && d[2] < ay1 && ay0 < d[4]) {
                         labels[((size_t)f * gh + cy) * gw + cx] = 1;
                         break;

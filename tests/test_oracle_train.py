@@ -17,7 +17,8 @@ def test_labels_closed_forms():
     b = np.array([[0, 40, 40, 50, 50],        # inside cell (1, 1)
                   [0, 0, 0, 32, 32],          # exactly cell (0, 0): half-open, touches nothing else
                   [1, 100, 200, 170, 256],    # spans cells x 3..5, y 6..7
-                  [1, 400, 10, 416, 20]],     # clipped edge cell x = 12 (covers 384..416)
+                  [1, 400, 10, 416, 20],      # clipped edge cell x = 12 (covers 384..416)
+                  [0, 300, 100, 300, 200]],   # empty (x0 == x1): intersects nothing
                  np.int32)
     lab = oracle.cell_labels(b, 2, 8, 13, 32, 416, 256)
     assert lab.shape == (2, 8, 13)
