@@ -173,6 +173,45 @@ otif_status otif_window_recall(const int32_t *boxes, int64_t nb, const otif_wind
                                unsigned long long *covered, cudaStream_t stream);
 
 /* ---------------------------------------------------------------------------
+ * §8(f) NEXT-3 — proxy training labels and training.
+ * "at each 32 x 32 cell, the label is 1 if there is some detection d_i in D(t) that
+ * intersects the cell, and 0 otherwise"; the model "should output a score
+ * close to 1 at cells that intersect a detection, and 0 at other cells".
+ * Loss: mean binary cross-entropy of sigmoid(z) over the cells of the batch (reading
+ * R26); optimiser: Adam (reading R27).  Training arithmetic is fp32 (weights,
+ * activations, gradients); reductions run in a fixed order (deterministic). */
+
+/* Labels: boxes [nb][5] int32 (frame, x0, y0, x1, y1), half-open pixels; cell (cy, cx)
+ * covers [cx*cell, (cx+1)*cell) x [cy*cell, (cy+1)*cell) clipped to the frame (R14).
+ * labels [n][gh][gw] u8 (0/1), overwritten.  Boxes with a frame outside [0, n) or an
+ * empty clipped area are ignored. */
+otif_status otif_cell_labels(const int32_t *boxes, int64_t nb, int32_t n, int32_t gh, int32_t gw,
+                             const otif_grid_desc *g, uint8_t *labels, cudaStream_t stream);
+
+/* Adam step t >= 1 on fp32 device arrays (reading R27):
+ * m = b1 m + (1-b1) g; v = b2 v + (1-b2) g^2; w -= lr (m/(1-b1^t)) / (sqrt(v/(1-b2^t)) + eps). */
+otif_status otif_adam_step(float *w, float *m, float *v, const float *g, int64_t count, int32_t t, float lr,
+                           float b1, float b2, float eps, cudaStream_t stream);
+
+/* A trainer owns fp32 master weights (initialised from the host blob, layout as in
+ * otif_proxy_create), Adam moments, gradients and the activations of up to max_batch
+ * frames.  Any widths (enc[i] >= 1, 1 <= dec <= 256), n_strided 1..5. */
+typedef struct otif_trainer otif_trainer;
+otif_status otif_trainer_create(const otif_proxy_desc *d, const float *weights, size_t n_weights,
+                                int32_t max_batch, otif_trainer **out);
+void otif_trainer_destroy(otif_trainer *t);
+/* Device views owned by the trainer: weights [n_weights], grads [n_weights]; output grid. */
+otif_status otif_trainer_params(const otif_trainer *t, float **weights, float **grads, size_t *n_weights,
+                                int32_t *gh, int32_t *gw);
+/* Forward + loss + backward of one batch: img [n, in_h, in_w, 3] u8 (device), labels
+ * [n, gh, gw] u8 (device) -> grads (overwritten), *loss = mean BCE (device float). */
+otif_status otif_trainer_backward(otif_trainer *t, const uint8_t *img, const uint8_t *labels, int32_t n,
+                                  float *loss, cudaStream_t stream);
+/* One Adam step (b1 0.9, b2 0.999, eps 1e-8) of the master weights with the current
+ * gradients; the step counter t is kept by the trainer. */
+otif_status otif_trainer_adam(otif_trainer *t, float lr, cudaStream_t stream);
+
+/* ---------------------------------------------------------------------------
  * §8(f) NEXT-4 — track refinement.  "we cluster tracks in S* prior to
  * inference, and construct a spatial index over cluster centers ... During inference,
  * we approximate the k-nearest neighbor lookup for a computed track s".

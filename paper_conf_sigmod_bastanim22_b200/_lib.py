@@ -99,6 +99,21 @@ def lib() -> ctypes.CDLL:
     L.otif_track_centers.restype = st
     L.otif_track_refine.argtypes = [P, P, i64, i32, P, P, i32, i32, f32, P, P, P]
     L.otif_track_refine.restype = st
+    L.otif_cell_labels.argtypes = [P, i64, i32, i32, i32, ctypes.POINTER(GridDesc), P, P]
+    L.otif_cell_labels.restype = st
+    L.otif_adam_step.argtypes = [P, P, P, P, i64, i32, f32, f32, f32, f32, P]
+    L.otif_adam_step.restype = st
+    L.otif_trainer_create.argtypes = [ctypes.POINTER(ProxyDesc), P, sz, i32, ctypes.POINTER(P)]
+    L.otif_trainer_create.restype = st
+    L.otif_trainer_destroy.argtypes = [P]
+    L.otif_trainer_destroy.restype = None
+    L.otif_trainer_params.argtypes = [P, ctypes.POINTER(P), ctypes.POINTER(P), ctypes.POINTER(sz),
+                                      ctypes.POINTER(i32), ctypes.POINTER(i32)]
+    L.otif_trainer_params.restype = st
+    L.otif_trainer_backward.argtypes = [P, P, P, i32, P, P]
+    L.otif_trainer_backward.restype = st
+    L.otif_trainer_adam.argtypes = [P, f32, P]
+    L.otif_trainer_adam.restype = st
     if hasattr(L, "otif_pipeline_create"):
         L.otif_pipeline_create.argtypes = [ctypes.POINTER(PipelineDesc), P, sz, ctypes.POINTER(P)]
         L.otif_pipeline_create.restype = st
@@ -133,6 +148,8 @@ EXPORTED = ("otif_status_str", "otif_last_error", "otif_version", "otif_resize",
             "otif_pipeline_run_device", "otif_pipeline_counters", "otif_pipeline_reset_counters",
             "otif_pipeline_set_timing", "otif_pipeline_stage_ms", "otif_choose_workspace_bytes",
             "otif_choose_window_sizes", "otif_window_recall", "otif_track_resample", "otif_dbscan_workspace_bytes",
-            "otif_track_dbscan", "otif_centers_workspace_bytes", "otif_track_centers", "otif_track_refine")
+            "otif_track_dbscan", "otif_centers_workspace_bytes", "otif_track_centers", "otif_track_refine",
+            "otif_cell_labels", "otif_adam_step", "otif_trainer_create", "otif_trainer_destroy", "otif_trainer_params",
+            "otif_trainer_backward", "otif_trainer_adam")
 STAGES = ("resize", "proxy_prep_e1", "conv_e2", "conv_e3", "conv_e4", "conv_e5", "conv_d1_head", "select",
           "pack", "append")

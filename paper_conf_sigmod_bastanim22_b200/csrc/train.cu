@@ -1,0 +1,505 @@
+// train.cu — §8(f) NEXT-3, proxy training labels and training on sm_100a.
+//
+//   labels_kernel    P:L139 label 1 at every cell a detection intersects (thread per box).
+//   sgemm_kernel<Op> one fp32 SIMT implicit-GEMM template (64 x 64 x 16 tiles, 4 x 4 per
+//                    thread) instantiated for the three convolution products of training:
+//                      FwdOp    y = ReLU(conv(x, W) + b)           M = pixels, N = Cout, K = 9 Cin
+//                      DgradOp  dx = conv^T(dy, W) ⊙ [x > 0]        M = input pixels, N = Cin, K = 9 Cout
+//                      WgradOp  dW | db = dy^T · im2col(x) | Σ dy   M = Cout, N = 9 Cin + 1, K = pixels
+//                    (split-K partials for WgradOp, reduced in a fixed order: deterministic).
+//   head_kernel      D2 (1x1, dec -> 1) + sigmoid + mean BCE (reading R26) + ∂/∂z, the D1
+//                    pre-activation gradient and per-warp D2 weight-gradient partials.
+//   adam_kernel      reading R27, fp32 master weights.
+//
+// Training runs in fp32 (weights, activations, gradients); the inference path keeps its
+// bf16 tcgen05 kernels and takes the trained weights through otif_proxy_create.  This is
+// the correctness-first cut of the training path: the convolution products run on the
+// CUDA cores, not yet on tcgen05.
+#include <math.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "common.cuh"
+
+namespace otif {
+namespace {
+
+constexpr int BM = 64, BN = 64, BK = 16, GT = 256;
+
+// ---- labels ----------------------------------------------------------------------------
+__global__ void labels_kernel(const int32_t *__restrict__ boxes, int64_t nb, int n, int gh, int gw, int cell,
+                              int frame_w, int frame_h, uint8_t *__restrict__ labels) {
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < nb; b += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t *d = boxes + 5 * b;
+        const int f = d[0];
+        if (f < 0 || f >= n) continue;
+        const int x0 = max(d[1], 0), y0 = max(d[2], 0), x1 = min(d[3], frame_w), y1 = min(d[4], frame_h);
+        if (x0 >= x1 || y0 >= y1) continue;
+        // cells [cx*cell, (cx+1)*cell) overlapping [x0, x1): cx in [x0/cell, (x1-1)/cell]
+        for (int cy = y0 / cell; cy <= (y1 - 1) / cell && cy < gh; cy++)
+            for (int cx = x0 / cell; cx <= (x1 - 1) / cell && cx < gw; cx++)
+                labels[((int64_t)f * gh + cy) * gw + cx] = 1;
+    }
+}
+
+// ---- generic SIMT GEMM -------------------------------------------------------------------
+// Op supplies: a(m, k), b(k, n) (0 outside), store(m, n, value, split), and the layout flags
+// A_KFAST / B_KFAST (true when consecutive k are contiguous in memory: the tile loaders
+// then walk k fastest, otherwise m / n fastest) for coalesced loads.
+template <class Op>
+__global__ void __launch_bounds__(GT) sgemm_kernel(Op op, int M, int N, int K, int k_split) {
+    __shared__ float As[BK][BM + 4];
+    __shared__ float Bs[BK][BN + 4];
+    const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+    const int m0 = blockIdx.x * BM, n0 = blockIdx.y * BN;
+    const int kb = blockIdx.z * k_split, ke = min(K, kb + k_split);
+    float acc[4][4] = {};
+    for (int k0 = kb; k0 < ke; k0 += BK) {
+#pragma unroll
+        for (int i = 0; i < 4; i++) {
+            const int e = tid + GT * i;
+            const int kk = Op::A_KFAST ? (e & (BK - 1)) : (e / BM);
+            const int mm = Op::A_KFAST ? (e / BK) : (e & (BM - 1));
+            const int m = m0 + mm, k = k0 + kk;
+            As[kk][mm] = (m < M && k < ke) ? op.a(m, k) : 0.f;
+        }
+#pragma unroll
+        for (int i = 0; i < 4; i++) {
+            const int e = tid + GT * i;
+            const int kk = Op::B_KFAST ? (e & (BK - 1)) : (e / BN);
+            const int nn = Op::B_KFAST ? (e / BK) : (e & (BN - 1));
+            const int n = n0 + nn, k = k0 + kk;
+            Bs[kk][nn] = (n < N && k < ke) ? op.b(k, n) : 0.f;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int kk = 0; kk < BK; kk++) {
+            float a[4], b[4];
+#pragma unroll
+            for (int i = 0; i < 4; i++) a[i] = As[kk][ty + 16 * i];
+#pragma unroll
+            for (int j = 0; j < 4; j++) b[j] = Bs[kk][tx + 16 * j];
+#pragma unroll
+            for (int i = 0; i < 4; i++)
+#pragma unroll
+                for (int j = 0; j < 4; j++) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        }
+        __syncthreads();
+    }
+#pragma unroll
+    for (int i = 0; i < 4; i++)
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            const int m = m0 + ty + 16 * i, n = n0 + tx + 16 * j;
+            if (m < M && n < N) op.store(m, n, acc[i][j], blockIdx.z);
+        }
+}
+
+struct ConvGeom {
+    int H, W, Cin, Ho, Wo, Cout, k, stride, pad;
+};
+
+template <typename T>
+__device__ __forceinline__ float act_in(const T *x, int64_t idx);
+template <>
+__device__ __forceinline__ float act_in<float>(const float *x, int64_t idx) { return x[idx]; }
+template <>
+__device__ __forceinline__ float act_in<uint8_t>(const uint8_t *x, int64_t idx) {
+    return ((float)x[idx] - 128.f) * (1.f / 128.f);           // (u - 128) / 128, exact in fp32
+}
+
+// y[m = (f, oy, ox), co] = ReLU(Σ_k im2col(x)[m, k] W[co, k] + b[co]),  k = (kh, kw, ci)
+template <typename T>
+struct FwdOp {
+    static constexpr bool A_KFAST = true, B_KFAST = true;
+    const T *x;
+    const float *w, *bias;
+    float *y;
+    ConvGeom g;
+    int relu;
+    __device__ float a(int m, int k) const {
+        const int hw = g.Ho * g.Wo, f = m / hw, r = m - f * hw, oy = r / g.Wo, ox = r - oy * g.Wo;
+        const int tap = k / g.Cin, ci = k - tap * g.Cin, kh = tap / g.k, kw = tap - kh * g.k;
+        const int iy = oy * g.stride - g.pad + kh, ix = ox * g.stride - g.pad + kw;
+        if (iy < 0 || iy >= g.H || ix < 0 || ix >= g.W) return 0.f;
+        return act_in<T>(x, (((int64_t)f * g.H + iy) * g.W + ix) * g.Cin + ci);
+    }
+    __device__ float b(int k, int n) const { return w[(int64_t)n * (g.k * g.k * g.Cin) + k]; }
+    __device__ void store(int m, int n, float v, int) const {
+        v += bias[n];
+        y[(int64_t)m * g.Cout + n] = relu ? fmaxf(v, 0.f) : v;
+    }
+};
+
+// dx[m = (f, iy, ix), ci] = Σ_{kh, kw, co} dy[f, oy, ox, co] W[co, kh, kw, ci] where
+// iy = oy*s - pad + kh, then ⊙ [x_post > 0] (the ReLU of the layer below): the result is
+// that layer's pre-activation gradient.  k = (kh, kw, co).
+struct DgradOp {
+    static constexpr bool A_KFAST = true, B_KFAST = false;
+    const float *dy, *w, *xpost;
+    float *dx;
+    ConvGeom g;
+    __device__ float a(int m, int k) const {
+        const int hw = g.H * g.W, f = m / hw, r = m - f * hw, iy = r / g.W, ix = r - iy * g.W;
+        const int tap = k / g.Cout, co = k - tap * g.Cout, kh = tap / g.k, kw = tap - kh * g.k;
+        const int ty = iy + g.pad - kh, tx = ix + g.pad - kw;
+        if (ty < 0 || tx < 0) return 0.f;
+        const int oy = ty / g.stride, ox = tx / g.stride;
+        if (oy * g.stride != ty || ox * g.stride != tx || oy >= g.Ho || ox >= g.Wo) return 0.f;
+        return dy[(((int64_t)f * g.Ho + oy) * g.Wo + ox) * g.Cout + co];
+    }
+    __device__ float b(int k, int n) const {
+        const int tap = k / g.Cout, co = k - tap * g.Cout;
+        return w[((int64_t)co * g.k * g.k + tap) * g.Cin + n];
+    }
+    __device__ void store(int m, int n, float v, int) const {
+        const int64_t i = (int64_t)m * g.Cin + n;
+        dx[i] = xpost[i] > 0.f ? v : 0.f;
+    }
+};
+
+// [dW | db][co, kk] = Σ_p dy[p, co] · (kk < K ? im2col(x)[p, kk] : 1), split over p.
+template <typename T>
+struct WgradOp {
+    static constexpr bool A_KFAST = false, B_KFAST = false;
+    const float *dy;
+    const T *x;
+    float *part;        // [split][Cout][K + 1]
+    ConvGeom g;
+    int Kw;             // k*k*Cin
+    __device__ float a(int m, int p) const { return dy[(int64_t)p * g.Cout + m]; }
+    __device__ float b(int p, int kk) const {
+        if (kk == Kw) return 1.f;
+        const int hw = g.Ho * g.Wo, f = p / hw, r = p - f * hw, oy = r / g.Wo, ox = r - oy * g.Wo;
+        const int tap = kk / g.Cin, ci = kk - tap * g.Cin, kh = tap / g.k, kw = tap - kh * g.k;
+        const int iy = oy * g.stride - g.pad + kh, ix = ox * g.stride - g.pad + kw;
+        if (iy < 0 || iy >= g.H || ix < 0 || ix >= g.W) return 0.f;
+        return act_in<T>(x, (((int64_t)f * g.H + iy) * g.W + ix) * g.Cin + ci);
+    }
+    __device__ void store(int m, int n, float v, int split) const {
+        part[((int64_t)split * g.Cout + m) * (Kw + 1) + n] = v;
+    }
+};
+
+// fixed-order sum of the split partials into the blob: W[co][kk] then b[co]
+__global__ void wgrad_reduce_kernel(const float *__restrict__ part, int splits, int cout, int kw,
+                                    float *__restrict__ grad) {
+    const int64_t total = (int64_t)cout * (kw + 1);
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+        float s = 0.f;
+        for (int sp = 0; sp < splits; sp++) s += part[(int64_t)sp * total + e];
+        const int co = (int)(e / (kw + 1)), kk = (int)(e - (int64_t)co * (kw + 1));
+        if (kk < kw)
+            grad[(int64_t)co * kw + kk] = s;
+        else
+            grad[(int64_t)cout * kw + co] = s;
+    }
+}
+
+// D2 + sigmoid + BCE (reading R26), warp per cell (grid-stride, fixed assignment):
+// z = b2 + Σ_c a[c] w2[c]; loss += softplus(z) - y z; dz = (sigmoid(z) - y) / M;
+// d_pre[c] = dz w2[c] [a[c] > 0]; per-warp partials of Σ dz a[c] (dW2), Σ dz (db2), loss.
+constexpr int kHeadWarps = 8;
+__global__ void __launch_bounds__(kHeadWarps * 32) head_kernel(const float *__restrict__ act, const float *__restrict__ w2,
+                                                               const uint8_t *__restrict__ labels, int64_t M, int dec,
+                                                               float *__restrict__ dpre, float *__restrict__ part) {
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const float b2 = w2[dec];
+    float dws[8] = {0, 0, 0, 0, 0, 0, 0, 0};      // channels lane + 32 i, dec <= 256
+    float dbs = 0.f, ls = 0.f;
+    const float invM = 1.f / (float)M;
+    for (int64_t cidx = gw; cidx < M; cidx += nw) {
+        const float *a = act + cidx * dec;
+        float z = 0.f;
+        for (int c = lane; c < dec; c += 32) z = fmaf(a[c], w2[c], z);
+        for (int s = 16; s > 0; s >>= 1) z += __shfl_xor_sync(0xffffffffu, z, s);
+        z += b2;
+        const float y = labels[cidx] ? 1.f : 0.f;
+        const float sp = z > 0.f ? z + log1pf(expf(-z)) : log1pf(expf(z));
+        const float dz = (1.f / (1.f + expf(-z)) - y) * invM;
+        ls += sp - y * z;
+        dbs += dz;
+#pragma unroll
+        for (int i = 0; i < 8; i++) {
+            const int c = lane + 32 * i;
+            if (c < dec) {
+                const float av = a[c];
+                dws[i] = fmaf(dz, av, dws[i]);
+                dpre[cidx * dec + c] = av > 0.f ? dz * w2[c] : 0.f;
+            }
+        }
+    }
+    float *o = part + gw * (dec + 2);
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+        const int c = lane + 32 * i;
+        if (c < dec) o[c] = dws[i];
+    }
+    if (lane == 0) {
+        o[dec] = dbs;
+        o[dec + 1] = ls;
+    }
+}
+
+// fixed-order reduction of the head partials -> grad (W2, b2) and the mean loss
+__global__ void head_reduce_kernel(const float *__restrict__ part, int64_t nwarps, int dec, int64_t M,
+                                   float *__restrict__ grad_w2, float *__restrict__ loss) {
+    for (int c = threadIdx.x; c < dec + 2; c += blockDim.x) {
+        float s = 0.f;
+        for (int64_t w = 0; w < nwarps; w++) s += part[w * (dec + 2) + c];
+        if (c <= dec)
+            grad_w2[c] = s;                       // W2[0..dec-1], then b2
+        else
+            *loss = s / (float)M;
+    }
+}
+
+__global__ void adam_kernel(float *__restrict__ w, float *__restrict__ m, float *__restrict__ v,
+                            const float *__restrict__ g, int64_t count, float lr, float b1, float b2, float eps,
+                            float c1, float c2) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x) {
+        const float gi = g[i];
+        const float mi = b1 * m[i] + (1.f - b1) * gi;
+        const float vi = b2 * v[i] + (1.f - b2) * gi * gi;
+        m[i] = mi;
+        v[i] = vi;
+        w[i] -= lr * (mi / c1) / (sqrtf(vi / c2) + eps);
+    }
+}
+
+template <class Op>
+otif_status run_gemm(const Op &op, int64_t M, int64_t N, int64_t K, int splits, cudaStream_t stream) {
+    if (M <= 0 || N <= 0) return OTIF_OK;
+    const int64_t k_split = round_up(cdiv(K, splits), BK);
+    const dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)splits);
+    sgemm_kernel<Op><<<grid, GT, 0, stream>>>(op, (int)M, (int)N, (int)K, (int)k_split);
+    OTIF_LAUNCH_CHECK();
+    return OTIF_OK;
+}
+
+}  // namespace
+}  // namespace otif
+
+using namespace otif;
+
+struct otif_trainer {
+    otif_proxy_desc d;
+    int max_batch = 0;
+    int sms = 0;
+    int cin[7], cout[7], ks[7], stride[7], hs[8], ws[8];
+    size_t woff[7];
+    size_t n_weights = 0;
+    float *w = nullptr, *m = nullptr, *v = nullptr, *grad = nullptr;
+    float *act[8] = {};          // act[1..6] fp32 NHWC post-ReLU; act[0] is the caller's u8 image
+    float *dbuf[2] = {};         // pre-activation gradients, ping-pong
+    float *part = nullptr;       // split-K / head partials
+    size_t part_floats = 0;
+    int64_t head_warps = 0;
+    int step = 0;
+};
+
+static int wgrad_splits(const otif_trainer *t, int L, int n) {
+    const int64_t pixels = (int64_t)n * t->hs[L + 1] * t->ws[L + 1];
+    const int64_t tiles = cdiv(t->cout[L], BM) * cdiv((int64_t)t->ks[L] * t->ks[L] * t->cin[L] + 1, BN);
+    int64_t s = cdiv(2 * (int64_t)t->sms, tiles);
+    s = std::min<int64_t>(s, std::max<int64_t>(1, pixels / 256));
+    return (int)std::max<int64_t>(1, std::min<int64_t>(s, 512));
+}
+
+extern "C" otif_status otif_cell_labels(const int32_t *boxes, int64_t nb, int32_t n, int32_t gh, int32_t gw,
+                                        const otif_grid_desc *g, uint8_t *labels, cudaStream_t stream) {
+    OTIF_REQUIRE(g && labels && (boxes || nb == 0), "otif_cell_labels: NULL argument");
+    OTIF_REQUIRE(n >= 0 && gh > 0 && gw > 0 && nb >= 0 && g->cell > 0 && g->frame_w > 0 && g->frame_h > 0,
+                 "otif_cell_labels: bad sizes");
+    otif_status st = check_device(nullptr);
+    if (st != OTIF_OK) return st;
+    if (n == 0) return OTIF_OK;
+    OTIF_CUDA(cudaMemsetAsync(labels, 0, (size_t)n * gh * gw, stream));
+    if (nb == 0) return OTIF_OK;
+    labels_kernel<<<(unsigned)std::min<int64_t>(cdiv(nb, 256), 4096), 256, 0, stream>>>(
+        boxes, nb, n, gh, gw, g->cell, g->frame_w, g->frame_h, labels);
+    OTIF_LAUNCH_CHECK();
+    return OTIF_OK;
+}
+
+extern "C" otif_status otif_adam_step(float *w, float *m, float *v, const float *g, int64_t count, int32_t t, float lr,
+                                      float b1, float b2, float eps, cudaStream_t stream) {
+    OTIF_REQUIRE(count >= 0 && t >= 1, "otif_adam_step: count=%lld t=%d", (long long)count, t);
+    if (count == 0) return OTIF_OK;
+    OTIF_REQUIRE(w && m && v && g, "otif_adam_step: NULL argument");
+    int sms = 0;
+    otif_status st = check_device(&sms);
+    if (st != OTIF_OK) return st;
+    const float c1 = (float)(1.0 - pow((double)b1, (double)t)), c2 = (float)(1.0 - pow((double)b2, (double)t));
+    adam_kernel<<<(unsigned)std::min<int64_t>(cdiv(count, 256), (int64_t)sms * 8), 256, 0, stream>>>(
+        w, m, v, g, count, lr, b1, b2, eps, c1, c2);
+    OTIF_LAUNCH_CHECK();
+    return OTIF_OK;
+}
+
+extern "C" otif_status otif_trainer_create(const otif_proxy_desc *d, const float *weights, size_t n_weights,
+                                           int32_t max_batch, otif_trainer **out) {
+    OTIF_REQUIRE(d && weights && out, "otif_trainer_create: NULL argument");
+    OTIF_REQUIRE(d->in_h > 0 && d->in_w > 0 && d->n_strided >= 1 && d->n_strided <= 5 && max_batch >= 1,
+                 "otif_trainer_create: in %dx%d n_strided %d max_batch %d", d->in_h, d->in_w, d->n_strided, max_batch);
+    for (int i = 0; i < 5; i++) OTIF_REQUIRE(d->enc[i] > 0, "otif_trainer_create: enc[%d]=%d", i, d->enc[i]);
+    OTIF_REQUIRE(d->dec > 0 && d->dec <= 256, "otif_trainer_create: dec=%d (1..256)", d->dec);
+    int sms = 0;
+    otif_status st = check_device(&sms);
+    if (st != OTIF_OK) return st;
+    otif_trainer *t = new otif_trainer();
+    t->d = *d;
+    t->max_batch = max_batch;
+    t->sms = sms;
+    int c = 3;
+    for (int L = 0; L < 7; L++) {
+        t->cin[L] = c;
+        t->cout[L] = L < 5 ? d->enc[L] : (L == 5 ? d->dec : 1);
+        t->ks[L] = L == 6 ? 1 : 3;
+        t->stride[L] = (L < 5 && L < d->n_strided) ? 2 : 1;
+        c = t->cout[L];
+    }
+    t->hs[0] = d->in_h;
+    t->ws[0] = d->in_w;
+    size_t off = 0, max_act = 0;
+    for (int L = 0; L < 7; L++) {
+        t->hs[L + 1] = (t->hs[L] + t->stride[L] - 1) / t->stride[L];
+        t->ws[L + 1] = (t->ws[L] + t->stride[L] - 1) / t->stride[L];
+        t->woff[L] = off;
+        off += (size_t)t->cout[L] * t->ks[L] * t->ks[L] * t->cin[L] + t->cout[L];
+        if (L < 6) max_act = std::max(max_act, (size_t)max_batch * t->hs[L + 1] * t->ws[L + 1] * t->cout[L]);
+    }
+    t->n_weights = off;
+    if (n_weights != off) {
+        delete t;
+        set_error("otif_trainer_create: n_weights %zu != %zu", n_weights, off);
+        return OTIF_EINVAL;
+    }
+    // partial buffers: max over layers of splits * Cout * (K + 1), and the head partials
+    size_t part = 0;
+    for (int L = 0; L < 6; L++) {
+        const size_t kw = (size_t)t->ks[L] * t->ks[L] * t->cin[L];
+        part = std::max(part, (size_t)wgrad_splits(t, L, max_batch) * t->cout[L] * (kw + 1));
+    }
+    t->head_warps = (int64_t)sms * 4 * kHeadWarps;
+    part = std::max(part, (size_t)t->head_warps * (t->d.dec + 2));
+    t->part_floats = part;
+    bool ok = cudaMalloc(&t->w, off * 4) == cudaSuccess && cudaMalloc(&t->m, off * 4) == cudaSuccess &&
+              cudaMalloc(&t->v, off * 4) == cudaSuccess && cudaMalloc(&t->grad, off * 4) == cudaSuccess &&
+              cudaMalloc(&t->part, part * 4) == cudaSuccess && cudaMalloc(&t->dbuf[0], max_act * 4) == cudaSuccess &&
+              cudaMalloc(&t->dbuf[1], max_act * 4) == cudaSuccess;
+    for (int L = 1; L <= 6 && ok; L++)
+        ok = cudaMalloc(&t->act[L], (size_t)max_batch * t->hs[L] * t->ws[L] * t->cout[L - 1] * 4) == cudaSuccess;
+    if (!ok) {
+        otif_trainer_destroy(t);
+        set_error("otif_trainer_create: device allocation failed");
+        return OTIF_ENOMEM;
+    }
+    if (cudaMemcpy(t->w, weights, off * 4, cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemset(t->m, 0, off * 4) != cudaSuccess || cudaMemset(t->v, 0, off * 4) != cudaSuccess ||
+        cudaMemset(t->grad, 0, off * 4) != cudaSuccess) {
+        otif_trainer_destroy(t);
+        set_error("otif_trainer_create: upload failed");
+        return OTIF_ECUDA;
+    }
+    *out = t;
+    return OTIF_OK;
+}
+
+extern "C" void otif_trainer_destroy(otif_trainer *t) {
+    if (!t) return;
+    cudaFree(t->w);
+    cudaFree(t->m);
+    cudaFree(t->v);
+    cudaFree(t->grad);
+    cudaFree(t->part);
+    for (int i = 0; i < 2; i++) cudaFree(t->dbuf[i]);
+    for (int L = 1; L <= 6; L++) cudaFree(t->act[L]);
+    delete t;
+}
+
+extern "C" otif_status otif_trainer_params(const otif_trainer *t, float **weights, float **grads, size_t *n_weights,
+                                           int32_t *gh, int32_t *gw) {
+    OTIF_REQUIRE(t, "otif_trainer_params: NULL trainer");
+    if (weights) *weights = t->w;
+    if (grads) *grads = t->grad;
+    if (n_weights) *n_weights = t->n_weights;
+    if (gh) *gh = t->hs[7];
+    if (gw) *gw = t->ws[7];
+    return OTIF_OK;
+}
+
+extern "C" otif_status otif_trainer_backward(otif_trainer *t, const uint8_t *img, const uint8_t *labels, int32_t n,
+                                             float *loss, cudaStream_t stream) {
+    OTIF_REQUIRE(t && img && labels && loss, "otif_trainer_backward: NULL argument");
+    OTIF_REQUIRE(n >= 1 && n <= t->max_batch, "otif_trainer_backward: n=%d (1..%d)", n, t->max_batch);
+    otif_status st = check_device(nullptr);
+    if (st != OTIF_OK) return st;
+    auto geom = [&](int L) {
+        ConvGeom g;
+        g.H = t->hs[L]; g.W = t->ws[L]; g.Cin = t->cin[L]; g.Ho = t->hs[L + 1]; g.Wo = t->ws[L + 1];
+        g.Cout = t->cout[L]; g.k = t->ks[L]; g.stride = t->stride[L]; g.pad = (t->ks[L] - 1) / 2;
+        return g;
+    };
+    // forward E1..D1 (D2 lives in the head kernel)
+    for (int L = 0; L < 6; L++) {
+        const ConvGeom g = geom(L);
+        const float *wl = t->w + t->woff[L];
+        const float *bl = wl + (size_t)g.Cout * g.k * g.k * g.Cin;
+        const int64_t M = (int64_t)n * g.Ho * g.Wo, K = (int64_t)g.k * g.k * g.Cin;
+        if (L == 0) {
+            FwdOp<uint8_t> op{img, wl, bl, t->act[1], g, 1};
+            st = run_gemm(op, M, g.Cout, K, 1, stream);
+        } else {
+            FwdOp<float> op{t->act[L], wl, bl, t->act[L + 1], g, 1};
+            st = run_gemm(op, M, g.Cout, K, 1, stream);
+        }
+        if (st != OTIF_OK) return st;
+    }
+    // head: loss, D2 gradient, D1 pre-activation gradient
+    const int dec = t->cout[5];
+    const int64_t cells = (int64_t)n * t->hs[7] * t->ws[7];
+    head_kernel<<<(unsigned)(t->head_warps / kHeadWarps), kHeadWarps * 32, 0, stream>>>(
+        t->act[6], t->w + t->woff[6], labels, cells, dec, t->dbuf[0], t->part);
+    OTIF_LAUNCH_CHECK();
+    head_reduce_kernel<<<1, 256, 0, stream>>>(t->part, t->head_warps, dec, cells, t->grad + t->woff[6], loss);
+    OTIF_LAUNCH_CHECK();
+    // backward D1 .. E1
+    int cur = 0;
+    for (int L = 5; L >= 0; L--) {
+        const ConvGeom g = geom(L);
+        const int kw = g.k * g.k * g.Cin;
+        const int64_t P = (int64_t)n * g.Ho * g.Wo;
+        const int splits = wgrad_splits(t, L, n);
+        if (L == 0) {
+            WgradOp<uint8_t> op{t->dbuf[cur], img, t->part, g, kw};
+            st = run_gemm(op, g.Cout, kw + 1, P, splits, stream);
+        } else {
+            WgradOp<float> op{t->dbuf[cur], t->act[L], t->part, g, kw};
+            st = run_gemm(op, g.Cout, kw + 1, P, splits, stream);
+        }
+        if (st != OTIF_OK) return st;
+        wgrad_reduce_kernel<<<(unsigned)std::min<int64_t>(cdiv((int64_t)g.Cout * (kw + 1), 256), 4096), 256, 0,
+                              stream>>>(t->part, splits, g.Cout, kw, t->grad + t->woff[L]);
+        OTIF_LAUNCH_CHECK();
+        if (L > 0) {
+            DgradOp op{t->dbuf[cur], t->w + t->woff[L], t->act[L], t->dbuf[cur ^ 1], g};
+            st = run_gemm(op, (int64_t)n * g.H * g.W, g.Cin, (int64_t)g.k * g.k * g.Cout, 1, stream);
+            if (st != OTIF_OK) return st;
+            cur ^= 1;
+        }
+    }
+    return OTIF_OK;
+}
+
+extern "C" otif_status otif_trainer_adam(otif_trainer *t, float lr, cudaStream_t stream) {
+    OTIF_REQUIRE(t, "otif_trainer_adam: NULL trainer");
+    t->step++;
+    return otif_adam_step(t->w, t->m, t->v, t->grad, (int64_t)t->n_weights, t->step, lr, 0.9f, 0.999f, 1e-8f,
+                          stream);
+}
