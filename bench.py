@@ -309,6 +309,35 @@ def run_otif(args):
         from scripts import tracks_bench
         next4 = tracks_bench.run(tracks_bench.tracks.C6, reps=5)
 
+    # §8(f) NEXT-3: proxy training steps (fp32 forward + backward + Adam) on
+    # 32 of this rank's C2 frames with ground-truth cell labels, timed with CUDA events
+    next3 = None
+    if not args.no_next3:
+        from paper_conf_sigmod_bastanim22_b200 import train as otif_train
+        sc = video.make_scene(wl, clip=rank)
+        tsel = [t for t in range(0, n, max(n // 64, 1)) if sc.gt_boxes(t)][:32]
+        bx = np.array([(i, *b) for i, t in enumerate(tsel) for b in sc.gt_boxes(t) if b[0] < b[2] and b[1] < b[3]],
+                      np.int32).reshape(-1, 5)
+        gh, gw = -(-wl.src_h // wl.cell), -(-wl.src_w // wl.cell)
+        lab = otif_train.otif_cell_labels(torch.from_numpy(bx).to(dev), len(tsel), (gh, gw), wl.src_w, wl.src_h,
+                                          wl.cell)
+        timg = otif.otif_resize(src[torch.tensor(tsel, device=dev)], wl.proxy_h, wl.proxy_w)
+        tr = otif_train.Trainer(wl.proxy_h, wl.proxy_w, wl.n_strided, weights.proxy_weights(), max_batch=len(tsel))
+        l0 = float(tr.step(timg, lab, 1e-3).item())
+        torch.cuda.synchronize()
+        t0e, t1e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0e.record()
+        for _ in range(args.steps):
+            lt = tr.step(timg, lab, 1e-3)
+        t1e.record()
+        torch.cuda.synchronize()
+        tms = t0e.elapsed_time(t1e) / args.steps
+        train_flop = 3 * 2 * (sum(macs) + head) * len(tsel)      # forward + dgrad + wgrad
+        next3 = {"what": "fp32 training step (forward, BCE head, dgrad, wgrad, Adam) on CUDA cores",
+                 "batch": len(tsel), "ms_per_step": tms, "train_frames_per_s": len(tsel) / (tms / 1e3),
+                 "tflops": train_flop / (tms / 1e3) / 1e12, "loss_first": l0, "loss_last": float(lt.item())}
+        del tr, timg, lab
+
     # end to end through the C ABI with HOST frames: pinned H2D + D2H inside the timed region
     e2e = None
     if not args.no_e2e:
@@ -362,6 +391,7 @@ def run_otif(args):
             "stages": stages,
             "perfect_proxy": perfect,
             "track_refinement": next4,
+            "proxy_training": next3,
             "cpu_baseline": cpu_baseline,
             "e2e": e2e,
             "gpu_launches": int(launches),
@@ -390,6 +420,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-perfect", action="store_true", help="skip the perfect-proxy (ground-truth mask) line")
     ap.add_argument("--no-next4", action="store_true", help="skip the NEXT-4 track-refinement line")
+    ap.add_argument("--no-next3", action="store_true", help="skip the NEXT-3 proxy-training line")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
