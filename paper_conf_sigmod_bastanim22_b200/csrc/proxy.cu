@@ -225,7 +225,13 @@ __global__ void __launch_bounds__(128) e1_umma_kernel(const __grid_constant__ E1
 // ---------------------------------------------------------------------------
 // E2..E5, D1: persistent warp-specialised implicit-GEMM conv on tcgen05
 // ---------------------------------------------------------------------------
-template <int MT>
+// SWAP (head layer, N = 128, MT = 2): the operands trade places — the weights are the
+// M = 128 operand and the 256 halo rows the N = 256 operand — so one M128 x N256 MMA
+// reads 12 KB of shared memory per 1 MFLOP instead of two M128 x N128 MMAs reading 16 KB
+// (N = 128 layers are shared-memory-bandwidth bound).  The accumulator is transposed
+// (TMEM lane = output channel, column = pixel); the head epilogue reduces the D2 dot
+// product across lanes (reduce-scatter shuffles) and across the 4 epilogue warps.
+template <int MT, bool SWAP = false>
 __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     const int warp = threadIdx.x >> 5;
@@ -246,6 +252,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(t_empty + 2);
     float *s_bias = reinterpret_cast<float *>(tmem_slot + 4);
     float *s_w2 = s_bias + 256;
+    float *s_red = s_w2 + 256;               // SWAP head: [4 warps][256 pixels] partial dots
 
     const uint32_t acc_cols = 2 * MT * p.N;  // two accumulator stages of MT sub-tiles x N columns
     const uint32_t tmem_cols = acc_cols <= 32 ? 32 : (acc_cols <= 64 ? 64 : (acc_cols <= 128 ? 128 : (acc_cols <= 256 ? 256 : 512)));
@@ -300,7 +307,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
     } else if (warp == 1) {
         // ===== MMA issuer (single thread) =====
         if (lane == 0) {
-            const uint32_t idesc = umma_idesc_bf16(kTileM, p.N);
+            const uint32_t idesc = SWAP ? umma_idesc_bf16(kTileM, kTileM * MT) : umma_idesc_bf16(kTileM, p.N);
             uint32_t as = 0, ap = 0, bs = 0, bp = 0, acc = 0, accp = 0;
             const uint32_t a_base = smem_u32(a_buf), b_base = smem_u32(b_buf);
             const uint32_t lbo_a = p.P * 16, lbo_b = p.N * 16;
@@ -321,11 +328,17 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                             const uint32_t b_stage = b_base + bs * b_bytes;
                             for (uint32_t s = 0; s < chunks / 2; s++) {
                                 const uint64_t bd = umma_desc(b_stage + 2 * s * lbo_b, lbo_b, 128);
-                                // the mt sub-tiles share this B stage: rows 128*m.. of the halo
+                                if (SWAP) {
+                                    // weights = M operand, the 128*MT halo rows = N operand
+                                    const uint64_t hd = umma_desc(a_tap + 2 * s * lbo_a, lbo_a, 128);
+                                    umma_bf16(d, bd, hd, idesc, accumulate);
+                                } else {
+                                    // the mt sub-tiles share this B stage: rows 128*m.. of the halo
 #pragma unroll
-                                for (int m = 0; m < MT; m++) {
-                                    uint64_t ad = umma_desc(a_tap + 2 * s * lbo_a + m * (kTileM * 16), lbo_a, 128);
-                                    umma_bf16(d + m * p.N, ad, bd, idesc, accumulate);
+                                    for (int m = 0; m < MT; m++) {
+                                        uint64_t ad = umma_desc(a_tap + 2 * s * lbo_a + m * (kTileM * 16), lbo_a, 128);
+                                        umma_bf16(d + m * p.N, ad, bd, idesc, accumulate);
+                                    }
                                 }
                                 accumulate = 1;
                             }
@@ -339,6 +352,58 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                 umma_commit(&t_full[acc]);
                 if (++acc == 2) { acc = 0; accp ^= 1; }
             }
+        }
+    } else if (SWAP && warp >= 4) {
+        // ===== head epilogue, transposed accumulator: lane = D1 channel, column = pixel =====
+        const int quarter = warp & 3;
+        const int ch = quarter * 32 + lane;
+        const float bias_c = s_bias[ch], w2_c = s_w2[ch];
+        const int r = threadIdx.x - 128;
+        uint32_t acc = 0, accp = 0;
+        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+            mbar_wait(&t_full[acc], accp);
+            tc_fence_after();
+            const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * (kTileM * MT);
+            for (int cc = 0; cc < kTileM * MT / 32; cc++) {
+                uint32_t v[32];
+                tmem_ld32(taddr + cc * 32, v);
+                float t[32];
+#pragma unroll
+                for (int j = 0; j < 32; j += 2) {
+                    const uint32_t pk = pack_bf16x2(fmaxf(__uint_as_float(v[j]) + bias_c, 0.0f),
+                                                    fmaxf(__uint_as_float(v[j + 1]) + bias_c, 0.0f));
+                    t[j] = w2_c * __uint_as_float(pk << 16);
+                    t[j + 1] = w2_c * __uint_as_float(pk & 0xFFFF0000u);
+                }
+                // reduce-scatter over the 32 channels of this warp: lane l ends with pixel l
+#pragma unroll
+                for (int sft = 16; sft >= 1; sft >>= 1) {
+                    const bool up = (lane & sft) != 0;
+#pragma unroll
+                    for (int j = 0; j < sft; j++) {
+                        const float send = up ? t[j] : t[j + sft];
+                        const float keep = up ? t[j + sft] : t[j];
+                        t[j] = keep + __shfl_xor_sync(0xffffffffu, send, sft);
+                    }
+                }
+                s_red[quarter * (kTileM * MT) + cc * 32 + lane] = t[0];
+            }
+            tc_fence_before();
+            mbar_arrive(&t_empty[acc]);
+            asm volatile("bar.sync 1, 128;" ::: "memory");
+            for (int px = r; px < kTileM * MT; px += 128) {
+                const float z = p.b2 + ((s_red[px] + s_red[kTileM * MT + px]) +
+                                        (s_red[2 * kTileM * MT + px] + s_red[3 * kTileM * MT + px]));
+                const int64_t q = (int64_t)tile * kTileM * MT + px;
+                const int f = (int)(q / p.fstride);
+                const int64_t rr = q - (int64_t)f * p.fstride;
+                const int oy = (int)(rr / p.pitch);
+                const int ox = (int)(rr - (int64_t)oy * p.pitch);
+                if (q < p.mtot && oy < p.out_h && ox < p.out_w)
+                    p.scores[((int64_t)f * p.out_h + oy) * p.out_w + ox] = 1.0f / (1.0f + expf(-z));
+            }
+            asm volatile("bar.sync 1, 128;" ::: "memory");
+            if (++acc == 2) { acc = 0; accp ^= 1; }
         }
     } else if (warp >= 4) {
         // ===== epilogue: TMEM -> regs -> bias, ReLU, bf16 -> next layer's layout =====
@@ -667,6 +732,7 @@ struct otif_proxy {
     float *w2_dev;                // [dec] bf16-rounded
     float b2;
     int num_sms;
+    int head_swap;                // swapped-operand head layer (default on; OTIF_HEAD_SWAP=0 for A/B runs)
     uint64_t plan_hash;
 };
 
@@ -758,7 +824,7 @@ static size_t plan_workspace(const otif_proxy *p, int n, Layout lay[5]) {
 static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
     size_t a = (size_t)(g.kb / 8) * g.P * 16;
     size_t b = (size_t)g.cout * g.kb * 2 / g.cg;
-    size_t fixed = (3 * kMaxStagesA + 3 * kMaxStagesB + 4) * 8 + 16 + 2 * 256 * 4 + 1024;
+    size_t fixed = (3 * kMaxStagesA + 3 * kMaxStagesB + 4) * 8 + 16 + 2 * 256 * 4 + 4 * 256 * 4 + 1024;
     size_t budget = 220 * 1024;
     sa = 2; sb = 2;
     // grow B (weights stream every tap) first, then A
@@ -870,7 +936,10 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         } else {
             int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
             if (grid < 1) grid = 1;
-            auto kern = g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>);
+            // head layer with N = 128: swapped operands (see conv_umma_kernel)
+            const bool swap = c.out_kind == 3 && g.mt == 2 && g.cout == 128 && p->head_swap;
+            auto kern = swap ? conv_umma_kernel<2, true>
+                             : (g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>));
             OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
             kern<<<grid, kConvThreads, smem, stream>>>(c);
         }
@@ -920,6 +989,10 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
     if (!p) return OTIF_ENOMEM;
     p->d = *d;
     p->num_sms = num_sms;
+    {
+        const char *e = getenv("OTIF_HEAD_SWAP");
+        p->head_swap = !(e && e[0] == '0');
+    }
     // spatial chain
     int h = d->in_h, w = d->in_w;
     int hs[7], wss[7];
