@@ -692,6 +692,434 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma2_kernel(const __gri
 }
 
 // ---------------------------------------------------------------------------
+// E1 fused into E2 (stride-2 E2 only).  E1's output never reaches HBM: per E2 tile
+// (M = 256 output positions of E2's parity-split input layout) the CTA
+//   1. stages the proxy-image rows the tile needs in shared memory ("slab": 4 image
+//      rows per plane row + 1; bulk copies, rows outside the frame filled with 128,
+//      i.e. x = 0 after normalisation = the zero padding of P:L135's convs);
+//   2. computes, one parity plane at a time ("plane job"), the E1 activations of the
+//      tile's A halo (P = 128 KT rows per plane) on the tensor cores: gather warps build
+//      the im2col rows from the slab as fp16 (u - 128) — exact integers — against fp16
+//      weights w * 2^s (exact: bf16 has 8 significant bits), so the fp32 accumulator is
+//      2^(s+7) times the bf16-path sum (power-of-two scaling commutes with rounding);
+//      epilogue warps apply acc * 2^-(s+7) + b, ReLU, bf16 RNE and write the rows into a
+//      plane buffer in E2's no-swizzle K-major A layout (pads exactly zero);
+//   3. runs E2's taps of that plane from the plane buffer (weights resident in shared
+//      memory) and drains the accumulators into E3's input layout.
+// Hand-offs are per plane job (a commit + wait round trip costs ~300-470 clk on B200,
+// scripts/micro/mma_rate.cu), and E1 and E2 MMAs come from two issuer warps so neither
+// chain stalls the other.  Roles (768 threads): warp 0 slab loader, warp 1 E1 MMA issuer,
+// warp 2 TMEM allocator, warp 3 E2 MMA issuer, warps 4-11 gather (2 warpgroups taking
+// alternate E1 M tiles), 12-19 E1 epilogue (likewise), 20-23 E2 epilogue.
+// Measured bound (ncu, C2): shared-memory bandwidth — N <= 64 MMAs read ~128 B/clk of
+// operands and the gather / epilogue stores share the same port.
+// TMEM: E2 accumulators 2 x 128 columns at 0, E1 accumulators 2 plane slots x 32 KT at 256.
+// ---------------------------------------------------------------------------
+constexpr int kE12Threads = 768;
+constexpr int kE12MaxPlaneBufs = 3;
+
+// n / d for 0 <= n < 2^31 by multiply-high (d fixed per launch)
+struct FastDiv {
+    uint32_t d, m, s;
+};
+static FastDiv make_fastdiv(uint32_t d) {
+    FastDiv f;
+    f.d = d;
+    f.s = 0;
+    while ((1ull << f.s) < d) f.s++;
+    f.m = (uint32_t)(((1ull << 32) * ((1ull << f.s) - d)) / d + 1);
+    return f;
+}
+__device__ __forceinline__ uint32_t fdiv(uint32_t n, const FastDiv &f) {
+    return (uint32_t)(((uint64_t)__umulhi(n, f.m) + n) >> f.s);
+}
+
+struct E12Params {
+    const uint8_t *img;         // u8 [n, hp, wp, 3]
+    int n, hp, wp, row_bytes;   // row_bytes = 3 wp
+    int h1, w1;                 // E1 output
+    int h2, w2, pitch;          // E2 output; pitch = w2 + 1
+    uint32_t fstride, mtot;     // E2 input layout (mtot + P < 2^31)
+    FastDiv div_pitch, div_rpf, div_fstride;  // / pitch, / (h2 + 1) plane rows per frame, / fstride
+    int P;                      // plane-buffer rows = 128 KT
+    int np;                     // plane buffers in the ring (2 or 3)
+    int na1;                    // A1 (im2col) plane stages (1 or 2)
+    int ntiles;
+    int slab_rows, slab_pitch;  // per slab buffer
+    int bulk;                   // image rows may be bulk-copied (16-B aligned rows)
+    int trace;                  // OTIF_E12_TRACE: CTA 0 prints per-role hand-off times (debug)
+    int group_ntaps[4], group_shift[4][9];
+    const uint16_t *wt1;        // fp16 [4 chunks][32 n][8]: K = kh*10 + kw*3 + c -> w * 2^s; K = kh*10 + 9 -> bias parts
+    const uint16_t *wt2;        // bf16 [9 taps in loop order][4 chunks][64 n][8], * 2^-(s+7)
+    const float *b2;
+    // destination: E3's input layout
+    int out_kind;
+    uint8_t *out;
+    int64_t out_lcap;
+    int out_c8, out_pitch;
+    int64_t out_fstride;
+};
+
+// E2-layout position q of a tile whose first plane row is g0: which of the 4 parity
+// planes hold an E1 pixel there (bit (rp << 1) | cp), and the slab byte offset of the
+// image sample at (row 2y - 1, column 2x - 1) for plane (0, 0) (the other planes add
+// 2 rp slab rows and 6 cp bytes).
+__device__ __forceinline__ void e12_decode(const E12Params &p, uint32_t q, uint32_t g0, uint32_t &vmask,
+                                           uint32_t &off) {
+    const uint32_t gr = fdiv(q, p.div_pitch);
+    const int j = (int)(q - gr * (uint32_t)p.pitch);
+    const int i = (int)(gr - fdiv(gr, p.div_rpf) * (uint32_t)(p.h2 + 1));
+    const bool in = q < p.mtot && i >= 1 && j >= 1;
+    const uint32_t r1 = 2 * i - 1 < p.h1, c1 = 2 * j - 1 < p.w1;
+    vmask = in ? (1u | (c1 << 1) | (r1 << 2) | ((r1 & c1) << 3)) : 0u;
+    off = 4 * (gr - g0) * (uint32_t)p.slab_pitch + 12 * (uint32_t)j + 1;
+}
+
+#ifdef OTIF_E12_TRACE_BUILD   // hand-off timeline of CTA 0 (nvcc -DOTIF_E12_TRACE_BUILD; OTIF_E12_TRACE=1)
+#define E12_TR(slot, col)                                                         \
+    do {                                                                          \
+        if (tr && (int)J < 16) tt[slot][J] = clock64();                           \
+    } while (0)
+#define E12_TR_DUMP(name, nslots)                                                                   \
+    do {                                                                                            \
+        if (tr)                                                                                     \
+            for (int j_ = 0; j_ < 16; j_++)                                                         \
+                printf("%s J=%2d %8lld %8lld %8lld\n", name, j_, tt[0][j_] - t00, (nslots) > 1 ? tt[1][j_] - t00 : 0ll, \
+                       (nslots) > 2 ? tt[2][j_] - t00 : 0ll);                                       \
+    } while (0)
+#define E12_TR_DECL                                                       \
+    const bool tr = (p.trace & 1) && blockIdx.x == 0 && ((threadIdx.x & 127) == 0 || threadIdx.x == 32 || threadIdx.x == 96); \
+    long long tt[3][16];                                                   \
+    const long long t00 = clock64();
+#else
+#define E12_TR(slot, col) do {} while (0)
+#define E12_TR_DUMP(name, nslots) do {} while (0)
+#define E12_TR_DECL
+#endif
+
+#define E12_WAIT_SLEEP(b, ph) (p.trace & 2 ? mbar_wait(b, ph) : mbar_wait_sleep(b, ph))
+template <int KT>
+__global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_constant__ E12Params p) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    constexpr int N2 = 64;
+    constexpr int MT = 2;
+    constexpr int P = 128 * KT;
+    constexpr uint32_t kW2Bytes = 9 * 4 * N2 * 16;     // 36,864
+    constexpr uint32_t kW1Bytes = 4 * 32 * 16;         // 2,048
+    constexpr uint32_t kA1Bytes = KT * 4 * 128 * 16;   // one plane's im2col rows
+    constexpr uint32_t kPlaneBytes = P * 64;           // one plane's E1 activations (E2's A)
+    const uint32_t slab_bytes = (uint32_t)p.slab_rows * p.slab_pitch;
+
+    uint8_t *w2_s = smem;
+    uint8_t *w1_s = w2_s + kW2Bytes;
+    uint8_t *a1_s = w1_s + kW1Bytes;
+    uint8_t *a2_s = a1_s + (size_t)p.na1 * kA1Bytes;
+    uint8_t *slab_s = a2_s + (size_t)p.np * kPlaneBytes;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(slab_s + 2 * (size_t)slab_bytes);
+    uint64_t *slab_full = bars, *slab_empty = bars + 2;
+    uint64_t *a1_full = bars + 4, *a1_empty = bars + 6;
+    uint64_t *e1_full = bars + 8, *e1_empty = bars + 10;
+    uint64_t *a2_full = bars + 12, *a2_empty = a2_full + kE12MaxPlaneBufs;
+    uint64_t *acc_full = a2_empty + kE12MaxPlaneBufs, *acc_empty = acc_full + 2;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acc_empty + 2);
+    float *s_b1 = reinterpret_cast<float *>(tmem_slot + 4);
+    float *s_b2 = s_b1 + 32;
+
+    // ---- prologue: barriers, TMEM, resident weights, slab pads = 128 ----
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < 2; i++) {
+            mbar_init(&slab_full[i], 1); mbar_init(&slab_empty[i], 256);
+            mbar_init(&a1_full[i], 256); mbar_init(&a1_empty[i], 1);
+            mbar_init(&e1_full[i], 1); mbar_init(&e1_empty[i], 256);
+            mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 128);
+        }
+        for (int i = 0; i < kE12MaxPlaneBufs; i++) { mbar_init(&a2_full[i], 256); mbar_init(&a2_empty[i], 1); }
+        fence_barrier_init();
+    }
+    if (warp == 2) tmem_alloc(tmem_slot, 512);
+    for (uint32_t i = threadIdx.x; i < kW2Bytes / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(w2_s)[i] = reinterpret_cast<const uint4 *>(p.wt2)[i];
+    for (uint32_t i = threadIdx.x; i < kW1Bytes / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(w1_s)[i] = reinterpret_cast<const uint4 *>(p.wt1)[i];
+    for (uint32_t i = threadIdx.x; i < 2 * slab_bytes / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(slab_s)[i] = make_uint4(0x80808080u, 0x80808080u, 0x80808080u, 0x80808080u);
+    if (threadIdx.x < N2) s_b2[threadIdx.x] = p.b2[threadIdx.x];
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // resident weights -> tensor core
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    const uint32_t rows_per_frame = (uint32_t)p.h2 + 1;   // plane rows per frame (row 0 = pad)
+    E12_TR_DECL
+
+    if (warp == 0) {
+        // ===== slab loader =====
+        uint32_t sb = 0, sp = 0;
+        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+            const uint32_t q0 = (uint32_t)tile * (128 * MT);
+            const uint32_t g0 = fdiv(q0, p.div_pitch);
+            E12_WAIT_SLEEP(&slab_empty[sb], sp ^ 1);
+            uint8_t *slab = slab_s + (size_t)sb * slab_bytes;
+            // slab row s: s = 0 -> image row 4(i0-1)-1 of plane row g0; s >= 1 -> plane row g0 + (s-1)/4, k = (s-1)%4
+            uint32_t my_bytes = 0;
+            for (int s = lane; s < p.slab_rows; s += 32) {
+                const uint32_t g = s == 0 ? g0 : g0 + (s - 1) / 4;
+                const int k = s == 0 ? -1 : (s - 1) % 4;
+                const uint32_t f = fdiv(g, p.div_rpf);
+                const int i = (int)(g - f * rows_per_frame);
+                const int y = 4 * (i - 1) + k;
+                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp) my_bytes += p.row_bytes;
+            }
+            if (p.bulk) {
+#pragma unroll
+                for (int o = 16; o >= 1; o >>= 1) my_bytes += __shfl_xor_sync(0xffffffffu, my_bytes, o);
+                if (lane == 0 && my_bytes) mbar_expect_tx(&slab_full[sb], my_bytes);
+                __syncwarp();
+            }
+            for (int s = lane; s < p.slab_rows; s += 32) {
+                const uint32_t g = s == 0 ? g0 : g0 + (s - 1) / 4;
+                const int k = s == 0 ? -1 : (s - 1) % 4;
+                const uint32_t f = fdiv(g, p.div_rpf);
+                const int i = (int)(g - f * rows_per_frame);
+                const int y = 4 * (i - 1) + k;
+                uint8_t *dst = slab + (size_t)s * p.slab_pitch;
+                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp) {
+                    const uint8_t *src = p.img + ((size_t)f * p.hp + y) * p.row_bytes;
+                    if (p.bulk) {
+                        bulk_g2s(dst + 16, src, p.row_bytes, &slab_full[sb]);
+                    } else {
+                        for (int b = 0; b < p.row_bytes; b++) dst[16 + b] = __ldg(src + b);
+                    }
+                } else {
+                    for (int b = 0; b < p.slab_pitch; b += 16)
+                        *reinterpret_cast<uint4 *>(dst + b) = make_uint4(0x80808080u, 0x80808080u, 0x80808080u, 0x80808080u);
+                }
+            }
+            __threadfence_block();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&slab_full[sb]);
+            if (++sb == 2) { sb = 0; sp ^= 1; }
+        }
+    } else if (warp == 1) {
+        // ===== E1 MMA issuer (whole warp, elected lane issues): one plane job per hand-off =====
+        const uint32_t idesc1 = umma_idesc_f16(128, 32);
+        const uint64_t a1d = umma_desc(smem_u32(a1_s), 2048, 128);
+        const uint64_t w1d = umma_desc(smem_u32(w1_s), 512, 128);
+        uint32_t J = 0;
+        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+            for (int g = 0; g < 4; g++, J++) {
+                const uint32_t s1 = (uint32_t)p.na1 == 1 ? 0 : (J & 1);
+                const uint32_t ph1 = (uint32_t)p.na1 == 1 ? (J & 1) : ((J >> 1) & 1);
+                mbar_wait(&a1_full[s1], ph1);
+                E12_TR(0, 0);
+                mbar_wait(&e1_empty[J & 1], ((J >> 1) & 1) ^ 1);
+                E12_TR(1, 0);
+                tc_fence_after();
+                const uint32_t d = tmem_base + 256 + (J & 1) * (32 * KT);
+#pragma unroll
+                for (int k = 0; k < KT; k++)
+#pragma unroll
+                    for (int s = 0; s < 2; s++)
+                        umma_bf16_warp(d + k * 32, a1d + ((s1 * kA1Bytes + k * 8192 + 2 * s * 2048) >> 4),
+                                       w1d + ((2 * s * 512) >> 4), idesc1, s);
+                umma_commit_warp(&a1_empty[s1]);
+                umma_commit_warp(&e1_full[J & 1]);
+                E12_TR(2, 0);
+            }
+        }
+        E12_TR_DUMP("E1MMA a1full e1empty issued", 3);
+    } else if (warp == 3) {
+        // ===== E2 MMA issuer (whole warp, elected lane issues) =====
+        const uint32_t idesc2 = umma_idesc_bf16(128, N2);
+        const uint64_t a2d = umma_desc(smem_u32(a2_s), P * 16, 128);
+        const uint64_t w2d = umma_desc(smem_u32(w2_s), N2 * 16, 128);
+        uint32_t pb = 0, pp = 0, acc = 0, accp = 0, J = 0;
+        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+            mbar_wait(&acc_empty[acc], accp ^ 1);
+            tc_fence_after();
+            const uint32_t d = tmem_base + acc * (MT * N2);
+            int pos = 0;
+            for (int g = 0; g < 4; g++, J++) {
+                E12_TR(0, 0);
+                mbar_wait(&a2_full[pb], pp);
+                E12_TR(1, 0);
+                tc_fence_after();
+                const uint64_t a = a2d + ((pb * kPlaneBytes) >> 4);
+                for (int t = 0; t < p.group_ntaps[g]; t++, pos++) {
+                    const uint64_t at = a + p.group_shift[g][t];          // +16 B per pixel of shift
+                    const uint64_t bt = w2d + ((pos * (4 * N2 * 16)) >> 4);
+#pragma unroll
+                    for (int s = 0; s < 2; s++)
+#pragma unroll
+                        for (int mm = 0; mm < MT; mm++)
+                            umma_bf16_warp(d + mm * N2, at + ((2 * s * P * 16 + mm * 2048) >> 4), bt + ((2 * s * N2 * 16) >> 4),
+                                           idesc2, (g == 0 && t == 0 && s == 0) ? 0u : 1u);
+                }
+                umma_commit_warp(&a2_empty[pb]);
+                E12_TR(2, 0);
+                if (++pb == (uint32_t)p.np) { pb = 0; pp ^= 1; }
+            }
+            umma_commit_warp(&acc_full[acc]);
+            if (++acc == 2) { acc = 0; accp ^= 1; }
+        }
+        E12_TR_DUMP("E2MMA start a2full issued", 3);
+    } else if (warp >= 4 && warp < 12) {
+        // ===== gather (2 warpgroups, alternate E1 M tiles): one im2col row per thread =====
+        const int wg = (warp - 4) >> 2;
+        const int row = (threadIdx.x - 128) & 127;
+        uint32_t J = 0, sb = 0, sp = 0;
+        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+            const uint32_t q0 = (uint32_t)tile * (128 * MT);
+            const uint32_t g0 = fdiv(q0, p.div_pitch);
+            uint32_t vm[KT], of[KT];
+#pragma unroll
+            for (int k = 0; k < KT; k++) e12_decode(p, q0 + k * 128 + row, g0, vm[k], of[k]);
+            E12_WAIT_SLEEP(&slab_full[sb], sp);
+            const uint8_t *slab = slab_s + (size_t)sb * slab_bytes;
+#pragma unroll
+            for (int g = 0; g < 4; g++, J++) {
+                const int rp = g >> 1, cp = g & 1;
+                const uint32_t s1 = (uint32_t)p.na1 == 1 ? 0 : (J & 1);
+                const uint32_t ph1 = (uint32_t)p.na1 == 1 ? (J & 1) : ((J >> 1) & 1);
+                if (wg == 0) E12_TR(0, 0);
+                E12_WAIT_SLEEP(&a1_empty[s1], ph1 ^ 1);
+                if (wg == 0) E12_TR(1, 0);
+#pragma unroll
+                for (int k = 0; k < KT; k++) {
+                    if ((int)((J * KT + k) & 1) != wg) continue;
+                    uint32_t wv[16];
+#pragma unroll
+                    for (int j = 0; j < 16; j++) wv[j] = 0;
+                    if ((vm[k] >> g) & 1) {
+                        const uint32_t b = of[k] + 2 * rp * p.slab_pitch + 6 * cp;
+                        const uint32_t sh = (b & 3) * 8;
+                        const uint32_t *wp = reinterpret_cast<const uint32_t *>(slab + (b & ~3u));
+                        uint32_t w[9];
+#pragma unroll
+                        for (int kh = 0; kh < 3; kh++) {
+                            const uint32_t *r = wp + kh * (p.slab_pitch >> 2);
+                            w[3 * kh] = r[0]; w[3 * kh + 1] = r[1]; w[3 * kh + 2] = r[2];
+                        }
+#pragma unroll
+                        for (int kh = 0; kh < 3; kh++) {
+                            const uint32_t w0 = w[3 * kh], w1 = w[3 * kh + 1], w2 = w[3 * kh + 2];
+                            const uint32_t a0 = __funnelshift_r(w0, w1, sh), a1 = __funnelshift_r(w1, w2, sh);
+                            wv[5 * kh + 0] = sub_f16x2(__byte_perm(a0, 0x64646464u, 0x4140), 0x64806480u);
+                            wv[5 * kh + 1] = sub_f16x2(__byte_perm(a0, 0x64646464u, 0x4342), 0x64806480u);
+                            wv[5 * kh + 2] = sub_f16x2(__byte_perm(a1, 0x64646464u, 0x4140), 0x64806480u);
+                            wv[5 * kh + 3] = sub_f16x2(__byte_perm(a1, 0x64646464u, 0x4342), 0x64806480u);
+                            // (u - 128, 128): the second half multiplies the bias part at K = 10 kh + 9
+                            wv[5 * kh + 4] = sub_f16x2(0x64006400u | ((w2 >> sh) & 0xFFu), 0x63006480u);
+                        }
+                    }
+                    uint8_t *dst = a1_s + s1 * kA1Bytes + k * 8192 + row * 16;
+#pragma unroll
+                    for (int c = 0; c < 4; c++)
+                        *reinterpret_cast<uint4 *>(dst + c * 2048) = make_uint4(wv[4 * c], wv[4 * c + 1], wv[4 * c + 2], wv[4 * c + 3]);
+                }
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_arrive(&a1_full[s1]);
+                if (wg == 0) E12_TR(2, 0);
+            }
+            mbar_arrive(&slab_empty[sb]);
+            if (++sb == 2) { sb = 0; sp ^= 1; }
+        }
+        if (wg == 0) E12_TR_DUMP("GATH start a1empty arrived", 3);
+    } else if (warp >= 12 && warp < 20) {
+        // ===== E1 epilogue (2 warpgroups, alternate E1 M tiles): TMEM -> ReLU, bf16 -> plane
+        // buffer (E2's A operand).  The accumulator already holds 2^(s+7) (E1 sum + bias);
+        // rounding to bf16 commutes with that power-of-two scale, which E2's weights undo.
+        // Positions without an E1 pixel have an all-zero A row, hence exactly zero here.
+        const int wg = (warp - 12) >> 2;
+        const int row = (threadIdx.x - 384) & 127;
+        const int quarter = warp & 3;
+        uint32_t J = 0, pb = 0, pp = 0;
+        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+#pragma unroll
+            for (int g = 0; g < 4; g++, J++) {
+                E12_WAIT_SLEEP(&a2_empty[pb], pp ^ 1);
+                if (wg == 0) E12_TR(0, 0);
+                mbar_wait(&e1_full[J & 1], (J >> 1) & 1);
+                if (wg == 0) E12_TR(1, 0);
+                tc_fence_after();
+                uint8_t *plane = a2_s + pb * kPlaneBytes;
+                const uint32_t tacc = tmem_base + ((uint32_t)(quarter * 32) << 16) + 256 + (J & 1) * (32 * KT);
+#pragma unroll
+                for (int k = 0; k < KT; k++) {
+                    if ((int)((J * KT + k) & 1) != wg) continue;
+                    uint32_t v[32];
+                    tmem_ld32(tacc + k * 32, v);
+                    uint32_t pk[16];
+#pragma unroll
+                    for (int j = 0; j < 16; j++) pk[j] = pack_bf16x2_relu(__uint_as_float(v[2 * j]), __uint_as_float(v[2 * j + 1]));
+                    uint8_t *dst = plane + (size_t)(k * 128 + row) * 16;
+#pragma unroll
+                    for (int c = 0; c < 4; c++)
+                        *reinterpret_cast<uint4 *>(dst + (size_t)c * P * 16) =
+                            make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+                }
+                tc_fence_before();
+                mbar_arrive(&e1_empty[J & 1]);
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_arrive(&a2_full[pb]);
+                if (wg == 0) E12_TR(2, 0);
+                if (++pb == (uint32_t)p.np) { pb = 0; pp ^= 1; }
+            }
+        }
+        if (wg == 0) E12_TR_DUMP("E1EP a2empty e1full arrived", 3);
+    } else if (warp >= 20) {
+        // ===== E2 epilogue: TMEM -> bias, ReLU, bf16 -> E3's input layout =====
+        const int row = threadIdx.x - 640;
+        const int quarter = warp & 3;
+        uint32_t acc = 0, accp = 0;
+        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+            E12_WAIT_SLEEP(&acc_full[acc], accp);
+            tc_fence_after();
+            for (int mm = 0; mm < MT; mm++) {
+                const uint32_t q = (uint32_t)tile * (128 * MT) + mm * 128 + row;
+                const uint32_t f = fdiv(q, p.div_fstride);
+                const uint32_t r = q - f * p.fstride;
+                const uint32_t oy = fdiv(r, p.div_pitch);
+                const int ox = (int)(r - oy * (uint32_t)p.pitch);
+                const bool valid = q < p.mtot && (int)oy < p.h2 && ox < p.w2;
+                int plane = 0;
+                const int64_t L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, (int)f, (int)oy, ox, plane);
+                const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * (MT * N2) + mm * N2;
+#pragma unroll
+                for (int cc = 0; cc < N2 / 32; cc++) {
+                    uint32_t v[32];
+                    tmem_ld32(taddr + cc * 32, v);
+                    if (valid) {
+                        uint32_t pk[16];
+#pragma unroll
+                        for (int j = 0; j < 16; j++)
+                            pk[j] = pack_bf16x2_relu(__uint_as_float(v[2 * j]) + s_b2[cc * 32 + 2 * j],
+                                                     __uint_as_float(v[2 * j + 1]) + s_b2[cc * 32 + 2 * j + 1]);
+#pragma unroll
+                        for (int c = 0; c < 4; c++) {
+                            uint8_t *dst = p.out + (((int64_t)plane * p.out_c8 + cc * 4 + c) * p.out_lcap + L) * 16;
+                            *reinterpret_cast<uint4 *>(dst) = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+                        }
+                    }
+                }
+            }
+            tc_fence_before();
+            mbar_arrive(&acc_empty[acc]);
+            if (++acc == 2) { acc = 0; accp ^= 1; }
+        }
+    }
+    __syncwarp();
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        tmem_dealloc(tmem_base, 512);
+    }
+}
+
+// ---------------------------------------------------------------------------
 // host side: plan, weight packing, launch
 // ---------------------------------------------------------------------------
 static uint16_t f32_to_bf16_rne(float f) {
@@ -733,6 +1161,12 @@ struct otif_proxy {
     float b2;
     int num_sms;
     int head_swap;                // swapped-operand head layer (default on; OTIF_HEAD_SWAP=0 for A/B runs)
+    // E1 fused into E2 (e12_umma_kernel); 0 = separate E1 kernel + E2 conv
+    int e12;
+    int e12_P, e12_np, e12_na1, e12_slab_rows, e12_slab_pitch;
+    size_t e12_smem;
+    uint16_t *e12_w1_dev;         // fp16 [4][32][8] = bf16(w1) * 2^s, K = kh*10 + kw*3 + c; bias parts at K = 9, 19, 29
+    uint16_t *e12_w2_dev;         // E2's packed bf16 weights * 2^-(s+7)
     uint64_t plan_hash;
 };
 
@@ -815,10 +1249,125 @@ static size_t plan_workspace(const otif_proxy *p, int n, Layout lay[5]) {
     size_t off = 256;  // tag header
     for (int i = 0; i < 5; i++) {
         lay[i] = input_layout(p->L[i], n);
+        if (i == 0 && p->e12 && (int64_t)n * p->L[0].fstride_unit + 4096 < (1ll << 31))
+            lay[i].bytes = 0;   // E1 output stays on chip (fused kernel)
         lay[i].offset = off;
         off += round_up(lay[i].bytes, 256);
     }
     return off;
+}
+
+// fp16 bits of v if v is exactly representable in fp16
+static bool f16_exact(float v, uint16_t *out) {
+    const uint16_t sign = signbit(v) ? 0x8000 : 0;
+    float a = fabsf(v);
+    if (a == 0.0f) { *out = sign; return true; }
+    if (!(a <= 65504.0f)) return false;
+    if (a >= ldexpf(1.0f, -14)) {
+        int ex;
+        float m = frexpf(a, &ex);                 // a = m 2^ex, m in [0.5, 1)
+        float frac = (m * 2.0f - 1.0f) * 1024.0f;  // a = (1 + frac/1024) 2^(ex-1)
+        if (frac != floorf(frac)) return false;
+        *out = (uint16_t)(sign | ((ex - 1 + 15) << 10) | (int)frac);
+        return true;
+    }
+    float q = ldexpf(a, 24);
+    if (q != floorf(q)) return false;
+    *out = (uint16_t)(sign | (int)q);
+    return true;
+}
+
+// Plan the fused E1+E2 kernel; returns false (separate kernels) when it does not apply.
+// round to 11 significant bits (fp16's precision; the range is checked by f16_exact)
+static float round_sig11(float x) {
+    if (x == 0.0f) return 0.0f;
+    int e;
+    const float m = frexpf(x, &e);
+    return ldexpf(rintf(ldexpf(m, 11)), e - 11);
+}
+
+// bf16 bits * 2^-k, if the result is an exact normal bf16 (or zero)
+static bool bf16_scale_exact(uint16_t b, int k, uint16_t *out) {
+    const int ex = (b >> 7) & 0xFF;
+    if (ex == 0) {
+        if (b & 0x7F) return false;
+        *out = b;
+        return true;
+    }
+    if (ex == 255 || ex - k < 1 || ex - k > 254) return false;
+    *out = (uint16_t)((b & 0x807F) | ((ex - k) << 7));
+    return true;
+}
+
+static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const float *b1 /* [32] */) {
+    if (const char *e = getenv("OTIF_E12")) {      // A/B runs only
+        if (e[0] == '0') return false;
+    }
+    const GemmLayer &g = p->L[0];
+    if (p->d.n_strided < 2 || g.kind != 2 || g.cin != 32 || g.cout != 64 || g.cg != 1) return false;
+    float maxabs = 0.0f;
+    for (int i = 0; i < 32 * 27; i++) maxabs = fmaxf(maxabs, fabsf(bf16_to_f32(f32_to_bf16_rne(w1[i]))));
+    int s = 0;
+    if (maxabs > 0.0f) {
+        int ex;
+        frexpf(32768.0f / maxabs, &ex);           // 2^(ex-1) <= 32768/maxabs < 2^ex
+        s = ex - 1;
+    }
+    if (s < -20 || s > 40) return false;
+    std::vector<uint16_t> wh(4 * 32 * 8, 0);
+    for (int o = 0; o < 32; o++)
+        for (int k = 0; k < 32; k++) {
+            const int kh = k / 10, slot = k % 10;
+            if (kh > 2 || slot > 8) continue;
+            const int kw = slot / 3, c = slot % 3;
+            const float v = ldexpf(bf16_to_f32(f32_to_bf16_rne(w1[((o * 3 + kh) * 3 + kw) * 3 + c])), s);
+            uint16_t h;
+            if (!f16_exact(v, &h)) return false;
+            wh[((k / 8) * 32 + o) * 8 + (k % 8)] = h;
+        }
+    // the bias rides in the MMA: A holds 128 at K = 9, 19, 29 (slot 9 of each kernel row),
+    // B holds b * 2^s split exactly into three fp16 parts, so acc = 2^(s+7) (sum + b)
+    for (int o = 0; o < 32; o++) {
+        const float x = ldexpf(b1[o], s);
+        if (ldexpf(x, -s) != b1[o]) return false;
+        const float hi = round_sig11(x), r = x - hi, mid = round_sig11(r), lo = r - mid;
+        const float parts[3] = {hi, mid, lo};
+        for (int kh = 0; kh < 3; kh++) {
+            uint16_t h;
+            if (!f16_exact(parts[kh], &h)) return false;
+            const int k = kh * 10 + 9;
+            wh[((k / 8) * 32 + o) * 8 + (k % 8)] = h;
+        }
+    }
+    // E2 reads E1's activations scaled by 2^(s+7): scale its weights by 2^-(s+7) (exact)
+    std::vector<uint16_t> w2((size_t)9 * 4 * 64 * 8);
+    if (cudaMemcpy(w2.data(), g.wpk_dev, w2.size() * 2, cudaMemcpyDeviceToHost) != cudaSuccess) return false;
+    for (auto &b : w2)
+        if (!bf16_scale_exact(b, s + 7, &b)) return false;
+    const int pitch = g.pitch;
+    const int P = (int)round_up(256 + pitch + 1, 128);
+    if (P / 128 < 3 || P / 128 > 4) return false;      // e12_umma_kernel<KT> instances
+    const int npr = (P - 1) / pitch + 2;
+    const int slab_rows = 4 * npr + 1;
+    const int slab_pitch = (int)round_up(16 + 3 * p->d.in_w + 32, 16);
+    const size_t fixed = 9 * 4 * 64 * 16 + 4 * 32 * 16 + 2 * (size_t)slab_rows * slab_pitch + 64 * 8 + 16 + 96 * 4 + 1024;
+    const size_t a1 = (size_t)P * 64, plane = (size_t)P * 64;
+    int np = 0, na1 = 0;
+    for (int cand_a1 = 2; cand_a1 >= 1 && !np; cand_a1--)
+        for (int cand = kE12MaxPlaneBufs; cand >= 2 && !np; cand--)
+            if (fixed + cand_a1 * a1 + cand * plane <= 227 * 1024) { np = cand; na1 = cand_a1; }
+    if (!np) return false;
+    if (cudaMalloc(&p->e12_w1_dev, wh.size() * 2) != cudaSuccess) return false;
+    cudaMemcpy(p->e12_w1_dev, wh.data(), wh.size() * 2, cudaMemcpyHostToDevice);
+    if (cudaMalloc(&p->e12_w2_dev, w2.size() * 2) != cudaSuccess) return false;
+    cudaMemcpy(p->e12_w2_dev, w2.data(), w2.size() * 2, cudaMemcpyHostToDevice);
+    p->e12_P = P;
+    p->e12_np = np;
+    p->e12_slab_rows = slab_rows;
+    p->e12_slab_pitch = slab_pitch;
+    p->e12_na1 = na1;
+    p->e12_smem = fixed + (size_t)na1 * a1 + (size_t)np * plane;
+    return true;
 }
 
 static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
@@ -867,8 +1416,42 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
     ws_tag_kernel<<<1, 1, 0, stream>>>(ws, tag);
     OTIF_LAUNCH_CHECK();
 
+    const bool e12 = p->e12 && (int64_t)n * p->L[0].fstride_unit + 4096 < (1ll << 31);
+    if (e12) {
+        // E1 fused into E2: one kernel writes E3's input
+        if (evs) OTIF_CUDA(cudaEventRecord(evs[0], stream));
+        const GemmLayer &g = p->L[0];
+        E12Params e;
+        memset(&e, 0, sizeof(e));
+        e.img = img; e.n = n; e.hp = p->d.in_h; e.wp = p->d.in_w; e.row_bytes = 3 * p->d.in_w;
+        e.h1 = p->e1_oh; e.w1 = p->e1_ow;
+        e.h2 = g.out_h; e.w2 = g.out_w; e.pitch = g.pitch;
+        e.fstride = (uint32_t)g.fstride_unit; e.mtot = (uint32_t)((int64_t)n * g.fstride_unit);
+        e.div_pitch = make_fastdiv((uint32_t)g.pitch);
+        e.div_rpf = make_fastdiv((uint32_t)g.out_h + 1);
+        e.div_fstride = make_fastdiv((uint32_t)g.fstride_unit);
+        e.P = p->e12_P; e.np = p->e12_np; e.na1 = p->e12_na1;
+        e.ntiles = (int)cdiv(e.mtot, 256);
+        e.slab_rows = p->e12_slab_rows; e.slab_pitch = p->e12_slab_pitch;
+        e.bulk = (e.row_bytes % 16 == 0) && (((uintptr_t)img & 15) == 0);
+        if (const char *x = getenv("OTIF_E12_TRACE")) e.trace = atoi(x);
+        for (int i = 0; i < 4; i++) {
+            e.group_ntaps[i] = g.group_ntaps[i];
+            for (int t = 0; t < 9; t++) e.group_shift[i][t] = g.group_shift[i][t];
+        }
+        e.wt1 = p->e12_w1_dev;
+        e.wt2 = p->e12_w2_dev; e.b2 = g.bias_dev;
+        e.out_kind = lay[1].kind; e.out = ws + lay[1].offset; e.out_lcap = lay[1].lcap;
+        e.out_c8 = lay[1].c8; e.out_pitch = lay[1].pitch; e.out_fstride = lay[1].fstride;
+        auto kern = e.P == 384 ? e12_umma_kernel<3> : e12_umma_kernel<4>;
+        OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->e12_smem));
+        const int grid = e.ntiles < p->num_sms ? e.ntiles : p->num_sms;
+        kern<<<grid, kE12Threads, p->e12_smem, stream>>>(e);
+        OTIF_LAUNCH_CHECK();
+        if (evs) OTIF_CUDA(cudaEventRecord(evs[1], stream));
+    }
     // E1
-    {
+    if (!e12) {
         E1Params e;
         e.img = img; e.n = n; e.h = p->d.in_h; e.w = p->d.in_w; e.oh = p->e1_oh; e.ow = p->e1_ow;
         e.bias = p->e1_b_dev;
@@ -883,7 +1466,7 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         if (evs) OTIF_CUDA(cudaEventRecord(evs[0], stream));
     }
     // E2..E5, D1
-    for (int li = 0; li < 5; li++) {
+    for (int li = e12 ? 1 : 0; li < 5; li++) {
         const GemmLayer &g = p->L[li];
         ConvParams c;
         memset(&c, 0, sizeof(c));
@@ -1081,6 +1664,7 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
             rc = OTIF_EUNSUPPORTED;
         }
     }
+    if (rc == OTIF_OK) p->e12 = plan_e12(p, weights + offs[0], weights + offs[0] + 32 * 27) ? 1 : 0;
     if (cudaGetLastError() != cudaSuccess && rc == OTIF_OK) rc = OTIF_ECUDA;
     if (rc != OTIF_OK) {
         otif_proxy_destroy(p);
@@ -1091,6 +1675,7 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
     mix(d->in_h); mix(d->in_w); mix(d->n_strided);
     for (int i = 0; i < 5; i++) mix(d->enc[i]);
     mix(d->dec);
+    mix(p->e12);
     p->plan_hash = hsh | 1;
     *out = p;
     return OTIF_OK;
@@ -1105,6 +1690,8 @@ extern "C" void otif_proxy_destroy(otif_proxy *p) {
     if (p->e1_w_dev) cudaFree(p->e1_w_dev);
     if (p->e1_b_dev) cudaFree(p->e1_b_dev);
     if (p->w2_dev) cudaFree(p->w2_dev);
+    if (p->e12_w1_dev) cudaFree(p->e12_w1_dev);
+    if (p->e12_w2_dev) cudaFree(p->e12_w2_dev);
     delete p;
 }
 

@@ -83,6 +83,35 @@ def test_proxy_parity(wl, n, blob):
         assert np.array_equal((got > np.float32(b))[far], (ref_bf16 > b)[far])
 
 
+# E1 fused into E2 (e12_umma_kernel: E1 activations computed on chip from a staged
+# image slab) vs the separate E1 + E2 kernels (OTIF_E12=0), on shapes that exercise odd
+# E1/E2 sizes (invalid parity-plane positions), rows that are not 16-B aligned (LSU slab
+# copies: 3*w % 16 != 0) and several strides.
+E12_CASES = [(67, 123, 3, 3), (64, 104, 3, 5), (45, 90, 2, 3), (33, 50, 5, 2), (135, 240, 3, 3), (90, 160, 4, 2)]
+
+
+@pytest.mark.parametrize("h,w,ns,n", E12_CASES, ids=[f"{c[0]}x{c[1]}s{c[2]}" for c in E12_CASES])
+def test_proxy_e1_fused_vs_separate(h, w, ns, n, blob, monkeypatch):
+    rng = np.random.default_rng(h * 1000 + w)
+    img = rng.integers(0, 256, (n, h, w, 3), dtype=np.uint8)
+    img[0, : h // 3] = 128                      # flat region (x = 0 after normalisation)
+    img[-1, :, : w // 4] = rng.integers(0, 2, (h, w // 4, 3)) * 255
+    fused = otif.Proxy(h, w, ns, blob)
+    monkeypatch.setenv("OTIF_E12", "0")
+    sep = otif.Proxy(h, w, ns, blob)
+    monkeypatch.delenv("OTIF_E12")
+    assert fused.workspace_bytes(n) < sep.workspace_bytes(n), "fused path not planned"
+    t = torch.from_numpy(img).cuda()
+    a = fused.score(t).cpu().numpy().astype(np.float64)
+    b = sep.score(t).cpu().numpy().astype(np.float64)
+    ref_none = oracle_scores(img, type("W", (), {"n_strided": ns})(), blob, oracle.QUANT_NONE)
+    assert np.abs(a - ref_none).max() <= 2e-2
+    assert np.abs(a - b).max() <= 1e-2
+    # the two paths differ only in the fp32 accumulation order of E1 (the fused path adds
+    # E1's bias inside the MMA), so bf16 roundings of E1 rarely differ
+    assert np.median(np.abs(a - b)) <= 1e-4
+
+
 def test_proxy_repeat_calls_reuse_workspace(blob):
     wl = configs.C1
     img = torch.from_numpy(oracle.resize(_frames(wl, 8).numpy(), wl.proxy_h, wl.proxy_w)).cuda()
