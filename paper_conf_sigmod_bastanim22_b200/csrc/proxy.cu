@@ -305,8 +305,8 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
             }
         }
     } else if (warp == 1) {
-        // ===== MMA issuer (single thread) =====
-        if (lane == 0) {
+        // ===== MMA issuer (whole warp, elected lane issues: descriptors stay warp-uniform) =====
+        {
             const uint32_t idesc = SWAP ? umma_idesc_bf16(kTileM, kTileM * MT) : umma_idesc_bf16(kTileM, p.N);
             uint32_t as = 0, ap = 0, bs = 0, bp = 0, acc = 0, accp = 0;
             const uint32_t a_base = smem_u32(a_buf), b_base = smem_u32(b_buf);
@@ -331,25 +331,25 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                                 if (SWAP) {
                                     // weights = M operand, the 128*MT halo rows = N operand
                                     const uint64_t hd = umma_desc(a_tap + 2 * s * lbo_a, lbo_a, 128);
-                                    umma_bf16(d, bd, hd, idesc, accumulate);
+                                    umma_bf16_warp(d, bd, hd, idesc, accumulate);
                                 } else {
                                     // the mt sub-tiles share this B stage: rows 128*m.. of the halo
 #pragma unroll
                                     for (int m = 0; m < MT; m++) {
                                         uint64_t ad = umma_desc(a_tap + 2 * s * lbo_a + m * (kTileM * 16), lbo_a, 128);
-                                        umma_bf16(d + m * p.N, ad, bd, idesc, accumulate);
+                                        umma_bf16_warp(d + m * p.N, ad, bd, idesc, accumulate);
                                     }
                                 }
                                 accumulate = 1;
                             }
-                            umma_commit(&b_empty[bs]);
+                            umma_commit_warp(&b_empty[bs]);
                             if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
                         }
-                        umma_commit(&a_empty[as]);
+                        umma_commit_warp(&a_empty[as]);
                         if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
                     }
                 }
-                umma_commit(&t_full[acc]);
+                umma_commit_warp(&t_full[acc]);
                 if (++acc == 2) { acc = 0; accp ^= 1; }
             }
         }
