@@ -248,7 +248,7 @@ __device__ void merge_update_mat(const SelectParams &p, Frame &F, int n, int lan
     __syncwarp();
 }
 
-__device__ void greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U) {
+__device__ bool greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U) {
     const int S = p.nmat;
     for (int q = lane; q < n * n; q += 32) {
         const int i = q / n, j = q - i * n;
@@ -271,6 +271,7 @@ __device__ void greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, 
             }
             if (Gv <= 0) break;
             merge_update_mat(p, F, n, lane, U, I, F.bj[I]);
+            if (F.sidx[I] == p.full) return true;  // exact full-frame exit (see select_kernel)
         }
         // phase B: lexicographically first pair of alive clusters whose placed windows overlap
         int mi = 0x7FFF, mj = 0x7FFF;
@@ -297,7 +298,90 @@ __device__ void greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, 
         }
         if (mi == 0x7FFF) break;
         merge_update_mat(p, F, n, lane, U, mi, mj);
+        if (F.sidx[mi] == p.full) return true;
     }
+    return false;
+}
+
+// Greedy grouping without the fit matrix (n > nmat or costs too large for the matrix):
+// row rescans.  Returns true on the exact full-frame exit (see select_kernel).
+__device__ bool greedy_rescan(const SelectParams &p, Frame &F, int n, int lane) {
+    while (true) {
+        for (int i = lane; i < n; i += 32)
+            if (F.alive[i]) rescan_row(p, F, n, i);
+        __syncwarp();
+        while (true) {  // phase A
+            long long G = kNoGain;
+            int I = 0x7FFF;
+            for (int i = lane; i < n; i += 32)
+                if (F.alive[i] && (F.bg[i] > G || (F.bg[i] == G && i < I))) { G = F.bg[i]; I = i; }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                long long og = __shfl_xor_sync(0xffffffffu, G, o);
+                int oi = __shfl_xor_sync(0xffffffffu, I, o);
+                if (og > G || (og == G && oi < I)) { G = og; I = oi; }
+            }
+            if (G <= 0) break;  // "once merging offers no further improvement" (strict)
+            const int J = F.bj[I];
+            __syncwarp();
+            if (lane == 0) {
+                F.cl[I] = runion(F.cl[I], F.cl[J]);
+                int s = fit_rect(p, F.cl[I]);
+                F.sidx[I] = (signed char)s;
+                F.cost[I] = p.cost[s];
+                F.alive[J] = 0;
+            }
+            __syncwarp();
+            if (F.sidx[I] == p.full) return true;
+            for (int i = lane; i < n; i += 32) {
+                if (!F.alive[i]) continue;
+                const int b = F.bj[i];
+                if (i == I || b == I || b == J) {
+                    rescan_row(p, F, n, i);
+                } else if (i < I) {
+                    long long g = F.cost[i] + F.cost[I] - p.cost[fit_rect(p, runion(F.cl[i], F.cl[I]))];
+                    if (g > F.bg[i] || (g == F.bg[i] && I < b)) { F.bg[i] = g; F.bj[i] = (short)I; }
+                }
+            }
+            __syncwarp();
+        }
+        // phase B: merge the lexicographically first pair whose placed windows overlap
+        int mi = 0x7FFF, mj = 0x7FFF;
+        for (int i = lane; i < n; i += 32) {
+            if (!F.alive[i]) continue;
+            int xi, yi, si = F.sidx[i];
+            place(p, F.cl[i], si, xi, yi);
+            for (int j = i + 1; j < n; j++) {
+                if (!F.alive[j]) continue;
+                int xj, yj, sj = F.sidx[j];
+                place(p, F.cl[j], sj, xj, yj);
+                if (xi < xj + p.sw[sj] && xj < xi + p.sw[si] && yi < yj + p.sh[sj] && yj < yi + p.sh[si]) {
+                    if (i < mi) { mi = i; mj = j; }
+                    break;
+                }
+            }
+            if (mi != 0x7FFF) break;  // later i of this lane are larger
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            int oi = __shfl_xor_sync(0xffffffffu, mi, o);
+            int oj = __shfl_xor_sync(0xffffffffu, mj, o);
+            if (oi < mi) { mi = oi; mj = oj; }
+        }
+        if (mi == 0x7FFF) break;
+        __syncwarp();
+        if (lane == 0) {
+            F.cl[mi] = runion(F.cl[mi], F.cl[mj]);
+            int s = fit_rect(p, F.cl[mi]);
+            F.sidx[mi] = (signed char)s;
+            F.cost[mi] = p.cost[s];
+            F.alive[mj] = 0;
+        }
+        __syncwarp();
+        if (F.sidx[mi] == p.full) return true;
+    }
+    return false;
+
 }
 
 __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_constant__ SelectParams p) {
@@ -429,80 +513,19 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
     }
 
     // --- grouping: phase A greedy merge, phase B disjointness (readings R7, R10) ---
-    if (p.nmat > 0 && n <= p.nmat) {
-        greedy_matrix(p, F, n, lane, base + p.gmat_offset);
-    } else
-    while (true) {
-        for (int i = lane; i < n; i += 32)
-            if (F.alive[i]) rescan_row(p, F, n, i);
-        __syncwarp();
-        while (true) {  // phase A
-            long long G = kNoGain;
-            int I = 0x7FFF;
-            for (int i = lane; i < n; i += 32)
-                if (F.alive[i] && (F.bg[i] > G || (F.bg[i] == G && i < I))) { G = F.bg[i]; I = i; }
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1) {
-                long long og = __shfl_xor_sync(0xffffffffu, G, o);
-                int oi = __shfl_xor_sync(0xffffffffu, I, o);
-                if (og > G || (og == G && oi < I)) { G = og; I = oi; }
-            }
-            if (G <= 0) break;  // "once merging offers no further improvement" (strict)
-            const int J = F.bj[I];
-            __syncwarp();
-            if (lane == 0) {
-                F.cl[I] = runion(F.cl[I], F.cl[J]);
-                int s = fit_rect(p, F.cl[I]);
-                F.sidx[I] = (signed char)s;
-                F.cost[I] = p.cost[s];
-                F.alive[J] = 0;
-            }
-            __syncwarp();
-            for (int i = lane; i < n; i += 32) {
-                if (!F.alive[i]) continue;
-                const int b = F.bj[i];
-                if (i == I || b == I || b == J) {
-                    rescan_row(p, F, n, i);
-                } else if (i < I) {
-                    long long g = F.cost[i] + F.cost[I] - p.cost[fit_rect(p, runion(F.cl[i], F.cl[I]))];
-                    if (g > F.bg[i] || (g == F.bg[i] && I < b)) { F.bg[i] = g; F.bj[i] = (short)I; }
-                }
-            }
-            __syncwarp();
-        }
-        // phase B: merge the lexicographically first pair whose placed windows overlap
-        int mi = 0x7FFF, mj = 0x7FFF;
-        for (int i = lane; i < n; i += 32) {
-            if (!F.alive[i]) continue;
-            int xi, yi, si = F.sidx[i];
-            place(p, F.cl[i], si, xi, yi);
-            for (int j = i + 1; j < n; j++) {
-                if (!F.alive[j]) continue;
-                int xj, yj, sj = F.sidx[j];
-                place(p, F.cl[j], sj, xj, yj);
-                if (xi < xj + p.sw[sj] && xj < xi + p.sw[si] && yi < yj + p.sh[sj] && yj < yi + p.sh[si]) {
-                    if (i < mi) { mi = i; mj = j; }
-                    break;
-                }
-            }
-            if (mi != 0x7FFF) break;  // later i of this lane are larger
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            int oi = __shfl_xor_sync(0xffffffffu, mi, o);
-            int oj = __shfl_xor_sync(0xffffffffu, mj, o);
-            if (oi < mi) { mi = oi; mj = oj; }
-        }
-        if (mi == 0x7FFF) break;
-        __syncwarp();
-        if (lane == 0) {
-            F.cl[mi] = runion(F.cl[mi], F.cl[mj]);
-            int s = fit_rect(p, F.cl[mi]);
-            F.sidx[mi] = (signed char)s;
-            F.cost[mi] = p.cost[s];
-            F.alive[mj] = 0;
-        }
-        __syncwarp();
+    // Exact full-frame exit: once a cluster's fit is the full frame (W' index p.full), the
+    // output is the single window (0, 0, Wd, Hd).  Its placement overlaps every other
+    // window, so phase B merges every cluster into it; a union containing it still fits
+    // p.full first (nothing cheaper contains the smaller rectangle); the final
+    // est = T_full is not > T_full, so the result is exactly the fallback window below.
+    bool full_hit = __any_sync(0xffffffffu, [&] {
+        bool h = false;
+        for (int c = lane; c < n; c += 32) h |= F.sidx[c] == p.full;
+        return h;
+    }());
+    if (!full_hit) {
+        if (p.nmat > 0 && n <= p.nmat) full_hit = greedy_matrix(p, F, n, lane, base + p.gmat_offset);
+        else full_hit = greedy_rescan(p, F, n, lane);
     }
 
     // --- emission: est(R), strict full-frame fallback (R11), (y, x) order (R15) ---
@@ -516,7 +539,7 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
         m += __shfl_xor_sync(0xffffffffu, m, o);
     }
     unsigned long long hsh = 0, pix = 0;
-    if (est > p.cost[p.full]) {
+    if (full_hit || est > p.cost[p.full]) {
         if (lane == 0) {
             otif_window w;
             w.frame = f; w.x = 0; w.y = 0; w.w = p.fw; w.h = p.fh; w.size_idx = p.orig[p.full];
