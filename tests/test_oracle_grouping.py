@@ -255,3 +255,31 @@ def test_select_windows_batch_order_and_offsets():
     # capacity overflow: total stays exact
     w2, c2, o2, t2 = oracle.select_windows(masks, 32, 416, 256, S, capacity=2)
     assert t2 == total and len(w2) == min(2, total)
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_full_fit_cluster_forces_full_frame(seed):
+    """The kernel's exact full-frame exit (select.cu): once ANY cluster's minimum-cost
+    fitting size is the full frame, the greedy's output is the single full-frame window
+    (phase B merges every other cluster into the full-frame placement; R10, R11).  Checked
+    on the oracle for masks whose components include one that only the full frame holds."""
+    rng = np.random.default_rng(seed)
+    fw, fh, cell = 960, 540, 32
+    gh, gw = -(-fh // cell), -(-fw // cell)
+    sizes = [(128, 128), (256, 256), (fw, fh)]
+    mask = (rng.random((gh, gw)) < rng.uniform(0.05, 0.3)).astype(np.uint8)
+    # a snake component wider than 256 px (so only the full frame contains it)
+    y = int(rng.integers(0, gh))
+    x0 = int(rng.integers(0, gw - 10))
+    mask[y, x0:x0 + int(rng.integers(9, gw - x0 + 1))] = 1
+    n, lab = oracle.components(mask, 4)
+    full_fit = False
+    for c in range(n):
+        ys, xs = np.nonzero(lab == c)
+        w = min(int(xs.max() + 1) * cell, fw) - int(xs.min()) * cell
+        h = min(int(ys.max() + 1) * cell, fh) - int(ys.min()) * cell
+        full_fit |= not any(sw >= w and sh >= h for sw, sh in sizes[:2])
+    assert full_fit
+    win = oracle.group_frame(mask, cell, fw, fh, sizes)
+    assert len(win) == 1
+    assert (int(win[0]["x"]), int(win[0]["y"]), int(win[0]["w"]), int(win[0]["h"])) == (0, 0, fw, fh)
