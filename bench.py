@@ -207,7 +207,7 @@ def run_otif(args):
     # device path: the whole clip is one device batch by default (every stage is one launch
     # over all frames, so latency-bound stages see enough frames to fill the SMs)
     batch = args.batch if args.batch > 0 else n
-    pipe = otif.Pipeline(wl, blob, b, max_batch=batch, proxy_batch=args.proxy_batch)
+    pipe = otif.Pipeline(wl, blob, b, max_batch=batch, proxy_batch=args.proxy_batch, overlap_chunks=args.overlap)
     stream = torch.cuda.current_stream()
     for _ in range(args.warmup):
         pipe.run_device(src)
@@ -419,6 +419,8 @@ def main():
     ap.add_argument("--batch", type=int, default=0, help="device batch (0 = whole clip)")
     ap.add_argument("--host-batch", type=int, default=512, help="device batch of the host (e2e) path")
     ap.add_argument("--proxy-batch", type=int, default=0, help="frames per resize+proxy launch (0 = batch)")
+    ap.add_argument("--overlap", type=int, default=0,
+                    help="chunks per device batch with resize/select/pack overlapped under the proxy (0 = serial)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--oracle-frames", type=int, default=32)
     ap.add_argument("--no-e2e", action="store_true")

@@ -286,6 +286,12 @@ typedef struct {
     int32_t batch_cap[8];       /* detector batch capacity per size, per device batch */
     int32_t proxy_batch;        /* frames per resize + proxy launch within a batch (0 = max_batch);
                                    small enough keeps each layer's activations L2-resident */
+    int32_t overlap_chunks;     /* >= 2: split each device batch into this many chunks and run the
+                                   memory-bound stages (resize of chunk c+1, select + pack of chunk
+                                   c-1) on a second stream while the tensor-bound proxy scores chunk c;
+                                   the proxy kernels then leave shared memory for co-resident resize /
+                                   pack CTAs.  Results are identical to the serial schedule (slots keep
+                                   the batch's emission order).  0 or 1 = serial (proxy_batch applies). */
 } otif_pipeline_desc;
 
 typedef struct otif_pipeline otif_pipeline;

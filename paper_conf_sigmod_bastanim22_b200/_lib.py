@@ -41,7 +41,8 @@ class PipelineDesc(ctypes.Structure):
     _fields_ = [("proxy", ProxyDesc), ("src_h", ctypes.c_int32), ("src_w", ctypes.c_int32),
                 ("det_h", ctypes.c_int32), ("det_w", ctypes.c_int32), ("grid", GridDesc),
                 ("threshold", ctypes.c_float), ("k", ctypes.c_int32), ("sizes", WSize * 8),
-                ("max_batch", ctypes.c_int32), ("batch_cap", ctypes.c_int32 * 8), ("proxy_batch", ctypes.c_int32)]
+                ("max_batch", ctypes.c_int32), ("batch_cap", ctypes.c_int32 * 8), ("proxy_batch", ctypes.c_int32),
+                ("overlap_chunks", ctypes.c_int32)]
 
 
 _lib = None

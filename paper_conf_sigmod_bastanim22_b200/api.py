@@ -174,9 +174,10 @@ class Pipeline:
 
     def __init__(self, workload, weights: np.ndarray, threshold: float, max_batch: int = 256,
                  batch_cap: Sequence[int] | None = None, connectivity: int = 4,
-                 enc=(32, 64, 128, 256, 256), dec=128, proxy_batch: int = 0):
+                 enc=(32, 64, 128, 256, 256), dec=128, proxy_batch: int = 0, overlap_chunks: int = 0):
         d = PipelineDesc()
         d.proxy_batch = int(proxy_batch)
+        d.overlap_chunks = int(overlap_chunks)
         d.proxy.in_h, d.proxy.in_w, d.proxy.n_strided = workload.proxy_h, workload.proxy_w, workload.n_strided
         for i, e in enumerate(enc):
             d.proxy.enc[i] = int(e)

@@ -31,13 +31,15 @@ struct PackParams {
     int bw[kMaxK], bh[kMaxK];
     int *slot;
     int *size_count;
+    int accumulate;   // internal (pipeline chunks): slots continue from size_count's current values
+    int stage_bytes;  // bulk ring stage size (<= kBulkStage)
 };
 
 __global__ void __launch_bounds__(1024) slot_kernel(const __grid_constant__ PackParams p) {
     __shared__ int s_warp_cnt[32][kMaxK];
     __shared__ int s_carry[kMaxK];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    if (threadIdx.x < kMaxK) s_carry[threadIdx.x] = 0;
+    if (threadIdx.x < kMaxK) s_carry[threadIdx.x] = (p.accumulate && threadIdx.x < p.k) ? p.size_count[threadIdx.x] : 0;
     __syncthreads();
     const int total = min(*p.total, p.capacity);
     for (int base = 0; base < total; base += blockDim.x) {
@@ -107,9 +109,9 @@ __device__ __forceinline__ uint4 load16u(const uint8_t *s0, uintptr_t src_end) {
 // global->shared (the window's rows of a chunk; a single copy when the window spans
 // full frame rows, so its bytes are contiguous) then shared->global into the packed
 // detector batch (contiguous).  Loads run kBulkLead chunks ahead of the stores.
-constexpr int kBulkStages = 3;
-constexpr int kBulkLead = 1;                 // <= kBulkStages - 1
-constexpr int kBulkStage = 16384;            // bytes per ring stage
+// STAGES ring stages, loads run STAGES - 2 chunks ahead of the stores (one stage is being
+// read by an in-flight store); stage size is a launch parameter (<= kBulkStage).
+constexpr int kBulkStage = 16384;            // largest ring stage (bytes)
 
 __device__ __forceinline__ void bulk_s2g(void *dst_gmem, const void *src_smem, uint32_t bytes) {
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst_gmem), "r"(smem_u32(src_smem)),
@@ -126,13 +128,15 @@ __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wa
 // One thread streams one window through the ring.  A window spanning full frame rows is
 // one contiguous byte range in the source: it moves in 16 KB chunks regardless of rows;
 // otherwise a chunk is as many whole rows as fit in a stage (one g2s per row).
+template <int kBulkStages>
 __device__ void pack_window_bulk(uint8_t *ring, uint64_t *bars, uint32_t &chunk_seq, const uint8_t *fbase, int sw,
-                                 const otif_window &w, uint8_t *dst) {
+                                 const otif_window &w, uint8_t *dst, uint32_t stage_bytes) {
+    constexpr int kBulkLead = kBulkStages - 2;
     const uint32_t row_bytes = (uint32_t)w.w * 3;
     const bool contiguous = (w.x == 0 && w.w == sw);
     const uint32_t total = (uint32_t)w.h * row_bytes;
-    const int rpc = (int)(kBulkStage / row_bytes);  // >= 1 (checked by the caller)
-    const uint32_t chunk_bytes = contiguous ? (uint32_t)kBulkStage : rpc * row_bytes;
+    const int rpc = (int)(stage_bytes / row_bytes);  // >= 1 (checked by the caller)
+    const uint32_t chunk_bytes = contiguous ? stage_bytes : rpc * row_bytes;
     const int nchunks = (int)((total + chunk_bytes - 1) / chunk_bytes);
     const uint8_t *wsrc = fbase + ((size_t)w.y * sw + w.x) * 3;
     const uint32_t base = chunk_seq;
@@ -143,7 +147,7 @@ __device__ void pack_window_bulk(uint8_t *ring, uint64_t *bars, uint32_t &chunk_
             bulk_wait_read<kBulkStages - kBulkLead - 1>();
             const uint32_t off = (uint32_t)i * chunk_bytes;
             const uint32_t bytes = min(chunk_bytes, total - off);
-            uint8_t *buf = ring + (size_t)s * kBulkStage;
+            uint8_t *buf = ring + (size_t)s * stage_bytes;
             mbar_arrive_expect_tx(&bars[s], bytes);
             if (contiguous) {
                 bulk_g2s(buf, wsrc + off, bytes, &bars[s]);
@@ -158,7 +162,7 @@ __device__ void pack_window_bulk(uint8_t *ring, uint64_t *bars, uint32_t &chunk_
             const uint32_t c = base + j, s = c % kBulkStages;
             mbar_wait(&bars[s], (c / kBulkStages) & 1);
             const uint32_t off = (uint32_t)j * chunk_bytes;
-            bulk_s2g(dst + off, ring + (size_t)s * kBulkStage, min(chunk_bytes, total - off));
+            bulk_s2g(dst + off, ring + (size_t)s * stage_bytes, min(chunk_bytes, total - off));
             bulk_commit();
         }
     }
@@ -166,8 +170,9 @@ __device__ void pack_window_bulk(uint8_t *ring, uint64_t *bars, uint32_t &chunk_
     bulk_wait_all();
 }
 
+template <int kBulkStages>
 __global__ void __launch_bounds__(128) pack_kernel(const __grid_constant__ PackParams p) {
-    extern __shared__ __align__(128) uint8_t ring[];  // kBulkStages x kBulkStage bytes
+    extern __shared__ __align__(128) uint8_t ring[];  // kBulkStages x p.stage_bytes
     __shared__ uint64_t bars[kBulkStages];
     if (threadIdx.x == 0) {
         for (int i = 0; i < kBulkStages; i++) mbar_init(&bars[i], 1);
@@ -184,10 +189,11 @@ __global__ void __launch_bounds__(128) pack_kernel(const __grid_constant__ PackP
         if (sl >= p.cap[s]) continue;
         uint8_t *dst = p.batch[s] + (size_t)sl * p.bh[s] * p.bw[s] * 3;
         const int row_bytes = w.w * 3;
-        if (identity && (row_bytes & 15) == 0 && row_bytes <= kBulkStage && (((uintptr_t)p.batch[s]) & 15) == 0 &&
+        if (identity && (row_bytes & 15) == 0 && row_bytes <= p.stage_bytes && (((uintptr_t)p.batch[s]) & 15) == 0 &&
             ((w.x * 3) & 15) == 0 && ((p.sw * 3) & 15) == 0 && (((uintptr_t)p.src) & 15) == 0) {
             if (threadIdx.x == 0)
-                pack_window_bulk(ring, bars, chunk_seq, p.src + (size_t)w.frame * p.sh * p.sw * 3, p.sw, w, dst);
+                pack_window_bulk<kBulkStages>(ring, bars, chunk_seq, p.src + (size_t)w.frame * p.sh * p.sw * 3, p.sw, w,
+                                              dst, (uint32_t)p.stage_bytes);
         } else if (identity && (row_bytes & 15) == 0 && (((uintptr_t)p.batch[s]) & 15) == 0) {
             const int per_row = row_bytes >> 4;
             const uint8_t *fbase = p.src + (size_t)w.frame * p.sh * p.sw * 3;
@@ -247,6 +253,51 @@ __global__ void __launch_bounds__(128) pack_kernel(const __grid_constant__ PackP
 
 using namespace otif;
 
+namespace otif {
+
+// internal entry (pipeline): accumulate = slots continue from size_count (chunked batches);
+// ctas = pack grid (0 = 6 per SM); stages 3 or 6; stage_bytes <= kBulkStage
+otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w,
+                        const otif_window *windows, const int32_t *total, int32_t capacity, const otif_wsize *sizes,
+                        int32_t k, uint8_t *const *batches, const int32_t *batch_cap, int32_t *slot,
+                        int32_t *size_count, cudaStream_t stream, int accumulate, int ctas, int stages,
+                        int stage_bytes) {
+    PackParams p;
+    memset(&p, 0, sizeof(p));
+    p.src = src; p.n = n; p.sh = src_h; p.sw = src_w; p.dh = det_h; p.dw = det_w;
+    p.src_bytes = (size_t)n * src_h * src_w * 3;
+    p.win = windows; p.total = total; p.capacity = capacity; p.k = k;
+    for (int s = 0; s < k; s++) {
+        OTIF_REQUIRE(sizes[s].w > 0 && sizes[s].h > 0 && sizes[s].w <= det_w && sizes[s].h <= det_h,
+                     "otif_pack_windows: size %d larger than the detector frame", s);
+        OTIF_REQUIRE(batch_cap[s] >= 0 && (batch_cap[s] == 0 || batches[s]), "otif_pack_windows: batch %d", s);
+        p.batch[s] = batches[s]; p.cap[s] = batch_cap[s]; p.bw[s] = sizes[s].w; p.bh[s] = sizes[s].h;
+    }
+    p.slot = slot; p.size_count = size_count;
+    p.accumulate = accumulate;
+    p.stage_bytes = stage_bytes > 0 && stage_bytes <= kBulkStage ? (stage_bytes & ~15) : kBulkStage;
+    int num_sms = 148;
+    check_device(&num_sms);
+    slot_kernel<<<1, 1024, 0, stream>>>(p);
+    OTIF_LAUNCH_CHECK();
+    if (capacity > 0) {
+        const int want = ctas > 0 ? ctas : num_sms * 6;
+        const int grid = capacity < want ? capacity : want;
+        const int smem = (stages == 6 ? 6 : 3) * p.stage_bytes;
+        if (stages == 6) {
+            OTIF_CUDA(cudaFuncSetAttribute(pack_kernel<6>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+            pack_kernel<6><<<grid, 128, smem, stream>>>(p);
+        } else {
+            OTIF_CUDA(cudaFuncSetAttribute(pack_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+            pack_kernel<3><<<grid, 128, smem, stream>>>(p);
+        }
+        OTIF_LAUNCH_CHECK();
+    }
+    return OTIF_OK;
+}
+
+}  // namespace otif
+
 extern "C" otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w, int32_t det_h,
                                          int32_t det_w, const otif_window *windows, const int32_t *total,
                                          int32_t capacity, const otif_wsize *sizes, int32_t k,
@@ -260,28 +311,6 @@ extern "C" otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t 
     OTIF_REQUIRE(src || n == 0, "otif_pack_windows: NULL src");
     otif_status st = check_device(nullptr);
     if (st != OTIF_OK) return st;
-    PackParams p;
-    memset(&p, 0, sizeof(p));
-    p.src = src; p.n = n; p.sh = src_h; p.sw = src_w; p.dh = det_h; p.dw = det_w;
-    p.src_bytes = (size_t)n * src_h * src_w * 3;
-    p.win = windows; p.total = total; p.capacity = capacity; p.k = k;
-    for (int s = 0; s < k; s++) {
-        OTIF_REQUIRE(sizes[s].w > 0 && sizes[s].h > 0 && sizes[s].w <= det_w && sizes[s].h <= det_h,
-                     "otif_pack_windows: size %d larger than the detector frame", s);
-        OTIF_REQUIRE(batch_cap[s] >= 0 && (batch_cap[s] == 0 || batches[s]), "otif_pack_windows: batch %d", s);
-        p.batch[s] = batches[s]; p.cap[s] = batch_cap[s]; p.bw[s] = sizes[s].w; p.bh[s] = sizes[s].h;
-    }
-    p.slot = slot; p.size_count = size_count;
-    int num_sms = 148;
-    check_device(&num_sms);
-    slot_kernel<<<1, 1024, 0, stream>>>(p);
-    OTIF_LAUNCH_CHECK();
-    if (capacity > 0) {
-        int grid = capacity < num_sms * 6 ? capacity : num_sms * 6;
-        const int smem = kBulkStages * kBulkStage;
-        OTIF_CUDA(cudaFuncSetAttribute(pack_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-        pack_kernel<<<grid, 128, smem, stream>>>(p);
-        OTIF_LAUNCH_CHECK();
-    }
-    return OTIF_OK;
+    return launch_pack(src, n, src_h, src_w, det_h, det_w, windows, total, capacity, sizes, k, batches, batch_cap,
+                       slot, size_count, stream, 0, 0, 3, kBulkStage);
 }

@@ -8,6 +8,15 @@
 // frames in flight to fill 148 SMs).  The detector batches stay on the device (the
 // detector runs there); windows, per-frame counts and counters are accumulated
 // on the device and copied back once per host call.
+//
+// Overlap mode (desc.overlap_chunks >= 2): the batch is split into chunks; the caller's
+// stream runs the tensor-bound proxy of chunk c while a second stream runs the
+// memory-bound stages — resize of chunk c+1, then select + pack of chunk c-1 — so HBM
+// traffic hides under the tensor-core work.  The proxy kernels then take a lower
+// shared-memory budget so that a pack (bulk-copy ring) or resize CTA fits on every SM
+// next to a proxy CTA.  Slots continue across the chunks (pack accumulates size_count),
+// so the detector batches hold the same windows in the same order as the serial schedule.
+#include <stdlib.h>
 #include <string.h>
 
 #include <new>
@@ -23,7 +32,14 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum);
+                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum, size_t smem_cap);
+otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w,
+                        const otif_window *windows, const int32_t *total, int32_t capacity, const otif_wsize *sizes,
+                        int32_t k, uint8_t *const *batches, const int32_t *batch_cap, int32_t *slot,
+                        int32_t *size_count, cudaStream_t stream, int accumulate, int ctas, int stages,
+                        int stage_bytes);
+otif_status proxy_set_smem_budget(otif_proxy *p, size_t budget);
+int proxy_launches(const otif_proxy *p);
 
 // timing stages: resize, proxy prep (tag + E1), E2, E3, E4, E5, D1+D2, select, pack, append
 constexpr int kStages = 10;
@@ -61,7 +77,7 @@ struct otif_pipeline {
     otif_proxy *proxy = nullptr;
     int gh = 0, gw = 0, cells = 0, cap_w = 0, pb = 0;
     uint8_t *src[2] = {nullptr, nullptr};
-    uint8_t *img = nullptr, *mask = nullptr, *proxy_ws = nullptr, *sel_ws = nullptr;
+    uint8_t *img = nullptr, *img2 = nullptr, *mask = nullptr, *proxy_ws = nullptr, *sel_ws = nullptr;
     size_t proxy_ws_bytes = 0, sel_ws_bytes = 0;
     float *scores = nullptr;
     otif_window *windows = nullptr;
@@ -76,27 +92,52 @@ struct otif_pipeline {
     int *out_total = nullptr;
     cudaStream_t s_compute = nullptr, s_copy = nullptr;
     cudaEvent_t ev_h2d[2] = {}, ev_free[2] = {};
-    // optional per-stage timing: an ordered log of (stage, event); the time between an
-    // event and its predecessor is charged to the event's stage (ST_START opens a span)
+    // overlap mode: chunking, the memory stream and its hand-off events
+    int chunks = 0, chunk = 0;
+    int pack_ctas = 0, pack_stages = 3, pack_stage_bytes = 16384;
+    size_t sel_smem_cap = 0;
+    cudaStream_t s_mem = nullptr;
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_resized[2] = {}, ev_scored[2] = {}, ev_imgfree[2] = {};
+    // optional per-stage timing: a log of spans (stage, start entry, end event); a span's
+    // time is charged to its stage (stage < 0: a start marker)
     int timing = 0;
     std::vector<cudaEvent_t> ev_pool;
-    std::vector<int> ev_stage;
+    std::vector<int> ev_stage, ev_from;
     size_t ev_used = 0;
     int64_t launches = 0;
 };
 
-static otif_status mark(otif_pipeline *p, int stage, cudaStream_t st, cudaEvent_t *out = nullptr) {
-    if (!p->timing) return OTIF_OK;
+// reserve a log entry (stage, from); its event is returned for the caller to record
+static int treserve(otif_pipeline *p, int stage, int from, cudaEvent_t *ev) {
     if (p->ev_pool.size() <= p->ev_used) {
         cudaEvent_t e;
-        OTIF_CUDA(cudaEventCreate(&e));
+        if (cudaEventCreate(&e) != cudaSuccess) return -1;
         p->ev_pool.push_back(e);
         p->ev_stage.push_back(0);
+        p->ev_from.push_back(-1);
     }
     p->ev_stage[p->ev_used] = stage;
-    if (out) *out = p->ev_pool[p->ev_used];
-    OTIF_CUDA(cudaEventRecord(p->ev_pool[p->ev_used++], st));
-    return OTIF_OK;
+    p->ev_from[p->ev_used] = from;
+    *ev = p->ev_pool[p->ev_used];
+    return (int)p->ev_used++;
+}
+
+// record a start marker on st; returns its entry (or -1 when timing is off)
+static int tmark(otif_pipeline *p, cudaStream_t st) {
+    if (!p->timing) return -1;
+    cudaEvent_t e;
+    int i = treserve(p, ST_START, -1, &e);
+    if (i >= 0) cudaEventRecord(e, st);
+    return i;
+}
+
+// close a span of `stage` opened at entry `from` (recorded on st); returns the new entry
+static int tspan(otif_pipeline *p, int stage, cudaStream_t st, int from) {
+    if (!p->timing || from < 0) return -1;
+    cudaEvent_t e;
+    int i = treserve(p, stage, from, &e);
+    if (i >= 0) cudaEventRecord(e, st);
+    return i;
 }
 
 #define RC(x)                           \
@@ -105,38 +146,92 @@ static otif_status mark(otif_pipeline *p, int stage, cudaStream_t st, cudaEvent_
         if (rc_ != OTIF_OK) return rc_; \
     } while (0)
 
+static otif_status run_proxy(otif_pipeline *p, const uint8_t *img, int mb, float *scores, cudaStream_t st) {
+    // six spans for the proxy (prep/E1, then each GEMM layer); launch_proxy records their
+    // end events at the actual points in the stream
+    cudaEvent_t evs[6];
+    int from = tmark(p, st);
+    for (int i = 0; i < 6 && p->timing; i++) from = treserve(p, ST_PREP + i, from, &evs[i]);
+    RC(launch_proxy(p->proxy, img, mb, scores, p->proxy_ws, p->proxy_ws_bytes, st, p->timing ? evs : nullptr));
+    p->launches += proxy_launches(p->proxy);
+    return OTIF_OK;
+}
+
+// select + pack (+ append) of frames [f0, f0 + nb) of the batch at src
+static otif_status run_select_pack(otif_pipeline *p, const uint8_t *src, int f0, int nb, int frame_base,
+                                   int accumulate, cudaStream_t st) {
+    const otif_pipeline_desc &d = p->d;
+    const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
+    int t0 = tmark(p, st);
+    RC(launch_select(p->scores + (size_t)f0 * p->cells, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k,
+                     p->mask + (size_t)f0 * p->cells, p->windows, p->cap_w, p->counts + f0, p->offsets + f0, p->total,
+                     p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base + f0, nullptr, p->sel_smem_cap));
+    t0 = tspan(p, ST_SELECT, st, t0);
+    RC(launch_pack(src + (size_t)f0 * frame_bytes, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total,
+                   p->cap_w, d.sizes, d.k, p->batches, d.batch_cap, p->slot, p->size_count, st, accumulate,
+                   p->pack_ctas, p->pack_stages, p->pack_stage_bytes));
+    t0 = tspan(p, ST_PACK, st, t0);
+    p->launches += 4;  // select 2, pack 2
+    if (p->out_win) {
+        append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts + f0, nb, frame_base + f0,
+                                          p->out_win, p->out_win_cap, p->out_counts, p->out_total);
+        OTIF_LAUNCH_CHECK();
+        p->launches += 1;
+        tspan(p, ST_APPEND, st, t0);
+    }
+    return OTIF_OK;
+}
+
 static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int frame_base, cudaStream_t st) {
     const otif_pipeline_desc &d = p->d;
     const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
-    cudaEvent_t evs[6];
-    for (int m0 = 0; m0 < nb; m0 += p->pb) {
-        const int mb = nb - m0 < p->pb ? nb - m0 : p->pb;
-        RC(mark(p, ST_START, st));
-        RC(otif_resize(src + (size_t)m0 * frame_bytes, mb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w, st));
-        RC(mark(p, ST_RESIZE, st));
-        // six log entries for the proxy (after E1, after each GEMM layer); launch_proxy
-        // re-records these events at their actual points in the stream
-        for (int i = 0; i < 6 && p->timing; i++) RC(mark(p, ST_PREP + i, st, &evs[i]));
-        RC(launch_proxy(p->proxy, p->img, mb, p->scores + (size_t)m0 * p->cells, p->proxy_ws, p->proxy_ws_bytes, st,
-                        p->timing ? evs : nullptr));
-        p->launches += 9;  // resize 1, proxy 8 (zero, tag, E1, 5 GEMM layers)
+    if (p->chunks < 2) {
+        for (int m0 = 0; m0 < nb; m0 += p->pb) {
+            const int mb = nb - m0 < p->pb ? nb - m0 : p->pb;
+            int t0 = tmark(p, st);
+            RC(otif_resize(src + (size_t)m0 * frame_bytes, mb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w, st));
+            tspan(p, ST_RESIZE, st, t0);
+            RC(run_proxy(p, p->img, mb, p->scores + (size_t)m0 * p->cells, st));
+            p->launches += 1;
+        }
+        return run_select_pack(p, src, 0, nb, frame_base, 0, st);
     }
-    RC(mark(p, ST_START, st));
-    RC(launch_select(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask, p->windows,
-                     p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base,
-                     nullptr));
-    RC(mark(p, ST_SELECT, st));
-    RC(otif_pack_windows(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
-                         p->batches, d.batch_cap, p->slot, p->size_count, st));
-    RC(mark(p, ST_PACK, st));
-    p->launches += 4;  // select 2, pack 2
-    if (p->out_win) {
-        append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts, nb, frame_base, p->out_win,
-                                          p->out_win_cap, p->out_counts, p->out_total);
-        OTIF_LAUNCH_CHECK();
+    // overlap: st = tensor stream (proxy), s_mem = memory stream (resize, select, pack)
+    cudaStream_t sm = p->s_mem;
+    uint8_t *img[2] = {p->img, p->img2};
+    const int cs = p->chunk;
+    const int nc = (nb + cs - 1) / cs;
+    OTIF_CUDA(cudaEventRecord(p->ev_fork, st));
+    OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_fork, 0));
+    for (int i = 0; i < 2; i++) OTIF_CUDA(cudaEventRecord(p->ev_imgfree[i], st));
+    auto resize_chunk = [&](int c) -> otif_status {
+        const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
+        OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_imgfree[c & 1], 0));
+        int t0 = tmark(p, sm);
+        RC(otif_resize(src + (size_t)c0 * frame_bytes, cn, d.src_h, d.src_w, img[c & 1], d.proxy.in_h, d.proxy.in_w, sm));
+        tspan(p, ST_RESIZE, sm, t0);
         p->launches += 1;
-        RC(mark(p, ST_APPEND, st));
+        OTIF_CUDA(cudaEventRecord(p->ev_resized[c & 1], sm));
+        return OTIF_OK;
+    };
+    auto select_chunk = [&](int c) -> otif_status {
+        const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
+        OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_scored[c & 1], 0));
+        return run_select_pack(p, src, c0, cn, frame_base, c > 0, sm);
+    };
+    RC(resize_chunk(0));
+    for (int c = 0; c < nc; c++) {
+        if (c + 1 < nc) RC(resize_chunk(c + 1));
+        if (c >= 1) RC(select_chunk(c - 1));
+        const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
+        OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_resized[c & 1], 0));
+        RC(run_proxy(p, img[c & 1], cn, p->scores + (size_t)c0 * p->cells, st));
+        OTIF_CUDA(cudaEventRecord(p->ev_scored[c & 1], st));
+        OTIF_CUDA(cudaEventRecord(p->ev_imgfree[c & 1], st));
     }
+    RC(select_chunk(nc - 1));
+    OTIF_CUDA(cudaEventRecord(p->ev_join, sm));
+    OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_join, 0));
     return OTIF_OK;
 }
 
@@ -173,12 +268,39 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     }
     const int B = d->max_batch;
     p->pb = (d->proxy_batch > 0 && d->proxy_batch < B) ? d->proxy_batch : B;
+    if (d->overlap_chunks >= 2) {
+        // A/B knobs (env, sweeps only): proxy smem budget, pack grid / ring, select CTA smem
+        auto envi = [](const char *k, long v) { const char *e = getenv(k); return e ? atol(e) : v; };
+        int num_sms = 148;
+        check_device(&num_sms);
+        p->chunks = d->overlap_chunks < B ? d->overlap_chunks : B;
+        p->chunk = (B + p->chunks - 1) / p->chunks;
+        p->pb = p->chunk;
+        p->pack_ctas = (int)envi("OTIF_OVL_PACK_CTAS", num_sms);
+        p->pack_stages = (int)envi("OTIF_OVL_PACK_STAGES", 3);
+        p->pack_stage_bytes = (int)envi("OTIF_OVL_PACK_STAGE", 12288);
+        p->sel_smem_cap = (size_t)envi("OTIF_OVL_SEL_SMEM", 36 * 1024);
+        const size_t budget = (size_t)envi("OTIF_OVL_PROXY_SMEM", 184 * 1024);
+        otif_status rc2 = proxy_set_smem_budget(p->proxy, budget);
+        if (rc2 != OTIF_OK) { otif_pipeline_destroy(p); return rc2; }
+    }
     p->cells = p->gh * p->gw;
     p->cap_w = B * ((p->cells + 1) / 2);
     const size_t src_bytes = (size_t)B * d->src_h * d->src_w * 3;
     PCUDA(cudaMalloc(&p->src[0], src_bytes));
     PCUDA(cudaMalloc(&p->src[1], src_bytes));
     PCUDA(cudaMalloc(&p->img, (size_t)p->pb * d->proxy.in_h * d->proxy.in_w * 3));
+    if (p->chunks >= 2) {
+        PCUDA(cudaMalloc(&p->img2, (size_t)p->pb * d->proxy.in_h * d->proxy.in_w * 3));
+        PCUDA(cudaStreamCreateWithFlags(&p->s_mem, cudaStreamNonBlocking));
+        PCUDA(cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming));
+        PCUDA(cudaEventCreateWithFlags(&p->ev_join, cudaEventDisableTiming));
+        for (int i = 0; i < 2; i++) {
+            PCUDA(cudaEventCreateWithFlags(&p->ev_resized[i], cudaEventDisableTiming));
+            PCUDA(cudaEventCreateWithFlags(&p->ev_scored[i], cudaEventDisableTiming));
+            PCUDA(cudaEventCreateWithFlags(&p->ev_imgfree[i], cudaEventDisableTiming));
+        }
+    }
     p->proxy_ws_bytes = otif_proxy_workspace_bytes(p->proxy, p->pb);
     PCUDA(cudaMalloc(&p->proxy_ws, p->proxy_ws_bytes));
     PCUDA(cudaMemset(p->proxy_ws, 0, p->proxy_ws_bytes));
@@ -213,7 +335,8 @@ extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     if (!p) return;
     if (p->s_compute) cudaStreamSynchronize(p->s_compute);
     if (p->s_copy) cudaStreamSynchronize(p->s_copy);
-    void *bufs[] = {p->src[0], p->src[1], p->img, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
+    if (p->s_mem) cudaStreamSynchronize(p->s_mem);
+    void *bufs[] = {p->src[0], p->src[1], p->img, p->img2, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
                     p->offsets, p->total, p->slot, p->size_count, p->ctr, p->out_win, p->out_counts, p->out_total};
     for (void *b : bufs)
         if (b) cudaFree(b);
@@ -226,6 +349,11 @@ extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     }
     if (p->s_compute) cudaStreamDestroy(p->s_compute);
     if (p->s_copy) cudaStreamDestroy(p->s_copy);
+    if (p->s_mem) cudaStreamDestroy(p->s_mem);
+    cudaEvent_t ovl[] = {p->ev_fork, p->ev_join, p->ev_resized[0], p->ev_resized[1], p->ev_scored[0], p->ev_scored[1],
+                         p->ev_imgfree[0], p->ev_imgfree[1]};
+    for (cudaEvent_t e : ovl)
+        if (e) cudaEventDestroy(e);
     if (p->proxy) otif_proxy_destroy(p->proxy);
     delete p;
 }
@@ -332,11 +460,12 @@ extern "C" otif_status otif_pipeline_stage_ms(otif_pipeline *p, float *ms, int32
     OTIF_REQUIRE(p && ms && n_ms >= kStages, "otif_pipeline_stage_ms: need %d entries", kStages);
     for (int s = 0; s < kStages; s++) ms[s] = 0.0f;
     if (p->ev_used > 0) OTIF_CUDA(cudaEventSynchronize(p->ev_pool[p->ev_used - 1]));
-    for (size_t i = 1; i < p->ev_used; i++) {
-        const int s = p->ev_stage[i];
-        if (s < 0) continue;  // a span start: no time charged
+    if (p->ev_used > 0) OTIF_CUDA(cudaDeviceSynchronize());  // spans live on two streams
+    for (size_t i = 0; i < p->ev_used; i++) {
+        const int s = p->ev_stage[i], from = p->ev_from[i];
+        if (s < 0 || from < 0) continue;  // a start marker: no time charged
         float t = 0.0f;
-        OTIF_CUDA(cudaEventElapsedTime(&t, p->ev_pool[i - 1], p->ev_pool[i]));
+        OTIF_CUDA(cudaEventElapsedTime(&t, p->ev_pool[from], p->ev_pool[i]));
         ms[s] += t;
     }
     if (launches) *launches = p->launches;

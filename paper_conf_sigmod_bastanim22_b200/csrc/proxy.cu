@@ -1164,7 +1164,10 @@ struct otif_proxy {
     // E1 fused into E2 (e12_umma_kernel); 0 = separate E1 kernel + E2 conv
     int e12;
     int e12_P, e12_np, e12_na1, e12_slab_rows, e12_slab_pitch;
-    size_t e12_smem;
+    size_t e12_smem, e12_fixed, e12_unit;
+    // shared-memory budget of one conv / E1+E2 CTA (default: the whole SM); a pipeline that
+    // runs memory-bound kernels next to the proxy lowers it so their CTAs stay co-resident
+    size_t smem_budget = 227 * 1024;
     uint16_t *e12_w1_dev;         // fp16 [4][32][8] = bf16(w1) * 2^s, K = kh*10 + kw*3 + c; bias parts at K = 9, 19, 29
     uint16_t *e12_w2_dev;         // E2's packed bf16 weights * 2^-(s+7)
     uint64_t plan_hash;
@@ -1299,6 +1302,17 @@ static bool bf16_scale_exact(uint16_t b, int k, uint16_t *out) {
     return true;
 }
 
+static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes, size_t budget = 220 * 1024);
+
+// deepest (im2col stages, plane buffers) of the E1+E2 kernel within `budget` bytes
+static bool e12_stages(size_t fixed, size_t unit, size_t budget, int &np, int &na1) {
+    np = 0; na1 = 0;
+    for (int cand_a1 = 2; cand_a1 >= 1 && !np; cand_a1--)
+        for (int cand = kE12MaxPlaneBufs; cand >= 2 && !np; cand--)
+            if (fixed + (size_t)(cand_a1 + cand) * unit <= budget) { np = cand; na1 = cand_a1; }
+    return np != 0;
+}
+
 static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const float *b1 /* [32] */) {
     if (const char *e = getenv("OTIF_E12")) {      // A/B runs only
         if (e[0] == '0') return false;
@@ -1353,10 +1367,7 @@ static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const f
     const size_t fixed = 9 * 4 * 64 * 16 + 4 * 32 * 16 + 2 * (size_t)slab_rows * slab_pitch + 64 * 8 + 16 + 96 * 4 + 1024;
     const size_t a1 = (size_t)P * 64, plane = (size_t)P * 64;
     int np = 0, na1 = 0;
-    for (int cand_a1 = 2; cand_a1 >= 1 && !np; cand_a1--)
-        for (int cand = kE12MaxPlaneBufs; cand >= 2 && !np; cand--)
-            if (fixed + cand_a1 * a1 + cand * plane <= 227 * 1024) { np = cand; na1 = cand_a1; }
-    if (!np) return false;
+    if (!e12_stages(fixed, a1, 227 * 1024, np, na1)) return false;
     if (cudaMalloc(&p->e12_w1_dev, wh.size() * 2) != cudaSuccess) return false;
     cudaMemcpy(p->e12_w1_dev, wh.data(), wh.size() * 2, cudaMemcpyHostToDevice);
     if (cudaMalloc(&p->e12_w2_dev, w2.size() * 2) != cudaSuccess) return false;
@@ -1367,14 +1378,47 @@ static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const f
     p->e12_slab_pitch = slab_pitch;
     p->e12_na1 = na1;
     p->e12_smem = fixed + (size_t)na1 * a1 + (size_t)np * plane;
+    p->e12_fixed = fixed;
+    p->e12_unit = a1;
     return true;
 }
 
-static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
+// kernel launches of one launch_proxy call (workspace zero + tag, E1+E2 fused or E1 and E2, E3..D1)
+int proxy_launches(const otif_proxy *p) { return p->e12 ? 7 : 8; }
+
+// Lower the per-CTA shared-memory budget of the proxy kernels (pipeline overlap mode):
+// the conv rings and the E1+E2 plane / im2col buffers shrink to fit.  Not thread-safe
+// against concurrent launches of the same proxy; the pipeline calls it once at create.
+otif_status proxy_set_smem_budget(otif_proxy *p, size_t budget) {
+    if (budget > 227 * 1024) budget = 227 * 1024;
+    for (int li = 0; li < 5; li++) {
+        int sa, sb;
+        size_t bytes;
+        conv_smem(p->L[li], sa, sb, bytes, budget);
+        if (bytes > budget) {
+            set_error("proxy_set_smem_budget: layer %d needs %zu B > %zu B", li + 2, bytes, budget);
+            return OTIF_EUNSUPPORTED;
+        }
+    }
+    if (p->e12) {
+        int np = 0, na1 = 0;
+        if (!e12_stages(p->e12_fixed, p->e12_unit, budget, np, na1)) {
+            set_error("proxy_set_smem_budget: E1+E2 needs more than %zu B", budget);
+            return OTIF_EUNSUPPORTED;
+        }
+        p->e12_np = np;
+        p->e12_na1 = na1;
+        p->e12_smem = p->e12_fixed + (size_t)(np + na1) * p->e12_unit;
+    }
+    p->smem_budget = budget;
+    return OTIF_OK;
+}
+
+static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes, size_t budget) {
     size_t a = (size_t)(g.kb / 8) * g.P * 16;
     size_t b = (size_t)g.cout * g.kb * 2 / g.cg;
     size_t fixed = (3 * kMaxStagesA + 3 * kMaxStagesB + 4) * 8 + 16 + 2 * 256 * 4 + 4 * 256 * 4 + 1024;
-    size_t budget = 220 * 1024;
+    if (budget > 220 * 1024) budget = 220 * 1024;
     sa = 2; sb = 2;
     // grow B (weights stream every tap) first, then A
     // a CTA pair recycles a stage over a longer loop (peer relay, multicast commit): deeper B ring
@@ -1497,7 +1541,7 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
             c.b2 = p->b2;
         }
         size_t smem;
-        conv_smem(g, c.stages_a, c.stages_b, smem);
+        conv_smem(g, c.stages_a, c.stages_b, smem, p->smem_budget);
         if (g.cg == 2) {
             const int pairs = p->num_sms / 2;
             const int clusters = c.ntiles < pairs ? (c.ntiles < 1 ? 1 : c.ntiles) : pairs;

@@ -341,6 +341,29 @@ def test_pipeline_host_vs_stages(wl, blob):
     assert list(sc) == [int((ref["size_idx"] == s).sum()) for s in range(len(wl.sizes))]
 
 
+@pytest.mark.parametrize("wl,chunks", [(configs.C2, 3), (configs.C1, 4), (configs.C3, 2)], ids=["C2", "C1", "C3"])
+def test_pipeline_overlap_matches_serial(wl, chunks, blob):
+    """Overlap mode (resize / select / pack of neighbouring chunks on a second stream while
+    the proxy scores a chunk) returns exactly the serial schedule's windows, per-frame counts,
+    per-size counts and device counters (incl. the order-independent window hash), over
+    several device batches with a ragged last chunk."""
+    b = threshold(wl.name, 0.7)
+    n = 75
+    src = video.frames(wl, n).contiguous()
+    ser = otif.Pipeline(wl, blob, b, max_batch=40)
+    ovl = otif.Pipeline(wl, blob, b, max_batch=40, overlap_chunks=chunks)
+    w0, c0, s0, t0 = ser.run_host(src)
+    w1, c1, s1, t1 = ovl.run_host(src)
+    assert t0 == t1 and np.array_equal(c0, c1) and list(s0) == list(s1)
+    assert np.array_equal(w0, w1)
+    src_d = src.cuda()
+    for pipe in (ser, ovl):
+        pipe.reset_counters()
+        pipe.run_device(src_d)
+    torch.cuda.synchronize()
+    assert torch.equal(ser.counters().cpu(), ovl.counters().cpu())
+
+
 def test_edge_cases():
     wl = configs.C1
     # n = 0 everywhere
