@@ -170,8 +170,8 @@ __device__ void pack_window_bulk(uint8_t *ring, uint64_t *bars, uint32_t &chunk_
     bulk_wait_all();
 }
 
-template <int kBulkStages>
-__global__ void __launch_bounds__(128) pack_kernel(const __grid_constant__ PackParams p) {
+template <int kBulkStages, int kThreads>
+__global__ void __launch_bounds__(kThreads) pack_kernel(const __grid_constant__ PackParams p) {
     extern __shared__ __align__(128) uint8_t ring[];  // kBulkStages x p.stage_bytes
     __shared__ uint64_t bars[kBulkStages];
     if (threadIdx.x == 0) {
@@ -256,12 +256,13 @@ using namespace otif;
 namespace otif {
 
 // internal entry (pipeline): accumulate = slots continue from size_count (chunked batches);
-// ctas = pack grid (0 = 6 per SM); stages 3 or 6; stage_bytes <= kBulkStage
+// ctas = pack grid (0 = 6 per SM); stages 3 or 6; stage_bytes <= kBulkStage; threads 128 or
+// 32 (one warp: few registers, so a CTA fits on an SM next to the 768-thread E1+E2 CTA)
 otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w,
                         const otif_window *windows, const int32_t *total, int32_t capacity, const otif_wsize *sizes,
                         int32_t k, uint8_t *const *batches, const int32_t *batch_cap, int32_t *slot,
                         int32_t *size_count, cudaStream_t stream, int accumulate, int ctas, int stages,
-                        int stage_bytes) {
+                        int stage_bytes, int threads) {
     PackParams p;
     memset(&p, 0, sizeof(p));
     p.src = src; p.n = n; p.sh = src_h; p.sw = src_w; p.dh = det_h; p.dw = det_w;
@@ -284,13 +285,10 @@ otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t sr
         const int want = ctas > 0 ? ctas : num_sms * 6;
         const int grid = capacity < want ? capacity : want;
         const int smem = (stages == 6 ? 6 : 3) * p.stage_bytes;
-        if (stages == 6) {
-            OTIF_CUDA(cudaFuncSetAttribute(pack_kernel<6>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-            pack_kernel<6><<<grid, 128, smem, stream>>>(p);
-        } else {
-            OTIF_CUDA(cudaFuncSetAttribute(pack_kernel<3>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-            pack_kernel<3><<<grid, 128, smem, stream>>>(p);
-        }
+        auto kern = stages == 6 ? (threads == 32 ? pack_kernel<6, 32> : pack_kernel<6, 128>)
+                                : (threads == 32 ? pack_kernel<3, 32> : pack_kernel<3, 128>);
+        OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        kern<<<grid, threads == 32 ? 32 : 128, smem, stream>>>(p);
         OTIF_LAUNCH_CHECK();
     }
     return OTIF_OK;
@@ -312,5 +310,5 @@ extern "C" otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t 
     otif_status st = check_device(nullptr);
     if (st != OTIF_OK) return st;
     return launch_pack(src, n, src_h, src_w, det_h, det_w, windows, total, capacity, sizes, k, batches, batch_cap,
-                       slot, size_count, stream, 0, 0, 3, kBulkStage);
+                       slot, size_count, stream, 0, 0, 3, kBulkStage, 128);
 }

@@ -37,7 +37,7 @@ otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t sr
                         const otif_window *windows, const int32_t *total, int32_t capacity, const otif_wsize *sizes,
                         int32_t k, uint8_t *const *batches, const int32_t *batch_cap, int32_t *slot,
                         int32_t *size_count, cudaStream_t stream, int accumulate, int ctas, int stages,
-                        int stage_bytes);
+                        int stage_bytes, int threads);
 otif_status proxy_set_smem_budget(otif_proxy *p, size_t budget);
 int proxy_launches(const otif_proxy *p);
 
@@ -94,7 +94,9 @@ struct otif_pipeline {
     cudaEvent_t ev_h2d[2] = {}, ev_free[2] = {};
     // overlap mode: chunking, the memory stream and its hand-off events
     int chunks = 0, chunk = 0;
-    int pack_ctas = 0, pack_stages = 3, pack_stage_bytes = 16384;
+    int pack_ctas = 0, pack_stages = 3, pack_stage_bytes = 16384, pack_threads = 128;
+    int ovl_mode = 0;   // 0: resize, select and pack on the memory stream; 1: pack only
+    int *totals = nullptr;  // [chunks] per-chunk window totals (overlap)
     size_t sel_smem_cap = 0;
     cudaStream_t s_mem = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_resized[2] = {}, ev_scored[2] = {}, ev_imgfree[2] = {};
@@ -157,24 +159,34 @@ static otif_status run_proxy(otif_pipeline *p, const uint8_t *img, int mb, float
     return OTIF_OK;
 }
 
-// select + pack (+ append) of frames [f0, f0 + nb) of the batch at src
-static otif_status run_select_pack(otif_pipeline *p, const uint8_t *src, int f0, int nb, int frame_base,
-                                   int accumulate, cudaStream_t st) {
+// select of frames [f0, f0 + nb) of the batch into window slice `wo` (capacity cap) and *tot
+static otif_status run_select(otif_pipeline *p, int f0, int nb, int frame_base, otif_window *wo, int cap, int *tot,
+                              cudaStream_t st) {
+    const otif_pipeline_desc &d = p->d;
+    int t0 = tmark(p, st);
+    RC(launch_select(p->scores + (size_t)f0 * p->cells, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k,
+                     p->mask + (size_t)f0 * p->cells, wo, cap, p->counts + f0, p->offsets + f0, tot, p->sel_ws,
+                     p->sel_ws_bytes, st, p->ctr, frame_base + f0, nullptr, p->sel_smem_cap));
+    tspan(p, ST_SELECT, st, t0);
+    p->launches += 2;
+    return OTIF_OK;
+}
+
+// pack (+ append) of those windows; accumulate = slots continue from earlier chunks
+static otif_status run_pack(otif_pipeline *p, const uint8_t *src, int f0, int nb, int frame_base,
+                            const otif_window *wo, int cap, const int *tot, int *slot, int accumulate,
+                            cudaStream_t st) {
     const otif_pipeline_desc &d = p->d;
     const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
     int t0 = tmark(p, st);
-    RC(launch_select(p->scores + (size_t)f0 * p->cells, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k,
-                     p->mask + (size_t)f0 * p->cells, p->windows, p->cap_w, p->counts + f0, p->offsets + f0, p->total,
-                     p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base + f0, nullptr, p->sel_smem_cap));
-    t0 = tspan(p, ST_SELECT, st, t0);
-    RC(launch_pack(src + (size_t)f0 * frame_bytes, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total,
-                   p->cap_w, d.sizes, d.k, p->batches, d.batch_cap, p->slot, p->size_count, st, accumulate,
-                   p->pack_ctas, p->pack_stages, p->pack_stage_bytes));
+    RC(launch_pack(src + (size_t)f0 * frame_bytes, nb, d.src_h, d.src_w, d.det_h, d.det_w, wo, tot, cap, d.sizes, d.k,
+                   p->batches, d.batch_cap, slot, p->size_count, st, accumulate, p->pack_ctas, p->pack_stages,
+                   p->pack_stage_bytes, p->pack_threads));
     t0 = tspan(p, ST_PACK, st, t0);
-    p->launches += 4;  // select 2, pack 2
+    p->launches += 2;
     if (p->out_win) {
-        append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts + f0, nb, frame_base + f0,
-                                          p->out_win, p->out_win_cap, p->out_counts, p->out_total);
+        append_kernel<<<1, 1024, 0, st>>>(wo, tot, cap, p->counts + f0, nb, frame_base + f0, p->out_win,
+                                          p->out_win_cap, p->out_counts, p->out_total);
         OTIF_LAUNCH_CHECK();
         p->launches += 1;
         tspan(p, ST_APPEND, st, t0);
@@ -194,7 +206,8 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
             RC(run_proxy(p, p->img, mb, p->scores + (size_t)m0 * p->cells, st));
             p->launches += 1;
         }
-        return run_select_pack(p, src, 0, nb, frame_base, 0, st);
+        RC(run_select(p, 0, nb, frame_base, p->windows, p->cap_w, p->total, st));
+        return run_pack(p, src, 0, nb, frame_base, p->windows, p->cap_w, p->total, p->slot, 0, st);
     }
     // overlap: st = tensor stream (proxy), s_mem = memory stream (resize, select, pack)
     cudaStream_t sm = p->s_mem;
@@ -214,22 +227,51 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
         OTIF_CUDA(cudaEventRecord(p->ev_resized[c & 1], sm));
         return OTIF_OK;
     };
-    auto select_chunk = [&](int c) -> otif_status {
+    // chunk c's windows, total and slots live in their own slices (no reuse hazard between
+    // the streams); pack keeps the emission order by running the chunks in order
+    const int per_frame = p->cap_w / d.max_batch;
+    auto select_chunk = [&](int c, cudaStream_t s) -> otif_status {
         const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
-        OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_scored[c & 1], 0));
-        return run_select_pack(p, src, c0, cn, frame_base, c > 0, sm);
+        return run_select(p, c0, cn, frame_base, p->windows + (size_t)c0 * per_frame, cn * per_frame, p->totals + c, s);
     };
-    RC(resize_chunk(0));
-    for (int c = 0; c < nc; c++) {
-        if (c + 1 < nc) RC(resize_chunk(c + 1));
-        if (c >= 1) RC(select_chunk(c - 1));
+    auto pack_chunk = [&](int c) -> otif_status {
         const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
-        OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_resized[c & 1], 0));
-        RC(run_proxy(p, img[c & 1], cn, p->scores + (size_t)c0 * p->cells, st));
-        OTIF_CUDA(cudaEventRecord(p->ev_scored[c & 1], st));
-        OTIF_CUDA(cudaEventRecord(p->ev_imgfree[c & 1], st));
+        return run_pack(p, src, c0, cn, frame_base, p->windows + (size_t)c0 * per_frame, cn * per_frame,
+                        p->totals + c, p->slot + (size_t)c0 * per_frame, c > 0, sm);
+    };
+    if (p->ovl_mode == 1) {
+        // tensor stream: resize, proxy, select per chunk; memory stream: pack of finished chunks
+        for (int c = 0; c < nc; c++) {
+            const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
+            int t0 = tmark(p, st);
+            RC(otif_resize(src + (size_t)c0 * frame_bytes, cn, d.src_h, d.src_w, img[0], d.proxy.in_h, d.proxy.in_w, st));
+            tspan(p, ST_RESIZE, st, t0);
+            p->launches += 1;
+            RC(run_proxy(p, img[0], cn, p->scores + (size_t)c0 * p->cells, st));
+            RC(select_chunk(c, st));
+            OTIF_CUDA(cudaEventRecord(p->ev_scored[c & 1], st));
+            OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_scored[c & 1], 0));
+            RC(pack_chunk(c));
+        }
+    } else {
+        RC(resize_chunk(0));
+        for (int c = 0; c < nc; c++) {
+            if (c + 1 < nc) RC(resize_chunk(c + 1));
+            if (c >= 1) {
+                OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_scored[(c - 1) & 1], 0));
+                RC(select_chunk(c - 1, sm));
+                RC(pack_chunk(c - 1));
+            }
+            const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
+            OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_resized[c & 1], 0));
+            RC(run_proxy(p, img[c & 1], cn, p->scores + (size_t)c0 * p->cells, st));
+            OTIF_CUDA(cudaEventRecord(p->ev_scored[c & 1], st));
+            OTIF_CUDA(cudaEventRecord(p->ev_imgfree[c & 1], st));
+        }
+        OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_scored[(nc - 1) & 1], 0));
+        RC(select_chunk(nc - 1, sm));
+        RC(pack_chunk(nc - 1));
     }
-    RC(select_chunk(nc - 1));
     OTIF_CUDA(cudaEventRecord(p->ev_join, sm));
     OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_join, 0));
     return OTIF_OK;
@@ -280,6 +322,9 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
         p->pack_stages = (int)envi("OTIF_OVL_PACK_STAGES", 3);
         p->pack_stage_bytes = (int)envi("OTIF_OVL_PACK_STAGE", 12288);
         p->sel_smem_cap = (size_t)envi("OTIF_OVL_SEL_SMEM", 36 * 1024);
+        p->pack_threads = (int)envi("OTIF_OVL_PACK_THREADS", 32);
+        p->ovl_mode = (int)envi("OTIF_OVL_MODE", 1);
+        if (p->ovl_mode == 1) p->sel_smem_cap = 0;   // select runs on the tensor stream between proxy launches
         const size_t budget = (size_t)envi("OTIF_OVL_PROXY_SMEM", 184 * 1024);
         otif_status rc2 = proxy_set_smem_budget(p->proxy, budget);
         if (rc2 != OTIF_OK) { otif_pipeline_destroy(p); return rc2; }
@@ -293,6 +338,7 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     if (p->chunks >= 2) {
         PCUDA(cudaMalloc(&p->img2, (size_t)p->pb * d->proxy.in_h * d->proxy.in_w * 3));
         PCUDA(cudaStreamCreateWithFlags(&p->s_mem, cudaStreamNonBlocking));
+        PCUDA(cudaMalloc(&p->totals, (size_t)(p->chunks + 1) * 4));
         PCUDA(cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming));
         PCUDA(cudaEventCreateWithFlags(&p->ev_join, cudaEventDisableTiming));
         for (int i = 0; i < 2; i++) {
@@ -336,7 +382,7 @@ extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     if (p->s_compute) cudaStreamSynchronize(p->s_compute);
     if (p->s_copy) cudaStreamSynchronize(p->s_copy);
     if (p->s_mem) cudaStreamSynchronize(p->s_mem);
-    void *bufs[] = {p->src[0], p->src[1], p->img, p->img2, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
+    void *bufs[] = {p->src[0], p->src[1], p->img, p->img2, p->totals, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
                     p->offsets, p->total, p->slot, p->size_count, p->ctr, p->out_win, p->out_counts, p->out_total};
     for (void *b : bufs)
         if (b) cudaFree(b);
