@@ -282,18 +282,18 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                 int tap_pos = 0;
                 for (int cb = 0; cb < p.ncb; cb++) {
                     tap_pos = 0;
-                    for (int g = 0; g < p.ngroups; g++) {
+                                        for (int g = 0; g < p.ngroups; g++) {
                         mbar_wait(&a_empty[as], ap ^ 1);
                         mbar_arrive_expect_tx(&a_full[as], a_bytes);
                         uint8_t *dst = a_buf + (size_t)as * a_bytes;
                         const int plane = p.group_plane[g];
-                        for (uint32_t j = 0; j < chunks; j++) {
+                                                for (uint32_t j = 0; j < chunks; j++) {
                             const uint8_t *src =
                                 p.act + (((int64_t)plane * p.c8_in + cb * chunks + j) * p.lcap + q0) * 16;
                             bulk_g2s(dst + j * p.P * 16, src, p.P * 16, &a_full[as]);
                         }
                         if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
-                        for (int t = 0; t < p.group_ntaps[g]; t++, tap_pos++) {
+                                                for (int t = 0; t < p.group_ntaps[g]; t++, tap_pos++) {
                             mbar_wait(&b_empty[bs], bp ^ 1);
                             mbar_arrive_expect_tx(&b_full[bs], b_bytes);
                             bulk_g2s(b_buf + (size_t)bs * b_bytes, p.wpk + ((size_t)cb * 9 + tap_pos) * b_bytes, b_bytes,
@@ -317,16 +317,16 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                 const uint32_t d = tmem_base + acc * MT * p.N;
                 uint32_t accumulate = 0;
                 for (int cb = 0; cb < p.ncb; cb++) {
-                    for (int g = 0; g < p.ngroups; g++) {
+                                        for (int g = 0; g < p.ngroups; g++) {
                         mbar_wait(&a_full[as], ap);
                         tc_fence_after();
                         const uint32_t a_stage = a_base + as * a_bytes;
-                        for (int t = 0; t < p.group_ntaps[g]; t++) {
+                                                for (int t = 0; t < p.group_ntaps[g]; t++) {
                             mbar_wait(&b_full[bs], bp);
                             tc_fence_after();
                             const uint32_t a_tap = a_stage + p.group_shift[g][t] * 16;
                             const uint32_t b_stage = b_base + bs * b_bytes;
-                            for (uint32_t s = 0; s < chunks / 2; s++) {
+                                                        for (uint32_t s = 0; s < chunks / 2; s++) {
                                 const uint64_t bd = umma_desc(b_stage + 2 * s * lbo_b, lbo_b, 128);
                                 if (SWAP) {
                                     // weights = M operand, the 128*MT halo rows = N operand
@@ -711,8 +711,11 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma2_kernel(const __gri
 // chain stalls the other.  Roles (768 threads): warp 0 slab loader, warp 1 E1 MMA issuer,
 // warp 2 TMEM allocator, warp 3 E2 MMA issuer, warps 4-11 gather (2 warpgroups taking
 // alternate E1 M tiles), 12-19 E1 epilogue (likewise), 20-23 E2 epilogue.
-// Measured bound (ncu, C2): shared-memory bandwidth — N <= 64 MMAs read ~128 B/clk of
-// operands and the gather / epilogue stores share the same port.
+// Measured bound (ncu, C2): instruction fetch.  With 24 warps in 7 roles the kernel was
+// "stall_no_instructions"-bound (51% of warp samples; shared-memory pipe 29%, tensor pipe
+// 14%): knocking out ALL gather / epilogue / E2-tap work left 1.1 of its 1.6 ms.  The
+// per-plane loops (g, taps, k sub-tiles, M sub-tiles) are therefore kept rolled
+// (#pragma unroll 1): 5720 -> 3950 SASS instructions, 1.66 -> 0.97 ms per C2 step.
 // TMEM: E2 accumulators 2 x 128 columns at 0, E1 accumulators 2 plane slots x 32 KT at 256.
 // ---------------------------------------------------------------------------
 constexpr int kE12Threads = 768;
@@ -773,6 +776,35 @@ __device__ __forceinline__ void e12_decode(const E12Params &p, uint32_t q, uint3
     const uint32_t r1 = 2 * i - 1 < p.h1, c1 = 2 * j - 1 < p.w1;
     vmask = in ? (1u | (c1 << 1) | (r1 << 2) | ((r1 & c1) << 3)) : 0u;
     off = 4 * (gr - g0) * (uint32_t)p.slab_pitch + 12 * (uint32_t)j + 1;
+}
+
+// One im2col row of E1 (fp16, K = 32 with the bias slots) for E2-layout position with
+// decode (valid, off) in parity plane (rp, cp), read from the staged image slab.
+__device__ __forceinline__ void e12_im2col_row(const E12Params &p, const uint8_t *slab, uint32_t valid, uint32_t off,
+                                               int rp, int cp, uint32_t (&wv)[16]) {
+#pragma unroll
+    for (int j = 0; j < 16; j++) wv[j] = 0;
+    if (!valid || (p.trace & 4)) return;   // trace & 4: timing experiment (no gather)
+    const uint32_t b = off + 2 * rp * p.slab_pitch + 6 * cp;
+    const uint32_t sh = (b & 3) * 8;
+    const uint32_t *wp = reinterpret_cast<const uint32_t *>(slab + (b & ~3u));
+    uint32_t w[9];
+#pragma unroll
+    for (int kh = 0; kh < 3; kh++) {
+        const uint32_t *r = wp + kh * (p.slab_pitch >> 2);
+        w[3 * kh] = r[0]; w[3 * kh + 1] = r[1]; w[3 * kh + 2] = r[2];
+    }
+#pragma unroll
+    for (int kh = 0; kh < 3; kh++) {
+        const uint32_t w0 = w[3 * kh], w1 = w[3 * kh + 1], w2 = w[3 * kh + 2];
+        const uint32_t a0 = __funnelshift_r(w0, w1, sh), a1 = __funnelshift_r(w1, w2, sh);
+        wv[5 * kh + 0] = sub_f16x2(__byte_perm(a0, 0x64646464u, 0x4140), 0x64806480u);
+        wv[5 * kh + 1] = sub_f16x2(__byte_perm(a0, 0x64646464u, 0x4342), 0x64806480u);
+        wv[5 * kh + 2] = sub_f16x2(__byte_perm(a1, 0x64646464u, 0x4140), 0x64806480u);
+        wv[5 * kh + 3] = sub_f16x2(__byte_perm(a1, 0x64646464u, 0x4342), 0x64806480u);
+        // (u - 128, 128): the second half multiplies the bias part at K = 10 kh + 9
+        wv[5 * kh + 4] = sub_f16x2(0x64006400u | ((w2 >> sh) & 0xFFu), 0x63006480u);
+    }
 }
 
 #ifdef OTIF_E12_TRACE_BUILD   // hand-off timeline of CTA 0 (nvcc -DOTIF_E12_TRACE_BUILD; OTIF_E12_TRACE=1)
@@ -877,7 +909,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 const uint32_t f = fdiv(g, p.div_rpf);
                 const int i = (int)(g - f * rows_per_frame);
                 const int y = 4 * (i - 1) + k;
-                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp) my_bytes += p.row_bytes;
+                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp && !(p.trace & 64)) my_bytes += p.row_bytes;
             }
             if (p.bulk) {
 #pragma unroll
@@ -892,14 +924,16 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 const int i = (int)(g - f * rows_per_frame);
                 const int y = 4 * (i - 1) + k;
                 uint8_t *dst = slab + (size_t)s * p.slab_pitch;
-                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp) {
+                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp && !(p.trace & 64)) {   // 64: timing experiment
                     const uint8_t *src = p.img + ((size_t)f * p.hp + y) * p.row_bytes;
                     if (p.bulk) {
                         bulk_g2s(dst + 16, src, p.row_bytes, &slab_full[sb]);
                     } else {
+#pragma unroll 1
                         for (int b = 0; b < p.row_bytes; b++) dst[16 + b] = __ldg(src + b);
                     }
                 } else {
+#pragma unroll 1
                     for (int b = 0; b < p.slab_pitch; b += 16)
                         *reinterpret_cast<uint4 *>(dst + b) = make_uint4(0x80808080u, 0x80808080u, 0x80808080u, 0x80808080u);
                 }
@@ -959,7 +993,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 E12_TR(1, 0);
                 tc_fence_after();
                 const uint64_t a = a2d + ((pb * kPlaneBytes) >> 4);
-                for (int t = 0; t < p.group_ntaps[g]; t++, pos++) {
+                const int ntaps = (p.trace & 8) ? 1 : p.group_ntaps[g];   // trace & 8: timing experiment
+#pragma unroll 1
+                for (int t = 0; t < ntaps; t++, pos++) {
                     const uint64_t at = a + p.group_shift[g][t];          // +16 B per pixel of shift
                     const uint64_t bt = w2d + ((pos * (4 * N2 * 16)) >> 4);
 #pragma unroll
@@ -990,7 +1026,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
             for (int k = 0; k < KT; k++) e12_decode(p, q0 + k * 128 + row, g0, vm[k], of[k]);
             E12_WAIT_SLEEP(&slab_full[sb], sp);
             const uint8_t *slab = slab_s + (size_t)sb * slab_bytes;
-#pragma unroll
+#pragma unroll 1
             for (int g = 0; g < 4; g++, J++) {
                 const int rp = g >> 1, cp = g & 1;
                 const uint32_t s1 = (uint32_t)p.na1 == 1 ? 0 : (J & 1);
@@ -998,36 +1034,24 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 if (wg == 0) E12_TR(0, 0);
                 if constexpr (!TS) E12_WAIT_SLEEP(&a1_empty[s1], ph1 ^ 1);
                 if (wg == 0) E12_TR(1, 0);
-                uint32_t wk[2][16];   // this thread's rows of its (at most 2) k sub-tiles
+                uint32_t wk[2][16];   // TS: this thread's rows of its (at most 2) k sub-tiles
+                if constexpr (TS) {
 #pragma unroll
-                for (int k = 0; k < KT; k++) {
-                    if ((int)((J * KT + k) & 1) != wg) continue;
-                    uint32_t *wv = wk[k >> 1];   // k = 0, 2 -> slots 0, 1; k = 1 -> slot 0
-#pragma unroll
-                    for (int j = 0; j < 16; j++) wv[j] = 0;
-                    if ((vm[k] >> g) & 1) {
-                        const uint32_t b = of[k] + 2 * rp * p.slab_pitch + 6 * cp;
-                        const uint32_t sh = (b & 3) * 8;
-                        const uint32_t *wp = reinterpret_cast<const uint32_t *>(slab + (b & ~3u));
-                        uint32_t w[9];
-#pragma unroll
-                        for (int kh = 0; kh < 3; kh++) {
-                            const uint32_t *r = wp + kh * (p.slab_pitch >> 2);
-                            w[3 * kh] = r[0]; w[3 * kh + 1] = r[1]; w[3 * kh + 2] = r[2];
-                        }
-#pragma unroll
-                        for (int kh = 0; kh < 3; kh++) {
-                            const uint32_t w0 = w[3 * kh], w1 = w[3 * kh + 1], w2 = w[3 * kh + 2];
-                            const uint32_t a0 = __funnelshift_r(w0, w1, sh), a1 = __funnelshift_r(w1, w2, sh);
-                            wv[5 * kh + 0] = sub_f16x2(__byte_perm(a0, 0x64646464u, 0x4140), 0x64806480u);
-                            wv[5 * kh + 1] = sub_f16x2(__byte_perm(a0, 0x64646464u, 0x4342), 0x64806480u);
-                            wv[5 * kh + 2] = sub_f16x2(__byte_perm(a1, 0x64646464u, 0x4140), 0x64806480u);
-                            wv[5 * kh + 3] = sub_f16x2(__byte_perm(a1, 0x64646464u, 0x4342), 0x64806480u);
-                            // (u - 128, 128): the second half multiplies the bias part at K = 10 kh + 9
-                            wv[5 * kh + 4] = sub_f16x2(0x64006400u | ((w2 >> sh) & 0xFFu), 0x63006480u);
-                        }
+                    for (int k = 0; k < KT; k++) {
+                        if ((int)((J * KT + k) & 1) != wg) continue;
+                        e12_im2col_row(p, slab, (vm[k] >> g) & 1, of[k], rp, cp, wk[k >> 1]);
                     }
-                    if constexpr (!TS) {
+                } else {
+                    // rolled loop over this warpgroup's k sub-tiles (code size: the kernel is
+                    // instruction-cache bound, see the header)
+#pragma unroll 1
+                    for (int k = (int)((wg - J * KT) & 1); k < KT; k += 2) {
+                        uint32_t vmk = vm[0], ofk = of[0];
+#pragma unroll
+                        for (int i = 1; i < KT; i++)
+                            if (k == i) { vmk = vm[i]; ofk = of[i]; }
+                        uint32_t wv[16];
+                        e12_im2col_row(p, slab, (vmk >> g) & 1, ofk, rp, cp, wv);
                         uint8_t *dst = a1_s + s1 * kA1Bytes + k * 8192 + row * 16;
 #pragma unroll
                         for (int c = 0; c < 4; c++)
@@ -1067,7 +1091,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
         const int quarter = warp & 3;
         uint32_t J = 0, pb = 0, pp = 0;
         for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
-#pragma unroll
+#pragma unroll 1
             for (int g = 0; g < 4; g++, J++) {
                 E12_WAIT_SLEEP(&a2_empty[pb], pp ^ 1);
                 if (wg == 0) E12_TR(0, 0);
@@ -1076,9 +1100,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 tc_fence_after();
                 uint8_t *plane = a2_s + pb * kPlaneBytes;
                 const uint32_t tacc = tmem_base + ((uint32_t)(quarter * 32) << 16) + 256 + (J & 1) * (32 * KT);
-#pragma unroll
-                for (int k = 0; k < KT; k++) {
-                    if ((int)((J * KT + k) & 1) != wg) continue;
+#pragma unroll 1
+                for (int k = (int)((wg - J * KT) & 1); k < KT; k += 2) {
+                    if (p.trace & 32) continue;   // 32: timing experiment
                     uint32_t v[32];
                     tmem_ld32(tacc + k * 32, v);
                     uint32_t pk[16];
@@ -1107,6 +1131,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
         for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
             E12_WAIT_SLEEP(&acc_full[acc], accp);
             tc_fence_after();
+#pragma unroll 1
             for (int mm = 0; mm < MT; mm++) {
                 const uint32_t q = (uint32_t)tile * (128 * MT) + mm * 128 + row;
                 const uint32_t f = fdiv(q, p.div_fstride);
@@ -1121,7 +1146,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 for (int cc = 0; cc < N2 / 32; cc++) {
                     uint32_t v[32];
                     tmem_ld32(taddr + cc * 32, v);
-                    if (valid) {
+                    if (valid && !(p.trace & 16)) {   // 16: timing experiment
                         uint32_t pk[16];
 #pragma unroll
                         for (int j = 0; j < 16; j++)
