@@ -87,6 +87,18 @@ class ClockSampler:
                                        "-lms", "50"], stdout=self.f, stderr=subprocess.DEVNULL)
         except Exception:
             self.p = None
+        # nvidia-smi needs a few hundred ms to start sampling: wait for its first line so the
+        # samples cover the timed region, and keep only the lines written after this point
+        self.skip = 0
+        t0 = time.time()
+        while self.p is not None and time.time() - t0 < 5.0:
+            self.f.flush()
+            with open(self.f.name) as fh:
+                n = len(fh.read().splitlines())
+            if n > 0:
+                self.skip = n
+                break
+            time.sleep(0.02)
 
     def stop(self):
         if self.p is None:
@@ -100,7 +112,10 @@ class ClockSampler:
         self.f.seek(0)
         sm, smax, reasons = [], [], set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for line in self.f.read().splitlines():
+        lines = self.f.read().splitlines()
+        if len(lines) > self.skip:
+            lines = lines[self.skip:]      # samples taken during the timed region
+        for line in lines:
             parts = [x.strip() for x in line.split(",")]
             if len(parts) < 9:
                 continue
@@ -413,7 +428,7 @@ def run_otif(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["otif", "reference"], default="otif")
     ap.add_argument("--batch", type=int, default=0, help="device batch (0 = whole clip)")
