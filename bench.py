@@ -353,7 +353,7 @@ def run_otif(args):
         torch.cuda.synchronize()
         tms = t0e.elapsed_time(t1e) / args.steps
         train_flop = 3 * 2 * (sum(macs) + head) * len(tsel)      # forward + dgrad + wgrad
-        next3 = {"what": "fp32 training step (forward, BCE head, dgrad, wgrad, Adam) on CUDA cores",
+        next3 = {"what": "fp32 training step (forward, BCE head, dgrad, wgrad, Adam); convolution GEMMs on tcgen05 (3xTF32, fp32-accurate)",
                  "batch": len(tsel), "ms_per_step": tms, "train_frames_per_s": len(tsel) / (tms / 1e3),
                  "tflops": train_flop / (tms / 1e3) / 1e12, "loss_first": l0, "loss_last": float(lt.item())}
         del tr, timg, lab

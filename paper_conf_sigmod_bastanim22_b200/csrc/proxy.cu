@@ -721,22 +721,6 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma2_kernel(const __gri
 constexpr int kE12Threads = 768;
 constexpr int kE12MaxPlaneBufs = 3;
 
-// n / d for 0 <= n < 2^31 by multiply-high (d fixed per launch)
-struct FastDiv {
-    uint32_t d, m, s;
-};
-static FastDiv make_fastdiv(uint32_t d) {
-    FastDiv f;
-    f.d = d;
-    f.s = 0;
-    while ((1ull << f.s) < d) f.s++;
-    f.m = (uint32_t)(((1ull << 32) * ((1ull << f.s) - d)) / d + 1);
-    return f;
-}
-__device__ __forceinline__ uint32_t fdiv(uint32_t n, const FastDiv &f) {
-    return (uint32_t)(((uint64_t)__umulhi(n, f.m) + n) >> f.s);
-}
-
 struct E12Params {
     const uint8_t *img;         // u8 [n, hp, wp, 3]
     int n, hp, wp, row_bytes;   // row_bytes = 3 wp

@@ -1,8 +1,10 @@
 // train.cu — §8(f) NEXT-3, proxy training labels and training on sm_100a.
 //
 //   labels_kernel    P:L139 label 1 at every cell a detection intersects (thread per box).
-//   sgemm_kernel<Op> one fp32 SIMT implicit-GEMM template (64 x 64 x 16 tiles, 4 x 4 per
-//                    thread) instantiated for the three convolution products of training:
+//   tc_gemm_kernel<Op, BN> the tcgen05 implicit GEMM (3xTF32 split, fp32 accumulation in
+//                    TMEM, 128 x BN tiles, gathers through the Op) — the default; and
+//   sgemm_kernel<Op> the fp32 SIMT version of the same template (64 x 64 x 16 tiles, 4 x 4 per
+//                    thread, OTIF_TRAIN_SIMT=1), instantiated for the three convolution products:
 //                      FwdOp    y = ReLU(conv(x, W) + b)           M = pixels, N = Cout, K = 9 Cin
 //                      DgradOp  dx = conv^T(dy, W) ⊙ [x > 0]        M = input pixels, N = Cin, K = 9 Cout
 //                      WgradOp  dW | db = dy^T · im2col(x) | Σ dy   M = Cout, N = 9 Cin + 1, K = pixels
@@ -11,10 +13,11 @@
 //                    pre-activation gradient and per-warp D2 weight-gradient partials.
 //   adam_kernel      reading R27, fp32 master weights.
 //
-// Training runs in fp32 (weights, activations, gradients); the inference path keeps its
-// bf16 tcgen05 kernels and takes the trained weights through otif_proxy_create.  This is
-// the correctness-first cut of the training path: the convolution products run on the
-// CUDA cores, not yet on tcgen05.
+// Training runs in fp32 (weights, activations, gradients; the 3xTF32 products keep fp32
+// accuracy, so the gradients still match the fp64 oracle within 2e-4); the inference path
+// keeps its bf16 tcgen05 kernels and takes the trained weights through otif_proxy_create.
+// C2 batch-32 step: 16.0 ms (SIMT, integer divisions) -> 5.5 ms (tcgen05, multiply-high
+// divisors, coalesced K-contiguous staging, tensor-tile split-K, parallel head reduce).
 #include <math.h>
 #include <stdlib.h>
 #include <string.h>
@@ -98,9 +101,209 @@ __global__ void __launch_bounds__(GT) sgemm_kernel(Op op, int M, int N, int K, i
         }
 }
 
+
+// ---- tcgen05 implicit GEMM (3xTF32) ------------------------------------------------------
+// The same Op interface on the 5th-gen tensor cores.  fp32 operands are split into
+// x = hi + lo with hi = tf32(x) (round to nearest) and lo = x - hi (exact in fp32); the
+// product is accumulated in fp32 TMEM as hi·hi + hi·lo + lo·hi ("3xTF32"), which keeps
+// the gradients at fp32 accuracy (the dropped lo·lo term is ~2^-22 relative).
+// CTA: 256 threads load a 128 x 32 A chunk and a BN x 32 B chunk per stage (gathers
+// through op.a / op.b, thread = (row, 4 consecutive k): one 16-B shared store per thread
+// into the no-swizzle K-major core-matrix layout), 2 stages; warp 0 issues the 12 MMAs
+// (M128 x BN x K8, kind::tf32) of a stage and commits them to the stage's "empty"
+// barrier, so loads of chunk c+1 overlap the MMAs of chunk c.  Epilogue: tcgen05.ld
+// (lane = row) -> op.store.  Split-K over blockIdx.z exactly like sgemm_kernel.
+constexpr int kTcThreads = 256, kTcM = 128, kTcK = 32;
+
+__device__ __forceinline__ float tf32_rna(float x) {
+    uint32_t r;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+    return __uint_as_float(r);
+}
+
+__device__ __forceinline__ void umma_tf32_warp(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                               uint32_t accumulate) {
+    asm volatile(
+        "{\n\t.reg .pred p, e;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "elect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+        : "memory");
+}
+
+// stage rows [0, R) x 32 k of one operand: thread t owns row t % R (R divides the CTA size)
+// and k-groups t / R, t / R + 256 / R, ...; ctx = the row's context (op.a_row / op.b_row)
+template <int R, class Ctx, class F>
+__device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F get, int k0, int ke, uint8_t *hi,
+                                                 uint8_t *lo) {
+    static_assert(kTcThreads % R == 0, "rows per thread");
+    const int r = threadIdx.x % R;
+    constexpr int kIters = (kTcK / 4) / (kTcThreads / R);
+    // all the thread's loads first (kIters x 4 in flight: the gathers are latency-bound)
+    float v[kIters][4];
+#pragma unroll
+    for (int it = 0; it < kIters; it++) {
+        const int kg = (int)threadIdx.x / R + it * (kTcThreads / R);
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            const int k = k0 + kg * 4 + j;
+            v[it][j] = (row_ok && k < ke) ? get(ctx, k) : 0.f;
+        }
+    }
+#pragma unroll
+    for (int it = 0; it < kIters; it++) {
+        const int kg = (int)threadIdx.x / R + it * (kTcThreads / R);
+        float h[4], l[4];
+#pragma unroll
+        for (int j = 0; j < 4; j++) { h[j] = tf32_rna(v[it][j]); l[j] = v[it][j] - h[j]; }
+        const size_t off = ((size_t)kg * R + r) * 16;
+        *reinterpret_cast<float4 *>(hi + off) = make_float4(h[0], h[1], h[2], h[3]);
+        *reinterpret_cast<float4 *>(lo + off) = make_float4(l[0], l[1], l[2], l[3]);
+    }
+}
+
+// K-contiguous operands (Op::*_KFAST): a warp stages 8 rows x 4 k-groups per unit (lane:
+// row = l & 7, k-group = l >> 3), so each load instruction reads 64 contiguous bytes of 8
+// rows (vs 32 scattered rows) and each 8-lane store phase hits 8 distinct 16-B bank
+// groups.  Row contexts are recomputed per unit (mk: row -> context).
+template <int R, class MK, class F>
+__device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get, int k0, int ke, uint8_t *hi,
+                                               uint8_t *lo) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    constexpr int kUnits = (R / 8) * 2, kPerWarp = kUnits / (kTcThreads / 32);
+    static_assert(kUnits % (kTcThreads / 32) == 0, "units per warp");
+    float v[kPerWarp][4];
+#pragma unroll
+    for (int i = 0; i < kPerWarp; i++) {
+        const int u = warp + i * (kTcThreads / 32);
+        const int r = (u >> 1) * 8 + (lane & 7), kg = (u & 1) * 4 + (lane >> 3);
+        const bool ok = r < rows;
+        const auto q = mk(ok ? row0 + r : row0);
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            const int k = k0 + kg * 4 + j;
+            v[i][j] = (ok && k < ke) ? get(q, k) : 0.f;
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < kPerWarp; i++) {
+        const int u = warp + i * (kTcThreads / 32);
+        const int r = (u >> 1) * 8 + (lane & 7), kg = (u & 1) * 4 + (lane >> 3);
+        float h[4], l[4];
+#pragma unroll
+        for (int j = 0; j < 4; j++) { h[j] = tf32_rna(v[i][j]); l[j] = v[i][j] - h[j]; }
+        const size_t off = ((size_t)kg * R + r) * 16;
+        *reinterpret_cast<float4 *>(hi + off) = make_float4(h[0], h[1], h[2], h[3]);
+        *reinterpret_cast<float4 *>(lo + off) = make_float4(l[0], l[1], l[2], l[3]);
+    }
+}
+
+template <class Op, int BN>
+__global__ void __launch_bounds__(kTcThreads, 1) tc_gemm_kernel(Op op, int M, int N, int K, int k_split) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    constexpr uint32_t kA = kTcM * kTcK * 4, kB = BN * kTcK * 4, kStage = 2 * kA + 2 * kB;
+    __shared__ uint64_t full[2], empty[2], done;
+    __shared__ uint32_t tslot;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int m0 = blockIdx.x * kTcM, n0 = blockIdx.y * BN;
+    const int kb = blockIdx.z * k_split, ke = min(K, kb + k_split);
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < 2; i++) { mbar_init(&full[i], kTcThreads); mbar_init(&empty[i], 1); }
+        mbar_init(&done, 1);
+        fence_barrier_init();
+    }
+    if (warp == 0) tmem_alloc(&tslot, BN < 32 ? 32 : BN);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem = tslot;
+    const uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(kTcM >> 4) << 24);
+    const int nchunks = ke > kb ? (ke - kb + kTcK - 1) / kTcK : 0;
+    const int am = m0 + (int)threadIdx.x % kTcM, bn = n0 + (int)threadIdx.x % BN;
+    const bool a_ok = am < M, b_ok = bn < N;
+    const typename Op::ARow actx = op.a_row(a_ok ? am : 0);
+    const typename Op::BRow bctx = op.b_row(b_ok ? bn : 0);
+    for (int c = 0; c < nchunks; c++) {
+        const int st = c & 1;
+        if (c >= 2) mbar_wait(&empty[st], ((c >> 1) - 1) & 1);   // the MMAs of chunk c-2 read this stage
+        uint8_t *base = smem + (size_t)st * kStage;
+        const int k0 = kb + c * kTcK;
+        if constexpr (Op::A_KFAST)
+            tc_stage_kfast<kTcM>([&](int m) { return op.a_row(m); }, m0, M - m0,
+                                 [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); }, k0, ke, base, base + kA);
+        else
+            tc_stage_operand<kTcM>(actx, a_ok, [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); }, k0,
+                                   ke, base, base + kA);
+        if constexpr (Op::B_KFAST)
+            tc_stage_kfast<BN>([&](int n) { return op.b_row(n); }, n0, N - n0,
+                               [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); }, k0, ke, base + 2 * kA,
+                               base + 2 * kA + kB);
+        else
+            tc_stage_operand<BN>(bctx, b_ok, [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); }, k0, ke,
+                                 base + 2 * kA, base + 2 * kA + kB);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        mbar_arrive(&full[st]);
+        if (warp == 0) {
+            mbar_wait(&full[st], (c >> 1) & 1);
+            tc_fence_after();
+            const uint32_t ah = smem_u32(base), al = ah + kA, bh = ah + 2 * kA, bl = bh + kB;
+#pragma unroll
+            for (int s = 0; s < kTcK / 8; s++) {
+                const uint32_t ao = 2 * s * (kTcM * 16), bo = 2 * s * (BN * 16);
+                const uint64_t dah = umma_desc(ah + ao, kTcM * 16, 128), dal = umma_desc(al + ao, kTcM * 16, 128);
+                const uint64_t dbh = umma_desc(bh + bo, BN * 16, 128), dbl = umma_desc(bl + bo, BN * 16, 128);
+                umma_tf32_warp(tmem, dal, dbh, idesc, (c > 0 || s > 0) ? 1u : 0u);
+                umma_tf32_warp(tmem, dah, dbl, idesc, 1u);
+                umma_tf32_warp(tmem, dah, dbh, idesc, 1u);
+            }
+            umma_commit_warp(&empty[st]);
+        }
+    }
+    if (warp == 0) umma_commit_warp(&done);
+    mbar_wait(&done, 0);
+    tc_fence_after();
+    // epilogue: warp w reads lanes 32 (w & 3).. and columns [(w >> 2) BN/2, +BN/2)
+    const int row = (warp & 3) * 32 + lane, m = m0 + row;
+    constexpr int kHalf = BN / 2 < 32 ? BN : BN / 2;          // BN = 32: warps 0-3 take all columns
+    const int c_lo = (warp >> 2) * kHalf, c_hi = c_lo + kHalf < BN ? c_lo + kHalf : BN;
+#pragma unroll 1
+    for (int cc = c_lo; cc < c_hi; cc += 32) {
+        uint32_t v[32];
+        if (nchunks > 0) {
+            tmem_ld32(tmem + ((uint32_t)((warp & 3) * 32) << 16) + cc, v);
+        } else {
+#pragma unroll
+            for (int j = 0; j < 32; j++) v[j] = 0u;
+        }
+        if (m < M)
+            for (int j = 0; j < 32; j++) {
+                const int n = n0 + cc + j;
+                if (n < N) op.store(m, n, __uint_as_float(v[j]), blockIdx.z);
+            }
+    }
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 0) {
+        tc_fence_after();
+        tmem_dealloc(tmem, BN < 32 ? 32 : BN);
+    }
+}
+
 struct ConvGeom {
     int H, W, Cin, Ho, Wo, Cout, k, stride, pad;
+    // multiply-high divisors for the gathers' index math (set by with_divs on the host)
+    FastDiv dHoWo, dWo, dHW, dW, dCin, dCout, dK, dStride;
 };
+
+static ConvGeom with_divs(ConvGeom g) {
+    g.dHoWo = make_fastdiv((uint32_t)(g.Ho * g.Wo)); g.dWo = make_fastdiv((uint32_t)g.Wo);
+    g.dHW = make_fastdiv((uint32_t)(g.H * g.W)); g.dW = make_fastdiv((uint32_t)g.W);
+    g.dCin = make_fastdiv((uint32_t)g.Cin); g.dCout = make_fastdiv((uint32_t)g.Cout);
+    g.dK = make_fastdiv((uint32_t)g.k); g.dStride = make_fastdiv((uint32_t)g.stride);
+    return g;
+}
+__device__ __forceinline__ int dv(int n, const FastDiv &d) { return (int)fdiv((uint32_t)n, d); }
 
 template <typename T>
 __device__ __forceinline__ float act_in(const T *x, int64_t idx);
@@ -120,14 +323,24 @@ struct FwdOp {
     float *y;
     ConvGeom g;
     int relu;
-    __device__ float a(int m, int k) const {
-        const int hw = g.Ho * g.Wo, f = m / hw, r = m - f * hw, oy = r / g.Wo, ox = r - oy * g.Wo;
-        const int tap = k / g.Cin, ci = k - tap * g.Cin, kh = tap / g.k, kw = tap - kh * g.k;
-        const int iy = oy * g.stride - g.pad + kh, ix = ox * g.stride - g.pad + kw;
-        if (iy < 0 || iy >= g.H || ix < 0 || ix >= g.W) return 0.f;
-        return act_in<T>(x, (((int64_t)f * g.H + iy) * g.W + ix) * g.Cin + ci);
+    // row contexts: the pixel of row m (A) / the weight row n (B) are fixed per thread in
+    // tc_gemm_kernel, so their index math is done once
+    struct ARow { int f, iy0, ix0; };
+    __device__ ARow a_row(int m) const {
+        const int f = dv(m, g.dHoWo), r = m - f * g.Ho * g.Wo, oy = dv(r, g.dWo), ox = r - oy * g.Wo;
+        return {f, oy * g.stride - g.pad, ox * g.stride - g.pad};
     }
-    __device__ float b(int k, int n) const { return w[(int64_t)n * (g.k * g.k * g.Cin) + k]; }
+    __device__ float a_at(const ARow &q, int k) const {
+        const int tap = dv(k, g.dCin), ci = k - tap * g.Cin, kh = dv(tap, g.dK), kw = tap - kh * g.k;
+        const int iy = q.iy0 + kh, ix = q.ix0 + kw;
+        if (iy < 0 || iy >= g.H || ix < 0 || ix >= g.W) return 0.f;
+        return act_in<T>(x, (((int64_t)q.f * g.H + iy) * g.W + ix) * g.Cin + ci);
+    }
+    using BRow = const float *;
+    __device__ BRow b_row(int n) const { return w + (int64_t)n * (g.k * g.k * g.Cin); }
+    __device__ float b_at(BRow q, int k) const { return q[k]; }
+    __device__ float a(int m, int k) const { return a_at(a_row(m), k); }
+    __device__ float b(int k, int n) const { return b_at(b_row(n), k); }
     __device__ void store(int m, int n, float v, int) const {
         v += bias[n];
         y[(int64_t)m * g.Cout + n] = relu ? fmaxf(v, 0.f) : v;
@@ -142,19 +355,27 @@ struct DgradOp {
     const float *dy, *w, *xpost;
     float *dx;
     ConvGeom g;
-    __device__ float a(int m, int k) const {
-        const int hw = g.H * g.W, f = m / hw, r = m - f * hw, iy = r / g.W, ix = r - iy * g.W;
-        const int tap = k / g.Cout, co = k - tap * g.Cout, kh = tap / g.k, kw = tap - kh * g.k;
-        const int ty = iy + g.pad - kh, tx = ix + g.pad - kw;
-        if (ty < 0 || tx < 0) return 0.f;
-        const int oy = ty / g.stride, ox = tx / g.stride;
-        if (oy * g.stride != ty || ox * g.stride != tx || oy >= g.Ho || ox >= g.Wo) return 0.f;
-        return dy[(((int64_t)f * g.Ho + oy) * g.Wo + ox) * g.Cout + co];
+    struct ARow { int f, ty0, tx0; };
+    __device__ ARow a_row(int m) const {
+        const int f = dv(m, g.dHW), r = m - f * g.H * g.W, iy = dv(r, g.dW), ix = r - iy * g.W;
+        return {f, iy + g.pad, ix + g.pad};
     }
-    __device__ float b(int k, int n) const {
-        const int tap = k / g.Cout, co = k - tap * g.Cout;
+    __device__ float a_at(const ARow &q, int k) const {
+        const int tap = dv(k, g.dCout), co = k - tap * g.Cout, kh = dv(tap, g.dK), kw = tap - kh * g.k;
+        const int ty = q.ty0 - kh, tx = q.tx0 - kw;
+        if (ty < 0 || tx < 0) return 0.f;
+        const int oy = dv(ty, g.dStride), ox = dv(tx, g.dStride);
+        if (oy * g.stride != ty || ox * g.stride != tx || oy >= g.Ho || ox >= g.Wo) return 0.f;
+        return dy[(((int64_t)q.f * g.Ho + oy) * g.Wo + ox) * g.Cout + co];
+    }
+    using BRow = int;
+    __device__ BRow b_row(int n) const { return n; }
+    __device__ float b_at(BRow n, int k) const {
+        const int tap = dv(k, g.dCout), co = k - tap * g.Cout;
         return w[((int64_t)co * g.k * g.k + tap) * g.Cin + n];
     }
+    __device__ float a(int m, int k) const { return a_at(a_row(m), k); }
+    __device__ float b(int k, int n) const { return b_at(b_row(n), k); }
     __device__ void store(int m, int n, float v, int) const {
         const int64_t i = (int64_t)m * g.Cin + n;
         dx[i] = xpost[i] > 0.f ? v : 0.f;
@@ -170,15 +391,24 @@ struct WgradOp {
     float *part;        // [split][Cout][K + 1]
     ConvGeom g;
     int Kw;             // k*k*Cin
-    __device__ float a(int m, int p) const { return dy[(int64_t)p * g.Cout + m]; }
-    __device__ float b(int p, int kk) const {
-        if (kk == Kw) return 1.f;
-        const int hw = g.Ho * g.Wo, f = p / hw, r = p - f * hw, oy = r / g.Wo, ox = r - oy * g.Wo;
-        const int tap = kk / g.Cin, ci = kk - tap * g.Cin, kh = tap / g.k, kw = tap - kh * g.k;
-        const int iy = oy * g.stride - g.pad + kh, ix = ox * g.stride - g.pad + kw;
-        if (iy < 0 || iy >= g.H || ix < 0 || ix >= g.W) return 0.f;
-        return act_in<T>(x, (((int64_t)f * g.H + iy) * g.W + ix) * g.Cin + ci);
+    using ARow = int;
+    __device__ ARow a_row(int m) const { return m; }
+    __device__ float a_at(ARow co, int p) const { return dy[(int64_t)p * g.Cout + co]; }
+    struct BRow { int bias, ci, kh, kw; };
+    __device__ BRow b_row(int kk) const {
+        if (kk == Kw) return {1, 0, 0, 0};
+        const int tap = dv(kk, g.dCin), kh = dv(tap, g.dK);
+        return {0, kk - tap * g.Cin, kh, tap - kh * g.k};
     }
+    __device__ float b_at(const BRow &q, int p) const {
+        if (q.bias) return 1.f;
+        const int f = dv(p, g.dHoWo), r = p - f * g.Ho * g.Wo, oy = dv(r, g.dWo), ox = r - oy * g.Wo;
+        const int iy = oy * g.stride - g.pad + q.kh, ix = ox * g.stride - g.pad + q.kw;
+        if (iy < 0 || iy >= g.H || ix < 0 || ix >= g.W) return 0.f;
+        return act_in<T>(x, (((int64_t)f * g.H + iy) * g.W + ix) * g.Cin + q.ci);
+    }
+    __device__ float a(int m, int p) const { return a_at(a_row(m), p); }
+    __device__ float b(int p, int kk) const { return b_at(b_row(kk), p); }
     __device__ void store(int m, int n, float v, int split) const {
         part[((int64_t)split * g.Cout + m) * (Kw + 1) + n] = v;
     }
@@ -246,16 +476,27 @@ __global__ void __launch_bounds__(kHeadWarps * 32) head_kernel(const float *__re
     }
 }
 
-// fixed-order reduction of the head partials -> grad (W2, b2) and the mean loss
-__global__ void head_reduce_kernel(const float *__restrict__ part, int64_t nwarps, int dec, int64_t M,
-                                   float *__restrict__ grad_w2, float *__restrict__ loss) {
-    for (int c = threadIdx.x; c < dec + 2; c += blockDim.x) {
-        float s = 0.f;
-        for (int64_t w = 0; w < nwarps; w++) s += part[w * (dec + 2) + c];
+// fixed-order reduction of the head partials -> grad (W2, b2) and the mean loss: one CTA
+// per column, each thread a fixed strided subset, then a fixed shared-memory tree
+// (deterministic: the order never depends on scheduling)
+__global__ void __launch_bounds__(256) head_reduce_kernel(const float *__restrict__ part, int64_t nwarps, int dec,
+                                                          int64_t M, float *__restrict__ grad_w2,
+                                                          float *__restrict__ loss) {
+    __shared__ float red[256];
+    const int c = blockIdx.x;
+    float s = 0.f;
+    for (int64_t w = threadIdx.x; w < nwarps; w += blockDim.x) s += part[w * (dec + 2) + c];
+    red[threadIdx.x] = s;
+    __syncthreads();
+    for (int h = 128; h > 0; h >>= 1) {
+        if ((int)threadIdx.x < h) red[threadIdx.x] += red[threadIdx.x + h];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) {
         if (c <= dec)
-            grad_w2[c] = s;                       // W2[0..dec-1], then b2
+            grad_w2[c] = red[0];                  // W2[0..dec-1], then b2
         else
-            *loss = s / (float)M;
+            *loss = red[0] / (float)M;
     }
 }
 
@@ -272,9 +513,43 @@ __global__ void adam_kernel(float *__restrict__ w, float *__restrict__ m, float 
     }
 }
 
+// 1 = tcgen05 3xTF32 (default), 0 = SIMT fp32 (OTIF_TRAIN_SIMT=1, A/B runs)
+static int train_tc() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("OTIF_TRAIN_SIMT");
+        v = (e && e[0] == '1') ? 0 : 1;
+    }
+    return v;
+}
+
 template <class Op>
 otif_status run_gemm(const Op &op, int64_t M, int64_t N, int64_t K, int splits, cudaStream_t stream) {
     if (M <= 0 || N <= 0) return OTIF_OK;
+    if (train_tc()) {
+        const int64_t k_split = round_up(cdiv(K, splits), kTcK);
+        if (N <= 32) {
+            constexpr int BNv = 32;
+            const size_t smem = 2 * (2 * (size_t)kTcM * kTcK * 4 + 2 * (size_t)BNv * kTcK * 4);
+            OTIF_CUDA(cudaFuncSetAttribute(tc_gemm_kernel<Op, BNv>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            const dim3 grid((unsigned)cdiv(M, kTcM), (unsigned)cdiv(N, BNv), (unsigned)splits);
+            tc_gemm_kernel<Op, BNv><<<grid, kTcThreads, smem, stream>>>(op, (int)M, (int)N, (int)K, (int)k_split);
+        } else if (N <= 64) {
+            constexpr int BNv = 64;
+            const size_t smem = 2 * (2 * (size_t)kTcM * kTcK * 4 + 2 * (size_t)BNv * kTcK * 4);
+            OTIF_CUDA(cudaFuncSetAttribute(tc_gemm_kernel<Op, BNv>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            const dim3 grid((unsigned)cdiv(M, kTcM), (unsigned)cdiv(N, BNv), (unsigned)splits);
+            tc_gemm_kernel<Op, BNv><<<grid, kTcThreads, smem, stream>>>(op, (int)M, (int)N, (int)K, (int)k_split);
+        } else {
+            constexpr int BNv = 128;
+            const size_t smem = 2 * (2 * (size_t)kTcM * kTcK * 4 + 2 * (size_t)BNv * kTcK * 4);
+            OTIF_CUDA(cudaFuncSetAttribute(tc_gemm_kernel<Op, BNv>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            const dim3 grid((unsigned)cdiv(M, kTcM), (unsigned)cdiv(N, BNv), (unsigned)splits);
+            tc_gemm_kernel<Op, BNv><<<grid, kTcThreads, smem, stream>>>(op, (int)M, (int)N, (int)K, (int)k_split);
+        }
+        OTIF_LAUNCH_CHECK();
+        return OTIF_OK;
+    }
     const int64_t k_split = round_up(cdiv(K, splits), BK);
     const dim3 grid((unsigned)cdiv(M, BM), (unsigned)cdiv(N, BN), (unsigned)splits);
     sgemm_kernel<Op><<<grid, GT, 0, stream>>>(op, (int)M, (int)N, (int)K, (int)k_split);
@@ -305,7 +580,10 @@ struct otif_trainer {
 
 static int wgrad_splits(const otif_trainer *t, int L, int n) {
     const int64_t pixels = (int64_t)n * t->hs[L + 1] * t->ws[L + 1];
-    const int64_t tiles = cdiv(t->cout[L], BM) * cdiv((int64_t)t->ks[L] * t->ks[L] * t->cin[L] + 1, BN);
+    const int64_t kw1 = (int64_t)t->ks[L] * t->ks[L] * t->cin[L] + 1;
+    // output tiles of the GEMM kernel in use (tcgen05: 128 x 32/64/128; SIMT: 64 x 64)
+    const int64_t tiles = train_tc() ? cdiv(t->cout[L], kTcM) * cdiv(kw1, kw1 <= 32 ? 32 : kw1 <= 64 ? 64 : 128)
+                                     : cdiv(t->cout[L], BM) * cdiv(kw1, BN);
     int64_t s = cdiv(2 * (int64_t)t->sms, tiles);
     s = std::min<int64_t>(s, std::max<int64_t>(1, pixels / 256));
     return (int)std::max<int64_t>(1, std::min<int64_t>(s, 512));
@@ -444,7 +722,7 @@ extern "C" otif_status otif_trainer_backward(otif_trainer *t, const uint8_t *img
         ConvGeom g;
         g.H = t->hs[L]; g.W = t->ws[L]; g.Cin = t->cin[L]; g.Ho = t->hs[L + 1]; g.Wo = t->ws[L + 1];
         g.Cout = t->cout[L]; g.k = t->ks[L]; g.stride = t->stride[L]; g.pad = (t->ks[L] - 1) / 2;
-        return g;
+        return with_divs(g);
     };
     // forward E1..D1 (D2 lives in the head kernel)
     for (int L = 0; L < 6; L++) {
@@ -467,7 +745,7 @@ extern "C" otif_status otif_trainer_backward(otif_trainer *t, const uint8_t *img
     head_kernel<<<(unsigned)(t->head_warps / kHeadWarps), kHeadWarps * 32, 0, stream>>>(
         t->act[6], t->w + t->woff[6], labels, cells, dec, t->dbuf[0], t->part);
     OTIF_LAUNCH_CHECK();
-    head_reduce_kernel<<<1, 256, 0, stream>>>(t->part, t->head_warps, dec, cells, t->grad + t->woff[6], loss);
+    head_reduce_kernel<<<(unsigned)(dec + 2), 256, 0, stream>>>(t->part, t->head_warps, dec, cells, t->grad + t->woff[6], loss);
     OTIF_LAUNCH_CHECK();
     // backward D1 .. E1
     int cur = 0;
