@@ -356,6 +356,13 @@ def run_otif(args):
         next3 = {"what": "fp32 training step (forward, BCE head, dgrad, wgrad, Adam); convolution GEMMs on tcgen05 (3xTF32, fp32-accurate)",
                  "batch": len(tsel), "ms_per_step": tms, "train_frames_per_s": len(tsel) / (tms / 1e3),
                  "tflops": train_flop / (tms / 1e3) / 1e12, "loss_first": l0, "loss_last": float(lt.item())}
+        # roofline of the training GEMMs: tf32 peak = measured sustained bf16 x the guide's
+        # nominal tf32/bf16 ratio (1.1 / 2.25); 3xTF32 issues 3 MMAs per useful product
+        tf32_peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))) * 1.1 / 2.25
+        next3["roofline"] = {"bound": "tensor", "unit": "TFLOP/s", "achieved": next3["tflops"],
+                             "peak": tf32_peak / 3.0, "frac": next3["tflops"] / (tf32_peak / 3.0),
+                             "peak_source": "measured bf16 sustained x 1.1/2.25 (tf32), / 3 (3xTF32 useful rate); "
+                                            "the step is bound by the implicit-GEMM gathers, not the MMAs"}
         del tr, timg, lab
 
     # end to end through the C ABI with HOST frames: pinned H2D + D2H inside the timed region

@@ -113,7 +113,13 @@ __global__ void __launch_bounds__(GT) sgemm_kernel(Op op, int M, int N, int K, i
 // (M128 x BN x K8, kind::tf32) of a stage and commits them to the stage's "empty"
 // barrier, so loads of chunk c+1 overlap the MMAs of chunk c.  Epilogue: tcgen05.ld
 // (lane = row) -> op.store.  Split-K over blockIdx.z exactly like sgemm_kernel.
-constexpr int kTcThreads = 256, kTcM = 128, kTcK = 32;
+#ifndef OTIF_TC_K
+#define OTIF_TC_K 16          // k per shared-memory stage (16: 3 CTAs per SM at BN = 128)
+#endif
+#ifndef OTIF_TC_MINB
+#define OTIF_TC_MINB 2
+#endif
+constexpr int kTcThreads = 256, kTcM = 128, kTcK = OTIF_TC_K;
 
 __device__ __forceinline__ float tf32_rna(float x) {
     uint32_t r;
@@ -139,7 +145,9 @@ __device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F 
                                                  uint8_t *lo) {
     static_assert(kTcThreads % R == 0, "rows per thread");
     const int r = threadIdx.x % R;
-    constexpr int kIters = (kTcK / 4) / (kTcThreads / R);
+    constexpr int kKG = kTcK / 4, kStep = kTcThreads / R;
+    constexpr int kIters = (kKG + kStep - 1) / kStep;
+    if ((int)threadIdx.x / R >= kKG) return;   // more threads than (row, k-group) units
     // all the thread's loads first (kIters x 4 in flight: the gathers are latency-bound)
     float v[kIters][4];
 #pragma unroll
@@ -148,12 +156,13 @@ __device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F 
 #pragma unroll
         for (int j = 0; j < 4; j++) {
             const int k = k0 + kg * 4 + j;
-            v[it][j] = (row_ok && k < ke) ? get(ctx, k) : 0.f;
+            v[it][j] = (row_ok && kg < kKG && k < ke) ? get(ctx, k) : 0.f;
         }
     }
 #pragma unroll
     for (int it = 0; it < kIters; it++) {
         const int kg = (int)threadIdx.x / R + it * (kTcThreads / R);
+        if (kg >= kKG) continue;
         float h[4], l[4];
 #pragma unroll
         for (int j = 0; j < 4; j++) { h[j] = tf32_rna(v[it][j]); l[j] = v[it][j] - h[j]; }
@@ -171,14 +180,15 @@ template <int R, class MK, class F>
 __device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get, int k0, int ke, uint8_t *hi,
                                                uint8_t *lo) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    constexpr int kUnits = (R / 8) * 2, kPerWarp = kUnits / (kTcThreads / 32);
-    static_assert(kUnits % (kTcThreads / 32) == 0, "units per warp");
+    constexpr int kGroups = kTcK / 16;                       // groups of 4 k-groups
+    constexpr int kUnits = (R / 8) * kGroups, kWarps = kTcThreads / 32;
+    constexpr int kPerWarp = (kUnits + kWarps - 1) / kWarps;
     float v[kPerWarp][4];
 #pragma unroll
     for (int i = 0; i < kPerWarp; i++) {
-        const int u = warp + i * (kTcThreads / 32);
-        const int r = (u >> 1) * 8 + (lane & 7), kg = (u & 1) * 4 + (lane >> 3);
-        const bool ok = r < rows;
+        const int u = warp + i * kWarps;
+        const int r = (u / kGroups) * 8 + (lane & 7), kg = (u % kGroups) * 4 + (lane >> 3);
+        const bool ok = u < kUnits && r < rows;
         const auto q = mk(ok ? row0 + r : row0);
 #pragma unroll
         for (int j = 0; j < 4; j++) {
@@ -188,8 +198,9 @@ __device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get,
     }
 #pragma unroll
     for (int i = 0; i < kPerWarp; i++) {
-        const int u = warp + i * (kTcThreads / 32);
-        const int r = (u >> 1) * 8 + (lane & 7), kg = (u & 1) * 4 + (lane >> 3);
+        const int u = warp + i * kWarps;
+        if (u >= kUnits) continue;
+        const int r = (u / kGroups) * 8 + (lane & 7), kg = (u % kGroups) * 4 + (lane >> 3);
         float h[4], l[4];
 #pragma unroll
         for (int j = 0; j < 4; j++) { h[j] = tf32_rna(v[i][j]); l[j] = v[i][j] - h[j]; }
@@ -200,7 +211,7 @@ __device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get,
 }
 
 template <class Op, int BN>
-__global__ void __launch_bounds__(kTcThreads, 1) tc_gemm_kernel(Op op, int M, int N, int K, int k_split) {
+__global__ void __launch_bounds__(kTcThreads, OTIF_TC_MINB) tc_gemm_kernel(Op op, int M, int N, int K, int k_split) {
     extern __shared__ __align__(1024) uint8_t smem[];
     constexpr uint32_t kA = kTcM * kTcK * 4, kB = BN * kTcK * 4, kStage = 2 * kA + 2 * kB;
     __shared__ uint64_t full[2], empty[2], done;
