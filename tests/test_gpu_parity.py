@@ -112,6 +112,22 @@ def test_proxy_e1_fused_vs_separate(h, w, ns, n, blob, monkeypatch):
     assert np.median(np.abs(a - b)) <= 1e-4
 
 
+@pytest.mark.parametrize("h,w,ns,n", [(135, 240, 3, 3), (67, 123, 3, 3), (45, 90, 2, 3)])
+def test_proxy_e12_ts_mode_matches_ss(h, w, ns, n, blob, monkeypatch):
+    """OTIF_E12_TS=1 (E1's im2col rows in TMEM, A-from-TMEM MMA) computes the same E1
+    sums (exact fp16 products, fp32 accumulation in the same K order) as the default
+    shared-memory operand path, so the scores are identical."""
+    rng = np.random.default_rng(h * 7 + w)
+    img = torch.from_numpy(rng.integers(0, 256, (n, h, w, 3), dtype=np.uint8)).cuda()
+    ss = otif.Proxy(h, w, ns, blob)
+    monkeypatch.setenv("OTIF_E12_TS", "1")
+    ts = otif.Proxy(h, w, ns, blob)
+    monkeypatch.delenv("OTIF_E12_TS")
+    a = ss.score(img).cpu().numpy()
+    b = ts.score(img).cpu().numpy()
+    assert np.array_equal(a, b)
+
+
 def test_proxy_repeat_calls_reuse_workspace(blob):
     wl = configs.C1
     img = torch.from_numpy(oracle.resize(_frames(wl, 8).numpy(), wl.proxy_h, wl.proxy_w)).cuda()
