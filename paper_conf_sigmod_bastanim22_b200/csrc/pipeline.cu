@@ -16,6 +16,7 @@
 // shared-memory budget so that a pack (bulk-copy ring) or resize CTA fits on every SM
 // next to a proxy CTA.  Slots continue across the chunks (pack accumulates size_count),
 // so the detector batches hold the same windows in the same order as the serial schedule.
+#include <cuda.h>
 #include <stdlib.h>
 #include <string.h>
 
@@ -40,6 +41,7 @@ otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t sr
                         int stage_bytes, int threads);
 otif_status proxy_set_smem_budget(otif_proxy *p, size_t budget);
 int proxy_launches(const otif_proxy *p);
+void proxy_set_num_sms(otif_proxy *p, int sms);
 
 // timing stages: resize, proxy prep (tag + E1), E2, E3, E4, E5, D1+D2, select, pack, append
 constexpr int kStages = 10;
@@ -72,6 +74,39 @@ __global__ void __launch_bounds__(1024) append_kernel(const otif_window *__restr
 
 using namespace otif;
 
+
+// Driver entry points of the green-context API, fetched through the runtime so that
+// libotif.so does not link libcuda (it must load on hosts without a driver).
+struct GreenApi {
+    CUresult (*DeviceGet)(CUdevice *, int);
+    CUresult (*DeviceGetDevResource)(CUdevice, CUdevResource *, CUdevResourceType);
+    CUresult (*DevSmResourceSplitByCount)(CUdevResource *, unsigned *, const CUdevResource *, CUdevResource *,
+                                          unsigned, unsigned);
+    CUresult (*DevResourceGenerateDesc)(CUdevResourceDesc *, CUdevResource *, unsigned);
+    CUresult (*GreenCtxCreate)(CUgreenCtx *, CUdevResourceDesc, CUdevice, unsigned);
+    CUresult (*GreenCtxStreamCreate)(CUstream *, CUgreenCtx, unsigned, int);
+    CUresult (*GreenCtxDestroy)(CUgreenCtx);
+};
+static const char *g_green_missing = "";
+static bool green_api(GreenApi &g) {
+    auto get = [](const char *name, void **fn) {
+        cudaDriverEntryPointQueryResult q = cudaDriverEntryPointSymbolNotFound;
+        *fn = nullptr;
+        if (cudaGetDriverEntryPointByVersion(name, fn, 12080, cudaEnableDefault, &q) != cudaSuccess || !*fn) {
+            cudaGetLastError();
+            if (cudaGetDriverEntryPoint(name, fn, cudaEnableDefault, &q) != cudaSuccess) cudaGetLastError();
+        }
+        if (!*fn) g_green_missing = name;
+        return *fn != nullptr;
+    };
+    return get("cuDeviceGet", (void **)&g.DeviceGet) && get("cuDeviceGetDevResource", (void **)&g.DeviceGetDevResource) &&
+           get("cuDevSmResourceSplitByCount", (void **)&g.DevSmResourceSplitByCount) &&
+           get("cuDevResourceGenerateDesc", (void **)&g.DevResourceGenerateDesc) &&
+           get("cuGreenCtxCreate", (void **)&g.GreenCtxCreate) &&
+           get("cuGreenCtxStreamCreate", (void **)&g.GreenCtxStreamCreate) &&
+           get("cuGreenCtxDestroy", (void **)&g.GreenCtxDestroy);
+}
+
 struct otif_pipeline {
     otif_pipeline_desc d;
     otif_proxy *proxy = nullptr;
@@ -99,6 +134,10 @@ struct otif_pipeline {
     int *totals = nullptr;  // [chunks] per-chunk window totals (overlap)
     size_t sel_smem_cap = 0;
     cudaStream_t s_mem = nullptr;
+    // partitioned overlap (OTIF_OVL_GREEN = SMs for the memory stages): two green contexts
+    // split the SMs; the proxy runs on s_tensor (its partition), resize/select/pack on s_mem
+    CUgreenCtx g_tensor = nullptr, g_mem = nullptr;
+    cudaStream_t s_tensor = nullptr;
     cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_resized[2] = {}, ev_scored[2] = {}, ev_imgfree[2] = {};
     // optional per-stage timing: a log of spans (stage, start entry, end event); a span's
     // time is charged to its stage (stage < 0: a start marker)
@@ -209,8 +248,15 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
         RC(run_select(p, 0, nb, frame_base, p->windows, p->cap_w, p->total, st));
         return run_pack(p, src, 0, nb, frame_base, p->windows, p->cap_w, p->total, p->slot, 0, st);
     }
-    // overlap: st = tensor stream (proxy), s_mem = memory stream (resize, select, pack)
+    // overlap: st = tensor stream (proxy), s_mem = memory stream (resize, select, pack); with
+    // an SM partition the proxy runs on the tensor partition's stream, joined back to st
     cudaStream_t sm = p->s_mem;
+    cudaStream_t caller = st;
+    if (p->s_tensor) {
+        OTIF_CUDA(cudaEventRecord(p->ev_fork, caller));
+        OTIF_CUDA(cudaStreamWaitEvent(p->s_tensor, p->ev_fork, 0));
+        st = p->s_tensor;
+    }
     uint8_t *img[2] = {p->img, p->img2};
     const int cs = p->chunk;
     const int nc = (nb + cs - 1) / cs;
@@ -274,6 +320,10 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
     }
     OTIF_CUDA(cudaEventRecord(p->ev_join, sm));
     OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_join, 0));
+    if (st != caller) {
+        OTIF_CUDA(cudaEventRecord(p->ev_join, st));
+        OTIF_CUDA(cudaStreamWaitEvent(caller, p->ev_join, 0));
+    }
     return OTIF_OK;
 }
 
@@ -325,9 +375,54 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
         p->pack_threads = (int)envi("OTIF_OVL_PACK_THREADS", 32);
         p->ovl_mode = (int)envi("OTIF_OVL_MODE", 1);
         if (p->ovl_mode == 1) p->sel_smem_cap = 0;   // select runs on the tensor stream between proxy launches
-        const size_t budget = (size_t)envi("OTIF_OVL_PROXY_SMEM", 184 * 1024);
-        otif_status rc2 = proxy_set_smem_budget(p->proxy, budget);
-        if (rc2 != OTIF_OK) { otif_pipeline_destroy(p); return rc2; }
+        const int green = (int)envi("OTIF_OVL_GREEN", 0);
+        if (green <= 0) {
+            const size_t budget = (size_t)envi("OTIF_OVL_PROXY_SMEM", 184 * 1024);
+            otif_status rc2 = proxy_set_smem_budget(p->proxy, budget);
+            if (rc2 != OTIF_OK) { otif_pipeline_destroy(p); return rc2; }
+        } else {
+            // SM partition instead of co-residence: the proxy keeps its full shared memory
+            p->ovl_mode = 0;
+            p->sel_smem_cap = 0;
+            p->pack_ctas = 0;
+            p->pack_threads = 128;
+            p->pack_stages = 3;
+            p->pack_stage_bytes = 16384;
+            int dev = 0;
+            PCUDA(cudaGetDevice(&dev));
+            GreenApi ga;
+            if (!green_api(ga)) {
+                set_error("otif_pipeline_create: green-context driver entry point %s unavailable", g_green_missing);
+                otif_pipeline_destroy(p);
+                return OTIF_EUNSUPPORTED;
+            }
+            CUdevice cdev;
+            CUdevResource all, parts[1], rest;
+            CUdevResourceDesc d_t, d_m;
+            unsigned nparts = 1;
+            const unsigned tensor_sms = (unsigned)((num_sms - green) / 8 * 8);
+            if (ga.DeviceGet(&cdev, dev) != CUDA_SUCCESS ||
+                ga.DeviceGetDevResource(cdev, &all, CU_DEV_RESOURCE_TYPE_SM) != CUDA_SUCCESS ||
+                ga.DevSmResourceSplitByCount(parts, &nparts, &all, &rest, 0, tensor_sms) != CUDA_SUCCESS || nparts != 1 ||
+                ga.DevResourceGenerateDesc(&d_t, &parts[0], 1) != CUDA_SUCCESS ||
+                ga.DevResourceGenerateDesc(&d_m, &rest, 1) != CUDA_SUCCESS ||
+                ga.GreenCtxCreate(&p->g_tensor, d_t, cdev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS ||
+                ga.GreenCtxCreate(&p->g_mem, d_m, cdev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS) {
+                set_error("otif_pipeline_create: green-context SM partition (%u + rest) failed", tensor_sms);
+                otif_pipeline_destroy(p);
+                return OTIF_EUNSUPPORTED;
+            }
+            CUstream st_t, st_m;
+            if (ga.GreenCtxStreamCreate(&st_t, p->g_tensor, CU_STREAM_NON_BLOCKING, 0) != CUDA_SUCCESS ||
+                ga.GreenCtxStreamCreate(&st_m, p->g_mem, CU_STREAM_NON_BLOCKING, 0) != CUDA_SUCCESS) {
+                set_error("otif_pipeline_create: green-context streams failed");
+                otif_pipeline_destroy(p);
+                return OTIF_EUNSUPPORTED;
+            }
+            p->s_tensor = (cudaStream_t)st_t;
+            p->s_mem = (cudaStream_t)st_m;
+            proxy_set_num_sms(p->proxy, (int)parts[0].sm.smCount);
+        }
     }
     p->cells = p->gh * p->gw;
     p->cap_w = B * ((p->cells + 1) / 2);
@@ -337,7 +432,7 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     PCUDA(cudaMalloc(&p->img, (size_t)p->pb * d->proxy.in_h * d->proxy.in_w * 3));
     if (p->chunks >= 2) {
         PCUDA(cudaMalloc(&p->img2, (size_t)p->pb * d->proxy.in_h * d->proxy.in_w * 3));
-        PCUDA(cudaStreamCreateWithFlags(&p->s_mem, cudaStreamNonBlocking));
+        if (!p->s_mem) PCUDA(cudaStreamCreateWithFlags(&p->s_mem, cudaStreamNonBlocking));
         PCUDA(cudaMalloc(&p->totals, (size_t)(p->chunks + 1) * 4));
         PCUDA(cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming));
         PCUDA(cudaEventCreateWithFlags(&p->ev_join, cudaEventDisableTiming));
@@ -395,7 +490,14 @@ extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     }
     if (p->s_compute) cudaStreamDestroy(p->s_compute);
     if (p->s_copy) cudaStreamDestroy(p->s_copy);
+    if (p->s_tensor) cudaStreamSynchronize(p->s_tensor);
     if (p->s_mem) cudaStreamDestroy(p->s_mem);
+    if (p->s_tensor) cudaStreamDestroy(p->s_tensor);
+    GreenApi ga;
+    if ((p->g_tensor || p->g_mem) && green_api(ga)) {
+        if (p->g_tensor) ga.GreenCtxDestroy(p->g_tensor);
+        if (p->g_mem) ga.GreenCtxDestroy(p->g_mem);
+    }
     cudaEvent_t ovl[] = {p->ev_fork, p->ev_join, p->ev_resized[0], p->ev_resized[1], p->ev_scored[0], p->ev_scored[1],
                          p->ev_imgfree[0], p->ev_imgfree[1]};
     for (cudaEvent_t e : ovl)

@@ -1427,6 +1427,12 @@ static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const f
     return true;
 }
 
+// SMs the persistent proxy kernels size their grids for (an SM partition of a green
+// context in the pipeline's partitioned overlap mode; default: the whole device)
+void proxy_set_num_sms(otif_proxy *p, int sms) {
+    if (sms > 0) p->num_sms = sms;
+}
+
 // kernel launches of one launch_proxy call (workspace zero + tag, E1+E2 fused or E1 and E2, E3..D1)
 int proxy_launches(const otif_proxy *p) { return p->e12 ? 7 : 8; }
 
