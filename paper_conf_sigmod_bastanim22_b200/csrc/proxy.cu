@@ -1126,6 +1126,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 int plane = 0;
                 const int64_t L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, (int)f, (int)oy, ox, plane);
                 const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * (MT * N2) + mm * N2;
+                // this row's first 8-channel chunk; chunks are lcap * 16 bytes apart
+                uint8_t *const row_out = p.out + ((int64_t)plane * p.out_c8 * p.out_lcap + L) * 16;
+                const int64_t chunk_stride = p.out_lcap * 16;
 #pragma unroll
                 for (int cc = 0; cc < N2 / 32; cc++) {
                     uint32_t v[32];
@@ -1137,10 +1140,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                             pk[j] = pack_bf16x2_relu(__uint_as_float(v[2 * j]) + s_b2[cc * 32 + 2 * j],
                                                      __uint_as_float(v[2 * j + 1]) + s_b2[cc * 32 + 2 * j + 1]);
 #pragma unroll
-                        for (int c = 0; c < 4; c++) {
-                            uint8_t *dst = p.out + (((int64_t)plane * p.out_c8 + cc * 4 + c) * p.out_lcap + L) * 16;
-                            *reinterpret_cast<uint4 *>(dst) = make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
-                        }
+                        for (int c = 0; c < 4; c++)
+                            *reinterpret_cast<uint4 *>(row_out + (cc * 4 + c) * chunk_stride) =
+                                make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
                     }
                 }
             }
