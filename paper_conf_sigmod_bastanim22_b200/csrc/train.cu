@@ -16,8 +16,9 @@
 // Training runs in fp32 (weights, activations, gradients; the 3xTF32 products keep fp32
 // accuracy, so the gradients still match the fp64 oracle within 2e-4); the inference path
 // keeps its bf16 tcgen05 kernels and takes the trained weights through otif_proxy_create.
-// C2 batch-32 step: 16.0 ms (SIMT, integer divisions) -> 5.5 ms (tcgen05, multiply-high
-// divisors, coalesced K-contiguous staging, tensor-tile split-K, parallel head reduce).
+// C2 batch-32 step: 16.0 ms (SIMT, integer divisions) -> 4.0 ms (tcgen05, multiply-high
+// divisors, coalesced K-contiguous staging with 16-B loads, 16-k stages at 2-3 CTAs per SM,
+// tensor-tile split-K, parallel head reduce).
 #include <math.h>
 #include <stdlib.h>
 #include <string.h>
@@ -176,9 +177,9 @@ __device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F 
 // row = l & 7, k-group = l >> 3), so each load instruction reads 64 contiguous bytes of 8
 // rows (vs 32 scattered rows) and each 8-lane store phase hits 8 distinct 16-B bank
 // groups.  Row contexts are recomputed per unit (mk: row -> context).
-template <int R, class MK, class F>
-__device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get, int k0, int ke, uint8_t *hi,
-                                               uint8_t *lo) {
+template <int R, class MK, class F, class F4>
+__device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get, F4 get4, bool vec, int k0, int ke,
+                                               uint8_t *hi, uint8_t *lo) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     constexpr int kGroups = kTcK / 16;                       // groups of 4 k-groups
     constexpr int kUnits = (R / 8) * kGroups, kWarps = kTcThreads / 32;
@@ -190,10 +191,15 @@ __device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get,
         const int r = (u / kGroups) * 8 + (lane & 7), kg = (u % kGroups) * 4 + (lane >> 3);
         const bool ok = u < kUnits && r < rows;
         const auto q = mk(ok ? row0 + r : row0);
+        const int kb4 = k0 + kg * 4;
+        if (vec && ok && kb4 + 4 <= ke) {
+            get4(q, kb4, v[i]);   // four consecutive k in one 16-B load
+        } else {
 #pragma unroll
-        for (int j = 0; j < 4; j++) {
-            const int k = k0 + kg * 4 + j;
-            v[i][j] = (ok && k < ke) ? get(q, k) : 0.f;
+            for (int j = 0; j < 4; j++) {
+                const int k = kb4 + j;
+                v[i][j] = (ok && k < ke) ? get(q, k) : 0.f;
+            }
         }
     }
 #pragma unroll
@@ -242,14 +248,17 @@ __global__ void __launch_bounds__(kTcThreads, OTIF_TC_MINB) tc_gemm_kernel(Op op
         const int k0 = kb + c * kTcK;
         if constexpr (Op::A_KFAST)
             tc_stage_kfast<kTcM>([&](int m) { return op.a_row(m); }, m0, M - m0,
-                                 [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); }, k0, ke, base, base + kA);
+                                 [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); },
+                                 [&](const typename Op::ARow &q, int k, float *v) { op.a_at4(q, k, v); }, op.a_vec(),
+                                 k0, ke, base, base + kA);
         else
             tc_stage_operand<kTcM>(actx, a_ok, [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); }, k0,
                                    ke, base, base + kA);
         if constexpr (Op::B_KFAST)
             tc_stage_kfast<BN>([&](int n) { return op.b_row(n); }, n0, N - n0,
-                               [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); }, k0, ke, base + 2 * kA,
-                               base + 2 * kA + kB);
+                               [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); },
+                               [&](const typename Op::BRow &q, int k, float *v) { op.b_at4(q, k, v); }, op.b_vec(), k0,
+                               ke, base + 2 * kA, base + 2 * kA + kB);
         else
             tc_stage_operand<BN>(bctx, b_ok, [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); }, k0, ke,
                                  base + 2 * kA, base + 2 * kA + kB);
@@ -352,6 +361,26 @@ struct FwdOp {
     __device__ float b_at(BRow q, int k) const { return q[k]; }
     __device__ float a(int m, int k) const { return a_at(a_row(m), k); }
     __device__ float b(int k, int n) const { return b_at(b_row(n), k); }
+    // 4 consecutive k (k % 4 == 0) in one 16-B load: same tap, consecutive channels when
+    // Cin % 4 == 0 (fp32 activations); the weights rows are K = 9 Cin long
+    __device__ bool a_vec() const { return sizeof(T) == 4 && g.Cin % 4 == 0 && (((uintptr_t)x) & 15) == 0; }
+    __device__ bool b_vec() const { return (g.k * g.k * g.Cin) % 4 == 0 && (((uintptr_t)w) & 15) == 0; }
+    __device__ void a_at4(const ARow &q, int k, float *v) const {
+        if constexpr (sizeof(T) == 4) {
+            const int tap = dv(k, g.dCin), ci = k - tap * g.Cin, kh = dv(tap, g.dK), kw = tap - kh * g.k;
+            const int iy = q.iy0 + kh, ix = q.ix0 + kw;
+            if (iy < 0 || iy >= g.H || ix < 0 || ix >= g.W) { v[0] = v[1] = v[2] = v[3] = 0.f; return; }
+            const float4 t = *reinterpret_cast<const float4 *>(
+                reinterpret_cast<const float *>(x) + (((int64_t)q.f * g.H + iy) * g.W + ix) * g.Cin + ci);
+            v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+        } else {
+            for (int j = 0; j < 4; j++) v[j] = a_at(q, k + j);
+        }
+    }
+    __device__ void b_at4(BRow q, int k, float *v) const {
+        const float4 t = *reinterpret_cast<const float4 *>(q + k);
+        v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+    }
     __device__ void store(int m, int n, float v, int) const {
         v += bias[n];
         y[(int64_t)m * g.Cout + n] = relu ? fmaxf(v, 0.f) : v;
@@ -384,6 +413,22 @@ struct DgradOp {
     __device__ float b_at(BRow n, int k) const {
         const int tap = dv(k, g.dCout), co = k - tap * g.Cout;
         return w[((int64_t)co * g.k * g.k + tap) * g.Cin + n];
+    }
+    // 4 consecutive k = 4 consecutive output channels of one tap (Cout % 4 == 0)
+    __device__ bool a_vec() const { return g.Cout % 4 == 0 && (((uintptr_t)dy) & 15) == 0; }
+    __device__ bool b_vec() const { return false; }
+    __device__ void a_at4(const ARow &q, int k, float *v) const {
+        const int tap = dv(k, g.dCout), co = k - tap * g.Cout, kh = dv(tap, g.dK), kw = tap - kh * g.k;
+        const int ty = q.ty0 - kh, tx = q.tx0 - kw;
+        v[0] = v[1] = v[2] = v[3] = 0.f;
+        if (ty < 0 || tx < 0) return;
+        const int oy = dv(ty, g.dStride), ox = dv(tx, g.dStride);
+        if (oy * g.stride != ty || ox * g.stride != tx || oy >= g.Ho || ox >= g.Wo) return;
+        const float4 t = *reinterpret_cast<const float4 *>(dy + (((int64_t)q.f * g.Ho + oy) * g.Wo + ox) * g.Cout + co);
+        v[0] = t.x; v[1] = t.y; v[2] = t.z; v[3] = t.w;
+    }
+    __device__ void b_at4(BRow n, int k, float *v) const {
+        for (int j = 0; j < 4; j++) v[j] = b_at(n, k + j);
     }
     __device__ float a(int m, int k) const { return a_at(a_row(m), k); }
     __device__ float b(int k, int n) const { return b_at(b_row(n), k); }
@@ -420,6 +465,10 @@ struct WgradOp {
     }
     __device__ float a(int m, int p) const { return a_at(a_row(m), p); }
     __device__ float b(int p, int kk) const { return b_at(b_row(kk), p); }
+    __device__ bool a_vec() const { return false; }
+    __device__ bool b_vec() const { return false; }
+    __device__ void a_at4(ARow q, int k, float *v) const { for (int j = 0; j < 4; j++) v[j] = a_at(q, k + j); }
+    __device__ void b_at4(const BRow &q, int k, float *v) const { for (int j = 0; j < 4; j++) v[j] = b_at(q, k + j); }
     __device__ void store(int m, int n, float v, int split) const {
         part[((int64_t)split * g.Cout + m) * (Kw + 1) + n] = v;
     }
