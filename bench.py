@@ -289,6 +289,13 @@ def run_otif(args):
     stages["pack"]["hbm_frac"] = stages["pack"]["gbs"] / hbm if stages["pack"]["gbs"] else None
     step_sum = sum(stage_ms.values())
     stages["conv_share_of_step"] = conv_ms / step_sum if step_sum else None
+    # HBM stages against the spec bandwidth too; grouping as ns/frame and share
+    for k in ("resize", "pack"):
+        if stages[k].get("gbs"):
+            stages[k]["hbm_frac_spec_8tbs"] = stages[k]["gbs"] / 8000.0
+    if stage_ms["select"] and frames_rank:
+        stages["select"]["ns_per_frame"] = stage_ms["select"] * 1e6 / frames_rank
+        stages["select"]["share_of_step"] = stage_ms["select"] / step_sum if step_sum else None
 
     # perfect-proxy line: stages 3-5 on ground-truth cell masks (mask_in), which
     # gives object-aligned windows instead of the random-init proxy's full-frame fallback
