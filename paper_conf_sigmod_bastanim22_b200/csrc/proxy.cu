@@ -719,6 +719,12 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma2_kernel(const __gri
 // TMEM: E2 accumulators 2 x 128 columns at 0, E1 accumulators 2 plane slots x 32 KT at 256.
 // ---------------------------------------------------------------------------
 constexpr int kE12Threads = 768;
+#ifndef OTIF_E12_ACC
+#define OTIF_E12_ACC 2        // E2 accumulator stages (A/B builds)
+#endif
+#ifndef OTIF_E12_E1SLOTS
+#define OTIF_E12_E1SLOTS 2    // E1 accumulator slots (A/B builds; 3 needs OTIF_E12_ACC=1)
+#endif
 constexpr int kE12MaxPlaneBufs = 3;
 
 struct E12Params {
@@ -822,7 +828,12 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
     // scripts/micro/ts_mma.cu) and the gather stores leave the shared-memory port.
     // TMEM: E2 acc 256 + E1 acc 2 x 96 + A1 48 columns = 496 (KT = 3 only).
     static_assert(!TS || KT == 3, "TMEM budget holds the A1 rows for KT = 3 only");
-    constexpr uint32_t kA1Col = 256 + 2 * 32 * KT;
+    // TMEM: E2 accumulators kAccStages x (MT x 64) at 0, E1 accumulators kE1Slots x 32 KT,
+    // then (TS) the A1 rows
+    constexpr int kAccStages = OTIF_E12_ACC, kE1Slots = OTIF_E12_E1SLOTS;
+    constexpr uint32_t kE1Col = kAccStages * 2 * 64;
+    constexpr uint32_t kA1Col = kE1Col + kE1Slots * 32 * KT;
+    static_assert(kA1Col + (TS ? 16 * KT : 0) <= 512, "TMEM budget");
     extern __shared__ __align__(1024) uint8_t smem[];
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -843,8 +854,8 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
     uint64_t *bars = reinterpret_cast<uint64_t *>(slab_s + 2 * (size_t)slab_bytes);
     uint64_t *slab_full = bars, *slab_empty = bars + 2;
     uint64_t *a1_full = bars + 4, *a1_empty = bars + 6;
-    uint64_t *e1_full = bars + 8, *e1_empty = bars + 10;
-    uint64_t *a2_full = bars + 12, *a2_empty = a2_full + kE12MaxPlaneBufs;
+    uint64_t *e1_full = bars + 8, *e1_empty = bars + 12;           // up to 4 slots each
+    uint64_t *a2_full = bars + 16, *a2_empty = a2_full + kE12MaxPlaneBufs;
     uint64_t *acc_full = a2_empty + kE12MaxPlaneBufs, *acc_empty = acc_full + 2;
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acc_empty + 2);
     float *s_b1 = reinterpret_cast<float *>(tmem_slot + 4);
@@ -855,9 +866,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
         for (int i = 0; i < 2; i++) {
             mbar_init(&slab_full[i], 1); mbar_init(&slab_empty[i], 256);
             mbar_init(&a1_full[i], 256); mbar_init(&a1_empty[i], 1);
-            mbar_init(&e1_full[i], 1); mbar_init(&e1_empty[i], 256);
             mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 128);
         }
+        for (int i = 0; i < kE1Slots; i++) { mbar_init(&e1_full[i], 1); mbar_init(&e1_empty[i], 256); }
         for (int i = 0; i < kE12MaxPlaneBufs; i++) { mbar_init(&a2_full[i], 256); mbar_init(&a2_empty[i], 1); }
         fence_barrier_init();
     }
@@ -939,10 +950,10 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 const uint32_t ph1 = (uint32_t)p.na1 == 1 ? (J & 1) : ((J >> 1) & 1);
                 mbar_wait(&a1_full[s1], ph1);
                 E12_TR(0, 0);
-                mbar_wait(&e1_empty[J & 1], ((J >> 1) & 1) ^ 1);
+                mbar_wait(&e1_empty[J % kE1Slots], ((J / kE1Slots) & 1) ^ 1);
                 E12_TR(1, 0);
                 tc_fence_after();
-                const uint32_t d = tmem_base + 256 + (J & 1) * (32 * KT);
+                const uint32_t d = tmem_base + kE1Col + (J % kE1Slots) * (32 * KT);
 #pragma unroll
                 for (int k = 0; k < KT; k++)
 #pragma unroll
@@ -955,7 +966,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                                            w1d + ((2 * s * 512) >> 4), idesc1, s);
                     }
                 umma_commit_warp(&a1_empty[s1]);
-                umma_commit_warp(&e1_full[J & 1]);
+                umma_commit_warp(&e1_full[J % kE1Slots]);
                 E12_TR(2, 0);
             }
         }
@@ -994,7 +1005,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 if (++pb == (uint32_t)p.np) { pb = 0; pp ^= 1; }
             }
             umma_commit_warp(&acc_full[acc]);
-            if (++acc == 2) { acc = 0; accp ^= 1; }
+            if (++acc == kAccStages) { acc = 0; accp ^= 1; }
         }
         E12_TR_DUMP("E2MMA start a2full issued", 3);
     } else if (warp >= 4 && warp < 12) {
@@ -1079,11 +1090,11 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
             for (int g = 0; g < 4; g++, J++) {
                 E12_WAIT_SLEEP(&a2_empty[pb], pp ^ 1);
                 if (wg == 0) E12_TR(0, 0);
-                mbar_wait(&e1_full[J & 1], (J >> 1) & 1);
+                mbar_wait(&e1_full[J % kE1Slots], (J / kE1Slots) & 1);
                 if (wg == 0) E12_TR(1, 0);
                 tc_fence_after();
                 uint8_t *plane = a2_s + pb * kPlaneBytes;
-                const uint32_t tacc = tmem_base + ((uint32_t)(quarter * 32) << 16) + 256 + (J & 1) * (32 * KT);
+                const uint32_t tacc = tmem_base + ((uint32_t)(quarter * 32) << 16) + kE1Col + (J % kE1Slots) * (32 * KT);
 #pragma unroll 1
                 for (int k = (int)((wg - J * KT) & 1); k < KT; k += 2) {
                     if (p.trace & 32) continue;   // 32: timing experiment
@@ -1099,7 +1110,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                             make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
                 }
                 tc_fence_before();
-                mbar_arrive(&e1_empty[J & 1]);
+                mbar_arrive(&e1_empty[J % kE1Slots]);
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
                 mbar_arrive(&a2_full[pb]);
                 if (wg == 0) E12_TR(2, 0);
@@ -1148,7 +1159,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
             }
             tc_fence_before();
             mbar_arrive(&acc_empty[acc]);
-            if (++acc == 2) { acc = 0; accp ^= 1; }
+            if (++acc == kAccStages) { acc = 0; accp ^= 1; }
         }
     }
     __syncwarp();
