@@ -135,3 +135,44 @@ def test_training_lowers_the_loss():
     for _ in range(60):
         last = float(tr.step(img, labels, 1e-3).item())
     assert last < 0.7 * first
+
+
+def test_simt_and_tensor_core_gemms_agree(tmp_path):
+    """The tcgen05 3xTF32 training GEMMs (default) and the fp32 SIMT GEMMs
+    (OTIF_TRAIN_SIMT=1, read once per process, hence a subprocess) give the same gradients
+    within fp32 accumulation-order error, on the full-width C1 case."""
+    import json
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import json, sys, numpy as np, torch
+sys.path.insert(0, sys.argv[1])
+import oracle
+from synth import configs, video, weights
+from paper_conf_sigmod_bastanim22_b200 import train
+wl = configs.C1
+img = oracle.resize(video.frames(wl, 2).numpy(), wl.proxy_h, wl.proxy_w)
+gh, gw = oracle.proxy_grid(wl.proxy_h, wl.proxy_w, wl.n_strided)
+lab = (np.arange(2 * gh * gw).reshape(2, gh, gw) % 3 == 0).astype(np.uint8)
+tr = train.Trainer(wl.proxy_h, wl.proxy_w, wl.n_strided, weights.proxy_weights(), max_batch=2)
+loss = float(tr.backward(torch.from_numpy(img).cuda(), torch.from_numpy(lab).cuda()).item())
+np.save(sys.argv[2], tr.grads_tensor().cpu().numpy())
+print(json.dumps({"loss": loss}))
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = {}
+    for mode in ("tc", "simt"):
+        env = dict(os.environ)
+        env.pop("OTIF_TRAIN_SIMT", None)
+        if mode == "simt":
+            env["OTIF_TRAIN_SIMT"] = "1"
+        path = str(tmp_path / f"{mode}.npy")
+        r = subprocess.run([sys.executable, "-c", code, root, path], env=env, capture_output=True, text=True,
+                           timeout=300)
+        assert r.returncode == 0, r.stderr[-2000:]
+        out[mode] = (json.loads(r.stdout.strip().splitlines()[-1])["loss"], np.load(path).astype(np.float64))
+    (l_tc, g_tc), (l_simt, g_simt) = out["tc"], out["simt"]
+    assert abs(l_tc - l_simt) <= 1e-5 * abs(l_simt)
+    for L, sl in enumerate(layer_slices(configs.ENC_WIDTHS, configs.DEC_WIDTH)):
+        assert rel_err(g_tc[sl], g_simt[sl]) < 2e-4, (L, rel_err(g_tc[sl], g_simt[sl]))
