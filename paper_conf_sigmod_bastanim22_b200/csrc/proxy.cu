@@ -798,15 +798,19 @@ __device__ __forceinline__ void e12_im2col_row(const E12Params &p, const uint8_t
 }
 
 #ifdef OTIF_E12_TRACE_BUILD   // hand-off timeline of CTA 0 (nvcc -DOTIF_E12_TRACE_BUILD; OTIF_E12_TRACE=1)
-#define E12_TR(slot, col)                                                         \
-    do {                                                                          \
-        if (tr && (int)J < 16) tt[slot][J] = clock64();                           \
+#ifndef OTIF_E12_TRACE_J0
+#define OTIF_E12_TRACE_J0 0   // first traced plane job (steady state: e.g. 200)
+#endif
+#define E12_TR(slot, col)                                                                                 \
+    do {                                                                                                  \
+        if (tr && (int)J >= OTIF_E12_TRACE_J0 && (int)J < OTIF_E12_TRACE_J0 + 16)                         \
+            tt[slot][J - OTIF_E12_TRACE_J0] = clock64();                                                  \
     } while (0)
 #define E12_TR_DUMP(name, nslots)                                                                   \
     do {                                                                                            \
         if (tr)                                                                                     \
             for (int j_ = 0; j_ < 16; j_++)                                                         \
-                printf("%s J=%2d %8lld %8lld %8lld\n", name, j_, tt[0][j_] - t00, (nslots) > 1 ? tt[1][j_] - t00 : 0ll, \
+                printf("%s t%d J=%2d %8lld %8lld %8lld\n", name, (int)threadIdx.x, j_, tt[0][j_] - t00, (nslots) > 1 ? tt[1][j_] - t00 : 0ll, \
                        (nslots) > 2 ? tt[2][j_] - t00 : 0ll);                                       \
     } while (0)
 #define E12_TR_DECL                                                       \
@@ -820,6 +824,8 @@ __device__ __forceinline__ void e12_im2col_row(const E12Params &p, const uint8_t
 #endif
 
 #define E12_WAIT_SLEEP(b, ph) (p.trace & 2 ? mbar_wait(b, ph) : mbar_wait_sleep(b, ph))
+// waits on the hand-off chain (gather <- a1_empty, E1 epilogue <- a2_empty): polling (bit 128 = sleep, A/B)
+#define E12_WAIT_CHAIN(b, ph) (p.trace & 128 ? mbar_wait_sleep(b, ph) : mbar_wait(b, ph))
 template <int KT, bool TS>
 __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_constant__ E12Params p) {
     // TS: E1's A operand (the im2col rows) lives in TMEM (columns kA1Col.., written by the
@@ -1026,9 +1032,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 const int rp = g >> 1, cp = g & 1;
                 const uint32_t s1 = (uint32_t)p.na1 == 1 ? 0 : (J & 1);
                 const uint32_t ph1 = (uint32_t)p.na1 == 1 ? (J & 1) : ((J >> 1) & 1);
-                if (wg == 0) E12_TR(0, 0);
-                if constexpr (!TS) E12_WAIT_SLEEP(&a1_empty[s1], ph1 ^ 1);
-                if (wg == 0) E12_TR(1, 0);
+                E12_TR(0, 0);
+                if constexpr (!TS) E12_WAIT_CHAIN(&a1_empty[s1], ph1 ^ 1);
+                E12_TR(1, 0);
                 uint32_t wk[2][16];   // TS: this thread's rows of its (at most 2) k sub-tiles
                 if constexpr (TS) {
 #pragma unroll
@@ -1070,12 +1076,12 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
                 }
                 mbar_arrive(&a1_full[s1]);
-                if (wg == 0) E12_TR(2, 0);
+                E12_TR(2, 0);
             }
             mbar_arrive(&slab_empty[sb]);
             if (++sb == 2) { sb = 0; sp ^= 1; }
         }
-        if (wg == 0) E12_TR_DUMP("GATH start a1empty arrived", 3);
+        E12_TR_DUMP("GATH start a1empty arrived", 3);
     } else if (warp >= 12 && warp < 20) {
         // ===== E1 epilogue (2 warpgroups, alternate E1 M tiles): TMEM -> ReLU, bf16 -> plane
         // buffer (E2's A operand).  The accumulator already holds 2^(s+7) (E1 sum + bias);
@@ -1088,10 +1094,10 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
         for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
 #pragma unroll 1
             for (int g = 0; g < 4; g++, J++) {
-                E12_WAIT_SLEEP(&a2_empty[pb], pp ^ 1);
-                if (wg == 0) E12_TR(0, 0);
+                E12_WAIT_CHAIN(&a2_empty[pb], pp ^ 1);
+                E12_TR(0, 0);
                 mbar_wait(&e1_full[J % kE1Slots], (J / kE1Slots) & 1);
-                if (wg == 0) E12_TR(1, 0);
+                E12_TR(1, 0);
                 tc_fence_after();
                 uint8_t *plane = a2_s + pb * kPlaneBytes;
                 const uint32_t tacc = tmem_base + ((uint32_t)(quarter * 32) << 16) + kE1Col + (J % kE1Slots) * (32 * KT);
@@ -1113,11 +1119,11 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 mbar_arrive(&e1_empty[J % kE1Slots]);
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
                 mbar_arrive(&a2_full[pb]);
-                if (wg == 0) E12_TR(2, 0);
+                E12_TR(2, 0);
                 if (++pb == (uint32_t)p.np) { pb = 0; pp ^= 1; }
             }
         }
-        if (wg == 0) E12_TR_DUMP("E1EP a2empty e1full arrived", 3);
+        E12_TR_DUMP("E1EP a2empty e1full arrived", 3);
     } else if (warp >= 20) {
         // ===== E2 epilogue: TMEM -> bias, ReLU, bf16 -> E3's input layout =====
         const int row = threadIdx.x - 640;

@@ -1,5 +1,5 @@
 set -e
-OTIF_NVCC_EXTRA=-DOTIF_E12_TRACE_BUILD python -c "from paper_conf_sigmod_bastanim22_b200 import build as b; b.build(force=True)"
+OTIF_NVCC_EXTRA="-DOTIF_E12_TRACE_BUILD ${TRACE_J0:+-DOTIF_E12_TRACE_J0=$TRACE_J0}" python -c "from paper_conf_sigmod_bastanim22_b200 import build as b; b.build(force=True)"
 for t in 1; do
   echo "== OTIF_E12_TRACE=$t"
   OTIF_E12_TRACE=$t python - <<'PY'
