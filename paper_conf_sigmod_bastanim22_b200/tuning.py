@@ -79,13 +79,16 @@ def proxy_sweep(frames: torch.Tensor, boxes: torch.Tensor, workloads: Sequence, 
         px = api.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, weights)
         img = api.otif_resize(frames, wl.proxy_h, wl.proxy_w)
         px.score(img)  # warm-up (workspace initialisation)
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        img = api.otif_resize(frames, wl.proxy_h, wl.proxy_w)
-        scores = px.score(img)
-        e1.record()
-        torch.cuda.synchronize()
-        t_proxy_ms = e0.elapsed_time(e1)
+        times = []
+        for _ in range(5):  # T_proxy,i: median of 5 device-timed resize + proxy passes
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            img = api.otif_resize(frames, wl.proxy_h, wl.proxy_w)
+            scores = px.score(img)
+            e1.record()
+            torch.cuda.synchronize()
+            times.append(e0.elapsed_time(e1))
+        t_proxy_ms = sorted(times)[len(times) // 2]
         for b in thresholds[wl.name]:
             r = api.otif_select_windows(scores, None, b, wl.src_w, wl.src_h, wl.cell, W, connectivity=connectivity)
             total = int(r["total"].item())
