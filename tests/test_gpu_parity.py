@@ -357,8 +357,9 @@ def test_pipeline_host_vs_stages(wl, blob):
     assert list(sc) == [int((ref["size_idx"] == s).sum()) for s in range(len(wl.sizes))]
 
 
+@pytest.mark.parametrize("green", [0, 32], ids=["coresident", "green32"])
 @pytest.mark.parametrize("wl,chunks", [(configs.C2, 3), (configs.C1, 4), (configs.C3, 2)], ids=["C2", "C1", "C3"])
-def test_pipeline_overlap_matches_serial(wl, chunks, blob):
+def test_pipeline_overlap_matches_serial(wl, chunks, green, blob, monkeypatch):
     """Overlap mode (resize / select / pack of neighbouring chunks on a second stream while
     the proxy scores a chunk) returns exactly the serial schedule's windows, per-frame counts,
     per-size counts and device counters (incl. the order-independent window hash), over
@@ -367,7 +368,10 @@ def test_pipeline_overlap_matches_serial(wl, chunks, blob):
     n = 75
     src = video.frames(wl, n).contiguous()
     ser = otif.Pipeline(wl, blob, b, max_batch=40)
+    if green:   # SM partition through two green contexts (read at create)
+        monkeypatch.setenv("OTIF_OVL_GREEN", str(green))
     ovl = otif.Pipeline(wl, blob, b, max_batch=40, overlap_chunks=chunks)
+    monkeypatch.delenv("OTIF_OVL_GREEN", raising=False)
     w0, c0, s0, t0 = ser.run_host(src)
     w1, c1, s1, t1 = ovl.run_host(src)
     assert t0 == t1 and np.array_equal(c0, c1) and list(s0) == list(s1)
