@@ -293,11 +293,12 @@ def test_end_to_end_c1(blob):
 
 
 # ------------------------------------------------------------------ full size (bench launch configuration)
-def test_full_size_c2_sampled(blob):
-    """C2 at its full size (4500 frames, one launch per stage as bench.py times it);
-    sampled frames are recomputed one by one on the oracle."""
-    wl = configs.C2
-    b = threshold("C2", 0.7)
+@pytest.mark.parametrize("wl", [configs.C2, configs.C3], ids=["C2", "C3"])
+def test_full_size_sampled(wl, blob):
+    """C2 (4500 960x540 frames) and C3 (3000 1920x1080 UAV frames, five window sizes) at
+    their full sizes, one launch per stage as bench.py times it; sampled frames are
+    recomputed one by one on the oracle."""
+    b = threshold(wl.name, 0.7)
     n = wl.n_frames
     src = torch.empty((n, wl.src_h, wl.src_w, 3), dtype=torch.uint8, device="cuda")
     video.make_scene(wl).render(range(n), out=src)
