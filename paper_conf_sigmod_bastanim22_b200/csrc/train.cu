@@ -438,6 +438,62 @@ struct DgradOp {
     }
 };
 
+// Stride-2 dgrad split by the parity (py, px) of the input pixel: only the taps with
+// kh = py + 1 (mod 2) and kw = px + 1 (mod 2) reach an output pixel (ty = iy + 1 - kh even),
+// so each class is a GEMM over ntap = 1, 2, 2 or 4 taps instead of 9 with 3/4 zeros
+// (M = that class's pixels, K = ntap x Cout).  Same sums as DgradOp without its zero terms.
+struct DgradParOp {
+    static constexpr bool A_KFAST = true, B_KFAST = false;
+    const float *dy, *w, *xpost;
+    float *dx;
+    ConvGeom g;
+    int py, px, Hc, Wc, ntap;
+    int tkh[4], tkw[4];
+    FastDiv dHWc, dWc, dCout;
+    struct ARow { int f, ty0, tx0; int64_t pix; };
+    __device__ ARow a_row(int m) const {
+        const int f = dv(m, dHWc), r = m - f * Hc * Wc, iyc = dv(r, dWc), ixc = r - iyc * Wc;
+        const int iy = 2 * iyc + py, ix = 2 * ixc + px;
+        return {f, iy + g.pad, ix + g.pad, ((int64_t)f * g.H + iy) * g.W + ix};
+    }
+    __device__ float a_at(const ARow &q, int k) const {
+        const int t = dv(k, dCout), co = k - t * g.Cout;
+        const int ty = q.ty0 - tkh[t], tx = q.tx0 - tkw[t];
+        if (ty < 0 || tx < 0) return 0.f;
+        const int oy = ty >> 1, ox = tx >> 1;
+        if (oy >= g.Ho || ox >= g.Wo) return 0.f;
+        return dy[(((int64_t)q.f * g.Ho + oy) * g.Wo + ox) * g.Cout + co];
+    }
+    using BRow = int;
+    __device__ BRow b_row(int n) const { return n; }
+    __device__ float b_at(BRow n, int k) const {
+        const int t = dv(k, dCout), co = k - t * g.Cout;
+        return w[((int64_t)co * g.k * g.k + tkh[t] * g.k + tkw[t]) * g.Cin + n];
+    }
+    __device__ float a(int m, int k) const { return a_at(a_row(m), k); }
+    __device__ float b(int k, int n) const { return b_at(b_row(n), k); }
+    __device__ bool a_vec() const { return g.Cout % 4 == 0 && (((uintptr_t)dy) & 15) == 0; }
+    __device__ bool b_vec() const { return false; }
+    __device__ void a_at4(const ARow &q, int k, float *v) const {
+        const int t = dv(k, dCout), co = k - t * g.Cout;
+        const int ty = q.ty0 - tkh[t], tx = q.tx0 - tkw[t];
+        v[0] = v[1] = v[2] = v[3] = 0.f;
+        if (ty < 0 || tx < 0) return;
+        const int oy = ty >> 1, ox = tx >> 1;
+        if (oy >= g.Ho || ox >= g.Wo) return;
+        const float4 x4 = *reinterpret_cast<const float4 *>(dy + (((int64_t)q.f * g.Ho + oy) * g.Wo + ox) * g.Cout + co);
+        v[0] = x4.x; v[1] = x4.y; v[2] = x4.z; v[3] = x4.w;
+    }
+    __device__ void b_at4(BRow n, int k, float *v) const {
+        for (int j = 0; j < 4; j++) v[j] = b_at(n, k + j);
+    }
+    __device__ void store(int m, int n, float v, int) const {
+        const int f = dv(m, dHWc), r = m - f * Hc * Wc, iyc = dv(r, dWc), ixc = r - iyc * Wc;
+        const int64_t i = (((int64_t)f * g.H + 2 * iyc + py) * g.W + 2 * ixc + px) * g.Cin + n;
+        dx[i] = xpost[i] > 0.f ? v : 0.f;
+    }
+};
+
 // [dW | db][co, kk] = Σ_p dy[p, co] · (kk < K ? im2col(x)[p, kk] : 1), split over p.
 template <typename T>
 struct WgradOp {
@@ -826,9 +882,32 @@ extern "C" otif_status otif_trainer_backward(otif_trainer *t, const uint8_t *img
                               stream>>>(t->part, splits, g.Cout, kw, t->grad + t->woff[L]);
         OTIF_LAUNCH_CHECK();
         if (L > 0) {
-            DgradOp op{t->dbuf[cur], t->w + t->woff[L], t->act[L], t->dbuf[cur ^ 1], g};
-            st = run_gemm(op, (int64_t)n * g.H * g.W, g.Cin, (int64_t)g.k * g.k * g.Cout, 1, stream);
-            if (st != OTIF_OK) return st;
+            if (g.stride == 2 && g.k == 3 && g.pad == 1 && train_tc()) {
+                // four parity classes of input pixels, each with its own tap subset
+                for (int py = 0; py < 2; py++)
+                    for (int px = 0; px < 2; px++) {
+                        DgradParOp op;
+                        op.dy = t->dbuf[cur]; op.w = t->w + t->woff[L]; op.xpost = t->act[L]; op.dx = t->dbuf[cur ^ 1];
+                        op.g = g; op.py = py; op.px = px;
+                        op.Hc = (g.H - py + 1) / 2; op.Wc = (g.W - px + 1) / 2;
+                        op.ntap = 0;
+                        for (int kh = 0; kh < 3; kh++)
+                            for (int kw = 0; kw < 3; kw++)
+                                if (((py + 1 - kh) & 1) == 0 && ((px + 1 - kw) & 1) == 0) {
+                                    op.tkh[op.ntap] = kh; op.tkw[op.ntap] = kw; op.ntap++;
+                                }
+                        op.dHWc = make_fastdiv((uint32_t)(op.Hc * op.Wc)); op.dWc = make_fastdiv((uint32_t)op.Wc);
+                        op.dCout = make_fastdiv((uint32_t)g.Cout);
+                        const int64_t Mc = (int64_t)n * op.Hc * op.Wc;
+                        if (Mc == 0) continue;
+                        st = run_gemm(op, Mc, g.Cin, (int64_t)op.ntap * g.Cout, 1, stream);
+                        if (st != OTIF_OK) return st;
+                    }
+            } else {
+                DgradOp op{t->dbuf[cur], t->w + t->woff[L], t->act[L], t->dbuf[cur ^ 1], g};
+                st = run_gemm(op, (int64_t)n * g.H * g.W, g.Cin, (int64_t)g.k * g.k * g.Cout, 1, stream);
+                if (st != OTIF_OK) return st;
+            }
             cur ^= 1;
         }
     }
