@@ -141,9 +141,9 @@ __device__ __forceinline__ void umma_tf32_warp(uint32_t tmem_d, uint64_t adesc, 
 
 // stage rows [0, R) x 32 k of one operand: thread t owns row t % R (R divides the CTA size)
 // and k-groups t / R, t / R + 256 / R, ...; ctx = the row's context (op.a_row / op.b_row)
-template <int R, class Ctx, class F>
-__device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F get, int k0, int ke, uint8_t *hi,
-                                                 uint8_t *lo) {
+template <int R, class Ctx, class F, class F4>
+__device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F get, F4 get4, bool vec, int k0, int ke,
+                                                 uint8_t *hi, uint8_t *lo) {
     static_assert(kTcThreads % R == 0, "rows per thread");
     const int r = threadIdx.x % R;
     constexpr int kKG = kTcK / 4, kStep = kTcThreads / R;
@@ -154,10 +154,15 @@ __device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F 
 #pragma unroll
     for (int it = 0; it < kIters; it++) {
         const int kg = (int)threadIdx.x / R + it * (kTcThreads / R);
+        const int kb4 = k0 + kg * 4;
+        if (vec && row_ok && kg < kKG && kb4 + 4 <= ke) {
+            get4(ctx, kb4, v[it]);   // four consecutive k with one index decomposition
+        } else {
 #pragma unroll
-        for (int j = 0; j < 4; j++) {
-            const int k = k0 + kg * 4 + j;
-            v[it][j] = (row_ok && kg < kKG && k < ke) ? get(ctx, k) : 0.f;
+            for (int j = 0; j < 4; j++) {
+                const int k = kb4 + j;
+                v[it][j] = (row_ok && kg < kKG && k < ke) ? get(ctx, k) : 0.f;
+            }
         }
     }
 #pragma unroll
@@ -252,16 +257,18 @@ __global__ void __launch_bounds__(kTcThreads, OTIF_TC_MINB) tc_gemm_kernel(Op op
                                  [&](const typename Op::ARow &q, int k, float *v) { op.a_at4(q, k, v); }, op.a_vec(),
                                  k0, ke, base, base + kA);
         else
-            tc_stage_operand<kTcM>(actx, a_ok, [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); }, k0,
-                                   ke, base, base + kA);
+            tc_stage_operand<kTcM>(actx, a_ok, [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); },
+                                   [&](const typename Op::ARow &q, int k, float *v) { op.a_at4(q, k, v); }, op.a_vec(),
+                                   k0, ke, base, base + kA);
         if constexpr (Op::B_KFAST)
             tc_stage_kfast<BN>([&](int n) { return op.b_row(n); }, n0, N - n0,
                                [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); },
                                [&](const typename Op::BRow &q, int k, float *v) { op.b_at4(q, k, v); }, op.b_vec(), k0,
                                ke, base + 2 * kA, base + 2 * kA + kB);
         else
-            tc_stage_operand<BN>(bctx, b_ok, [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); }, k0, ke,
-                                 base + 2 * kA, base + 2 * kA + kB);
+            tc_stage_operand<BN>(bctx, b_ok, [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); },
+                                 [&](const typename Op::BRow &q, int k, float *v) { op.b_at4(q, k, v); }, op.b_vec(),
+                                 k0, ke, base + 2 * kA, base + 2 * kA + kB);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mbar_arrive(&full[st]);
         if (warp == 0) {
@@ -522,9 +529,20 @@ struct WgradOp {
     __device__ float a(int m, int p) const { return a_at(a_row(m), p); }
     __device__ float b(int p, int kk) const { return b_at(b_row(kk), p); }
     __device__ bool a_vec() const { return false; }
-    __device__ bool b_vec() const { return false; }
+    __device__ bool b_vec() const { return true; }   // 4 consecutive pixels: one decomposition, then steps
     __device__ void a_at4(ARow q, int k, float *v) const { for (int j = 0; j < 4; j++) v[j] = a_at(q, k + j); }
-    __device__ void b_at4(const BRow &q, int k, float *v) const { for (int j = 0; j < 4; j++) v[j] = b_at(q, k + j); }
+    __device__ void b_at4(const BRow &q, int p, float *v) const {
+        if (q.bias) { v[0] = v[1] = v[2] = v[3] = 1.f; return; }
+        int f = dv(p, g.dHoWo), r = p - f * g.Ho * g.Wo, oy = dv(r, g.dWo), ox = r - oy * g.Wo;
+#pragma unroll
+        for (int j = 0; j < 4; j++) {
+            const int iy = oy * g.stride - g.pad + q.kh, ix = ox * g.stride - g.pad + q.kw;
+            v[j] = (iy < 0 || iy >= g.H || ix < 0 || ix >= g.W)
+                       ? 0.f
+                       : act_in<T>(x, (((int64_t)f * g.H + iy) * g.W + ix) * g.Cin + q.ci);
+            if (++ox == g.Wo) { ox = 0; if (++oy == g.Ho) { oy = 0; f++; } }
+        }
+    }
     __device__ void store(int m, int n, float v, int split) const {
         part[((int64_t)split * g.Cout + m) * (Kw + 1) + n] = v;
     }
