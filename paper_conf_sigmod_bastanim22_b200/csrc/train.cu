@@ -24,6 +24,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <type_traits>
 #include <vector>
 
 #include "common.cuh"
@@ -140,38 +141,55 @@ __device__ __forceinline__ void umma_tf32_warp(uint32_t tmem_d, uint64_t adesc, 
 }
 
 // stage rows [0, R) x 32 k of one operand: thread t owns row t % R (R divides the CTA size)
-// and k-groups t / R, t / R + 256 / R, ...; ctx = the row's context (op.a_row / op.b_row)
+// and k-groups t / R, t / R + 256 / R, ...; ctx = the row's context (op.a_row / op.b_row).
+// Split into a load half (gathers into registers) and a store half (tf32 split + 16-B
+// shared stores) so the kernel can keep the next chunks' gathers in flight (OTIF_TC_PREFETCH).
+template <int R>
+struct TcRowsRegs {
+    static constexpr int kN = (kTcK / 4 + kTcThreads / R - 1) / (kTcThreads / R);
+    float v[kN][4];
+};
+template <int R>
+struct TcKfastRegs {
+    static constexpr int kN = ((R / 8) * (kTcK / 16) + kTcThreads / 32 - 1) / (kTcThreads / 32);
+    float v[kN][4];
+};
+
 template <int R, class Ctx, class F, class F4>
-__device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F get, F4 get4, bool vec, int k0, int ke,
-                                                 uint8_t *hi, uint8_t *lo) {
+__device__ __forceinline__ void tc_load_operand(const Ctx &ctx, bool row_ok, F get, F4 get4, bool vec, int k0, int ke,
+                                                TcRowsRegs<R> &g) {
     static_assert(kTcThreads % R == 0, "rows per thread");
-    const int r = threadIdx.x % R;
-    constexpr int kKG = kTcK / 4, kStep = kTcThreads / R;
-    constexpr int kIters = (kKG + kStep - 1) / kStep;
+    constexpr int kKG = kTcK / 4, kStep = kTcThreads / R, kIters = TcRowsRegs<R>::kN;
     if ((int)threadIdx.x / R >= kKG) return;   // more threads than (row, k-group) units
     // all the thread's loads first (kIters x 4 in flight: the gathers are latency-bound)
-    float v[kIters][4];
 #pragma unroll
     for (int it = 0; it < kIters; it++) {
-        const int kg = (int)threadIdx.x / R + it * (kTcThreads / R);
+        const int kg = (int)threadIdx.x / R + it * kStep;
         const int kb4 = k0 + kg * 4;
         if (vec && row_ok && kg < kKG && kb4 + 4 <= ke) {
-            get4(ctx, kb4, v[it]);   // four consecutive k with one index decomposition
+            get4(ctx, kb4, g.v[it]);   // four consecutive k with one index decomposition
         } else {
 #pragma unroll
             for (int j = 0; j < 4; j++) {
                 const int k = kb4 + j;
-                v[it][j] = (row_ok && kg < kKG && k < ke) ? get(ctx, k) : 0.f;
+                g.v[it][j] = (row_ok && kg < kKG && k < ke) ? get(ctx, k) : 0.f;
             }
         }
     }
+}
+
+template <int R>
+__device__ __forceinline__ void tc_store_operand(const TcRowsRegs<R> &g, uint8_t *hi, uint8_t *lo) {
+    constexpr int kKG = kTcK / 4, kStep = kTcThreads / R, kIters = TcRowsRegs<R>::kN;
+    const int r = threadIdx.x % R;
+    if ((int)threadIdx.x / R >= kKG) return;
 #pragma unroll
     for (int it = 0; it < kIters; it++) {
-        const int kg = (int)threadIdx.x / R + it * (kTcThreads / R);
+        const int kg = (int)threadIdx.x / R + it * kStep;
         if (kg >= kKG) continue;
         float h[4], l[4];
 #pragma unroll
-        for (int j = 0; j < 4; j++) { h[j] = tf32_rna(v[it][j]); l[j] = v[it][j] - h[j]; }
+        for (int j = 0; j < 4; j++) { h[j] = tf32_rna(g.v[it][j]); l[j] = g.v[it][j] - h[j]; }
         const size_t off = ((size_t)kg * R + r) * 16;
         *reinterpret_cast<float4 *>(hi + off) = make_float4(h[0], h[1], h[2], h[3]);
         *reinterpret_cast<float4 *>(lo + off) = make_float4(l[0], l[1], l[2], l[3]);
@@ -183,13 +201,11 @@ __device__ __forceinline__ void tc_stage_operand(const Ctx &ctx, bool row_ok, F 
 // rows (vs 32 scattered rows) and each 8-lane store phase hits 8 distinct 16-B bank
 // groups.  Row contexts are recomputed per unit (mk: row -> context).
 template <int R, class MK, class F, class F4>
-__device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get, F4 get4, bool vec, int k0, int ke,
-                                               uint8_t *hi, uint8_t *lo) {
+__device__ __forceinline__ void tc_load_kfast(MK mk, int row0, int rows, F get, F4 get4, bool vec, int k0, int ke,
+                                              TcKfastRegs<R> &g) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     constexpr int kGroups = kTcK / 16;                       // groups of 4 k-groups
-    constexpr int kUnits = (R / 8) * kGroups, kWarps = kTcThreads / 32;
-    constexpr int kPerWarp = (kUnits + kWarps - 1) / kWarps;
-    float v[kPerWarp][4];
+    constexpr int kUnits = (R / 8) * kGroups, kWarps = kTcThreads / 32, kPerWarp = TcKfastRegs<R>::kN;
 #pragma unroll
     for (int i = 0; i < kPerWarp; i++) {
         const int u = warp + i * kWarps;
@@ -198,15 +214,22 @@ __device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get,
         const auto q = mk(ok ? row0 + r : row0);
         const int kb4 = k0 + kg * 4;
         if (vec && ok && kb4 + 4 <= ke) {
-            get4(q, kb4, v[i]);   // four consecutive k in one 16-B load
+            get4(q, kb4, g.v[i]);   // four consecutive k in one 16-B load
         } else {
 #pragma unroll
             for (int j = 0; j < 4; j++) {
                 const int k = kb4 + j;
-                v[i][j] = (ok && k < ke) ? get(q, k) : 0.f;
+                g.v[i][j] = (ok && k < ke) ? get(q, k) : 0.f;
             }
         }
     }
+}
+
+template <int R>
+__device__ __forceinline__ void tc_store_kfast(const TcKfastRegs<R> &g, uint8_t *hi, uint8_t *lo) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    constexpr int kGroups = kTcK / 16;
+    constexpr int kUnits = (R / 8) * kGroups, kWarps = kTcThreads / 32, kPerWarp = TcKfastRegs<R>::kN;
 #pragma unroll
     for (int i = 0; i < kPerWarp; i++) {
         const int u = warp + i * kWarps;
@@ -214,12 +237,16 @@ __device__ __forceinline__ void tc_stage_kfast(MK mk, int row0, int rows, F get,
         const int r = (u / kGroups) * 8 + (lane & 7), kg = (u % kGroups) * 4 + (lane >> 3);
         float h[4], l[4];
 #pragma unroll
-        for (int j = 0; j < 4; j++) { h[j] = tf32_rna(v[i][j]); l[j] = v[i][j] - h[j]; }
+        for (int j = 0; j < 4; j++) { h[j] = tf32_rna(g.v[i][j]); l[j] = g.v[i][j] - h[j]; }
         const size_t off = ((size_t)kg * R + r) * 16;
         *reinterpret_cast<float4 *>(hi + off) = make_float4(h[0], h[1], h[2], h[3]);
         *reinterpret_cast<float4 *>(lo + off) = make_float4(l[0], l[1], l[2], l[3]);
     }
 }
+
+#ifndef OTIF_TC_PREFETCH
+#define OTIF_TC_PREFETCH 1    // 1: two register sets, chunk c+2's gathers issued while c+1's are in flight
+#endif
 
 template <class Op, int BN>
 __global__ void __launch_bounds__(kTcThreads, OTIF_TC_MINB) tc_gemm_kernel(Op op, int M, int N, int K, int k_split) {
@@ -246,31 +273,43 @@ __global__ void __launch_bounds__(kTcThreads, OTIF_TC_MINB) tc_gemm_kernel(Op op
     const bool a_ok = am < M, b_ok = bn < N;
     const typename Op::ARow actx = op.a_row(a_ok ? am : 0);
     const typename Op::BRow bctx = op.b_row(b_ok ? bn : 0);
-    for (int c = 0; c < nchunks; c++) {
+    using ARegs = typename std::conditional<Op::A_KFAST, TcKfastRegs<kTcM>, TcRowsRegs<kTcM>>::type;
+    using BRegs = typename std::conditional<Op::B_KFAST, TcKfastRegs<BN>, TcRowsRegs<BN>>::type;
+    auto load = [&](int c, ARegs &ra, BRegs &rb) {
+        const int k0 = kb + c * kTcK;
+        if constexpr (Op::A_KFAST)
+            tc_load_kfast<kTcM>([&](int m) { return op.a_row(m); }, m0, M - m0,
+                                [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); },
+                                [&](const typename Op::ARow &q, int k, float *v) { op.a_at4(q, k, v); }, op.a_vec(),
+                                k0, ke, ra);
+        else
+            tc_load_operand<kTcM>(actx, a_ok, [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); },
+                                  [&](const typename Op::ARow &q, int k, float *v) { op.a_at4(q, k, v); }, op.a_vec(),
+                                  k0, ke, ra);
+        if constexpr (Op::B_KFAST)
+            tc_load_kfast<BN>([&](int n) { return op.b_row(n); }, n0, N - n0,
+                              [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); },
+                              [&](const typename Op::BRow &q, int k, float *v) { op.b_at4(q, k, v); }, op.b_vec(), k0,
+                              ke, rb);
+        else
+            tc_load_operand<BN>(bctx, b_ok, [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); },
+                                [&](const typename Op::BRow &q, int k, float *v) { op.b_at4(q, k, v); }, op.b_vec(),
+                                k0, ke, rb);
+    };
+    // store chunk c's registers into its stage, hand the stage to the MMA warp; `next`
+    // issues the gathers of a later chunk into the registers just freed (before warp 0
+    // waits on the stage barrier), so they overlap the hand-off
+    auto stage = [&](int c, ARegs &ra, BRegs &rb, int next) {
         const int st = c & 1;
         if (c >= 2) mbar_wait(&empty[st], ((c >> 1) - 1) & 1);   // the MMAs of chunk c-2 read this stage
         uint8_t *base = smem + (size_t)st * kStage;
-        const int k0 = kb + c * kTcK;
-        if constexpr (Op::A_KFAST)
-            tc_stage_kfast<kTcM>([&](int m) { return op.a_row(m); }, m0, M - m0,
-                                 [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); },
-                                 [&](const typename Op::ARow &q, int k, float *v) { op.a_at4(q, k, v); }, op.a_vec(),
-                                 k0, ke, base, base + kA);
-        else
-            tc_stage_operand<kTcM>(actx, a_ok, [&](const typename Op::ARow &q, int k) { return op.a_at(q, k); },
-                                   [&](const typename Op::ARow &q, int k, float *v) { op.a_at4(q, k, v); }, op.a_vec(),
-                                   k0, ke, base, base + kA);
-        if constexpr (Op::B_KFAST)
-            tc_stage_kfast<BN>([&](int n) { return op.b_row(n); }, n0, N - n0,
-                               [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); },
-                               [&](const typename Op::BRow &q, int k, float *v) { op.b_at4(q, k, v); }, op.b_vec(), k0,
-                               ke, base + 2 * kA, base + 2 * kA + kB);
-        else
-            tc_stage_operand<BN>(bctx, b_ok, [&](const typename Op::BRow &q, int k) { return op.b_at(q, k); },
-                                 [&](const typename Op::BRow &q, int k, float *v) { op.b_at4(q, k, v); }, op.b_vec(),
-                                 k0, ke, base + 2 * kA, base + 2 * kA + kB);
+        if constexpr (Op::A_KFAST) tc_store_kfast<kTcM>(ra, base, base + kA);
+        else tc_store_operand<kTcM>(ra, base, base + kA);
+        if constexpr (Op::B_KFAST) tc_store_kfast<BN>(rb, base + 2 * kA, base + 2 * kA + kB);
+        else tc_store_operand<BN>(rb, base + 2 * kA, base + 2 * kA + kB);
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mbar_arrive(&full[st]);
+        if (next < nchunks) load(next, ra, rb);
         if (warp == 0) {
             mbar_wait(&full[st], (c >> 1) & 1);
             tc_fence_after();
@@ -286,7 +325,30 @@ __global__ void __launch_bounds__(kTcThreads, OTIF_TC_MINB) tc_gemm_kernel(Op op
             }
             umma_commit_warp(&empty[st]);
         }
+    };
+#if OTIF_TC_PREFETCH
+    {
+        ARegs ra0, ra1;
+        BRegs rb0, rb1;
+        if (nchunks > 0) load(0, ra0, rb0);
+        if (nchunks > 1) load(1, ra1, rb1);
+#pragma unroll 1
+        for (int c = 0; c < nchunks; c += 2) {
+            stage(c, ra0, rb0, c + 2);
+            if (c + 1 < nchunks) stage(c + 1, ra1, rb1, c + 3);
+        }
     }
+#else
+    {
+        ARegs ra;
+        BRegs rb;
+#pragma unroll 1
+        for (int c = 0; c < nchunks; c++) {
+            load(c, ra, rb);
+            stage(c, ra, rb, nchunks);
+        }
+    }
+#endif
     if (warp == 0) umma_commit_warp(&done);
     mbar_wait(&done, 0);
     tc_fence_after();
