@@ -326,7 +326,21 @@ __global__ void __launch_bounds__(kTcThreads, OTIF_TC_MINB) tc_gemm_kernel(Op op
             umma_commit_warp(&empty[st]);
         }
     };
-#if OTIF_TC_PREFETCH
+#if OTIF_TC_PREFETCH >= 2
+    {   // three register sets (A/B variant)
+        ARegs ra0, ra1, ra2;
+        BRegs rb0, rb1, rb2;
+        if (nchunks > 0) load(0, ra0, rb0);
+        if (nchunks > 1) load(1, ra1, rb1);
+        if (nchunks > 2) load(2, ra2, rb2);
+#pragma unroll 1
+        for (int c = 0; c < nchunks; c += 3) {
+            stage(c, ra0, rb0, c + 3);
+            if (c + 1 < nchunks) stage(c + 1, ra1, rb1, c + 4);
+            if (c + 2 < nchunks) stage(c + 2, ra2, rb2, c + 5);
+        }
+    }
+#elif OTIF_TC_PREFETCH
     {
         ARegs ra0, ra1;
         BRegs rb0, rb1;
