@@ -788,13 +788,16 @@ struct otif_trainer {
     int step = 0;
 };
 
+#ifndef OTIF_WGRAD_WAVES
+#define OTIF_WGRAD_WAVES 3     // split-K CTAs per SM targeted by the weight-gradient GEMMs
+#endif
 static int wgrad_splits(const otif_trainer *t, int L, int n) {
     const int64_t pixels = (int64_t)n * t->hs[L + 1] * t->ws[L + 1];
     const int64_t kw1 = (int64_t)t->ks[L] * t->ks[L] * t->cin[L] + 1;
     // output tiles of the GEMM kernel in use (tcgen05: 128 x 32/64/128; SIMT: 64 x 64)
     const int64_t tiles = train_tc() ? cdiv(t->cout[L], kTcM) * cdiv(kw1, kw1 <= 32 ? 32 : kw1 <= 64 ? 64 : 128)
                                      : cdiv(t->cout[L], BM) * cdiv(kw1, BN);
-    int64_t s = cdiv(2 * (int64_t)t->sms, tiles);
+    int64_t s = cdiv(OTIF_WGRAD_WAVES * (int64_t)t->sms, tiles);
     s = std::min<int64_t>(s, std::max<int64_t>(1, pixels / 256));
     return (int)std::max<int64_t>(1, std::min<int64_t>(s, 512));
 }
