@@ -15,6 +15,9 @@ GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 BAND = 1e-3  # "except for cells whose oracle score lies within 1e-3 of the threshold" (north_star)
 
 
+THRESHOLD_NAMES = tuple(json.load(open(os.path.join(GOLDEN, "thresholds.json")))["workloads"].keys())
+
+
 def threshold(name: str, q: float = 0.7) -> float:
     d = json.load(open(os.path.join(GOLDEN, "thresholds.json")))
     return d["workloads"][name][str(q)]["B"]

@@ -3,13 +3,15 @@ identical inputs, then end to end.  Criteria (north_star / SURVEY §8(c)):
   resize & pack pixels within 1 LSB (identity crops byte-exact); proxy scores within
   2e-2 of the quant=none oracle; masks bit-exact vs the quant=bf16 oracle except cells
   within 1e-3 of the threshold; windows bit-exact given the same mask."""
+import zlib
+
 import numpy as np
 import pytest
 import torch
 
 import oracle
 from synth import configs, video, weights
-from tests.helpers import BAND, as_tuples, oracle_scores, threshold, windows_np
+from tests.helpers import BAND, THRESHOLD_NAMES, as_tuples, oracle_scores, threshold, windows_np
 
 pytestmark = pytest.mark.gpu
 
@@ -63,6 +65,7 @@ PROXY_CASES = [
     (configs.C3, 2),         # S = 16 (c = 64, r = 1/4)
     (configs.C4_SWEEP[2], 2),  # S = 4 (r = 1/8, c = 32): only E1, E2 strided
     (configs.C4_SWEEP[3], 2),  # S = 32 (r = 1/2, c = 64): all five strided (the paper's case)
+    (configs.C1.with_(name="C1s2", cell=8), 2),  # S = 2 (n_strided = 1): E2 stride 1, separate E1 kernel
 ]
 
 
@@ -78,7 +81,9 @@ def test_proxy_parity(wl, n, blob):
     assert np.abs(got - ref_none).max() <= 2e-2
     # masks: bit-exact outside the 1e-3 band around each frozen threshold
     for q in (0.5, 0.7, 0.9):
-        b = threshold(wl.name if wl.name in ("C1", "C2", "C3") else wl.name, q)
+        # frozen thresholds (R5); a workload without one takes the q-quantile of these
+        # oracle scores (oracle-derived, as R5 prescribes)
+        b = threshold(wl.name, q) if wl.name in THRESHOLD_NAMES else float(np.float32(np.quantile(ref_bf16, q)))
         far = np.abs(ref_bf16 - b) > BAND
         assert np.array_equal((got > np.float32(b))[far], (ref_bf16 > b)[far])
 
@@ -161,7 +166,8 @@ SELECT_CASES = [(configs.C1, 4), (configs.C2, 4), (configs.C3, 4), (configs.C4_S
 
 @pytest.mark.parametrize("wl,conn", SELECT_CASES, ids=[f"{c[0].name}-{c[1]}" for c in SELECT_CASES])
 def test_select_windows_mask_parity(wl, conn):
-    rng = np.random.default_rng(hash(wl.name) % 1000 + conn)
+    seed = zlib.crc32(wl.name.encode()) + conn       # stable across processes (no str-hash salt)
+    rng = np.random.default_rng(seed)
     gh, gw = -(-wl.src_h // wl.cell), -(-wl.src_w // wl.cell)
     masks = _random_masks(rng, 60, gh, gw)
     # add ground-truth masks of the workload's own video (perfect proxy)
@@ -172,10 +178,10 @@ def test_select_windows_mask_parity(wl, conn):
     r = otif.otif_select_windows(None, torch.from_numpy(masks).cuda(), 0.0, wl.src_w, wl.src_h, wl.cell,
                                  wl.sizes, connectivity=conn, want_mask=True)
     total = int(r["total"].item())
-    assert total == ref_t
-    assert np.array_equal(r["counts"].cpu().numpy(), ref_c)
-    assert np.array_equal(r["offsets"].cpu().numpy(), ref_o)
-    assert as_tuples(windows_np(r["windows"], total)) == as_tuples(ref_w)
+    assert total == ref_t, f"seed={seed}"
+    assert np.array_equal(r["counts"].cpu().numpy(), ref_c), f"seed={seed}"
+    assert np.array_equal(r["offsets"].cpu().numpy(), ref_o), f"seed={seed}"
+    assert as_tuples(windows_np(r["windows"], total)) == as_tuples(ref_w), f"seed={seed}"
     assert np.array_equal(r["mask"].cpu().numpy(), masks)
 
 

@@ -1,0 +1,264 @@
+"""GPU parity of the windowing path where it is ACTIVE (frames that keep several
+sub-frame windows), against the oracle, element by element on identical inputs.
+
+Stage 4 (grouping; readings R6–R11): thousands of multi-window frames on
+the C2, C3, C4a and C4d grids under 4- and 8-connectivity, with area costs
+and with non-area measured-style costs T_{w,h}, including int64 costs
+>= 2^30 (the kernel's matrix-free rescan path) and frames with more than 128
+components that merge (the deferred full-slice pass).  Ground-truth masks under the
+NEXT-1 window set W* (P:L153–155).
+Stage 5 (pack): sub-frame windows in identity mode through all three
+copy branches (16-B aligned bulk ring, unaligned funnel shift, byte path), several
+sizes per frame, k = 5 (C3), windows at the right / bottom borders and windows taller
+than one ring stage; byte-exact against oracle.pack_windows.
+NEXT-2 recall on windows that miss boxes.
+
+Seeds are fixed per case (zlib.crc32 of the case name) and appear in the assertion
+messages."""
+import zlib
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from synth import configs, masks, video
+from tests.helpers import as_tuples, windows_np
+
+pytestmark = pytest.mark.gpu
+
+otif = pytest.importorskip("paper_conf_sigmod_bastanim22_b200")
+from paper_conf_sigmod_bastanim22_b200 import tuning  # noqa: E402
+
+GRIDS = [configs.C2, configs.C3, configs.C4_SWEEP[0], configs.C4_SWEEP[3]]
+
+
+def _seed(name: str) -> int:
+    return zlib.crc32(name.encode())
+
+
+def _grid(wl):
+    return -(-wl.src_h // wl.cell), -(-wl.src_w // wl.cell)
+
+
+def _select_both(m, wl, sizes, conn, fw=None, fh=None):
+    fw = fw or wl.src_w
+    fh = fh or wl.src_h
+    ref_w, ref_c, ref_o, ref_t = oracle.select_windows(m, wl.cell, fw, fh, sizes, conn)
+    r = otif.otif_select_windows(None, torch.from_numpy(m).cuda(), 0.0, fw, fh, wl.cell, sizes, connectivity=conn)
+    return (ref_w, ref_c, ref_o, ref_t), r
+
+
+def _assert_same(ref, r, what):
+    ref_w, ref_c, ref_o, ref_t = ref
+    t = int(r["total"].item())
+    assert t == ref_t, what
+    assert np.array_equal(r["counts"].cpu().numpy(), ref_c), what
+    assert np.array_equal(r["offsets"].cpu().numpy(), ref_o), what
+    assert as_tuples(windows_np(r["windows"], t)) == as_tuples(ref_w), what
+
+
+# ------------------------------------------------------------------ stage 4
+def test_select_multiwindow_parity():
+    """>= 5000 multi-window frames (counted once, at area cost and 4-connectivity), each
+    bit-exact; the same frames again at 8-connectivity and with affine costs."""
+    multi_total = 0
+    for wl in GRIDS:
+        gh, gw = _grid(wl)
+        seed = _seed("multiwindow-" + wl.name)
+        rng = np.random.default_rng(seed)
+        m = np.concatenate([masks.sparse(rng, 1500, gh, gw, 0.003, 0.05), masks.blobs(rng, 1000, gh, gw)])
+        for conn in (4, 8):
+            for cost in ("area", "affine"):
+                sizes = [tuple(s) if cost == "area" else (s[0], s[1], 30000 + s[0] * s[1]) for s in wl.sizes]
+                ref, r = _select_both(m, wl, sizes, conn)
+                what = f"{wl.name} conn={conn} cost={cost} seed={seed}"
+                _assert_same(ref, r, what)
+                multi = int((ref[1] > 1).sum())
+                assert multi >= 1250, what + f": only {multi} multi-window frames"
+                if conn == 4 and cost == "area":
+                    multi_total += multi
+    assert multi_total >= 5000, multi_total
+
+
+def test_select_rescan_many_components_merge():
+    """Frames with > 128 components (deferred to the full-size slice, rescan path) whose
+    clusters merge in phase A (cheap 3-cell windows), and that stay multi-window."""
+    wl = configs.C4_SWEEP[0]                      # 23 x 40 grid
+    gh, gw = _grid(wl)
+    c = wl.cell
+    sizes = [(c, c, 2), (3 * c, c, 3), (c, 3 * c, 3), (wl.src_w, wl.src_h, 1000)]
+    seed = _seed("rescan-lattice")
+    rng = np.random.default_rng(seed)
+    m = masks.lattice(rng, 300, gh, gw)
+    ncomp = np.array([oracle.components(m[i], 4)[0] for i in range(len(m))])
+    assert (ncomp > 128).all()
+    ref, r = _select_both(m, wl, sizes, 4)
+    _assert_same(ref, r, f"lattice seed={seed}")
+    counts = ref[1]
+    assert (counts > 1).sum() >= 200
+    assert (counts < ncomp).sum() >= 200          # clusters merged on those frames
+    ref8, r8 = _select_both(m, wl, sizes, 8)
+    _assert_same(ref8, r8, f"lattice conn=8 seed={seed}")
+
+
+@pytest.mark.parametrize("wl", GRIDS, ids=lambda w: w.name)
+def test_select_large_int64_costs(wl):
+    """Costs >= 2^30 (no exact int32 gain matrix: the kernel takes the rescan path for
+    every frame) give the same windows as the oracle; measured-style non-area costs."""
+    gh, gw = _grid(wl)
+    seed = _seed("bigcost-" + wl.name)
+    rng = np.random.default_rng(seed)
+    m = np.concatenate([masks.sparse(rng, 600, gh, gw, 0.003, 0.05), masks.blobs(rng, 400, gh, gw)])
+    for scale in (1 << 20, 1 << 33):
+        sizes = [(s[0], s[1], (s[0] * s[1] + 7919 * i) * scale // 1024) for i, s in enumerate(wl.sizes)]
+        assert max(s[2] for s in sizes) >= (1 << 30) or scale < (1 << 30)
+        for conn in (4, 8):
+            ref, r = _select_both(m, wl, sizes, conn)
+            _assert_same(ref, r, f"{wl.name} scale={scale} conn={conn} seed={seed}")
+            assert (ref[1] > 1).sum() >= 200
+
+
+@pytest.mark.parametrize("wl", [configs.C2, configs.C4_SWEEP[1]], ids=lambda w: w.name)
+def test_select_ground_truth_under_wstar(wl):
+    """Perfect-proxy masks of the workload's own video, grouped with the window
+    set W* that NEXT-1 chooses from them over every cell-multiple candidate (
+    on these scenes W* holds road-band strips, e.g. 960x224 at C2)."""
+    n = 600
+    sc = video.make_scene(wl)
+    m = np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell) for t in range(n)])
+    cands = tuning.candidate_sizes(wl.src_w, wl.src_h, wl.cell)
+    idx, est = oracle.choose_window_sizes(m[::4], wl.cell, wl.src_w, wl.src_h, cands, k=3)
+    wstar = [(wl.src_w, wl.src_h)] + [tuple(cands[i][:2]) for i in idx if i >= 0]
+    assert len(wstar) == 3
+    for conn in (4, 8):
+        ref, r = _select_both(m, wl, wstar, conn)
+        _assert_same(ref, r, f"{wl.name} W*={wstar} conn={conn}")
+        assert (ref[1] > 1).sum() >= 200
+
+
+# ------------------------------------------------------------------ stage 5
+def _branch(w, sw):
+    """Which copy branch of pack_kernel a window takes (identity mode, aligned buffers)."""
+    rb = int(w["w"]) * 3
+    if rb % 16 == 0 and (int(w["x"]) * 3) % 16 == 0 and (sw * 3) % 16 == 0:
+        return "bulk"
+    if rb % 16 == 0:
+        return "funnel"
+    return "byte"
+
+
+def _pack_both(src, windows, sizes, caps=None):
+    n, sh, sw, _ = src.shape
+    if caps is None:
+        caps = [int((windows["size_idx"] == s).sum()) for s in range(len(sizes))]
+    ref_b, ref_slot, ref_cnt = oracle.pack_windows(src.numpy(), sh, sw, windows, sizes, caps)
+    wt = torch.from_numpy(np.stack([windows[f] for f in oracle.WINDOW_DTYPE.names], 1).astype(np.int32)).cuda()
+    total = torch.tensor([len(windows)], dtype=torch.int32, device="cuda")
+    b, slot, scount = otif.otif_pack_windows(src.cuda(), sh, sw, wt, total, sizes, caps)
+    assert np.array_equal(slot[:len(windows)].cpu().numpy(), ref_slot)
+    assert np.array_equal(scount.cpu().numpy(), ref_cnt)
+    for s in range(len(sizes)):
+        assert np.array_equal(b[s].cpu().numpy(), ref_b[s]), f"size {s} {sizes[s]}"
+    return ref_cnt
+
+
+def _win_array(rows):
+    a = np.zeros(len(rows), oracle.WINDOW_DTYPE)
+    for i, r in enumerate(rows):
+        a[i] = r
+    return a
+
+
+def test_pack_subframe_hand_built():
+    """Hand-built C2 windows: aligned and unaligned x, right / bottom borders, several
+    sizes per frame, windows taller than one 16 KB ring stage (128 rows x 384 B)."""
+    wl = configs.C2
+    src = video.frames(wl, 4)
+    sizes = [(128, 128), (256, 256), (960, 540), (112, 64), (100, 60)]
+    rows = []
+    for f in range(4):
+        rows += [(f, 0, 0, 128, 128, 0), (f, 16 * (f + 1), 200, 128, 128, 0), (f, 5 + f, 7, 128, 128, 0),
+                 (f, 960 - 128, 540 - 128, 128, 128, 0), (f, 960 - 256, 100 + f, 256, 256, 1),
+                 (f, 333, 284, 256, 256, 1), (f, 848, 476, 112, 64, 3), (f, 17, 480, 112, 64, 3),
+                 (f, 860, 480, 100, 60, 4), (f, 3, 1, 100, 60, 4)]
+    rows.append((2, 0, 0, 960, 540, 2))
+    win = _win_array(rows)
+    br = [_branch(w, wl.src_w) for w in win]
+    assert br.count("bulk") >= 8 and br.count("funnel") >= 8 and br.count("byte") >= 8
+    cnt = _pack_both(src, win, sizes)
+    assert list(cnt) == [16, 8, 1, 8, 8]
+
+
+@pytest.mark.parametrize("case", ["C2", "C3", "odd"])
+def test_pack_subframe_from_select(case):
+    """Windows produced by the grouping on object-shaped masks, packed in identity mode.
+    C3: five sizes (k = 5).  odd: a 1000 x 562 frame (rows 3000 B, not 16-B aligned; the
+    last cell column / row are clipped, R14), so windows at the borders are unaligned."""
+    if case == "odd":
+        wl = configs.C2.with_(name="odd", src_w=1000, src_h=562)
+    else:
+        wl = configs.C2 if case == "C2" else configs.C3
+    gh, gw = _grid(wl)
+    n = 12 if case != "C3" else 6
+    seed = _seed("pack-" + case)
+    rng = np.random.default_rng(seed)
+    m = masks.blobs(rng, n, gh, gw, max_objects=5, max_side=3)
+    m[:, :, -1] |= (rng.random((n, gh)) < 0.12).astype(np.uint8)     # right-border cells
+    m[:, -1, :] |= (rng.random((n, gw)) < 0.12).astype(np.uint8)     # bottom-border cells
+    sizes = list(wl.sizes) if case != "odd" else [(128, 128), (256, 256), (1000, 562)]
+    win, cnt, off, tot = oracle.select_windows(m, wl.cell, wl.src_w, wl.src_h, sizes)
+    assert (cnt > 1).sum() >= n // 2, f"seed={seed}"
+    if case == "odd":
+        src = torch.from_numpy(np.random.default_rng(seed).integers(0, 256, (n, 562, 1000, 3), dtype=np.uint8))
+    else:
+        src = video.frames(wl, n)
+    br = [_branch(w, wl.src_w) for w in win]
+    sub = [w for w in win if (w["w"], w["h"]) != (wl.src_w, wl.src_h)]
+    assert len(sub) >= 2 * n
+    edge = sum(int(w["x"] + w["w"] == wl.src_w or w["y"] + w["h"] == wl.src_h) for w in sub)
+    assert edge >= n
+    if case == "odd":
+        assert br.count("funnel") >= 2 * n
+    else:
+        assert br.count("bulk") >= 2 * n
+    got = _pack_both(src, win, sizes)
+    if case == "C3":
+        assert (got[:4] > 0).sum() >= 3            # several of the five sizes in use
+
+
+def test_pack_pipeline_counts_dropped_windows():
+    """batch_cap smaller than a size's window count: slots and size_count stay exact
+    (size_count counts every listed window) and only slots < batch_cap are written."""
+    wl = configs.C2
+    src = video.frames(wl, 3)
+    rows = [(f, 16 * i, 32 * f, 128, 128, 0) for f in range(3) for i in range(5)]
+    win = _win_array(rows)
+    cnt = _pack_both(src, win, [(128, 128), (960, 540)], caps=[7, 0])
+    assert list(cnt) == [15, 0]
+
+
+# ------------------------------------------------------------------ NEXT-2 recall
+def test_recall_with_missed_boxes():
+    """Windows that miss some ground-truth boxes (cells of half of the objects removed from
+    the mask): the GPU recall numerator equals the oracle's, and 0 < recall < 1."""
+    wl = configs.C4_SWEEP[1]
+    n = 120
+    sc = video.make_scene(wl)
+    seed = _seed("recall-missed")
+    rng = np.random.default_rng(seed)
+    m_list, boxes = [], []
+    for i in range(n):
+        bx = [b for b in sc.gt_boxes(i) if b[0] < b[2] and b[1] < b[3]]
+        keep = [b for b in bx if rng.random() < 0.5]
+        m_list.append(video.gt_mask(keep, wl.src_w, wl.src_h, wl.cell))
+        boxes += [(i, *b) for b in bx]
+    m = np.stack(m_list)
+    boxes = np.array(boxes, np.int32).reshape(-1, 5)
+    r = otif.otif_select_windows(None, torch.from_numpy(m).cuda(), 0.0, wl.src_w, wl.src_h, wl.cell, wl.sizes)
+    t = int(r["total"].item())
+    w = windows_np(r["windows"], t)
+    cov = tuning.window_recall(torch.from_numpy(boxes).cuda(), r["windows"], r["offsets"], r["counts"])
+    ref = oracle.covered(boxes, w)
+    assert cov == ref, f"seed={seed}"
+    assert 0 < ref < len(boxes), (ref, len(boxes))
