@@ -1,5 +1,5 @@
 #!/usr/bin/env python
-"""bench.py — OTIF proxy + windowing hot path on B200: frames/s, roofline, CPU oracle baseline.
+"""bench.py — OTIF proxy + windowing hot path on B200: frames/s, rooflines, CPU oracle baseline.
 
 A "step" is one pass of the whole hot path (resize -> proxy CNN -> threshold ->
 connected components + window selection -> crop/pack) over the BASELINE.json configs[1]
@@ -9,16 +9,25 @@ larger than the 126 MB L2, so no L2 flush is needed between steps).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl otif|reference]
 
-N > 1 runs under torchrun (one process per GPU, NCCL): every rank processes its own
-4500-frame shard of clips (weak scaling, no data-path collective); per-rank counters are
-combined with one all_gather at the end.  --impl reference times the CPU oracle
-(oracle/, plain fp64 C) on the host cores on a bounded sample of the same workload.
+N > 1: one process per GPU over NCCL.  Without torchrun in the environment the script
+re-launches itself under `torch.distributed.run` (127.0.0.1).  Every rank processes its
+own 4500-frame clip set (weak scaling, no data-path collective); per-rank counters are
+combined with one all_gather at the end.  The "c5" object runs the fixed 8-hour corpus
+(480 one-minute clips) sharded by contiguous clip ranges.
+
+Beside the headline line (random-init proxy, north_star) the JSON carries: the other
+BASELINE configs (C1, C3, C4b, C4d) with their own rooflines and oracle samples, the
+windowing-active path (trained proxy + the NEXT-1 window set W*, and the perfect proxy
+under W*), the NEXT-3 / NEXT-4 rows, e2e through the C ABI with host buffers, and the
+oracle timed on the host cores.  --impl reference times the CPU oracle (oracle/, plain
+fp64 C) on a bounded sample of the same workload.
 """
 from __future__ import annotations
 
 import argparse
 import json
 import os
+import socket
 import subprocess
 import sys
 import tempfile
@@ -49,8 +58,8 @@ def threshold_for(name: str, q: float = 0.7) -> float:
 
 
 def conv_macs_per_frame(wl, enc, dec):
-    """Algorithmic MACs of the tensor-core layers E2..E5, D1 (and E1, D2) per frame:
-    Ho*Wo*Cout*Cin*k^2 with Ho = ceil(Hi/2) for strided layers (P:L135 shape, reading R1/R2)."""
+    """Algorithmic MACs of E1..E5, D1 per frame: Ho*Wo*Cout*Cin*k^2 with Ho = ceil(Hi/2) for
+    strided layers (P:L135 shape, readings R1/R2); and the D2 head's MACs."""
     h, w, c = wl.proxy_h, wl.proxy_w, 3
     layers = []
     for i in range(6):
@@ -133,13 +142,13 @@ class ClockSampler:
 
 
 # --------------------------------------------------------------------------- CPU oracle leg
-def oracle_frames_per_s(wl, frames_u8: np.ndarray, threshold: float, cores: int):
+def oracle_frames_per_s(wl, frames_u8: np.ndarray, threshold: float, cores: int, blob=None, sizes=None):
     """Time the oracle (as it stands) on a bounded sample: resize, proxy (quant=bf16),
     threshold, grouping and pack per frame, one frame per task over `cores` threads."""
     import oracle
     from synth import configs, weights
-    blob = weights.proxy_weights()
-    sizes = [tuple(s) for s in wl.sizes]
+    blob = weights.proxy_weights() if blob is None else blob
+    sizes = [tuple(s) for s in (wl.sizes if sizes is None else sizes)]
 
     def one(i):
         f = frames_u8[i:i + 1]
@@ -156,6 +165,15 @@ def oracle_frames_per_s(wl, frames_u8: np.ndarray, threshold: float, cores: int)
         list(ex.map(one, range(n)))
     dt = time.perf_counter() - t0
     return n / dt, dt
+
+
+def cpu_baseline_for(wl, thr, n, cores):
+    from synth import video
+    frames = video.frames(wl, n).numpy()
+    fps, dt = oracle_frames_per_s(wl, frames, thr, cores)
+    return {"value": fps, "unit": "frames/s", "cores": cores, "kind": "oracle",
+            "sample": f"first {n} {wl.name} frames, full path per frame (resize, fp64 proxy quant=bf16, threshold, "
+                      f"grouping, pack), one frame per task on {cores} threads, {dt:.1f} s wall"}
 
 
 def run_reference(args):
@@ -191,6 +209,118 @@ def run_reference(args):
     return 0
 
 
+# --------------------------------------------------------------------------- GPU measurement helpers
+def measure_pipeline(otif, wl, blob, thr, src, steps, warmup, sizes=None, caps=None, batch=None):
+    """Whole path (otif_pipeline_run_device) over the device-resident frames `src`: warm-up,
+    then `steps` timed passes bracketed by CUDA events on the launching stream; per-stage
+    event times, kernel launches and device counters."""
+    import torch
+    n = src.shape[0]
+    pipe = otif.Pipeline(wl, blob, thr, max_batch=batch or n, sizes=sizes, batch_cap=caps)
+    stream = torch.cuda.current_stream()
+    for _ in range(warmup):
+        pipe.run_device(src)
+    torch.cuda.synchronize()
+    pipe.reset_counters()
+    pipe.set_timing(True)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        pipe.run_device(src)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms_total = e0.elapsed_time(e1)
+    stage_ms, launches = pipe.stage_ms()
+    ctr = pipe.counters()
+    out = {"pipe": pipe, "ms_total": ms_total, "stage_ms": stage_ms, "launches": launches, "ctr": ctr,
+           "frames": n * steps, "steps": steps}
+    return out
+
+
+CONV_STAGES = ["proxy_prep_e1", "conv_e2", "conv_e3", "conv_e4", "conv_e5", "conv_d1_head"]
+
+
+def rooflines(wl, m, peaks, peak_src, traffic=None):
+    """Per-kernel rooflines of one measured pipeline: the proxy convolutions (tensor) against
+    the measured bf16 burst peak (the timed regions are well under a second, at the
+    maximum SM clock) with the sustained peak beside it; resize and pack (HBM) against
+    the measured copy bandwidth; the grouping as ns/frame and share of the step."""
+    from synth import configs
+    sm = m["stage_ms"]
+    frames = int(m["ctr"][0].item())
+    steps = m["steps"]
+    macs, head = conv_macs_per_frame(wl, configs.ENC_WIDTHS, configs.DEC_WIDTH)
+    conv_ms = sum(sm[s] for s in CONV_STAGES)
+    conv_flops = 2.0 * sum(macs) * frames
+    tflops = conv_flops / (conv_ms / 1e3) / 1e12 if conv_ms > 0 else 0.0
+    burst = float(peaks.get("bf16_tflops"))
+    sustained = float(peaks.get("bf16_tflops_sustained", burst))
+    per_layer = {}
+    for i, s in enumerate(CONV_STAGES[1:]):
+        fl = 2.0 * (macs[i + 1] + (macs[0] if i == 0 else 0)) * frames
+        ms = sm[s] + (sm["proxy_prep_e1"] if i == 0 else 0.0)
+        name = "conv_e1_e2" if i == 0 else s
+        per_layer[name] = {"ms_per_step": ms / steps, "tflops": fl / (ms / 1e3) / 1e12 if ms > 0 else None,
+                           "frac_burst": fl / (ms / 1e3) / 1e12 / burst if ms > 0 else None}
+    hbm = float(peaks.get("hbm_gbs"))
+    rs_bytes = resize_bytes_per_frame(wl) * frames
+    pk_bytes = 2.0 * 3 * int(m["ctr"][14].item())
+    step_sum = sum(sm.values())
+    conv = {"bound": "tensor", "achieved": tflops, "peak": burst, "unit": "TFLOP/s", "frac": tflops / burst,
+            "frac_vs_sustained": tflops / sustained, "traffic": traffic,
+            "peak_source": peak_src + ": bf16 burst (cuBLAS 8192^3 best of 10 at the max SM clock); "
+                                      "sustained (4 s loop under the power cap) beside it",
+            "algorithmic": f"2 x {sum(macs) / 1e6:.1f} MMAC/frame (E1..D1) x {frames // steps} frames per launch set",
+            "layers": per_layer, "ms_per_step": conv_ms / steps, "share_of_step": conv_ms / step_sum}
+    out = {"conv": conv}
+    for k, byts in (("resize", rs_bytes), ("pack", pk_bytes)):
+        ms = sm[k]
+        gbs = byts / (ms / 1e3) / 1e9 if ms > 0 else None
+        out[k] = {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm if gbs else None,
+                  "frac_spec_8tbs": gbs / 8000.0 if gbs else None, "bytes_per_step": byts / steps,
+                  "ms_per_step": ms / steps}
+    out["select"] = {"ms_per_step": sm["select"] / steps, "ns_per_frame": sm["select"] * 1e6 / max(frames, 1),
+                     "share_of_step": sm["select"] / step_sum if step_sum else None}
+    return out
+
+
+def window_stats(m, wl, sizes):
+    c = m["ctr"].cpu().tolist()
+    frames = c[0]
+    full_idx = [i for i, s in enumerate(sizes) if (int(s[0]), int(s[1])) == (wl.src_w, wl.src_h)]
+    full = sum(c[5 + i] for i in full_idx)
+    return {"windows_per_frame": c[2] / max(frames, 1), "fallback_share": full / max(frames, 1),
+            "window_area_fraction": c[3] / max(frames * wl.src_w * wl.src_h, 1),
+            "per_size": c[5:5 + len(sizes)], "dropped_windows": c[13], "positive_cell_fraction":
+            c[1] / max(frames * (-(-wl.src_h // wl.cell)) * (-(-wl.src_w // wl.cell)), 1)}
+
+
+def caps_for(wl, sizes, n, per_frame=8):
+    """Detector batch capacities: one full-frame slot per frame; per_frame slots of each
+    smaller size (bounded by how many such windows fit in a frame)."""
+    out = []
+    for s in sizes:
+        if (int(s[0]), int(s[1])) == (wl.src_w, wl.src_h):
+            out.append(n)
+        else:
+            fit = max(1, (wl.src_w // int(s[0])) * (wl.src_h // int(s[1])))
+            out.append(n * min(per_frame, fit))
+    return out
+
+
+def choose_wstar(otif_tuning, wl, clip, n, k, dev):
+    """NEXT-1 on the GPU: W* from the perfect-proxy masks of n frames of `clip`."""
+    import torch
+    from synth import video
+    sc = video.make_scene(wl, clip=clip)
+    masks = torch.from_numpy(np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell)
+                                       for t in range(n)])).to(dev)
+    cands = otif_tuning.candidate_sizes(wl.src_w, wl.src_h, wl.cell)
+    chosen, sums, idx = otif_tuning.choose_window_sizes(masks, wl.src_w, wl.src_h, wl.cell, cands, k=k)
+    return [tuple(int(v) for v in c[:2]) for c in chosen], sums
+
+
 # --------------------------------------------------------------------------- GPU leg
 def run_otif(args):
     import torch
@@ -199,13 +329,24 @@ def run_otif(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}")
+    nccl = None
     if world > 1:
+        # communicator init lines (rank count per communicator) go to stderr, not the JSON stdout
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        nccl = {"backend": dist.get_backend(), "comm_nranks": dist.get_world_size(),
+                "nccl_version": ".".join(str(v) for v in torch.cuda.nccl.version())}
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
 
     import paper_conf_sigmod_bastanim22_b200 as otif
+    from paper_conf_sigmod_bastanim22_b200 import dist as odist
+    from paper_conf_sigmod_bastanim22_b200 import tuning as otif_tuning
     from synth import configs, video, weights
 
     wl = configs.C2
@@ -213,57 +354,27 @@ def run_otif(args):
     blob = weights.proxy_weights()
     b = threshold_for(wl.name)
     peaks, peak_src = load_peaks()
+    cores = len(os.sched_getaffinity(0))
+    extras = (world == 1 or rank == 0) and not args.headline_only
 
-    # this rank's shard: its own 4500-frame clip set (weak scaling; clip seeds by rank)
+    # this rank's shard: its own 4500-frame clip (weak scaling; clip seeds by rank)
     src = torch.empty((n, wl.src_h, wl.src_w, 3), dtype=torch.uint8, device=dev)
     video.make_scene(wl, clip=rank).render(range(n), out=src)
     torch.cuda.synchronize()
 
-    # device path: the whole clip is one device batch by default (every stage is one launch
-    # over all frames, so latency-bound stages see enough frames to fill the SMs)
-    batch = args.batch if args.batch > 0 else n
-    pipe = otif.Pipeline(wl, blob, b, max_batch=batch, proxy_batch=args.proxy_batch, overlap_chunks=args.overlap)
-    stream = torch.cuda.current_stream()
-    for _ in range(args.warmup):
-        pipe.run_device(src)
-    torch.cuda.synchronize()
-    pipe.reset_counters()
-    pipe.set_timing(True)
-
+    # ---- headline: C2, random-init proxy (north_star), one device batch of 4500 frames
     sampler = ClockSampler(local)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for _ in range(args.steps):
-        pipe.run_device(src)
-    e1.record(stream)
-    torch.cuda.synchronize()
+    m = measure_pipeline(otif, wl, blob, b, src, args.steps, args.warmup, batch=args.batch or None)
     if world > 1:
         dist.barrier()
     clocks = sampler.stop()
-    ms_total = e0.elapsed_time(e1)
-    stage_ms, launches = pipe.stage_ms()
-    ctr = pipe.counters()
-    from paper_conf_sigmod_bastanim22_b200 import dist as odist
-    ms_max = odist.max_over_ranks(ms_total, dev)
-    gathered = odist.gather_counters(ctr)
-    ms_step = ms_max / args.steps
+    ms_max = odist.max_over_ranks(m["ms_total"], dev)
+    gathered = odist.gather_counters(m["ctr"])
     frames_total = int(gathered[:, 0].sum().item())
     value = frames_total / (ms_max / 1000.0)
-
-    # roofline: the proxy's tcgen05 convolution kernels (E1+E2 fused, E3..E5, D1)
-    macs, head = conv_macs_per_frame(wl, configs.ENC_WIDTHS, configs.DEC_WIDTH)
-    frames_rank = int(ctr[0].item())
-    # every proxy conv runs on tcgen05: E1 (fused into E2's kernel, e12_umma_kernel, when it
-    # applies; else its own kernel, timed in the prep stage) and E2..E5, D1 (conv_umma_kernel)
-    conv_stage = ["proxy_prep_e1", "conv_e2", "conv_e3", "conv_e4", "conv_e5", "conv_d1_head"]
-    conv_ms = sum(stage_ms[s] for s in conv_stage)
-    conv_flops = 2.0 * sum(macs) * frames_rank
-    achieved_tflops = conv_flops / (conv_ms / 1000.0) / 1e12 if conv_ms > 0 else 0.0
-    peak_t = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
-    n_batches = -(-n // batch) * args.steps
     traffic = None
     prof = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if os.path.exists(prof):
@@ -271,79 +382,110 @@ def run_otif(args):
             traffic = json.load(open(prof)).get("conv_dram_bytes_per_batch")
         except Exception:
             traffic = None
-    per_layer = {}
-    for i, s in enumerate(conv_stage[1:]):
-        fl = 2.0 * (macs[i + 1] + (macs[0] if i == 0 else 0)) * frames_rank
-        ms = stage_ms[s] + (stage_ms["proxy_prep_e1"] if i == 0 else 0.0)
-        if i == 0:
-            s = "conv_e1_e2"
-        per_layer[s] = {"ms_per_launch": ms / n_batches,
-                        "tflops": fl / (ms / 1000.0) / 1e12 if ms > 0 else None}
-    hbm = float(peaks.get("hbm_gbs"))
-    rs_bytes = resize_bytes_per_frame(wl) * frames_rank
-    pk_bytes = 2.0 * 3 * int(ctr[3].item())
-    stages = {k: {"ms_per_step": v / args.steps} for k, v in stage_ms.items()}
-    stages["resize"]["gbs"] = rs_bytes / (stage_ms["resize"] / 1000.0) / 1e9 if stage_ms["resize"] else None
-    stages["resize"]["hbm_frac"] = stages["resize"]["gbs"] / hbm if stages["resize"]["gbs"] else None
-    stages["pack"]["gbs"] = pk_bytes / (stage_ms["pack"] / 1000.0) / 1e9 if stage_ms["pack"] else None
-    stages["pack"]["hbm_frac"] = stages["pack"]["gbs"] / hbm if stages["pack"]["gbs"] else None
-    step_sum = sum(stage_ms.values())
-    stages["conv_share_of_step"] = conv_ms / step_sum if step_sum else None
-    # HBM stages against the spec bandwidth too; grouping as ns/frame and share
-    for k in ("resize", "pack"):
-        if stages[k].get("gbs"):
-            stages[k]["hbm_frac_spec_8tbs"] = stages[k]["gbs"] / 8000.0
-    if stage_ms["select"] and frames_rank:
-        stages["select"]["ns_per_frame"] = stage_ms["select"] * 1e6 / frames_rank
-        stages["select"]["share_of_step"] = stage_ms["select"] / step_sum if step_sum else None
+    rl = rooflines(wl, m, peaks, peak_src, traffic)
+    launches = m["launches"]
+    m["pipe"].close()
 
-    # perfect-proxy line: stages 3-5 on ground-truth cell masks (mask_in), which
-    # gives object-aligned windows instead of the random-init proxy's full-frame fallback
-    perfect = None
-    if not args.no_perfect:
+    objs = {}
+    # ---- the other BASELINE configs, each with its own rooflines and oracle sample
+    if extras and not args.no_configs:
+        cfg = {}
+        for cw, nfr in ((configs.C1, None), (configs.C3, None), (configs.C4_SWEEP[1], None), (configs.C4_SWEEP[3], None)):
+            nn = nfr or cw.n_frames
+            s2 = torch.empty((nn, cw.src_h, cw.src_w, 3), dtype=torch.uint8, device=dev)
+            video.make_scene(cw).render(range(nn), out=s2)
+            thr = threshold_for(cw.name)
+            steps_c = max(args.steps, int(np.ceil(2000.0 / nn)) if nn < 1000 else args.steps)
+            mc = measure_pipeline(otif, cw, blob, thr, s2, steps_c, args.warmup)
+            r = rooflines(cw, mc, peaks, peak_src)
+            cfg[cw.name] = {"workload": f"{cw.src_w}x{cw.src_h} {cw.scene}, {nn} frames, proxy {cw.proxy_w}x{cw.proxy_h} "
+                                        f"(S={cw.stride}), {cw.cell}-px cells, W={[list(x) for x in cw.sizes]}",
+                            "frames_per_s": mc["frames"] / (mc["ms_total"] / 1e3),
+                            "ms_per_step": mc["ms_total"] / steps_c, "steps": steps_c, "threshold_q": 0.7,
+                            "roofline": r, "windows": window_stats(mc, cw, cw.sizes), "gpu_launches": mc["launches"],
+                            "cpu_baseline": None if args.no_cpu_baseline else
+                            cpu_baseline_for(cw, thr, min(args.oracle_frames, nn), cores)}
+            mc["pipe"].close()
+            del s2
+            torch.cuda.empty_cache()
+        objs["configs"] = cfg
+
+    # ---- windowing active: the NEXT-3-trained C2 proxy and the perfect proxy under W*
+    if extras and not args.no_windowing:
+        from scripts import train_proxy
+        t0 = time.time()
+        tw, tinfo = train_proxy.train_weights(wl, steps=args.train_steps, batch=32, clip=1)
+        wstar3, sums3 = choose_wstar(otif_tuning, wl, 1, 600, 3, dev)
+        wstar5, sums5 = choose_wstar(otif_tuning, wl, 1, 600, 5, dev)
+        prep_s = time.time() - t0
+        win = {"what": "C2 clip 0 (4500 frames) through the whole path with the proxy trained by NEXT-3 (P:L137-141) "
+                       "on clip 1 and the window set W* chosen by NEXT-1 (P:L153-155) from clip 1's ground-truth "
+                       "masks; B = 0.5 on the trained scores",
+               "train": {k: tinfo[k] for k in ("steps", "batch", "ms_per_step", "loss")},
+               "W*_k3": [list(x) for x in wstar3], "W*_k5": [list(x) for x in wstar5], "prep_s": prep_s}
+        for tag, W in (("k3", wstar3), ("k5", wstar5)):
+            caps = caps_for(wl, W, n)
+            mw = measure_pipeline(otif, wl, tw, 0.5, src, args.steps, args.warmup, sizes=W, caps=caps)
+            win[tag] = {"frames_per_s": mw["frames"] / (mw["ms_total"] / 1e3), "ms_per_step": mw["ms_total"] / args.steps,
+                        "windows": window_stats(mw, wl, W), "roofline": rooflines(wl, mw, peaks, peak_src),
+                        "batch_cap": caps}
+            mw["pipe"].close()
+            torch.cuda.empty_cache()
+        # perfect proxy: stages 3-5 on the ground-truth cell masks of clip 0 under W*
         sc = video.make_scene(wl, clip=rank)
         masks = torch.from_numpy(np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell)
                                            for t in range(n)])).to(dev)
-        caps = [n if (s[0], s[1]) == (wl.src_w, wl.src_h) else 8 * n for s in wl.sizes]
-
-        def perfect_step():
-            r = otif.otif_select_windows(None, masks, 0.0, wl.src_w, wl.src_h, wl.cell, wl.sizes)
-            otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], wl.sizes, caps)
-            return r
-
-        for _ in range(2):
-            perfect_step()
-        torch.cuda.synchronize()
-        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        p0.record()
-        for _ in range(args.steps):
-            r = perfect_step()
-        p1.record()
-        torch.cuda.synchronize()
-        pms = p0.elapsed_time(p1) / args.steps
-        tot = int(r["total"].item())
-        wins = r["windows"][:tot].cpu().numpy()
-        px = int((wins[:, 3].astype(np.int64) * wins[:, 4]).sum()) if tot else 0
-        perfect = {"what": "select (mask_in = ground-truth cells) + pack per step; allocations inside",
-                   "frames_per_s": n / (pms / 1000.0), "ms_per_step": pms, "windows_per_frame": tot / n,
-                   "window_area_fraction": px / (n * wl.src_w * wl.src_h),
-                   "pack_bytes_per_step": 2 * 3 * px}
+        pp = {}
+        for tag, W in (("default_W", list(wl.sizes)), ("W*_k3", wstar3), ("W*_k5", wstar5)):
+            caps = caps_for(wl, W, n)
+            r = otif.otif_select_windows(None, masks, 0.0, wl.src_w, wl.src_h, wl.cell, W)
+            otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], W, caps)
+            torch.cuda.synchronize()
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+            sel_ms = pk_ms = 0.0
+            for _ in range(args.steps):
+                ev[0].record()
+                r = otif.otif_select_windows(None, masks, 0.0, wl.src_w, wl.src_h, wl.cell, W)
+                ev[1].record()
+                bt, slot, scount = otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], W, caps)
+                ev[2].record()
+                torch.cuda.synchronize()
+                sel_ms += ev[0].elapsed_time(ev[1])
+                pk_ms += ev[1].elapsed_time(ev[2])
+                del bt
+            tot = int(r["total"].item())
+            wins = r["windows"][:tot].cpu().numpy()
+            px = int((wins[:, 3].astype(np.int64) * wins[:, 4]).sum()) if tot else 0
+            full = int(((wins[:, 3] == wl.src_w) & (wins[:, 4] == wl.src_h)).sum()) if tot else 0
+            sc_np = scount.cpu().numpy()
+            pp[tag] = {"W": [list(x) for x in W], "windows_per_frame": tot / n, "fallback_share": full / n,
+                       "window_area_fraction": px / (n * wl.src_w * wl.src_h), "per_size": sc_np.tolist(),
+                       "dropped_windows": int(np.maximum(sc_np - np.array(caps), 0).sum()),
+                       "select_ns_per_frame": sel_ms / args.steps * 1e6 / n,
+                       "select_ms_per_step": sel_ms / args.steps, "pack_ms_per_step": pk_ms / args.steps,
+                       "pack_gbs": 2 * 3 * px / (pk_ms / args.steps / 1e3) / 1e9 if pk_ms > 0 else None,
+                       "est_sum": int(r["est_sum"].item())}
+            pp[tag]["pack_hbm_frac"] = pp[tag]["pack_gbs"] / float(peaks["hbm_gbs"]) if pp[tag]["pack_gbs"] else None
+        win["perfect_proxy"] = pp
         del masks
+        objs["windowing_active"] = win
 
-    # §8(f) NEXT-4: track index over S* + refinement of gap-16 query tracks (C6)
-    next4 = None
-    if not args.no_next4:
+    # ---- C5: the 8-hour corpus (480 one-minute clips x 450 frames), contiguous
+    # clip ranges per rank, per-clip device counters and hashes, strong scaling
+    if not args.no_c5:
+        objs["c5"] = run_c5(otif, odist, configs, video, blob, b, dev, world, rank, args)
+
+    # ---- NEXT-4: track index over S* + refinement of gap-16 query tracks (C6)
+    if extras and not args.no_next4:
         from scripts import tracks_bench
-        next4 = tracks_bench.run(tracks_bench.tracks.C6, reps=5)
+        objs["track_refinement"] = tracks_bench.run(tracks_bench.tracks.C6, reps=5)
 
-    # §8(f) NEXT-3: proxy training steps (fp32 forward + backward + Adam) on
-    # 32 of this rank's C2 frames with ground-truth cell labels, timed with CUDA events
-    next3 = None
-    if not args.no_next3:
+    # ---- NEXT-3: proxy training steps (fp32 forward + backward + Adam)
+    if extras and not args.no_next3:
         from paper_conf_sigmod_bastanim22_b200 import train as otif_train
         sc = video.make_scene(wl, clip=rank)
         tsel = [t for t in range(0, n, max(n // 64, 1)) if sc.gt_boxes(t)][:32]
-        bx = np.array([(i, *b) for i, t in enumerate(tsel) for b in sc.gt_boxes(t) if b[0] < b[2] and b[1] < b[3]],
+        bx = np.array([(i, *bb) for i, t in enumerate(tsel) for bb in sc.gt_boxes(t) if bb[0] < bb[2] and bb[1] < bb[3]],
                       np.int32).reshape(-1, 5)
         gh, gw = -(-wl.src_h // wl.cell), -(-wl.src_w // wl.cell)
         lab = otif_train.otif_cell_labels(torch.from_numpy(bx).to(dev), len(tsel), (gh, gw), wl.src_w, wl.src_h,
@@ -359,33 +501,34 @@ def run_otif(args):
         t1e.record()
         torch.cuda.synchronize()
         tms = t0e.elapsed_time(t1e) / args.steps
+        macs, head = conv_macs_per_frame(wl, configs.ENC_WIDTHS, configs.DEC_WIDTH)
         train_flop = 3 * 2 * (sum(macs) + head) * len(tsel)      # forward + dgrad + wgrad
-        next3 = {"what": "fp32 training step (forward, BCE head, dgrad, wgrad, Adam); convolution GEMMs on tcgen05 (3xTF32, fp32-accurate)",
-                 "batch": len(tsel), "ms_per_step": tms, "train_frames_per_s": len(tsel) / (tms / 1e3),
-                 "tflops": train_flop / (tms / 1e3) / 1e12, "loss_first": l0, "loss_last": float(lt.item())}
-        # roofline of the training GEMMs: tf32 peak = measured sustained bf16 x the guide's
-        # nominal tf32/bf16 ratio (1.1 / 2.25); 3xTF32 issues 3 MMAs per useful product
-        tf32_peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))) * 1.1 / 2.25
-        next3["roofline"] = {"bound": "tensor", "unit": "TFLOP/s", "achieved": next3["tflops"],
-                             "peak": tf32_peak / 3.0, "frac": next3["tflops"] / (tf32_peak / 3.0),
-                             "peak_source": "measured bf16 sustained x 1.1/2.25 (tf32), / 3 (3xTF32 useful rate); "
-                                            "the step is bound by the implicit-GEMM gathers, not the MMAs"}
+        nx3 = {"what": "fp32 training step (forward, BCE head, dgrad, wgrad, Adam); convolution GEMMs on tcgen05 "
+                       "(3xTF32, fp32-accurate)", "batch": len(tsel), "ms_per_step": tms,
+               "train_frames_per_s": len(tsel) / (tms / 1e3), "tflops": train_flop / (tms / 1e3) / 1e12,
+               "loss_first": l0, "loss_last": float(lt.item())}
+        # tf32 peak = measured bf16 burst x the guide's nominal tf32/bf16 ratio (1.1 / 2.25);
+        # 3xTF32 issues 3 MMAs per useful product
+        tf32_peak = float(peaks.get("bf16_tflops")) * 1.1 / 2.25
+        nx3["roofline"] = {"bound": "tensor", "unit": "TFLOP/s", "achieved": nx3["tflops"], "peak": tf32_peak / 3.0,
+                           "frac": nx3["tflops"] / (tf32_peak / 3.0),
+                           "peak_source": "measured bf16 burst x 1.1/2.25 (tf32), / 3 (3xTF32 useful rate); "
+                                          "the step is bound by the implicit-GEMM gathers, not the MMAs"}
+        objs["proxy_training"] = nx3
         del tr, timg, lab
 
-    # end to end through the C ABI with HOST frames: pinned H2D + D2H inside the timed region
+    # ---- end to end through the C ABI with HOST frames: pinned H2D + D2H inside the timed region
     e2e = None
     if not args.no_e2e:
-        # pinned host copy of this rank's clip (7.0 GB); if the host cannot pin that much
-        # (8 ranks on one node), fall back to the first 1024 frames of the clip
         e2e_frames = n
         try:
             host = torch.empty(src.shape, dtype=torch.uint8, pin_memory=True)
         except RuntimeError:
+            # the host cannot pin 7 GB per rank (8 ranks on one node): first 1024 frames
             e2e_frames = min(n, 1024)
             host = torch.empty((e2e_frames,) + tuple(src.shape[1:]), dtype=torch.uint8, pin_memory=True)
         host.copy_(src[:e2e_frames])
         del src
-        pipe.close()
         torch.cuda.empty_cache()
         pipe = otif.Pipeline(wl, blob, b, max_batch=args.host_batch)
         pipe.run_host(host)  # warm-up (allocates the output arrays)
@@ -395,56 +538,107 @@ def run_otif(args):
             t0 = time.perf_counter()
             last = pipe.run_host(host)
             times.append(time.perf_counter() - t0)
-        win, counts, sc, tot = last
+        win_, counts, sc_, tot = last
         tmax = odist.max_over_ranks(max(times), dev)
         e2e = {"value": world * e2e_frames / tmax, "unit": "frames/s",
                "h2d_bytes_per_step": int(host.numel()),
-               "d2h_bytes_per_step": int(4 + 4 * e2e_frames + 24 * tot + 8 * (5 + len(wl.sizes))),
+               "d2h_bytes_per_step": int(4 + 4 * e2e_frames + 24 * tot + 8 * 15),
                "frames_per_step_per_gpu": e2e_frames,
-               "api": "otif_pipeline_run_host (C ABI), pinned host frames, 2 streams"}
+               "api": "otif_pipeline_run_host (C ABI), pinned host frames, 2 streams (PCIe-bound)"}
+        pipe.close()
 
     cpu_baseline = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        from synth import video as v2
-        cores = len(os.sched_getaffinity(0))
-        frames = v2.frames(wl, args.oracle_frames).numpy()
-        fps, dt = oracle_frames_per_s(wl, frames, b, cores)
-        cpu_baseline = {"value": fps, "unit": "frames/s", "cores": cores, "kind": "oracle",
-                        "sample": f"first {args.oracle_frames} C2 frames, full path (resize, fp64 proxy quant=bf16, "
-                                  f"threshold, grouping, pack), one frame per task, {dt:.1f} s wall"}
+        cpu_baseline = cpu_baseline_for(wl, b, args.oracle_frames, cores)
 
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "frames/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms_max / args.steps, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
             "config": {"workload": "C2: 960x540 traffic-camera clip, 10 min @30 fps sampled every 4th frame "
                                    "(4500 frames per GPU), proxy at 1/4 res (240x135), 32x32-px cells (17x30 grid)",
-                       "frames_per_step_per_gpu": n, "batch": batch, "W": [list(s) for s in wl.sizes],
+                       "frames_per_step_per_gpu": n, "batch": args.batch or n, "W": [list(s) for s in wl.sizes],
                        "threshold": b, "threshold_q": 0.7, "proxy": "E1-E5 (32,64,128,256,256) + D1 128 + D2 1, "
                        "random init PCG64(20220612)", "l2": "inputs (7.0 GB/GPU) exceed the 126 MB L2; no flush",
                        "parallelism": f"dp{world} (clip-sharded)"},
-            "roofline": {"bound": "tensor", "kernel": "proxy convs on tcgen05: e12_umma_kernel (E1 fused into E2) + conv_umma_kernel (E3..E5, D1)",
-                         "achieved": achieved_tflops, "peak": peak_t, "unit": "TFLOP/s",
-                         "frac": achieved_tflops / peak_t if peak_t else None, "traffic": traffic,
-                         "peak_source": peak_src + " bf16 sustained", "per_launch": "5 launches per batch of "
-                         f"{batch} frames (E1+E2 fused: the prep stage holds only the workspace tag); achieved = algorithmic FLOPs of E1..D1 / event-timed duration",
-                         "layers": per_layer},
-            "stages": stages,
-            "perfect_proxy": perfect,
-            "track_refinement": next4,
-            "proxy_training": next3,
+            "roofline": dict(rl["conv"], kernel="proxy convs on tcgen05: e12_umma_kernel (E1 fused into E2) + "
+                                                "conv_umma_kernel (E3..E5, D1+D2 head)",
+                             per_launch="5 launches per batch of 4500 frames; achieved = algorithmic FLOPs of "
+                                        "E1..D1 / CUDA-event time of those launches on the pipeline stream"),
+            "stages": {k: v for k, v in rl.items() if k != "conv"},
+            **objs,
             "cpu_baseline": cpu_baseline,
             "e2e": e2e,
             "gpu_launches": int(launches),
             "clocks": clocks,
+            "nccl": nccl,
             "counters": odist.combine(gathered),
         }
         print(json.dumps(line), flush=True)
-    pipe.close()
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def run_c5(otif, odist, configs, video, blob, b, dev, world, rank, args):
+    """C5: 480 clips x 450 frames (216,000 frames, 336 GB of u8: larger than HBM), every rank
+    renders the same 8-clip pool and clip k reads pool slot k mod 8; rank r
+    takes clips shard_clips(480, G, r).  One pipeline call per clip (frame_base = the
+    clip's global first frame, so window hashes are keyed by the global frame); its
+    device counters are snapshotted per clip and reset.  Time = max over ranks."""
+    import torch
+    import torch.distributed as dist
+    wl = configs.C5
+    fpc = configs.C5_FRAMES_PER_CLIP
+    n_clips = configs.C5_CLIPS if args.c5_clips <= 0 else args.c5_clips
+    pool = torch.empty((configs.C5_POOL_CLIPS * fpc, wl.src_h, wl.src_w, 3), dtype=torch.uint8, device=dev)
+    for j in range(configs.C5_POOL_CLIPS):
+        video.make_scene(wl, clip=j).render(range(fpc), out=pool[j * fpc:(j + 1) * fpc])
+    pipe = otif.Pipeline(wl, blob, b, max_batch=fpc)
+    clips = odist.shard_clips(n_clips, world, rank)
+
+    def run_clip(k):
+        j = k % configs.C5_POOL_CLIPS
+        pipe.run_device(pool[j * fpc:(j + 1) * fpc], frame_base=k * fpc)
+        c = pipe.counters()
+        pipe.reset_counters()
+        return c
+
+    for k in list(clips)[:2]:     # warm-up
+        run_clip(k)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    times, per_clip = [], None
+    for _ in range(args.c5_passes):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        per_clip = odist.run_corpus(clips, run_clip)
+        e1.record()
+        torch.cuda.synchronize()
+        times.append(e0.elapsed_time(e1))
+    if world > 1:
+        dist.barrier()
+    ms = odist.max_over_ranks(float(np.mean(times)), dev)
+    allc = odist.gather_clip_counters(per_clip.to(dev), n_clips, per_clip.shape[1])
+    digest = odist.corpus_digest(allc)
+    pipe.close()
+    del pool
+    torch.cuda.empty_cache()
+    return {"what": f"{n_clips} one-minute 960x540 clips x {fpc} sampled frames (P:L99, P:L244), 8-clip pool, "
+                    f"contiguous clip ranges per rank; one pipeline call per clip",
+            "frames_per_s": n_clips * fpc / (ms / 1e3), "ms_per_pass": ms, "passes": args.c5_passes,
+            "scaling": "strong (fixed corpus)", "clips_per_rank": len(clips), "corpus": digest}
+
+
+def _free_port() -> int:
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
 
 
 def main():
@@ -455,19 +649,31 @@ def main():
     ap.add_argument("--impl", choices=["otif", "reference"], default="otif")
     ap.add_argument("--batch", type=int, default=0, help="device batch (0 = whole clip)")
     ap.add_argument("--host-batch", type=int, default=512, help="device batch of the host (e2e) path")
-    ap.add_argument("--proxy-batch", type=int, default=0, help="frames per resize+proxy launch (0 = batch)")
-    ap.add_argument("--overlap", type=int, default=0,
-                    help="chunks per device batch with resize/select/pack overlapped under the proxy (0 = serial)")
     ap.add_argument("--e2e-steps", type=int, default=2)
-    ap.add_argument("--oracle-frames", type=int, default=32)
+    ap.add_argument("--oracle-frames", type=int, default=64)
+    ap.add_argument("--train-steps", type=int, default=400)
+    ap.add_argument("--c5-clips", type=int, default=0, help="C5 clips (0 = the full 480)")
+    ap.add_argument("--c5-passes", type=int, default=2)
+    ap.add_argument("--headline-only", action="store_true", help="only the C2 headline (+ e2e / cpu baseline)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--no-perfect", action="store_true", help="skip the perfect-proxy (ground-truth mask) line")
+    ap.add_argument("--no-configs", action="store_true", help="skip the C1 / C3 / C4b / C4d objects")
+    ap.add_argument("--no-windowing", action="store_true", help="skip the trained-proxy / perfect-proxy objects")
+    ap.add_argument("--no-c5", action="store_true", help="skip the C5 corpus object")
     ap.add_argument("--no-next4", action="store_true", help="skip the NEXT-4 track-refinement line")
     ap.add_argument("--no-next3", action="store_true", help="skip the NEXT-3 proxy-training line")
     args = ap.parse_args()
     if args.warmup < 3:
         ap.error("--warmup must be >= 3")
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # one process per GPU: re-launch under torchrun on this node (NCCL over NVLink)
+        env = dict(os.environ)
+        env.setdefault("NCCL_DEBUG", "INFO")
+        env.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        env.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr=127.0.0.1", f"--master-port={_free_port()}", os.path.abspath(__file__)] + sys.argv[1:]
+        return subprocess.call(cmd, env=env)
     if args.impl == "reference":
         return run_reference(args)
     return run_otif(args)

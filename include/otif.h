@@ -117,6 +117,9 @@ otif_status otif_proxy_score(const otif_proxy *p, const uint8_t *img, int32_t n,
  * compacted across the batch in (frame, y, x) order; frame_count[n], frame_offset[n]
  * (exclusive prefix), total[1].  total and counts are exact even when windows beyond
  * `capacity` are dropped; capacity = n*ceil(gh*gw/2) can never overflow.
+ * est_sum [1] int64 (device, optional, may be NULL): set to Σ_t est(R_t) over the n
+ * frames, est(R) = Σ_{r in R} T_{r.w, r.h} (the runtime estimate the tuner
+ * sums) — computed with the grouping, no second pass.
  * Limits: gh*gw <= 8192.  workspace: >= otif_select_workspace_bytes(n, gh, gw). */
 typedef struct { int32_t frame_w, frame_h, cell, connectivity; /* 4 or 8 */ } otif_grid_desc;
 size_t otif_select_workspace_bytes(int32_t n, int32_t gh, int32_t gw);
@@ -125,7 +128,7 @@ otif_status otif_select_windows(const float *scores, const uint8_t *mask_in, flo
                                 const otif_wsize *sizes, int32_t k,
                                 uint8_t *mask_out, otif_window *windows, int32_t capacity,
                                 int32_t *frame_count, int32_t *frame_offset, int32_t *total,
-                                void *workspace, size_t ws_bytes, cudaStream_t stream);
+                                void *workspace, size_t ws_bytes, cudaStream_t stream, int64_t *est_sum);
 
 /* ---------------------------------------------------------------------------
  * Stage 5 — crop / resample / pack (the detector is initialised "at each of
@@ -284,14 +287,7 @@ typedef struct {
     otif_wsize sizes[8];
     int32_t max_batch;          /* frames per device batch (one select / pack launch each) */
     int32_t batch_cap[8];       /* detector batch capacity per size, per device batch */
-    int32_t proxy_batch;        /* frames per resize + proxy launch within a batch (0 = max_batch);
-                                   small enough keeps each layer's activations L2-resident */
-    int32_t overlap_chunks;     /* >= 2: split each device batch into this many chunks and run the
-                                   memory-bound stages (resize of chunk c+1, select + pack of chunk
-                                   c-1) on a second stream while the tensor-bound proxy scores chunk c;
-                                   the proxy kernels then leave shared memory for co-resident resize /
-                                   pack CTAs.  Results are identical to the serial schedule (slots keep
-                                   the batch's emission order).  0 or 1 = serial (proxy_batch applies). */
+    int32_t proxy_batch;        /* frames per resize + proxy launch within a batch (0 = max_batch) */
 } otif_pipeline_desc;
 
 typedef struct otif_pipeline otif_pipeline;
@@ -303,15 +299,18 @@ otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *src_host, in
                                    int32_t *frame_count_out, int32_t *total_out,
                                    int32_t *size_count_out);
 /* Same path on frames already resident in device memory, enqueued on `stream`
- * without any host synchronisation.  Windows and detector batches of each device
- * batch stay in the pipeline's device buffers (overwritten batch by batch); the
- * counters below accumulate on the device across calls until reset. */
-otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t *src_dev, int32_t n,
+ * without any host synchronisation.  frame_base = global index of src_dev[0] (the
+ * window hash keys windows by global frame, so a corpus sharded over ranks or clips
+ * hashes identically).  Windows and detector batches of each device batch stay in
+ * the pipeline's device buffers (overwritten batch by batch); the counters below
+ * accumulate on the device across calls until reset. */
+otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t *src_dev, int32_t n, int64_t frame_base,
                                      cudaStream_t stream);
-/* Device pointer to int64[5 + k] counters accumulated since create/reset (run_host
- * resets them at its start): frames, positive cells, windows, window pixels, an
- * order-independent hash of all windows (sum of 64-bit mixes of (frame,x,y,w,h,s)),
- * then windows per size. */
+/* Device pointer to int64[15] counters accumulated since create/reset (run_host
+ * resets them at its start): [0] frames, [1] positive cells, [2] windows, [3] window
+ * pixels, [4] an order-independent hash of all windows (wrapping sum of 64-bit mixes
+ * of (global frame, x, y, w, h, s)), [5 + s] windows of size s (8 slots), [13] windows
+ * dropped because their slot exceeded batch_cap[s], [14] pixels of the windows packed. */
 const int64_t *otif_pipeline_counters(const otif_pipeline *p);
 otif_status otif_pipeline_reset_counters(otif_pipeline *p, cudaStream_t stream);
 /* Per-stage device timing (CUDA events recorded between the stage launches on the

@@ -41,8 +41,7 @@ class PipelineDesc(ctypes.Structure):
     _fields_ = [("proxy", ProxyDesc), ("src_h", ctypes.c_int32), ("src_w", ctypes.c_int32),
                 ("det_h", ctypes.c_int32), ("det_w", ctypes.c_int32), ("grid", GridDesc),
                 ("threshold", ctypes.c_float), ("k", ctypes.c_int32), ("sizes", WSize * 8),
-                ("max_batch", ctypes.c_int32), ("batch_cap", ctypes.c_int32 * 8), ("proxy_batch", ctypes.c_int32),
-                ("overlap_chunks", ctypes.c_int32)]
+                ("max_batch", ctypes.c_int32), ("batch_cap", ctypes.c_int32 * 8), ("proxy_batch", ctypes.c_int32)]
 
 
 _lib = None
@@ -76,7 +75,7 @@ def lib() -> ctypes.CDLL:
     L.otif_select_workspace_bytes.argtypes = [i32, i32, i32]
     L.otif_select_workspace_bytes.restype = sz
     L.otif_select_windows.argtypes = [P, P, ctypes.c_float, i32, i32, i32, ctypes.POINTER(GridDesc), P, i32,
-                                      P, P, i32, P, P, P, P, sz, P]
+                                      P, P, i32, P, P, P, P, sz, P, P]
     L.otif_select_windows.restype = st
     L.otif_pack_windows.argtypes = [P, i32, i32, i32, i32, i32, P, P, i32, P, i32, P, P, P, P, P]
     L.otif_pack_windows.restype = st
@@ -122,7 +121,7 @@ def lib() -> ctypes.CDLL:
         L.otif_pipeline_destroy.restype = None
         L.otif_pipeline_run_host.argtypes = [P, P, i32, P, i32, P, P, P]
         L.otif_pipeline_run_host.restype = st
-        L.otif_pipeline_run_device.argtypes = [P, P, i32, P]
+        L.otif_pipeline_run_device.argtypes = [P, P, i32, ctypes.c_int64, P]
         L.otif_pipeline_run_device.restype = st
         L.otif_pipeline_counters.argtypes = [P]
         L.otif_pipeline_counters.restype = P

@@ -124,7 +124,8 @@ class Proxy:
 def otif_select_windows(scores: torch.Tensor | None, mask_in: torch.Tensor | None, threshold: float,
                         frame_w: int, frame_h: int, cell: int, sizes, connectivity: int = 4,
                         capacity: int | None = None, want_mask: bool = False, stream=None):
-    """-> dict(windows int32[capacity, 6], counts int32[n], offsets int32[n], total int32[1], mask u8|None)."""
+    """-> dict(windows int32[capacity, 6], counts int32[n], offsets int32[n], total int32[1], mask u8|None,
+    est_sum int64[1] = Σ_t est(R_t) (computed by the grouping kernel))."""
     t = scores if scores is not None else mask_in
     _require_cuda(t)
     n, gh, gw = t.shape
@@ -136,6 +137,7 @@ def otif_select_windows(scores: torch.Tensor | None, mask_in: torch.Tensor | Non
     offsets = torch.empty(n, dtype=torch.int32, device=dev)
     total = torch.zeros(1, dtype=torch.int32, device=dev)
     mask = torch.empty((n, gh, gw), dtype=torch.uint8, device=dev) if want_mask else None
+    est_sum = torch.zeros(1, dtype=torch.int64, device=dev)
     ws_bytes = int(lib().otif_select_workspace_bytes(n, gh, gw))
     ws = torch.empty(max(ws_bytes, 256) + 256, dtype=torch.uint8, device=dev)
     g = GridDesc(frame_w, frame_h, cell, connectivity)
@@ -143,8 +145,8 @@ def otif_select_windows(scores: torch.Tensor | None, mask_in: torch.Tensor | Non
     check(lib().otif_select_windows(_ptr(scores), _ptr(mask_in), ctypes.c_float(threshold), n, gh, gw,
                                     ctypes.byref(g), ws_sizes, len(sizes), _ptr(mask), _ptr(windows), capacity,
                                     _ptr(counts), _ptr(offsets), _ptr(total), _ptr(ws), ws.numel(),
-                                    _stream(stream)), "otif_select_windows")
-    return dict(windows=windows, counts=counts, offsets=offsets, total=total, mask=mask)
+                                    _stream(stream), _ptr(est_sum)), "otif_select_windows")
+    return dict(windows=windows, counts=counts, offsets=offsets, total=total, mask=mask, est_sum=est_sum)
 
 
 # ---------------------------------------------------------------- stage 5
@@ -174,10 +176,11 @@ class Pipeline:
 
     def __init__(self, workload, weights: np.ndarray, threshold: float, max_batch: int = 256,
                  batch_cap: Sequence[int] | None = None, connectivity: int = 4,
-                 enc=(32, 64, 128, 256, 256), dec=128, proxy_batch: int = 0, overlap_chunks: int = 0):
+                 enc=(32, 64, 128, 256, 256), dec=128, proxy_batch: int = 0, sizes=None):
+        """sizes: W as [(w, h)] or [(w, h, cost)] (default: the workload's own W)."""
         d = PipelineDesc()
         d.proxy_batch = int(proxy_batch)
-        d.overlap_chunks = int(overlap_chunks)
+        sizes = list(workload.sizes) if sizes is None else list(sizes)
         d.proxy.in_h, d.proxy.in_w, d.proxy.n_strided = workload.proxy_h, workload.proxy_w, workload.n_strided
         for i, e in enumerate(enc):
             d.proxy.enc[i] = int(e)
@@ -186,20 +189,22 @@ class Pipeline:
         d.det_h, d.det_w = workload.src_h, workload.src_w
         d.grid = GridDesc(workload.src_w, workload.src_h, workload.cell, connectivity)
         d.threshold = float(threshold)
-        d.k = len(workload.sizes)
-        for i, s in enumerate(workload.sizes):
+        d.k = len(sizes)
+        for i, s in enumerate(sizes):
             d.sizes[i].w, d.sizes[i].h = int(s[0]), int(s[1])
             d.sizes[i].cost = int(s[2]) if len(s) > 2 else int(s[0]) * int(s[1])
         d.max_batch = int(max_batch)
         if batch_cap is None:
             # a full-frame window is the only window of its frame; smaller sizes get headroom
             caps = [max_batch if (int(w[0]), int(w[1])) == (workload.src_w, workload.src_h) else max_batch * 4
-                    for w in workload.sizes]
+                    for w in sizes]
         else:
             caps = batch_cap
         for i in range(d.k):
             d.batch_cap[i] = int(caps[i])
         self.k = d.k
+        self.sizes = sizes
+        self.batch_cap = [int(c) for c in caps]
         self.desc = d
         w = np.ascontiguousarray(weights, np.float32)
         self._w = w
@@ -226,15 +231,17 @@ class Pipeline:
         t = int(total[0])
         return win[:min(t, cap)], counts, sc, t
 
-    def run_device(self, frames: torch.Tensor, stream=None):
+    def run_device(self, frames: torch.Tensor, frame_base: int = 0, stream=None):
+        """frames: device u8 [n, H, W, 3]; frame_base = global index of frames[0] (window hash key)."""
         _require_cuda(frames)
-        check(lib().otif_pipeline_run_device(self.handle, _ptr(frames), frames.shape[0], _stream(stream)),
-              "otif_pipeline_run_device")
+        check(lib().otif_pipeline_run_device(self.handle, _ptr(frames), frames.shape[0], int(frame_base),
+                                             _stream(stream)), "otif_pipeline_run_device")
 
     def counters(self) -> torch.Tensor:
-        """int64 [5 + k] device counters: frames, positive cells, windows, window pixels, hash, per-size."""
+        """int64 [15] device counters: frames, positive cells, windows, window pixels, window hash,
+        windows per size [8], windows dropped for batch_cap, pixels of the windows packed."""
         ptr = lib().otif_pipeline_counters(self.handle)
-        n = 5 + self.k
+        n = 15
         # wrap the device pointer without copying (read via a torch tensor view)
         return _device_view_i64(ptr, n)
 

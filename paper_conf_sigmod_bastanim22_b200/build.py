@@ -4,6 +4,7 @@ from __future__ import annotations
 import glob
 import os
 import subprocess
+from concurrent.futures import ThreadPoolExecutor
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
@@ -28,17 +29,21 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not needs_build():
         return LIB
     nvcc = os.environ.get("NVCC", "nvcc")
-    objs = []
-    for src in sources():
+    extra = os.environ.get("OTIF_NVCC_EXTRA", "").split()   # e.g. -DOTIF_E12_TRACE_BUILD (debug builds)
+
+    def compile_one(src):
         obj = os.path.join(CSRC, os.path.basename(src)[:-3] + ".o")
-        extra = os.environ.get("OTIF_NVCC_EXTRA", "").split()   # e.g. -DOTIF_E12_TRACE_BUILD (debug builds)
         cmd = [nvcc] + NVCC_FLAGS + extra + ["-c", src, "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError(f"nvcc failed for {src}:\n{r.stderr}")
         if verbose:
             print(r.stderr)
-        objs.append(obj)
+        return obj
+
+    # one nvcc per translation unit, in parallel
+    with ThreadPoolExecutor(max(1, min(len(sources()), os.cpu_count() or 1))) as ex:
+        objs = list(ex.map(compile_one, sources()))
     cmd = [nvcc, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", LIB] + objs
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:

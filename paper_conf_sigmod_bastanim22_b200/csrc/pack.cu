@@ -31,7 +31,7 @@ struct PackParams {
     int bw[kMaxK], bh[kMaxK];
     int *slot;
     int *size_count;
-    int accumulate;   // internal (pipeline chunks): slots continue from size_count's current values
+    unsigned long long *ctr_pack;  // internal (pipeline): [0] windows dropped for batch_cap, [1] packed pixels
     int stage_bytes;  // bulk ring stage size (<= kBulkStage)
 };
 
@@ -39,9 +39,10 @@ __global__ void __launch_bounds__(1024) slot_kernel(const __grid_constant__ Pack
     __shared__ int s_warp_cnt[32][kMaxK];
     __shared__ int s_carry[kMaxK];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    if (threadIdx.x < kMaxK) s_carry[threadIdx.x] = (p.accumulate && threadIdx.x < p.k) ? p.size_count[threadIdx.x] : 0;
+    if (threadIdx.x < kMaxK) s_carry[threadIdx.x] = 0;
     __syncthreads();
     const int total = min(*p.total, p.capacity);
+    unsigned long long dropped = 0, packed_px = 0;
     for (int base = 0; base < total; base += blockDim.x) {
         const int g = base + threadIdx.x;
         const int s = g < total ? p.win[g].size_idx : -1;
@@ -56,6 +57,8 @@ __global__ void __launch_bounds__(1024) slot_kernel(const __grid_constant__ Pack
             int pre = s_carry[s];
             for (int w = 0; w < warp; w++) pre += s_warp_cnt[w][s];
             p.slot[g] = pre + rank;
+            if (pre + rank < p.cap[s]) packed_px += (unsigned long long)p.win[g].w * p.win[g].h;
+            else dropped++;
         }
         __syncthreads();
         if (threadIdx.x < p.k) {
@@ -67,6 +70,16 @@ __global__ void __launch_bounds__(1024) slot_kernel(const __grid_constant__ Pack
     }
     // size_count counts every listed window, including those dropped for batch_cap
     if (threadIdx.x < p.k) p.size_count[threadIdx.x] = s_carry[threadIdx.x];
+    if (p.ctr_pack) {
+        for (int o = 16; o > 0; o >>= 1) {
+            dropped += __shfl_xor_sync(0xffffffffu, dropped, o);
+            packed_px += __shfl_xor_sync(0xffffffffu, packed_px, o);
+        }
+        if (lane == 0 && (dropped | packed_px)) {
+            atomicAdd(&p.ctr_pack[0], dropped);
+            atomicAdd(&p.ctr_pack[1], packed_px);
+        }
+    }
 }
 
 __device__ __forceinline__ uint32_t fshift(uint32_t lo, uint32_t hi, uint32_t sh_bytes) {
@@ -111,7 +124,8 @@ __device__ __forceinline__ uint4 load16u(const uint8_t *s0, uintptr_t src_end) {
 // detector batch (contiguous).  Loads run kBulkLead chunks ahead of the stores.
 // STAGES ring stages, loads run STAGES - 2 chunks ahead of the stores (one stage is being
 // read by an in-flight store); stage size is a launch parameter (<= kBulkStage).
-constexpr int kBulkStage = 16384;            // largest ring stage (bytes)
+constexpr int kBulkStage = 16384;            // ring stage (bytes)
+constexpr int kPackStages = 3;
 
 __device__ __forceinline__ void bulk_s2g(void *dst_gmem, const void *src_smem, uint32_t bytes) {
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst_gmem), "r"(smem_u32(src_smem)),
@@ -255,14 +269,12 @@ using namespace otif;
 
 namespace otif {
 
-// internal entry (pipeline): accumulate = slots continue from size_count (chunked batches);
-// ctas = pack grid (0 = 6 per SM); stages 3 or 6; stage_bytes <= kBulkStage; threads 128 or
-// 32 (one warp: few registers, so a CTA fits on an SM next to the 768-thread E1+E2 CTA)
+// internal entry; ctr_pack (pipeline, may be NULL): device counters of dropped windows
+// and packed pixels, accumulated
 otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w,
                         const otif_window *windows, const int32_t *total, int32_t capacity, const otif_wsize *sizes,
                         int32_t k, uint8_t *const *batches, const int32_t *batch_cap, int32_t *slot,
-                        int32_t *size_count, cudaStream_t stream, int accumulate, int ctas, int stages,
-                        int stage_bytes, int threads) {
+                        int32_t *size_count, cudaStream_t stream, unsigned long long *ctr_pack) {
     PackParams p;
     memset(&p, 0, sizeof(p));
     p.src = src; p.n = n; p.sh = src_h; p.sw = src_w; p.dh = det_h; p.dw = det_w;
@@ -275,20 +287,20 @@ otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t sr
         p.batch[s] = batches[s]; p.cap[s] = batch_cap[s]; p.bw[s] = sizes[s].w; p.bh[s] = sizes[s].h;
     }
     p.slot = slot; p.size_count = size_count;
-    p.accumulate = accumulate;
-    p.stage_bytes = stage_bytes > 0 && stage_bytes <= kBulkStage ? (stage_bytes & ~15) : kBulkStage;
+    p.ctr_pack = ctr_pack;
+    p.stage_bytes = kBulkStage;
     int num_sms = 148;
     check_device(&num_sms);
     slot_kernel<<<1, 1024, 0, stream>>>(p);
     OTIF_LAUNCH_CHECK();
     if (capacity > 0) {
-        const int want = ctas > 0 ? ctas : num_sms * 6;
+        // persistent grid: 6 CTAs per SM (3 x 16 KB rings each), one window per CTA at a time
+        const int want = num_sms * 6;
         const int grid = capacity < want ? capacity : want;
-        const int smem = (stages == 6 ? 6 : 3) * p.stage_bytes;
-        auto kern = stages == 6 ? (threads == 32 ? pack_kernel<6, 32> : pack_kernel<6, 128>)
-                                : (threads == 32 ? pack_kernel<3, 32> : pack_kernel<3, 128>);
+        const int smem = kPackStages * p.stage_bytes;
+        auto kern = pack_kernel<kPackStages, 128>;
         OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-        kern<<<grid, threads == 32 ? 32 : 128, smem, stream>>>(p);
+        kern<<<grid, 128, smem, stream>>>(p);
         OTIF_LAUNCH_CHECK();
     }
     return OTIF_OK;
@@ -310,5 +322,5 @@ extern "C" otif_status otif_pack_windows(const uint8_t *src, int32_t n, int32_t 
     otif_status st = check_device(nullptr);
     if (st != OTIF_OK) return st;
     return launch_pack(src, n, src_h, src_w, det_h, det_w, windows, total, capacity, sizes, k, batches, batch_cap,
-                       slot, size_count, stream, 0, 0, 3, kBulkStage, 128);
+                       slot, size_count, stream, nullptr);
 }

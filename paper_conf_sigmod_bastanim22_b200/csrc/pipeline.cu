@@ -2,21 +2,14 @@
 // buffers, a compute stream and a copy stream, the batch loop, and result accumulation.
 //
 // A device batch (max_batch frames) runs resize + proxy in mini-batches of proxy_batch
-// frames — small enough that each layer's activations stay resident in the 126 MB L2
-// for the next layer — writing the scores of the whole batch; then one select launch and
-// one pack launch cover the whole batch (the latency-bound grouping needs thousands of
-// frames in flight to fill 148 SMs).  The detector batches stay on the device (the
-// detector runs there); windows, per-frame counts and counters are accumulated
-// on the device and copied back once per host call.
-//
-// Overlap mode (desc.overlap_chunks >= 2): the batch is split into chunks; the caller's
-// stream runs the tensor-bound proxy of chunk c while a second stream runs the
-// memory-bound stages — resize of chunk c+1, then select + pack of chunk c-1 — so HBM
-// traffic hides under the tensor-core work.  The proxy kernels then take a lower
-// shared-memory budget so that a pack (bulk-copy ring) or resize CTA fits on every SM
-// next to a proxy CTA.  Slots continue across the chunks (pack accumulates size_count),
-// so the detector batches hold the same windows in the same order as the serial schedule.
-#include <cuda.h>
+// frames, writing the scores of the whole batch; then one select launch and one pack
+// launch cover the whole batch (the latency-bound grouping needs thousands of frames in
+// flight to fill 148 SMs).  The detector batches stay on the device (the detector runs
+// there); windows, per-frame counts and counters are accumulated on the device
+// and copied back once per host call.  Host runs stage the frames of batch b+1 (copy
+// stream, pinned host memory) while batch b computes.  Every stage is bracketed by an
+// NVTX range (visible in nsys / ncu --nvtx) and, when timing is on, by CUDA events.
+#include <nvtx3/nvToolsExt.h>
 #include <stdlib.h>
 #include <string.h>
 
@@ -33,27 +26,27 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum, size_t smem_cap);
+                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum);
 otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w,
                         const otif_window *windows, const int32_t *total, int32_t capacity, const otif_wsize *sizes,
                         int32_t k, uint8_t *const *batches, const int32_t *batch_cap, int32_t *slot,
-                        int32_t *size_count, cudaStream_t stream, int accumulate, int ctas, int stages,
-                        int stage_bytes, int threads);
-otif_status proxy_set_smem_budget(otif_proxy *p, size_t budget);
+                        int32_t *size_count, cudaStream_t stream, unsigned long long *ctr_pack);
 int proxy_launches(const otif_proxy *p);
-void proxy_set_num_sms(otif_proxy *p, int sms);
 
 // timing stages: resize, proxy prep (tag + E1), E2, E3, E4, E5, D1+D2, select, pack, append
 constexpr int kStages = 10;
 enum { ST_START = -1, ST_RESIZE = 0, ST_PREP = 1, ST_SELECT = 7, ST_PACK = 8, ST_APPEND = 9 };
 
-// counters: [0] frames, [1] positive cells, [2] windows, [3] window pixels,
-//           [4] order-independent window hash (sum of 64-bit mixes), [5 + s] windows of size s
+// counters (otif.h): [0] frames, [1] positive cells, [2] windows, [3] window pixels,
+// [4] order-independent window hash, [5 + s] windows of size s (s < 8),
+// [13] windows dropped for batch_cap, [14] pixels of the windows actually packed
 constexpr int kCtrFixed = 5;
+constexpr int kCtrPack = kCtrFixed + 8;
+constexpr int kCtrTotal = kCtrPack + 2;
 
 // Host runs only: append one batch's windows (frame index rebased to the global frame)
 // and per-frame counts to the run's output arrays.  (The counters are accumulated by
-// the select kernel itself.)
+// the select and slot kernels themselves.)
 __global__ void __launch_bounds__(1024) append_kernel(const otif_window *__restrict__ win, const int *__restrict__ total,
                                                       int capacity, const int *__restrict__ counts, int nb,
                                                       int frame_base, otif_window *out_win, int out_cap,
@@ -74,45 +67,12 @@ __global__ void __launch_bounds__(1024) append_kernel(const otif_window *__restr
 
 using namespace otif;
 
-
-// Driver entry points of the green-context API, fetched through the runtime so that
-// libotif.so does not link libcuda (it must load on hosts without a driver).
-struct GreenApi {
-    CUresult (*DeviceGet)(CUdevice *, int);
-    CUresult (*DeviceGetDevResource)(CUdevice, CUdevResource *, CUdevResourceType);
-    CUresult (*DevSmResourceSplitByCount)(CUdevResource *, unsigned *, const CUdevResource *, CUdevResource *,
-                                          unsigned, unsigned);
-    CUresult (*DevResourceGenerateDesc)(CUdevResourceDesc *, CUdevResource *, unsigned);
-    CUresult (*GreenCtxCreate)(CUgreenCtx *, CUdevResourceDesc, CUdevice, unsigned);
-    CUresult (*GreenCtxStreamCreate)(CUstream *, CUgreenCtx, unsigned, int);
-    CUresult (*GreenCtxDestroy)(CUgreenCtx);
-};
-static const char *g_green_missing = "";
-static bool green_api(GreenApi &g) {
-    auto get = [](const char *name, void **fn) {
-        cudaDriverEntryPointQueryResult q = cudaDriverEntryPointSymbolNotFound;
-        *fn = nullptr;
-        if (cudaGetDriverEntryPointByVersion(name, fn, 12080, cudaEnableDefault, &q) != cudaSuccess || !*fn) {
-            cudaGetLastError();
-            if (cudaGetDriverEntryPoint(name, fn, cudaEnableDefault, &q) != cudaSuccess) cudaGetLastError();
-        }
-        if (!*fn) g_green_missing = name;
-        return *fn != nullptr;
-    };
-    return get("cuDeviceGet", (void **)&g.DeviceGet) && get("cuDeviceGetDevResource", (void **)&g.DeviceGetDevResource) &&
-           get("cuDevSmResourceSplitByCount", (void **)&g.DevSmResourceSplitByCount) &&
-           get("cuDevResourceGenerateDesc", (void **)&g.DevResourceGenerateDesc) &&
-           get("cuGreenCtxCreate", (void **)&g.GreenCtxCreate) &&
-           get("cuGreenCtxStreamCreate", (void **)&g.GreenCtxStreamCreate) &&
-           get("cuGreenCtxDestroy", (void **)&g.GreenCtxDestroy);
-}
-
 struct otif_pipeline {
     otif_pipeline_desc d;
     otif_proxy *proxy = nullptr;
     int gh = 0, gw = 0, cells = 0, cap_w = 0, pb = 0;
-    uint8_t *src[2] = {nullptr, nullptr};
-    uint8_t *img = nullptr, *img2 = nullptr, *mask = nullptr, *proxy_ws = nullptr, *sel_ws = nullptr;
+    uint8_t *src[2] = {nullptr, nullptr};   // host-run staging (allocated by the first host run)
+    uint8_t *img = nullptr, *mask = nullptr, *proxy_ws = nullptr, *sel_ws = nullptr;
     size_t proxy_ws_bytes = 0, sel_ws_bytes = 0;
     float *scores = nullptr;
     otif_window *windows = nullptr;
@@ -127,18 +87,6 @@ struct otif_pipeline {
     int *out_total = nullptr;
     cudaStream_t s_compute = nullptr, s_copy = nullptr;
     cudaEvent_t ev_h2d[2] = {}, ev_free[2] = {};
-    // overlap mode: chunking, the memory stream and its hand-off events
-    int chunks = 0, chunk = 0;
-    int pack_ctas = 0, pack_stages = 3, pack_stage_bytes = 16384, pack_threads = 128;
-    int ovl_mode = 0;   // 0: resize, select and pack on the memory stream; 1: pack only
-    int *totals = nullptr;  // [chunks] per-chunk window totals (overlap)
-    size_t sel_smem_cap = 0;
-    cudaStream_t s_mem = nullptr;
-    // partitioned overlap (OTIF_OVL_GREEN = SMs for the memory stages): two green contexts
-    // split the SMs; the proxy runs on s_tensor (its partition), resize/select/pack on s_mem
-    CUgreenCtx g_tensor = nullptr, g_mem = nullptr;
-    cudaStream_t s_tensor = nullptr;
-    cudaEvent_t ev_fork = nullptr, ev_join = nullptr, ev_resized[2] = {}, ev_scored[2] = {}, ev_imgfree[2] = {};
     // optional per-stage timing: a log of spans (stage, start entry, end event); a span's
     // time is charged to its stage (stage < 0: a start marker)
     int timing = 0;
@@ -187,7 +135,15 @@ static int tspan(otif_pipeline *p, int stage, cudaStream_t st, int from) {
         if (rc_ != OTIF_OK) return rc_; \
     } while (0)
 
+// NVTX range for the host-side enqueue of one stage (nsys shows it on the CPU timeline
+// and, with CUDA trace, correlates it with the stage's kernels)
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
+
 static otif_status run_proxy(otif_pipeline *p, const uint8_t *img, int mb, float *scores, cudaStream_t st) {
+    NvtxRange r("otif.proxy");
     // six spans for the proxy (prep/E1, then each GEMM layer); launch_proxy records their
     // end events at the actual points in the stream
     cudaEvent_t evs[6];
@@ -198,131 +154,42 @@ static otif_status run_proxy(otif_pipeline *p, const uint8_t *img, int mb, float
     return OTIF_OK;
 }
 
-// select of frames [f0, f0 + nb) of the batch into window slice `wo` (capacity cap) and *tot
-static otif_status run_select(otif_pipeline *p, int f0, int nb, int frame_base, otif_window *wo, int cap, int *tot,
-                              cudaStream_t st) {
-    const otif_pipeline_desc &d = p->d;
-    int t0 = tmark(p, st);
-    RC(launch_select(p->scores + (size_t)f0 * p->cells, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k,
-                     p->mask + (size_t)f0 * p->cells, wo, cap, p->counts + f0, p->offsets + f0, tot, p->sel_ws,
-                     p->sel_ws_bytes, st, p->ctr, frame_base + f0, nullptr, p->sel_smem_cap));
-    tspan(p, ST_SELECT, st, t0);
-    p->launches += 2;
-    return OTIF_OK;
-}
-
-// pack (+ append) of those windows; accumulate = slots continue from earlier chunks
-static otif_status run_pack(otif_pipeline *p, const uint8_t *src, int f0, int nb, int frame_base,
-                            const otif_window *wo, int cap, const int *tot, int *slot, int accumulate,
-                            cudaStream_t st) {
+static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int frame_base, cudaStream_t st) {
     const otif_pipeline_desc &d = p->d;
     const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
+    for (int m0 = 0; m0 < nb; m0 += p->pb) {
+        const int mb = nb - m0 < p->pb ? nb - m0 : p->pb;
+        {
+            NvtxRange r("otif.resize");
+            int t0 = tmark(p, st);
+            RC(otif_resize(src + (size_t)m0 * frame_bytes, mb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w,
+                           st));
+            tspan(p, ST_RESIZE, st, t0);
+            p->launches += 1;
+        }
+        RC(run_proxy(p, p->img, mb, p->scores + (size_t)m0 * p->cells, st));
+    }
+    {
+        NvtxRange r("otif.select");
+        int t0 = tmark(p, st);
+        RC(launch_select(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask, p->windows,
+                         p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base,
+                         nullptr));
+        tspan(p, ST_SELECT, st, t0);
+        p->launches += 2;
+    }
+    NvtxRange r("otif.pack");
     int t0 = tmark(p, st);
-    RC(launch_pack(src + (size_t)f0 * frame_bytes, nb, d.src_h, d.src_w, d.det_h, d.det_w, wo, tot, cap, d.sizes, d.k,
-                   p->batches, d.batch_cap, slot, p->size_count, st, accumulate, p->pack_ctas, p->pack_stages,
-                   p->pack_stage_bytes, p->pack_threads));
+    RC(launch_pack(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
+                   p->batches, d.batch_cap, p->slot, p->size_count, st, p->ctr + kCtrPack));
     t0 = tspan(p, ST_PACK, st, t0);
     p->launches += 2;
     if (p->out_win) {
-        append_kernel<<<1, 1024, 0, st>>>(wo, tot, cap, p->counts + f0, nb, frame_base + f0, p->out_win,
+        append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts, nb, frame_base, p->out_win,
                                           p->out_win_cap, p->out_counts, p->out_total);
         OTIF_LAUNCH_CHECK();
         p->launches += 1;
         tspan(p, ST_APPEND, st, t0);
-    }
-    return OTIF_OK;
-}
-
-static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int frame_base, cudaStream_t st) {
-    const otif_pipeline_desc &d = p->d;
-    const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
-    if (p->chunks < 2) {
-        for (int m0 = 0; m0 < nb; m0 += p->pb) {
-            const int mb = nb - m0 < p->pb ? nb - m0 : p->pb;
-            int t0 = tmark(p, st);
-            RC(otif_resize(src + (size_t)m0 * frame_bytes, mb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w, st));
-            tspan(p, ST_RESIZE, st, t0);
-            RC(run_proxy(p, p->img, mb, p->scores + (size_t)m0 * p->cells, st));
-            p->launches += 1;
-        }
-        RC(run_select(p, 0, nb, frame_base, p->windows, p->cap_w, p->total, st));
-        return run_pack(p, src, 0, nb, frame_base, p->windows, p->cap_w, p->total, p->slot, 0, st);
-    }
-    // overlap: st = tensor stream (proxy), s_mem = memory stream (resize, select, pack); with
-    // an SM partition the proxy runs on the tensor partition's stream, joined back to st
-    cudaStream_t sm = p->s_mem;
-    cudaStream_t caller = st;
-    if (p->s_tensor) {
-        OTIF_CUDA(cudaEventRecord(p->ev_fork, caller));
-        OTIF_CUDA(cudaStreamWaitEvent(p->s_tensor, p->ev_fork, 0));
-        st = p->s_tensor;
-    }
-    uint8_t *img[2] = {p->img, p->img2};
-    const int cs = p->chunk;
-    const int nc = (nb + cs - 1) / cs;
-    OTIF_CUDA(cudaEventRecord(p->ev_fork, st));
-    OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_fork, 0));
-    for (int i = 0; i < 2; i++) OTIF_CUDA(cudaEventRecord(p->ev_imgfree[i], st));
-    auto resize_chunk = [&](int c) -> otif_status {
-        const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
-        OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_imgfree[c & 1], 0));
-        int t0 = tmark(p, sm);
-        RC(otif_resize(src + (size_t)c0 * frame_bytes, cn, d.src_h, d.src_w, img[c & 1], d.proxy.in_h, d.proxy.in_w, sm));
-        tspan(p, ST_RESIZE, sm, t0);
-        p->launches += 1;
-        OTIF_CUDA(cudaEventRecord(p->ev_resized[c & 1], sm));
-        return OTIF_OK;
-    };
-    // chunk c's windows, total and slots live in their own slices (no reuse hazard between
-    // the streams); pack keeps the emission order by running the chunks in order
-    const int per_frame = p->cap_w / d.max_batch;
-    auto select_chunk = [&](int c, cudaStream_t s) -> otif_status {
-        const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
-        return run_select(p, c0, cn, frame_base, p->windows + (size_t)c0 * per_frame, cn * per_frame, p->totals + c, s);
-    };
-    auto pack_chunk = [&](int c) -> otif_status {
-        const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
-        return run_pack(p, src, c0, cn, frame_base, p->windows + (size_t)c0 * per_frame, cn * per_frame,
-                        p->totals + c, p->slot + (size_t)c0 * per_frame, c > 0, sm);
-    };
-    if (p->ovl_mode == 1) {
-        // tensor stream: resize, proxy, select per chunk; memory stream: pack of finished chunks
-        for (int c = 0; c < nc; c++) {
-            const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
-            int t0 = tmark(p, st);
-            RC(otif_resize(src + (size_t)c0 * frame_bytes, cn, d.src_h, d.src_w, img[0], d.proxy.in_h, d.proxy.in_w, st));
-            tspan(p, ST_RESIZE, st, t0);
-            p->launches += 1;
-            RC(run_proxy(p, img[0], cn, p->scores + (size_t)c0 * p->cells, st));
-            RC(select_chunk(c, st));
-            OTIF_CUDA(cudaEventRecord(p->ev_scored[c & 1], st));
-            OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_scored[c & 1], 0));
-            RC(pack_chunk(c));
-        }
-    } else {
-        RC(resize_chunk(0));
-        for (int c = 0; c < nc; c++) {
-            if (c + 1 < nc) RC(resize_chunk(c + 1));
-            if (c >= 1) {
-                OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_scored[(c - 1) & 1], 0));
-                RC(select_chunk(c - 1, sm));
-                RC(pack_chunk(c - 1));
-            }
-            const int c0 = c * cs, cn = nb - c0 < cs ? nb - c0 : cs;
-            OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_resized[c & 1], 0));
-            RC(run_proxy(p, img[c & 1], cn, p->scores + (size_t)c0 * p->cells, st));
-            OTIF_CUDA(cudaEventRecord(p->ev_scored[c & 1], st));
-            OTIF_CUDA(cudaEventRecord(p->ev_imgfree[c & 1], st));
-        }
-        OTIF_CUDA(cudaStreamWaitEvent(sm, p->ev_scored[(nc - 1) & 1], 0));
-        RC(select_chunk(nc - 1, sm));
-        RC(pack_chunk(nc - 1));
-    }
-    OTIF_CUDA(cudaEventRecord(p->ev_join, sm));
-    OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_join, 0));
-    if (st != caller) {
-        OTIF_CUDA(cudaEventRecord(p->ev_join, st));
-        OTIF_CUDA(cudaStreamWaitEvent(caller, p->ev_join, 0));
     }
     return OTIF_OK;
 }
@@ -346,6 +213,7 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     OTIF_REQUIRE(d->src_h > 0 && d->src_w > 0 && d->det_h > 0 && d->det_w > 0, "otif_pipeline_create: sizes");
     OTIF_REQUIRE(d->grid.frame_w == d->det_w && d->grid.frame_h == d->det_h,
                  "otif_pipeline_create: grid frame must be the detector resolution");
+    for (int s = 0; s < d->k; s++) OTIF_REQUIRE(d->batch_cap[s] >= 0, "otif_pipeline_create: batch_cap[%d] < 0", s);
     otif_pipeline *p = new (std::nothrow) otif_pipeline();
     if (!p) return OTIF_ENOMEM;
     p->d = *d;
@@ -360,88 +228,9 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     }
     const int B = d->max_batch;
     p->pb = (d->proxy_batch > 0 && d->proxy_batch < B) ? d->proxy_batch : B;
-    if (d->overlap_chunks >= 2) {
-        // A/B knobs (env, sweeps only): proxy smem budget, pack grid / ring, select CTA smem
-        auto envi = [](const char *k, long v) { const char *e = getenv(k); return e ? atol(e) : v; };
-        int num_sms = 148;
-        check_device(&num_sms);
-        p->chunks = d->overlap_chunks < B ? d->overlap_chunks : B;
-        p->chunk = (B + p->chunks - 1) / p->chunks;
-        p->pb = p->chunk;
-        p->pack_ctas = (int)envi("OTIF_OVL_PACK_CTAS", num_sms);
-        p->pack_stages = (int)envi("OTIF_OVL_PACK_STAGES", 3);
-        p->pack_stage_bytes = (int)envi("OTIF_OVL_PACK_STAGE", 12288);
-        p->sel_smem_cap = (size_t)envi("OTIF_OVL_SEL_SMEM", 36 * 1024);
-        p->pack_threads = (int)envi("OTIF_OVL_PACK_THREADS", 32);
-        p->ovl_mode = (int)envi("OTIF_OVL_MODE", 1);
-        if (p->ovl_mode == 1) p->sel_smem_cap = 0;   // select runs on the tensor stream between proxy launches
-        const int green = (int)envi("OTIF_OVL_GREEN", 0);
-        if (green <= 0) {
-            const size_t budget = (size_t)envi("OTIF_OVL_PROXY_SMEM", 184 * 1024);
-            otif_status rc2 = proxy_set_smem_budget(p->proxy, budget);
-            if (rc2 != OTIF_OK) { otif_pipeline_destroy(p); return rc2; }
-        } else {
-            // SM partition instead of co-residence: the proxy keeps its full shared memory
-            p->ovl_mode = 0;
-            p->sel_smem_cap = 0;
-            p->pack_ctas = 0;
-            p->pack_threads = 128;
-            p->pack_stages = 3;
-            p->pack_stage_bytes = 16384;
-            int dev = 0;
-            PCUDA(cudaGetDevice(&dev));
-            GreenApi ga;
-            if (!green_api(ga)) {
-                set_error("otif_pipeline_create: green-context driver entry point %s unavailable", g_green_missing);
-                otif_pipeline_destroy(p);
-                return OTIF_EUNSUPPORTED;
-            }
-            CUdevice cdev;
-            CUdevResource all, parts[1], rest;
-            CUdevResourceDesc d_t, d_m;
-            unsigned nparts = 1;
-            const unsigned tensor_sms = (unsigned)((num_sms - green) / 8 * 8);
-            if (ga.DeviceGet(&cdev, dev) != CUDA_SUCCESS ||
-                ga.DeviceGetDevResource(cdev, &all, CU_DEV_RESOURCE_TYPE_SM) != CUDA_SUCCESS ||
-                ga.DevSmResourceSplitByCount(parts, &nparts, &all, &rest, 0, tensor_sms) != CUDA_SUCCESS || nparts != 1 ||
-                ga.DevResourceGenerateDesc(&d_t, &parts[0], 1) != CUDA_SUCCESS ||
-                ga.DevResourceGenerateDesc(&d_m, &rest, 1) != CUDA_SUCCESS ||
-                ga.GreenCtxCreate(&p->g_tensor, d_t, cdev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS ||
-                ga.GreenCtxCreate(&p->g_mem, d_m, cdev, CU_GREEN_CTX_DEFAULT_STREAM) != CUDA_SUCCESS) {
-                set_error("otif_pipeline_create: green-context SM partition (%u + rest) failed", tensor_sms);
-                otif_pipeline_destroy(p);
-                return OTIF_EUNSUPPORTED;
-            }
-            CUstream st_t, st_m;
-            if (ga.GreenCtxStreamCreate(&st_t, p->g_tensor, CU_STREAM_NON_BLOCKING, 0) != CUDA_SUCCESS ||
-                ga.GreenCtxStreamCreate(&st_m, p->g_mem, CU_STREAM_NON_BLOCKING, 0) != CUDA_SUCCESS) {
-                set_error("otif_pipeline_create: green-context streams failed");
-                otif_pipeline_destroy(p);
-                return OTIF_EUNSUPPORTED;
-            }
-            p->s_tensor = (cudaStream_t)st_t;
-            p->s_mem = (cudaStream_t)st_m;
-            proxy_set_num_sms(p->proxy, (int)parts[0].sm.smCount);
-        }
-    }
     p->cells = p->gh * p->gw;
     p->cap_w = B * ((p->cells + 1) / 2);
-    const size_t src_bytes = (size_t)B * d->src_h * d->src_w * 3;
-    PCUDA(cudaMalloc(&p->src[0], src_bytes));
-    PCUDA(cudaMalloc(&p->src[1], src_bytes));
     PCUDA(cudaMalloc(&p->img, (size_t)p->pb * d->proxy.in_h * d->proxy.in_w * 3));
-    if (p->chunks >= 2) {
-        PCUDA(cudaMalloc(&p->img2, (size_t)p->pb * d->proxy.in_h * d->proxy.in_w * 3));
-        if (!p->s_mem) PCUDA(cudaStreamCreateWithFlags(&p->s_mem, cudaStreamNonBlocking));
-        PCUDA(cudaMalloc(&p->totals, (size_t)(p->chunks + 1) * 4));
-        PCUDA(cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming));
-        PCUDA(cudaEventCreateWithFlags(&p->ev_join, cudaEventDisableTiming));
-        for (int i = 0; i < 2; i++) {
-            PCUDA(cudaEventCreateWithFlags(&p->ev_resized[i], cudaEventDisableTiming));
-            PCUDA(cudaEventCreateWithFlags(&p->ev_scored[i], cudaEventDisableTiming));
-            PCUDA(cudaEventCreateWithFlags(&p->ev_imgfree[i], cudaEventDisableTiming));
-        }
-    }
     p->proxy_ws_bytes = otif_proxy_workspace_bytes(p->proxy, p->pb);
     PCUDA(cudaMalloc(&p->proxy_ws, p->proxy_ws_bytes));
     PCUDA(cudaMemset(p->proxy_ws, 0, p->proxy_ws_bytes));
@@ -458,8 +247,8 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     for (int s = 0; s < d->k; s++)
         if (d->batch_cap[s] > 0)
             PCUDA(cudaMalloc(&p->batches[s], (size_t)d->batch_cap[s] * d->sizes[s].w * d->sizes[s].h * 3));
-    PCUDA(cudaMalloc(&p->ctr, (kCtrFixed + 8) * 8));
-    PCUDA(cudaMemset(p->ctr, 0, (kCtrFixed + 8) * 8));
+    PCUDA(cudaMalloc(&p->ctr, kCtrTotal * 8));
+    PCUDA(cudaMemset(p->ctr, 0, kCtrTotal * 8));
     PCUDA(cudaMalloc(&p->out_total, 4));
     PCUDA(cudaStreamCreateWithFlags(&p->s_compute, cudaStreamNonBlocking));
     PCUDA(cudaStreamCreateWithFlags(&p->s_copy, cudaStreamNonBlocking));
@@ -476,8 +265,7 @@ extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     if (!p) return;
     if (p->s_compute) cudaStreamSynchronize(p->s_compute);
     if (p->s_copy) cudaStreamSynchronize(p->s_copy);
-    if (p->s_mem) cudaStreamSynchronize(p->s_mem);
-    void *bufs[] = {p->src[0], p->src[1], p->img, p->img2, p->totals, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
+    void *bufs[] = {p->src[0], p->src[1], p->img, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
                     p->offsets, p->total, p->slot, p->size_count, p->ctr, p->out_win, p->out_counts, p->out_total};
     for (void *b : bufs)
         if (b) cudaFree(b);
@@ -490,23 +278,16 @@ extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     }
     if (p->s_compute) cudaStreamDestroy(p->s_compute);
     if (p->s_copy) cudaStreamDestroy(p->s_copy);
-    if (p->s_tensor) cudaStreamSynchronize(p->s_tensor);
-    if (p->s_mem) cudaStreamDestroy(p->s_mem);
-    if (p->s_tensor) cudaStreamDestroy(p->s_tensor);
-    GreenApi ga;
-    if ((p->g_tensor || p->g_mem) && green_api(ga)) {
-        if (p->g_tensor) ga.GreenCtxDestroy(p->g_tensor);
-        if (p->g_mem) ga.GreenCtxDestroy(p->g_mem);
-    }
-    cudaEvent_t ovl[] = {p->ev_fork, p->ev_join, p->ev_resized[0], p->ev_resized[1], p->ev_scored[0], p->ev_scored[1],
-                         p->ev_imgfree[0], p->ev_imgfree[1]};
-    for (cudaEvent_t e : ovl)
-        if (e) cudaEventDestroy(e);
     if (p->proxy) otif_proxy_destroy(p->proxy);
     delete p;
 }
 
 static otif_status ensure_outputs(otif_pipeline *p, int n, int cap_windows) {
+    if (!p->src[0]) {   // double-buffered host staging, first host run only
+        const size_t bytes = (size_t)p->d.max_batch * p->d.src_h * p->d.src_w * 3;
+        OTIF_CUDA(cudaMalloc(&p->src[0], bytes));
+        OTIF_CUDA(cudaMalloc(&p->src[1], bytes));
+    }
     if (n > p->out_counts_cap) {
         if (p->out_counts) cudaFree(p->out_counts);
         p->out_counts = nullptr;
@@ -527,11 +308,12 @@ extern "C" otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *s
                                               int32_t *total_out, int32_t *size_count_out) {
     OTIF_REQUIRE(p && (src_host || n == 0) && n >= 0 && cap_windows >= 0, "otif_pipeline_run_host: bad arguments");
     OTIF_REQUIRE(total_out, "otif_pipeline_run_host: NULL total_out");
+    NvtxRange range("otif.pipeline_run_host");
     RC(ensure_outputs(p, n > 0 ? n : 1, cap_windows > 0 ? cap_windows : 1));
     const otif_pipeline_desc &d = p->d;
     const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
     OTIF_CUDA(cudaMemsetAsync(p->out_total, 0, 4, p->s_compute));
-    OTIF_CUDA(cudaMemsetAsync(p->ctr, 0, (kCtrFixed + 8) * 8, p->s_compute));
+    OTIF_CUDA(cudaMemsetAsync(p->ctr, 0, kCtrTotal * 8, p->s_compute));
     // the copy stream must not overwrite a src buffer before the compute stream is done with it
     for (int i = 0; i < 2; i++) OTIF_CUDA(cudaEventRecord(p->ev_free[i], p->s_compute));
     const int cap_saved = p->out_win_cap;
@@ -555,7 +337,7 @@ extern "C" otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *s
     OTIF_CUDA(cudaMemcpyAsync(&total, p->out_total, 4, cudaMemcpyDeviceToHost, p->s_compute));
     if (frame_count_out && n > 0)
         OTIF_CUDA(cudaMemcpyAsync(frame_count_out, p->out_counts, (size_t)n * 4, cudaMemcpyDeviceToHost, p->s_compute));
-    unsigned long long ctr[kCtrFixed + 8];
+    unsigned long long ctr[kCtrTotal];
     OTIF_CUDA(cudaMemcpyAsync(ctr, p->ctr, sizeof(ctr), cudaMemcpyDeviceToHost, p->s_compute));
     OTIF_CUDA(cudaStreamSynchronize(p->s_compute));
     const int keep = total < cap_windows ? total : cap_windows;
@@ -568,8 +350,10 @@ extern "C" otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *s
 }
 
 extern "C" otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t *src_dev, int32_t n,
-                                                cudaStream_t stream) {
-    OTIF_REQUIRE(p && (src_dev || n == 0) && n >= 0, "otif_pipeline_run_device: bad arguments");
+                                                int64_t frame_base, cudaStream_t stream) {
+    OTIF_REQUIRE(p && (src_dev || n == 0) && n >= 0 && frame_base >= 0 && frame_base + n < (1ll << 31),
+                 "otif_pipeline_run_device: bad arguments");
+    NvtxRange range("otif.pipeline_run_device");
     const size_t frame_bytes = (size_t)p->d.src_h * p->d.src_w * 3;
     // device runs keep no per-frame outputs beyond the current batch: counters only
     otif_window *ow = p->out_win;
@@ -579,7 +363,7 @@ extern "C" otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t 
     otif_status rc = OTIF_OK;
     for (int f0 = 0; f0 < n && rc == OTIF_OK; f0 += p->d.max_batch) {
         const int nb = n - f0 < p->d.max_batch ? n - f0 : p->d.max_batch;
-        rc = run_batch(p, src_dev + (size_t)f0 * frame_bytes, nb, f0, stream);
+        rc = run_batch(p, src_dev + (size_t)f0 * frame_bytes, nb, (int)(frame_base + f0), stream);
     }
     p->out_win = ow;
     p->out_counts = oc;
@@ -592,7 +376,7 @@ extern "C" const int64_t *otif_pipeline_counters(const otif_pipeline *p) {
 
 extern "C" otif_status otif_pipeline_reset_counters(otif_pipeline *p, cudaStream_t stream) {
     OTIF_REQUIRE(p, "otif_pipeline_reset_counters: NULL");
-    OTIF_CUDA(cudaMemsetAsync(p->ctr, 0, (kCtrFixed + 8) * 8, stream));
+    OTIF_CUDA(cudaMemsetAsync(p->ctr, 0, kCtrTotal * 8, stream));
     return OTIF_OK;
 }
 
@@ -608,7 +392,6 @@ extern "C" otif_status otif_pipeline_stage_ms(otif_pipeline *p, float *ms, int32
     OTIF_REQUIRE(p && ms && n_ms >= kStages, "otif_pipeline_stage_ms: need %d entries", kStages);
     for (int s = 0; s < kStages; s++) ms[s] = 0.0f;
     if (p->ev_used > 0) OTIF_CUDA(cudaEventSynchronize(p->ev_pool[p->ev_used - 1]));
-    if (p->ev_used > 0) OTIF_CUDA(cudaDeviceSynchronize());  // spans live on two streams
     for (size_t i = 0; i < p->ev_used; i++) {
         const int s = p->ev_stage[i], from = p->ev_from[i];
         if (s < 0 || from < 0) continue;  // a start marker: no time charged

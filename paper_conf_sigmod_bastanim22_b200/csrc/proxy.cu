@@ -469,229 +469,6 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
 }
 
 // ---------------------------------------------------------------------------
-// The same implicit GEMM on a CTA PAIR (cluster of 2, tcgen05 cta_group::2): one M=256
-// MMA spans both SMs — each CTA holds 128 rows of A (its own halo) and HALF of the N
-// columns of B, so per-SM shared-memory operand traffic and weight streaming halve
-// (N=128 layers are otherwise shared-memory-bandwidth bound).  The leader (rank 0)
-// issues the MMAs and commits them to both CTAs' barriers (multicast); the peer's MMA
-// warp relays "stage full" to the leader (remote mbarrier arrive); both epilogues
-// drain their own TMEM and report to the leader's accumulator-empty barrier.
-// Weights are packed [cb][tap][half][chunk][N/2][8].
-// ---------------------------------------------------------------------------
-template <int MT>
-__global__ void __launch_bounds__(kConvThreads, 1) conv_umma2_kernel(const __grid_constant__ ConvParams p) {
-    extern __shared__ __align__(1024) uint8_t smem[];
-    const int warp = threadIdx.x >> 5;
-    const int lane = threadIdx.x & 31;
-    const uint32_t rank = cluster_ctarank();
-    const int cluster = blockIdx.x >> 1, nclusters = gridDim.x >> 1;
-
-    const uint32_t chunks = p.kb >> 3;
-    const uint32_t a_bytes = chunks * p.P * 16;
-    const uint32_t nh = (uint32_t)p.N / 2;           // B rows held by this CTA
-    const uint32_t b_bytes = nh * p.kb * 2;
-    uint8_t *a_buf = smem;
-    uint8_t *b_buf = a_buf + (size_t)p.stages_a * a_bytes;
-    uint64_t *bars = reinterpret_cast<uint64_t *>(b_buf + (size_t)p.stages_b * b_bytes);
-    uint64_t *a_full = bars;
-    uint64_t *a_empty = a_full + kMaxStagesA;
-    uint64_t *b_full = a_empty + kMaxStagesA;
-    uint64_t *b_empty = b_full + kMaxStagesB;
-    uint64_t *a_peer = b_empty + kMaxStagesB;        // leader: peer's A stage landed
-    uint64_t *b_peer = a_peer + kMaxStagesA;         // leader: peer's B stage landed
-    uint64_t *t_full = b_peer + kMaxStagesB;
-    uint64_t *t_empty = t_full + 2;
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(t_empty + 2);
-    float *s_bias = reinterpret_cast<float *>(tmem_slot + 4);
-    float *s_w2 = s_bias + 256;
-
-    const uint32_t acc_cols = 2 * MT * p.N;
-    const uint32_t tmem_cols = acc_cols <= 32 ? 32 : (acc_cols <= 64 ? 64 : (acc_cols <= 128 ? 128 : (acc_cols <= 256 ? 256 : 512)));
-    const int npairs = p.ntiles;                     // pair tiles of 2 x 128*MT rows
-
-    if (threadIdx.x == 0) {
-        for (int i = 0; i < p.stages_a; i++) { mbar_init(&a_full[i], 1); mbar_init(&a_empty[i], 1); mbar_init(&a_peer[i], 1); }
-        for (int i = 0; i < p.stages_b; i++) { mbar_init(&b_full[i], 1); mbar_init(&b_empty[i], 1); mbar_init(&b_peer[i], 1); }
-        for (int i = 0; i < 2; i++) { mbar_init(&t_full[i], 1); mbar_init(&t_empty[i], 129);  /* 128 local + 1 from the peer */ }
-        fence_barrier_init();
-    }
-    if (warp == 2) tmem_alloc2(tmem_slot, tmem_cols);
-    for (int i = threadIdx.x; i < p.N; i += blockDim.x) {
-        s_bias[i] = p.bias[i];
-        if (p.out_kind == 3) s_w2[i] = p.w2[i];
-    }
-    tc_fence_before();
-    __syncthreads();
-    cluster_sync();  // both CTAs' barriers initialised before any remote arrive
-    tc_fence_after();
-    const uint32_t tmem_base = *tmem_slot;
-
-    if (warp == 0) {
-        // ===== producer (both CTAs): own halo rows and own half of the weights =====
-        if (lane == 0) {
-            uint32_t as = 0, ap = 0, bs = 0, bp = 0;
-            for (int pt = cluster; pt < npairs; pt += nclusters) {
-                const int64_t q0 = ((int64_t)pt * 2 + rank) * kTileM * MT;
-                for (int cb = 0; cb < p.ncb; cb++) {
-                    int tap_pos = 0;
-                    for (int g = 0; g < p.ngroups; g++) {
-                        mbar_wait(&a_empty[as], ap ^ 1);
-                        mbar_arrive_expect_tx(&a_full[as], a_bytes);
-                        uint8_t *dst = a_buf + (size_t)as * a_bytes;
-                        const int plane = p.group_plane[g];
-                        for (uint32_t j = 0; j < chunks; j++) {
-                            const uint8_t *src =
-                                p.act + (((int64_t)plane * p.c8_in + cb * chunks + j) * p.lcap + q0) * 16;
-                            bulk_g2s(dst + j * p.P * 16, src, p.P * 16, &a_full[as]);
-                        }
-                        if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
-                        for (int t = 0; t < p.group_ntaps[g]; t++, tap_pos++) {
-                            mbar_wait(&b_empty[bs], bp ^ 1);
-                            mbar_arrive_expect_tx(&b_full[bs], b_bytes);
-                            bulk_g2s(b_buf + (size_t)bs * b_bytes,
-                                     p.wpk + (((size_t)cb * 9 + tap_pos) * 2 + rank) * b_bytes, b_bytes, &b_full[bs]);
-                            if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
-                        }
-                    }
-                }
-            }
-        }
-    } else if (warp == 1 && rank == 1) {
-        // ===== peer: relay "stage full" to the leader's a_peer / b_peer =====
-        if (lane == 0) {
-            uint32_t as = 0, ap = 0, bs = 0, bp = 0;
-            const uint32_t a_peer0 = mapa_shared(smem_u32(a_peer), 0), b_peer0 = mapa_shared(smem_u32(b_peer), 0);
-            for (int pt = cluster; pt < npairs; pt += nclusters) {
-                for (int cb = 0; cb < p.ncb; cb++) {
-                    for (int g = 0; g < p.ngroups; g++) {
-                        mbar_wait(&a_full[as], ap);
-                        mbar_arrive_cluster(a_peer0 + as * 8);
-                        if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
-                        for (int t = 0; t < p.group_ntaps[g]; t++) {
-                            mbar_wait(&b_full[bs], bp);
-                            mbar_arrive_cluster(b_peer0 + bs * 8);
-                            if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
-                        }
-                    }
-                }
-            }
-        }
-    } else if (warp == 1) {
-        // ===== leader: MMA issuer for the pair (single thread) =====
-        if (lane == 0) {
-            const uint32_t idesc = umma_idesc_bf16(2 * kTileM, p.N);
-            uint32_t as = 0, ap = 0, bs = 0, bp = 0, acc = 0, accp = 0;
-            const uint32_t a_base = smem_u32(a_buf), b_base = smem_u32(b_buf);
-            const uint32_t lbo_a = p.P * 16, lbo_b = nh * 16;
-            for (int pt = cluster; pt < npairs; pt += nclusters) {
-                mbar_wait_cluster(&t_empty[acc], accp ^ 1);
-                tc_fence_after();
-                const uint32_t d = tmem_base + acc * MT * p.N;
-                uint32_t accumulate = 0;
-                for (int cb = 0; cb < p.ncb; cb++) {
-                    for (int g = 0; g < p.ngroups; g++) {
-                        mbar_wait(&a_full[as], ap);
-                        mbar_wait_cluster(&a_peer[as], ap);
-                        tc_fence_after();
-                        const uint32_t a_stage = a_base + as * a_bytes;
-                        for (int t = 0; t < p.group_ntaps[g]; t++) {
-                            mbar_wait(&b_full[bs], bp);
-                            mbar_wait_cluster(&b_peer[bs], bp);
-                            tc_fence_after();
-                            const uint32_t a_tap = a_stage + p.group_shift[g][t] * 16;
-                            const uint32_t b_stage = b_base + bs * b_bytes;
-                            for (uint32_t s = 0; s < chunks / 2; s++) {
-                                const uint64_t bd = umma_desc(b_stage + 2 * s * lbo_b, lbo_b, 128);
-#pragma unroll
-                                for (int m = 0; m < MT; m++) {
-                                    uint64_t ad = umma_desc(a_tap + 2 * s * lbo_a + m * (kTileM * 16), lbo_a, 128);
-                                    umma2_bf16(d + m * p.N, ad, bd, idesc, accumulate);
-                                }
-                                accumulate = 1;
-                            }
-                            umma2_commit_mc(&b_empty[bs], 0x3);
-                            if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
-                        }
-                        umma2_commit_mc(&a_empty[as], 0x3);
-                        if (++as == (uint32_t)p.stages_a) { as = 0; ap ^= 1; }
-                    }
-                }
-                umma2_commit_mc(&t_full[acc], 0x3);
-                if (++acc == 2) { acc = 0; accp ^= 1; }
-            }
-        }
-    } else if (warp >= 4) {
-        // ===== epilogue (both CTAs): own 128 TMEM lanes = own rows =====
-        const int row = threadIdx.x - 128;
-        const int quarter = warp & 3;
-        const uint32_t t_empty0 = mapa_shared(smem_u32(t_empty), 0);
-        uint32_t acc = 0, accp = 0;
-        for (int pt = cluster; pt < npairs; pt += nclusters) {
-            mbar_wait(&t_full[acc], accp);
-            tc_fence_after();
-            for (int m = 0; m < MT; m++) {
-                const int64_t q = ((int64_t)pt * 2 + rank) * kTileM * MT + m * kTileM + row;
-                const int f = (int)(q / p.fstride);
-                const int64_t r = q - (int64_t)f * p.fstride;
-                const int oy = (int)(r / p.pitch);
-                const int ox = (int)(r - (int64_t)oy * p.pitch);
-                const bool valid = q < p.mtot && oy < p.out_h && ox < p.out_w;
-                int plane = 0;
-                int64_t L = 0;
-                if (p.out_kind != 3) L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, f, oy, ox, plane);
-                const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + (acc * MT + m) * p.N;
-                float z = p.b2;
-                for (int cc = 0; cc < p.N / 32; cc++) {
-                    uint32_t v[32];
-                    tmem_ld32(taddr + cc * 32, v);
-                    uint32_t pk[16];
-#pragma unroll
-                    for (int j = 0; j < 16; j++) {
-                        float a = fmaxf(__uint_as_float(v[2 * j]) + s_bias[cc * 32 + 2 * j], 0.0f);
-                        float b = fmaxf(__uint_as_float(v[2 * j + 1]) + s_bias[cc * 32 + 2 * j + 1], 0.0f);
-                        pk[j] = pack_bf16x2(a, b);
-                    }
-                    if (p.out_kind == 3) {
-#pragma unroll
-                        for (int j = 0; j < 16; j++) {
-                            float a = __uint_as_float(pk[j] << 16);
-                            float b = __uint_as_float(pk[j] & 0xFFFF0000u);
-                            z = fmaf(s_w2[cc * 32 + 2 * j], a, z);
-                            z = fmaf(s_w2[cc * 32 + 2 * j + 1], b, z);
-                        }
-                    } else if (valid) {
-#pragma unroll
-                        for (int c = 0; c < 4; c++) {
-                            uint8_t *dst = p.out + (((int64_t)plane * p.out_c8 + cc * 4 + c) * p.out_lcap + L) * 16;
-                            *reinterpret_cast<uint4 *>(dst) =
-                                make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
-                        }
-                    }
-                }
-                if (p.out_kind == 3 && valid)
-                    p.scores[((int64_t)f * p.out_h + oy) * p.out_w + ox] = 1.0f / (1.0f + expf(-z));
-            }
-            tc_fence_before();
-            if (rank == 0) {
-                mbar_arrive(&t_empty[acc]);
-            } else {  // one cluster-scope release for the whole peer epilogue
-                asm volatile("bar.sync 1, 128;" ::: "memory");
-                if (row == 0) mbar_arrive_cluster(t_empty0 + acc * 8);
-            }
-            if (++acc == 2) { acc = 0; accp ^= 1; }
-        }
-    }
-    __syncwarp();
-    tc_fence_before();
-    __syncthreads();
-    cluster_sync();  // the peer's smem / TMEM stay alive until the pair's last MMA drained
-    if (warp == 2) {
-        tc_fence_after();
-        tmem_dealloc2(tmem_base, tmem_cols);
-    }
-}
-
-// ---------------------------------------------------------------------------
 // E1 fused into E2 (stride-2 E2 only).  E1's output never reaches HBM: per E2 tile
 // (M = 256 output positions of E2's parity-split input layout) the CTA
 //   1. stages the proxy-image rows the tile needs in shared memory ("slab": 4 image
@@ -753,6 +530,15 @@ struct E12Params {
     int64_t out_fstride;
 };
 
+// Trace / knock-out bits (OTIF_E12_TRACE, read at launch) exist only in a trace build
+// (nvcc -DOTIF_E12_TRACE_BUILD); in the release library they are the constant 0, so no
+// environment variable can change what the shipped kernel computes.
+#ifdef OTIF_E12_TRACE_BUILD
+#define E12_BITS (p.trace)
+#else
+#define E12_BITS 0
+#endif
+
 // E2-layout position q of a tile whose first plane row is g0: which of the 4 parity
 // planes hold an E1 pixel there (bit (rp << 1) | cp), and the slab byte offset of the
 // image sample at (row 2y - 1, column 2x - 1) for plane (0, 0) (the other planes add
@@ -774,7 +560,7 @@ __device__ __forceinline__ void e12_im2col_row(const E12Params &p, const uint8_t
                                                int rp, int cp, uint32_t (&wv)[16]) {
 #pragma unroll
     for (int j = 0; j < 16; j++) wv[j] = 0;
-    if (!valid || (p.trace & 4)) return;   // trace & 4: timing experiment (no gather)
+    if (!valid || (E12_BITS & 4)) return;   // trace & 4: timing experiment (no gather)
     const uint32_t b = off + 2 * rp * p.slab_pitch + 6 * cp;
     const uint32_t sh = (b & 3) * 8;
     const uint32_t *wp = reinterpret_cast<const uint32_t *>(slab + (b & ~3u));
@@ -814,7 +600,7 @@ __device__ __forceinline__ void e12_im2col_row(const E12Params &p, const uint8_t
                        (nslots) > 2 ? tt[2][j_] - t00 : 0ll);                                       \
     } while (0)
 #define E12_TR_DECL                                                       \
-    const bool tr = (p.trace & 1) && blockIdx.x == 0 && ((threadIdx.x & 127) == 0 || threadIdx.x == 32 || threadIdx.x == 96); \
+    const bool tr = (E12_BITS & 1) && blockIdx.x == 0 && ((threadIdx.x & 127) == 0 || threadIdx.x == 32 || threadIdx.x == 96); \
     long long tt[3][16];                                                   \
     const long long t00 = clock64();
 #else
@@ -823,23 +609,15 @@ __device__ __forceinline__ void e12_im2col_row(const E12Params &p, const uint8_t
 #define E12_TR_DECL
 #endif
 
-#define E12_WAIT_SLEEP(b, ph) (p.trace & 2 ? mbar_wait(b, ph) : mbar_wait_sleep(b, ph))
+#define E12_WAIT_SLEEP(b, ph) (E12_BITS & 2 ? mbar_wait(b, ph) : mbar_wait_sleep(b, ph))
 // waits on the hand-off chain (gather <- a1_empty, E1 epilogue <- a2_empty): polling (bit 128 = sleep, A/B)
-#define E12_WAIT_CHAIN(b, ph) (p.trace & 128 ? mbar_wait_sleep(b, ph) : mbar_wait(b, ph))
-template <int KT, bool TS>
+#define E12_WAIT_CHAIN(b, ph) (E12_BITS & 128 ? mbar_wait_sleep(b, ph) : mbar_wait(b, ph))
+template <int KT>
 __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_constant__ E12Params p) {
-    // TS: E1's A operand (the im2col rows) lives in TMEM (columns kA1Col.., written by the
-    // gather warps with tcgen05.st, lane = row) instead of shared memory: the E1 MMA then
-    // reads only its B operand from shared memory (M128 N32 K16: 17 vs 40 clk per MMA,
-    // scripts/micro/ts_mma.cu) and the gather stores leave the shared-memory port.
-    // TMEM: E2 acc 256 + E1 acc 2 x 96 + A1 48 columns = 496 (KT = 3 only).
-    static_assert(!TS || KT == 3, "TMEM budget holds the A1 rows for KT = 3 only");
-    // TMEM: E2 accumulators kAccStages x (MT x 64) at 0, E1 accumulators kE1Slots x 32 KT,
-    // then (TS) the A1 rows
+    // TMEM: E2 accumulators kAccStages x (MT x 64) at 0, E1 accumulators kE1Slots x 32 KT
     constexpr int kAccStages = OTIF_E12_ACC, kE1Slots = OTIF_E12_E1SLOTS;
     constexpr uint32_t kE1Col = kAccStages * 2 * 64;
-    constexpr uint32_t kA1Col = kE1Col + kE1Slots * 32 * KT;
-    static_assert(kA1Col + (TS ? 16 * KT : 0) <= 512, "TMEM budget");
+    static_assert(kE1Col + kE1Slots * 32 * KT <= 512, "TMEM budget");
     extern __shared__ __align__(1024) uint8_t smem[];
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -855,7 +633,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
     uint8_t *w2_s = smem;
     uint8_t *w1_s = w2_s + kW2Bytes;
     uint8_t *a1_s = w1_s + kW1Bytes;
-    uint8_t *a2_s = a1_s + (TS ? (size_t)0 : (size_t)p.na1 * kA1Bytes);
+    uint8_t *a2_s = a1_s + (size_t)p.na1 * kA1Bytes;
     uint8_t *slab_s = a2_s + (size_t)p.np * kPlaneBytes;
     uint64_t *bars = reinterpret_cast<uint64_t *>(slab_s + 2 * (size_t)slab_bytes);
     uint64_t *slab_full = bars, *slab_empty = bars + 2;
@@ -910,7 +688,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 const uint32_t f = fdiv(g, p.div_rpf);
                 const int i = (int)(g - f * rows_per_frame);
                 const int y = 4 * (i - 1) + k;
-                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp && !(p.trace & 64)) my_bytes += p.row_bytes;
+                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp && !(E12_BITS & 64)) my_bytes += p.row_bytes;
             }
             if (p.bulk) {
 #pragma unroll
@@ -925,7 +703,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 const int i = (int)(g - f * rows_per_frame);
                 const int y = 4 * (i - 1) + k;
                 uint8_t *dst = slab + (size_t)s * p.slab_pitch;
-                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp && !(p.trace & 64)) {   // 64: timing experiment
+                if ((int)f < p.n && i >= 1 && y >= 0 && y < p.hp && !(E12_BITS & 64)) {   // 64: timing experiment
                     const uint8_t *src = p.img + ((size_t)f * p.hp + y) * p.row_bytes;
                     if (p.bulk) {
                         bulk_g2s(dst + 16, src, p.row_bytes, &slab_full[sb]);
@@ -964,11 +742,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 for (int k = 0; k < KT; k++)
 #pragma unroll
                     for (int s = 0; s < 2; s++) {
-                        if constexpr (TS)
-                            umma_ts_warp(d + k * 32, tmem_base + kA1Col + k * 16 + s * 8, w1d + ((2 * s * 512) >> 4),
-                                         idesc1, s);
-                        else
-                            umma_bf16_warp(d + k * 32, a1d + ((s1 * kA1Bytes + k * 8192 + 2 * s * 2048) >> 4),
+                        umma_bf16_warp(d + k * 32, a1d + ((s1 * kA1Bytes + k * 8192 + 2 * s * 2048) >> 4),
                                            w1d + ((2 * s * 512) >> 4), idesc1, s);
                     }
                 umma_commit_warp(&a1_empty[s1]);
@@ -994,7 +768,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 E12_TR(1, 0);
                 tc_fence_after();
                 const uint64_t a = a2d + ((pb * kPlaneBytes) >> 4);
-                const int ntaps = (p.trace & 8) ? 1 : p.group_ntaps[g];   // trace & 8: timing experiment
+                const int ntaps = (E12_BITS & 8) ? 1 : p.group_ntaps[g];   // trace & 8: timing experiment
 #pragma unroll 1
                 for (int t = 0; t < ntaps; t++, pos++) {
                     const uint64_t at = a + p.group_shift[g][t];          // +16 B per pixel of shift
@@ -1033,16 +807,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 const uint32_t s1 = (uint32_t)p.na1 == 1 ? 0 : (J & 1);
                 const uint32_t ph1 = (uint32_t)p.na1 == 1 ? (J & 1) : ((J >> 1) & 1);
                 E12_TR(0, 0);
-                if constexpr (!TS) E12_WAIT_CHAIN(&a1_empty[s1], ph1 ^ 1);
+                E12_WAIT_CHAIN(&a1_empty[s1], ph1 ^ 1);
                 E12_TR(1, 0);
-                uint32_t wk[2][16];   // TS: this thread's rows of its (at most 2) k sub-tiles
-                if constexpr (TS) {
-#pragma unroll
-                    for (int k = 0; k < KT; k++) {
-                        if ((int)((J * KT + k) & 1) != wg) continue;
-                        e12_im2col_row(p, slab, (vm[k] >> g) & 1, of[k], rp, cp, wk[k >> 1]);
-                    }
-                } else {
+                {
                     // rolled loop over this warpgroup's k sub-tiles (code size: the kernel is
                     // instruction-cache bound, see the header)
 #pragma unroll 1
@@ -1059,22 +826,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                             *reinterpret_cast<uint4 *>(dst + c * 2048) = make_uint4(wv[4 * c], wv[4 * c + 1], wv[4 * c + 2], wv[4 * c + 3]);
                     }
                 }
-                if constexpr (TS) {
-                    // the rows are computed; now wait for the E1 MMAs of the previous job to
-                    // release the single A1 buffer and store them into this warp's TMEM lanes
-                    E12_WAIT_SLEEP(&a1_empty[0], (J & 1) ^ 1);
-                    tc_fence_after();
-                    const uint32_t lanes = (uint32_t)(row & ~31) << 16;
-#pragma unroll
-                    for (int k = 0; k < KT; k++) {
-                        if ((int)((J * KT + k) & 1) != wg) continue;
-                        tmem_st16(tmem_base + lanes + kA1Col + k * 16, wk[k >> 1]);
-                    }
-                    tmem_wait_st();
-                    tc_fence_before();
-                } else {
-                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-                }
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
                 mbar_arrive(&a1_full[s1]);
                 E12_TR(2, 0);
             }
@@ -1103,7 +855,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 const uint32_t tacc = tmem_base + ((uint32_t)(quarter * 32) << 16) + kE1Col + (J % kE1Slots) * (32 * KT);
 #pragma unroll 1
                 for (int k = (int)((wg - J * KT) & 1); k < KT; k += 2) {
-                    if (p.trace & 32) continue;   // 32: timing experiment
+                    if (E12_BITS & 32) continue;   // 32: timing experiment
                     uint32_t v[32];
                     tmem_ld32(tacc + k * 32, v);
                     uint32_t pk[16];
@@ -1150,7 +902,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 for (int cc = 0; cc < N2 / 32; cc++) {
                     uint32_t v[32];
                     tmem_ld32(taddr + cc * 32, v);
-                    if (valid && !(p.trace & 16)) {   // 16: timing experiment
+                    if (valid && !(E12_BITS & 16)) {   // 16: timing experiment
                         uint32_t pk[16];
 #pragma unroll
                         for (int j = 0; j < 16; j++)
@@ -1201,7 +953,7 @@ struct GemmLayer {
     int64_t fstride_unit;         // per-frame pixels of the input layout
     int max_shift;
     int ngroups, group_plane[4], group_ntaps[4], group_shift[4][9], group_tap[4][9];
-    int kb, ncb, P, mt, cg;   // cg: 1 = single CTA, 2 = CTA pair (cta_group::2)
+    int kb, ncb, P, mt;
     uint8_t *wpk_dev;
     float *bias_dev;
 };
@@ -1218,15 +970,10 @@ struct otif_proxy {
     float *w2_dev;                // [dec] bf16-rounded
     float b2;
     int num_sms;
-    int head_swap;                // swapped-operand head layer (default on; OTIF_HEAD_SWAP=0 for A/B runs)
     // E1 fused into E2 (e12_umma_kernel); 0 = separate E1 kernel + E2 conv
     int e12;
     int e12_P, e12_np, e12_na1, e12_slab_rows, e12_slab_pitch;
-    int e12_ts;                   // E1's A operand in TMEM (KT = 3; OTIF_E12_TS=0 for A/B runs)
     size_t e12_smem, e12_fixed, e12_unit;
-    // shared-memory budget of one conv / E1+E2 CTA (default: the whole SM); a pipeline that
-    // runs memory-bound kernels next to the proxy lowers it so their CTAs stay co-resident
-    size_t smem_budget = 227 * 1024;
     uint16_t *e12_w1_dev;         // fp16 [4][32][8] = bf16(w1) * 2^s, K = kh*10 + kw*3 + c; bias parts at K = 9, 19, 29
     uint16_t *e12_w2_dev;         // E2's packed bf16 weights * 2^-(s+7)
     uint64_t plan_hash;
@@ -1279,17 +1026,9 @@ static void build_layer(GemmLayer &g, int cin, int cout, int stride, int in_h, i
     // mt sub-tiles of 128 rows per CTA tile so that every tap issues >= 256 columns of MMA
     // work (mt * N = 256): amortises the per-stage barrier and copy overheads of small N
     g.mt = cout >= 256 ? 1 : (cout >= 128 ? 2 : 4);
-    // CTA pairs (cta_group::2) would halve per-SM operand traffic for N >= 128, but with
-    // the relayed stage hand-off they measured 1.3-1.7x SLOWER than single CTAs on B200
-    // (profiles/r01_cta_pair.md); single CTAs are the default, pairs opt-in for tuning.
-    g.cg = 1;
-    if (const char *e = getenv("OTIF_CONV_CG")) {  // tuning experiments only
-        if (atoi(e) == 2 && cout >= 128) g.cg = 2;
-    }
-    if (const char *e = getenv("OTIF_CONV_MT_MAX")) {  // tuning experiments only
-        int cap = atoi(e);
-        if (cap >= 1 && g.mt > cap) g.mt = cap;
-    }
+    // (CTA pairs, cta_group::2 with M = 256, measured 1.3-1.7x slower than single CTAs here
+    // because every stage hand-off is relayed through the peer's mbarrier:
+    // profiles/r01_cta_pair.md; not built)
     g.P = (int)round_up(kTileM * g.mt + g.max_shift, 8);
 }
 
@@ -1300,7 +1039,7 @@ static Layout input_layout(const GemmLayer &g, int n) {
     l.pitch = g.pitch;
     l.fstride = g.fstride_unit;
     int64_t mtot = (int64_t)n * g.fstride_unit;
-    l.lcap = round_up(round_up(mtot, (int64_t)kTileM * g.mt * g.cg) + g.max_shift + 8, 16);
+    l.lcap = round_up(round_up(mtot, (int64_t)kTileM * g.mt) + g.max_shift + 8, 16);
     l.c8 = g.cin / 8;
     l.bytes = (size_t)l.planes * l.c8 * l.lcap * 16;
     l.offset = 0;
@@ -1361,24 +1100,20 @@ static bool bf16_scale_exact(uint16_t b, int k, uint16_t *out) {
     return true;
 }
 
-static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes, size_t budget = 220 * 1024);
+static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes);
 
-// deepest (im2col stages, plane buffers) of the E1+E2 kernel within `budget` bytes; in TS
-// mode the im2col rows live in TMEM (one buffer, no shared memory)
-static bool e12_stages(size_t fixed, size_t unit, size_t budget, int &np, int &na1, bool ts) {
+// deepest (im2col stages, plane buffers) of the E1+E2 kernel within `budget` bytes
+static bool e12_stages(size_t fixed, size_t unit, size_t budget, int &np, int &na1) {
     np = 0; na1 = 0;
-    for (int cand_a1 = ts ? 1 : 2; cand_a1 >= 1 && !np; cand_a1--)
+    for (int cand_a1 = 2; cand_a1 >= 1 && !np; cand_a1--)
         for (int cand = kE12MaxPlaneBufs; cand >= 2 && !np; cand--)
-            if (fixed + (size_t)((ts ? 0 : cand_a1) + cand) * unit <= budget) { np = cand; na1 = cand_a1; }
+            if (fixed + (size_t)(cand_a1 + cand) * unit <= budget) { np = cand; na1 = cand_a1; }
     return np != 0;
 }
 
 static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const float *b1 /* [32] */) {
-    if (const char *e = getenv("OTIF_E12")) {      // A/B runs only
-        if (e[0] == '0') return false;
-    }
     const GemmLayer &g = p->L[0];
-    if (p->d.n_strided < 2 || g.kind != 2 || g.cin != 32 || g.cout != 64 || g.cg != 1) return false;
+    if (p->d.n_strided < 2 || g.kind != 2 || g.cin != 32 || g.cout != 64) return false;
     float maxabs = 0.0f;
     for (int i = 0; i < 32 * 27; i++) maxabs = fmaxf(maxabs, fabsf(bf16_to_f32(f32_to_bf16_rne(w1[i]))));
     int s = 0;
@@ -1426,10 +1161,8 @@ static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const f
     const int slab_pitch = (int)round_up(16 + 3 * p->d.in_w + 32, 16);
     const size_t fixed = 9 * 4 * 64 * 16 + 4 * 32 * 16 + 2 * (size_t)slab_rows * slab_pitch + 64 * 8 + 16 + 96 * 4 + 1024;
     const size_t a1 = (size_t)P * 64, plane = (size_t)P * 64;
-    // measured 1.75 vs 1.66 ms on the C2 step (latency, not the shared-memory port, bounds E1+E2), so opt-in
-    const bool ts = P / 128 == 3 && getenv("OTIF_E12_TS") && getenv("OTIF_E12_TS")[0] == '1';
     int np = 0, na1 = 0;
-    if (!e12_stages(fixed, a1, 227 * 1024, np, na1, ts)) return false;
+    if (!e12_stages(fixed, a1, 227 * 1024, np, na1)) return false;
     if (cudaMalloc(&p->e12_w1_dev, wh.size() * 2) != cudaSuccess) return false;
     cudaMemcpy(p->e12_w1_dev, wh.data(), wh.size() * 2, cudaMemcpyHostToDevice);
     if (cudaMalloc(&p->e12_w2_dev, w2.size() * 2) != cudaSuccess) return false;
@@ -1439,59 +1172,24 @@ static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const f
     p->e12_slab_rows = slab_rows;
     p->e12_slab_pitch = slab_pitch;
     p->e12_na1 = na1;
-    p->e12_smem = fixed + (size_t)(ts ? 0 : na1) * a1 + (size_t)np * plane;
-    p->e12_ts = ts ? 1 : 0;
+    p->e12_smem = fixed + (size_t)na1 * a1 + (size_t)np * plane;
     p->e12_fixed = fixed;
     p->e12_unit = a1;
     return true;
 }
 
-// SMs the persistent proxy kernels size their grids for (an SM partition of a green
-// context in the pipeline's partitioned overlap mode; default: the whole device)
-void proxy_set_num_sms(otif_proxy *p, int sms) {
-    if (sms > 0) p->num_sms = sms;
-}
-
 // kernel launches of one launch_proxy call (workspace zero + tag, E1+E2 fused or E1 and E2, E3..D1)
 int proxy_launches(const otif_proxy *p) { return p->e12 ? 7 : 8; }
 
-// Lower the per-CTA shared-memory budget of the proxy kernels (pipeline overlap mode):
-// the conv rings and the E1+E2 plane / im2col buffers shrink to fit.  Not thread-safe
-// against concurrent launches of the same proxy; the pipeline calls it once at create.
-otif_status proxy_set_smem_budget(otif_proxy *p, size_t budget) {
-    if (budget > 227 * 1024) budget = 227 * 1024;
-    for (int li = 0; li < 5; li++) {
-        int sa, sb;
-        size_t bytes;
-        conv_smem(p->L[li], sa, sb, bytes, budget);
-        if (bytes > budget) {
-            set_error("proxy_set_smem_budget: layer %d needs %zu B > %zu B", li + 2, bytes, budget);
-            return OTIF_EUNSUPPORTED;
-        }
-    }
-    if (p->e12) {
-        int np = 0, na1 = 0;
-        if (!e12_stages(p->e12_fixed, p->e12_unit, budget, np, na1, p->e12_ts != 0)) {
-            set_error("proxy_set_smem_budget: E1+E2 needs more than %zu B", budget);
-            return OTIF_EUNSUPPORTED;
-        }
-        p->e12_np = np;
-        p->e12_na1 = na1;
-        p->e12_smem = p->e12_fixed + (size_t)(np + (p->e12_ts ? 0 : na1)) * p->e12_unit;
-    }
-    p->smem_budget = budget;
-    return OTIF_OK;
-}
-
-static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes, size_t budget) {
+static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
     size_t a = (size_t)(g.kb / 8) * g.P * 16;
-    size_t b = (size_t)g.cout * g.kb * 2 / g.cg;
+    size_t b = (size_t)g.cout * g.kb * 2;
     size_t fixed = (3 * kMaxStagesA + 3 * kMaxStagesB + 4) * 8 + 16 + 2 * 256 * 4 + 4 * 256 * 4 + 1024;
-    if (budget > 220 * 1024) budget = 220 * 1024;
+    const size_t budget = 220 * 1024;
     sa = 2; sb = 2;
-    // grow B (weights stream every tap) first, then A
-    // a CTA pair recycles a stage over a longer loop (peer relay, multicast commit): deeper B ring
-    const int sb_max = g.cg == 2 ? kMaxStagesB : 6;
+    // grow B (weights stream every tap) first, then A (deeper rings measured no faster,
+    // DESIGN.md §11)
+    const int sb_max = 6;
     while (sb < kMaxStagesB && sa * a + (sb + 1) * b + fixed <= budget && sb < sb_max) sb++;
     while (sa < kMaxStagesA && (sa + 1) * a + sb * b + fixed <= budget && sa < 3) sa++;
     bytes = sa * a + sb * b + fixed;
@@ -1547,7 +1245,9 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         e.ntiles = (int)cdiv(e.mtot, 256);
         e.slab_rows = p->e12_slab_rows; e.slab_pitch = p->e12_slab_pitch;
         e.bulk = (e.row_bytes % 16 == 0) && (((uintptr_t)img & 15) == 0);
+#ifdef OTIF_E12_TRACE_BUILD
         if (const char *x = getenv("OTIF_E12_TRACE")) e.trace = atoi(x);
+#endif
         for (int i = 0; i < 4; i++) {
             e.group_ntaps[i] = g.group_ntaps[i];
             for (int t = 0; t < 9; t++) e.group_shift[i][t] = g.group_shift[i][t];
@@ -1556,8 +1256,7 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         e.wt2 = p->e12_w2_dev; e.b2 = g.bias_dev;
         e.out_kind = lay[1].kind; e.out = ws + lay[1].offset; e.out_lcap = lay[1].lcap;
         e.out_c8 = lay[1].c8; e.out_pitch = lay[1].pitch; e.out_fstride = lay[1].fstride;
-        auto kern = e.P == 384 ? (p->e12_ts ? e12_umma_kernel<3, true> : e12_umma_kernel<3, false>)
-                               : e12_umma_kernel<4, false>;
+        auto kern = e.P == 384 ? e12_umma_kernel<3> : e12_umma_kernel<4>;
         OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->e12_smem));
         const int grid = e.ntiles < p->num_sms ? e.ntiles : p->num_sms;
         kern<<<grid, kE12Threads, p->e12_smem, stream>>>(e);
@@ -1595,7 +1294,7 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         }
         c.wpk = g.wpk_dev; c.bias = g.bias_dev; c.N = g.cout;
         c.mtot = (int64_t)n * g.fstride_unit;
-        c.ntiles = (int)cdiv(c.mtot, (int64_t)kTileM * g.mt * g.cg);  // pair tiles when cg == 2
+        c.ntiles = (int)cdiv(c.mtot, (int64_t)kTileM * g.mt);
         c.pitch = g.pitch; c.fstride = g.fstride_unit; c.out_h = g.out_h; c.out_w = g.out_w;
         if (li < 4) {
             c.out_kind = lay[li + 1].kind;
@@ -1611,35 +1310,15 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
             c.b2 = p->b2;
         }
         size_t smem;
-        conv_smem(g, c.stages_a, c.stages_b, smem, p->smem_budget);
-        if (g.cg == 2) {
-            const int pairs = p->num_sms / 2;
-            const int clusters = c.ntiles < pairs ? (c.ntiles < 1 ? 1 : c.ntiles) : pairs;
-            auto kern = g.mt == 4 ? conv_umma2_kernel<4> : (g.mt == 2 ? conv_umma2_kernel<2> : conv_umma2_kernel<1>);
-            OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            cudaLaunchConfig_t cfg = {};
-            cfg.gridDim = dim3(2 * clusters);
-            cfg.blockDim = dim3(kConvThreads);
-            cfg.dynamicSmemBytes = smem;
-            cfg.stream = stream;
-            cudaLaunchAttribute attr[1];
-            attr[0].id = cudaLaunchAttributeClusterDimension;
-            attr[0].val.clusterDim.x = 2;
-            attr[0].val.clusterDim.y = 1;
-            attr[0].val.clusterDim.z = 1;
-            cfg.attrs = attr;
-            cfg.numAttrs = 1;
-            OTIF_CUDA(cudaLaunchKernelEx(&cfg, kern, c));
-        } else {
-            int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
-            if (grid < 1) grid = 1;
-            // head layer with N = 128: swapped operands (see conv_umma_kernel)
-            const bool swap = c.out_kind == 3 && g.mt == 2 && g.cout == 128 && p->head_swap;
-            auto kern = swap ? conv_umma_kernel<2, true>
-                             : (g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>));
-            OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-            kern<<<grid, kConvThreads, smem, stream>>>(c);
-        }
+        conv_smem(g, c.stages_a, c.stages_b, smem);
+        int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
+        if (grid < 1) grid = 1;
+        // head layer with N = 128: swapped operands (see conv_umma_kernel)
+        const bool swap = c.out_kind == 3 && g.mt == 2 && g.cout == 128;
+        auto kern = swap ? conv_umma_kernel<2, true>
+                         : (g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>));
+        OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        kern<<<grid, kConvThreads, smem, stream>>>(c);
         OTIF_LAUNCH_CHECK();
         if (evs) OTIF_CUDA(cudaEventRecord(evs[1 + li], stream));
     }
@@ -1686,10 +1365,6 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
     if (!p) return OTIF_ENOMEM;
     p->d = *d;
     p->num_sms = num_sms;
-    {
-        const char *e = getenv("OTIF_HEAD_SWAP");
-        p->head_swap = !(e && e[0] == '0');
-    }
     // spatial chain
     int h = d->in_h, w = d->in_w;
     int hs[7], wss[7];
@@ -1744,10 +1419,7 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
                             for (int e = 0; e < 8; e++) {
                                 int ci = cb * g.kb + j * 8 + e;
                                 float v = W[(((size_t)nn * 3 + kh) * 3 + kw) * g.cin + ci];
-                                // cg == 2: [cb][tap][half][chunk][N/2][8] (each CTA of a pair streams its half)
-                                const int nh = g.cout / g.cg, half = nn / nh, nl = nn - half * nh;
-                                pk[(((((size_t)cb * 9 + pos) * g.cg + half) * chunks + j) * nh + nl) * 8 + e] =
-                                    f32_to_bf16_rne(v);
+                                pk[((((size_t)cb * 9 + pos) * chunks + j) * g.cout + nn) * 8 + e] = f32_to_bf16_rne(v);
                             }
                 }
         }

@@ -669,7 +669,7 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum, size_t smem_cap) {
+                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum) {
     SelectParams p;
     memset(&p, 0, sizeof(p));
     p.scores = scores; p.mask_in = mask_in; p.thr = threshold;
@@ -719,8 +719,7 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
         p.from_list = pass;
         p.nmat = small_costs ? (int)round_up(ccap < kMatMax ? ccap : kMatMax, 8) : 0;
         p.frame_bytes = sel_frame_bytes(gh, gw, ccap, p.nmat, &p.gmat_offset);
-        // smem_cap (pipeline overlap mode): CTAs small enough to sit next to a proxy CTA
-        const size_t cap_bytes = smem_cap > 0 && smem_cap < 200 * 1024 ? smem_cap : 200 * 1024;
+        const size_t cap_bytes = 200 * 1024;
         int warps = (int)(cap_bytes / p.frame_bytes);
         warps = warps < 1 ? 1 : (warps > kSelWarpsMax ? kSelWarpsMax : warps);
         if (pass == 0) {  // spread small batches over the SMs rather than packing frames into few CTAs
@@ -784,9 +783,11 @@ extern "C" otif_status otif_select_windows(const float *scores, const uint8_t *m
                                            int32_t gh, int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes,
                                            int32_t k, uint8_t *mask_out, otif_window *windows, int32_t capacity,
                                            int32_t *frame_count, int32_t *frame_offset, int32_t *total,
-                                           void *workspace, size_t ws_bytes, cudaStream_t stream) {
+                                           void *workspace, size_t ws_bytes, cudaStream_t stream,
+                                           int64_t *est_sum) {
     otif_status st = validate_select(scores, mask_in, n, gh, gw, g, sizes, k, capacity);
     if (st != OTIF_OK) return st;
+    if (est_sum) OTIF_CUDA(cudaMemsetAsync(est_sum, 0, 8, stream));
     if (n == 0) {
         if (total) OTIF_CUDA(cudaMemsetAsync(total, 0, 4, stream));
         return OTIF_OK;
@@ -797,5 +798,6 @@ extern "C" otif_status otif_select_windows(const float *scores, const uint8_t *m
     st = check_device(nullptr);
     if (st != OTIF_OK) return st;
     return launch_select(scores, mask_in, threshold, n, gh, gw, g, sizes, k, mask_out, windows, capacity, frame_count,
-                         frame_offset, total, workspace, ws_bytes, stream, nullptr, 0, nullptr, 0);
+                         frame_offset, total, workspace, ws_bytes, stream, nullptr, 0,
+                         reinterpret_cast<unsigned long long *>(est_sum));
 }

@@ -723,14 +723,13 @@ __global__ void adam_kernel(float *__restrict__ w, float *__restrict__ m, float 
     }
 }
 
-// 1 = tcgen05 3xTF32 (default), 0 = SIMT fp32 (OTIF_TRAIN_SIMT=1, A/B runs)
+// 1 = tcgen05 3xTF32 (default), 0 = SIMT fp32 (A/B builds: nvcc -DOTIF_TRAIN_SIMT)
 static int train_tc() {
-    static int v = -1;
-    if (v < 0) {
-        const char *e = getenv("OTIF_TRAIN_SIMT");
-        v = (e && e[0] == '1') ? 0 : 1;
-    }
-    return v;
+#ifdef OTIF_TRAIN_SIMT
+    return 0;
+#else
+    return 1;
+#endif
 }
 
 template <class Op>

@@ -18,7 +18,7 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum, size_t smem_cap = 0);
+                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum);
 otif_status validate_select(const float *scores, const uint8_t *mask_in, int32_t n, int32_t gh, int32_t gw,
                             const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, int32_t capacity);
 size_t select_workspace_bytes(int32_t n, int32_t gh, int32_t gw);

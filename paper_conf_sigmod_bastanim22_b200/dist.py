@@ -3,6 +3,9 @@
 one all_gather of per-rank int64 counters at the end."""
 from __future__ import annotations
 
+import hashlib
+from typing import Callable
+
 import torch
 import torch.distributed as dist
 
@@ -34,8 +37,12 @@ def combine(gathered: torch.Tensor) -> dict:
     """Totals over ranks; the window hash is a sum of 64-bit mixes, so it combines by
     wrapping addition and is independent of how clips were sharded."""
     tot = gathered.sum(0).tolist()
-    return {"frames": tot[0], "positive_cells": tot[1], "windows": tot[2], "window_pixels": tot[3],
-            "window_hash": int(tot[4]) & ((1 << 64) - 1), "per_size": tot[5:]}
+    out = {"frames": tot[0], "positive_cells": tot[1], "windows": tot[2], "window_pixels": tot[3],
+           "window_hash": int(tot[4]) & ((1 << 64) - 1), "per_size": tot[5:13]}
+    if len(tot) >= 15:   # pipeline counters: windows dropped for batch_cap, pixels packed
+        out["dropped_windows"] = tot[13]
+        out["packed_pixels"] = tot[14]
+    return out
 
 
 def max_over_ranks(value: float, device="cpu") -> float:
@@ -44,3 +51,42 @@ def max_over_ranks(value: float, device="cpu") -> float:
     if dist.is_available() and dist.is_initialized():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+def run_corpus(clips: range, run_clip: Callable[[int], torch.Tensor]) -> torch.Tensor:
+    """The shard loop: run_clip(k) processes clip k and returns its int64 counters [C]
+    (device or host); -> [len(clips), C] in clip order."""
+    rows = [run_clip(k) for k in clips]
+    if not rows:
+        return torch.zeros((0, 0), dtype=torch.int64)
+    return torch.stack(rows)
+
+
+def gather_clip_counters(per_clip: torch.Tensor, n_clips: int, width: int, group=None) -> torch.Tensor:
+    """Per-clip counters of every rank -> [n_clips, width] on every rank, in clip order.
+    Ranks hold contiguous clip ranges (shard_clips), so the gathered blocks concatenate
+    in rank order; shards are padded to ceil(n_clips / world) rows for one all_gather."""
+    dev = per_clip.device if per_clip.numel() else torch.device("cpu")
+    if not dist.is_available() or not dist.is_initialized():
+        return per_clip.reshape(-1, width).clone()
+    world = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    mx = -(-n_clips // world)
+    mine = torch.zeros((mx, width), dtype=torch.int64, device=dev)
+    got = len(shard_clips(n_clips, world, rank))
+    if got:
+        mine[:got] = per_clip.reshape(got, width)
+    flat = gather_counters(mine.reshape(-1), group)            # [world, mx * width]
+    parts = [flat[r].reshape(mx, width)[:len(shard_clips(n_clips, world, r))] for r in range(world)]
+    return torch.cat(parts)
+
+
+def corpus_digest(clip_counters: torch.Tensor) -> dict:
+    """Totals over the corpus plus a digest of the ordered per-clip window hashes: both are
+    independent of how the clips were sharded (the check of SURVEY §8(e))."""
+    c = clip_counters.cpu()
+    tot = combine(c) if c.numel() else {}
+    hashes = [int(h) & ((1 << 64) - 1) for h in c[:, 4].tolist()] if c.numel() else []
+    tot["clips"] = len(hashes)
+    tot["per_clip_hash_sha256"] = hashlib.sha256(b"".join(h.to_bytes(8, "little") for h in hashes)).hexdigest()
+    return tot

@@ -74,8 +74,7 @@ def proxy_sweep(frames: torch.Tensor, boxes: torch.Tensor, workloads: Sequence, 
     n = frames.shape[0]
     nb = boxes.shape[0]
     for wl in workloads:
-        W = list(sizes) if sizes is not None else [tuple(s) + (s[0] * s[1],) for s in wl.sizes]
-        cost = {i: (s[2] if len(s) > 2 else s[0] * s[1]) for i, s in enumerate(W)}
+        W = list(sizes) if sizes is not None else list(wl.sizes)
         px = api.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, weights)
         img = api.otif_resize(frames, wl.proxy_h, wl.proxy_w)
         px.score(img)  # warm-up (workspace initialisation)
@@ -92,10 +91,7 @@ def proxy_sweep(frames: torch.Tensor, boxes: torch.Tensor, workloads: Sequence, 
         for b in thresholds[wl.name]:
             r = api.otif_select_windows(scores, None, b, wl.src_w, wl.src_h, wl.cell, W, connectivity=connectivity)
             total = int(r["total"].item())
-            win = r["windows"][:total]
-            sidx = win[:, 5].long()
-            costs = torch.tensor([cost[i] for i in range(len(W))], dtype=torch.int64, device=frames.device)
-            est = int(costs[sidx].sum().item()) if total else 0
+            est = int(r["est_sum"].item())          # Σ_t est(R_t), summed by the grouping kernel
             cov = window_recall(boxes, r["windows"], r["offsets"], r["counts"])
             rows.append({"setting": wl.name, "proxy_w": wl.proxy_w, "proxy_h": wl.proxy_h, "cell": wl.cell,
                          "threshold": b, "t_proxy_ms": t_proxy_ms, "est_detector_cost": est, "windows": total,

@@ -44,46 +44,56 @@ def evaluate(wl, w, frames, boxes, threshold=0.5):
             "window_area_fraction": area}
 
 
+def train_weights(wl, steps=300, batch=32, lr=1e-3, n_train=1024, clip=0):
+    """Train one proxy on clip `clip` of workload wl (frames with at least one detection,
+    P:L139; labels P:L139; BCE + Adam, readings R26/R27) from the random init.
+    -> (trained fp32 weight blob, info dict with the loss curve and ms per step)."""
+    rng = np.random.default_rng(wl.seed + 7919 * clip)
+    sc = video.make_scene(wl, clip=clip)
+    cand = [t for t in range(n_train) if len(sc.gt_boxes(t)) > 0]
+    frames = video.frames(wl, n_train, device="cuda", clip=clip)
+    img_all = otif.otif_resize(frames, wl.proxy_h, wl.proxy_w)
+    del frames
+    gh, gw = -(-wl.src_h // wl.cell), -(-wl.src_w // wl.cell)
+    lab_all = train.otif_cell_labels(torch.from_numpy(boxes_for(wl, range(n_train), clip)).cuda(), n_train,
+                                     (gh, gw), wl.src_w, wl.src_h, wl.cell)
+    cand_t = torch.tensor(cand, device="cuda")
+    w0 = weights.proxy_weights()
+    tr = train.Trainer(wl.proxy_h, wl.proxy_w, wl.n_strided, w0, max_batch=batch)
+    order = [cand_t[torch.from_numpy(rng.choice(len(cand), batch, replace=False)).cuda()] for _ in range(steps)]
+    losses = []
+    tr.step(img_all[order[0]], lab_all[order[0]], lr)      # warm-up (not timed)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for s in range(1, steps):
+        idx = order[s]
+        loss = tr.step(img_all[idx], lab_all[idx], lr)
+        if s % 25 == 0 or s == steps - 1:
+            losses.append((s, loss.clone()))
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / max(steps - 1, 1)
+    w = tr.weights()
+    del tr, img_all, lab_all
+    torch.cuda.empty_cache()
+    info = {"setting": wl.name, "proxy": f"{wl.proxy_w}x{wl.proxy_h}", "cell": wl.cell, "batch": batch,
+            "steps": steps, "train_clip": clip, "ms_per_step": ms, "train_frames_per_s": batch / (ms / 1e3),
+            "loss": [(s, float(l.item())) for s, l in losses]}
+    return w, info
+
+
 def run(settings, steps, batch, lr=1e-3, n_train=1024, n_eval=128):
     out = []
     for wl in settings:
-        # training frames: sampled frames with at least one detection, clip 0
-        rng = np.random.default_rng(wl.seed)
-        sc = video.make_scene(wl, clip=0)
-        cand = [t for t in range(n_train) if len(sc.gt_boxes(t)) > 0]
-        frames = video.frames(wl, n_train, device="cuda", clip=0)
-        img_all = otif.otif_resize(frames, wl.proxy_h, wl.proxy_w)
-        del frames
-        gh, gw = -(-wl.src_h // wl.cell), -(-wl.src_w // wl.cell)
-        lab_all = train.otif_cell_labels(torch.from_numpy(boxes_for(wl, range(n_train), 0)).cuda(), n_train,
-                                         (gh, gw), wl.src_w, wl.src_h, wl.cell)
-        cand_t = torch.tensor(cand, device="cuda")
-        w0 = weights.proxy_weights()
-        tr = train.Trainer(wl.proxy_h, wl.proxy_w, wl.n_strided, w0, max_batch=batch)
-        order = [cand_t[torch.from_numpy(rng.choice(len(cand), batch, replace=False)).cuda()] for _ in range(steps)]
-        losses = []
-        tr.step(img_all[order[0]], lab_all[order[0]], lr)      # warm-up (not timed)
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record()
-        for s in range(1, steps):
-            idx = order[s]
-            loss = tr.step(img_all[idx], lab_all[idx], lr)
-            if s % 25 == 0 or s == steps - 1:
-                losses.append((s, loss.clone()))
-        e1.record()
-        torch.cuda.synchronize()
-        ms = e0.elapsed_time(e1) / max(steps - 1, 1)
+        w, info = train_weights(wl, steps, batch, lr, n_train, clip=0)
         # held-out evaluation: clip 1
         ev_frames = video.frames(wl, n_eval, device="cuda", clip=1)
         ev_boxes = torch.from_numpy(boxes_for(wl, range(n_eval), 1)).cuda()
-        trained = evaluate(wl, tr.weights(), ev_frames, ev_boxes)
-        rand = evaluate(wl, w0, ev_frames, ev_boxes)
-        out.append({"setting": wl.name, "proxy": f"{wl.proxy_w}x{wl.proxy_h}", "cell": wl.cell, "batch": batch,
-                    "steps": steps, "ms_per_step": ms, "train_frames_per_s": batch / (ms / 1e3),
-                    "loss": [(s, float(l.item())) for s, l in losses],
-                    "held_out_threshold_0.5": {"trained": trained, "random_init": rand}})
-        del tr, img_all, lab_all
+        trained = evaluate(wl, w, ev_frames, ev_boxes)
+        rand = evaluate(wl, weights.proxy_weights(), ev_frames, ev_boxes)
+        info["held_out_threshold_0.5"] = {"trained": trained, "random_init": rand}
+        out.append(info)
         torch.cuda.empty_cache()
     return out
 

@@ -59,10 +59,10 @@ def test_status_strings_and_validation_without_gpu(libotif):
     g = _lib.GridDesc(416, 256, 32, 4)
     sizes = (_lib.WSize * 1)(_lib.WSize(64, 64, 4096))
     rc = L.otif_select_windows(None, ctypes.c_void_p(1), ctypes.c_float(0.5), 1, 8, 13, ctypes.byref(g), sizes, 1,
-                               None, None, 0, None, None, None, None, 0, None)
+                               None, None, 0, None, None, None, None, 0, None, None)
     assert rc == _lib.EINVAL and b"full frame" in L.otif_last_error()
     rc = L.otif_select_windows(None, ctypes.c_void_p(1), ctypes.c_float(0.5), 1, 8, 12, ctypes.byref(g), sizes, 1,
-                               None, None, 0, None, None, None, None, 0, None)
+                               None, None, 0, None, None, None, None, 0, None, None)
     assert rc == _lib.EINVAL and b"grid" in L.otif_last_error()
     d = _lib.ProxyDesc()
     d.in_h, d.in_w, d.n_strided, d.dec = 64, 104, 6, 128

@@ -24,9 +24,10 @@ def test_shard_clips_partition():
 
 
 def _per_clip_counters(clip: int) -> torch.Tensor:
-    # deterministic fake per-clip counters (frames, pos, windows, pixels, hash, s0, s1, s2)
+    # deterministic fake per-clip pipeline counters (otif.h layout, 15 int64: frames, pos,
+    # windows, pixels, hash, 8 per-size, dropped, packed pixels) standing in for run_clip
     g = torch.Generator().manual_seed(clip)
-    v = torch.randint(0, 1000, (8,), generator=g, dtype=torch.int64)
+    v = torch.randint(0, 1000, (15,), generator=g, dtype=torch.int64)
     v[0] = 450
     v[4] = (clip * 0x9E3779B97F4A7C15) & 0x7FFFFFFFFFFFFFFF
     return v
@@ -36,12 +37,14 @@ def _worker(rank, world, port, n_clips, out):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    ctr = torch.zeros(8, dtype=torch.int64)
-    for c in odist.shard_clips(n_clips, world, rank):
-        ctr += _per_clip_counters(c)
+    # the real shard loop (bench.py C5) with a CPU stand-in for the per-clip pipeline call
+    clips = odist.shard_clips(n_clips, world, rank)
+    per_clip = odist.run_corpus(clips, _per_clip_counters)
+    ctr = per_clip.sum(0) if len(clips) else torch.zeros(15, dtype=torch.int64)
     g = odist.gather_counters(ctr)
+    allc = odist.gather_clip_counters(per_clip, n_clips, 15)
     t = odist.max_over_ranks(float(rank + 1))
-    out[rank] = (g.clone(), t, odist.combine(g))
+    out[rank] = (g.clone(), t, odist.combine(g), allc.clone(), odist.corpus_digest(allc))
     dist.barrier()
     dist.destroy_process_group()
 
@@ -54,20 +57,21 @@ def _free_port():
     return p
 
 
-@pytest.mark.parametrize("world", [2])
-def test_gloo_gather_and_sharding_invariance(world):
-    n_clips = 10
+@pytest.mark.parametrize("world,n_clips", [(2, 10), (3, 10), (2, 1)])
+def test_gloo_gather_and_sharding_invariance(world, n_clips):
     mgr = mp.Manager()
     out = mgr.dict()
     mp.spawn(_worker, args=(world, _free_port(), n_clips, out), nprocs=world, join=True)
-    ref = sum(_per_clip_counters(c) for c in range(n_clips))
+    ref_rows = torch.stack([_per_clip_counters(c) for c in range(n_clips)])
+    ref = ref_rows.sum(0)
+    single = odist.corpus_digest(odist.run_corpus(range(n_clips), _per_clip_counters))
     for r in range(world):
-        g, t, tot = out[r]
-        assert g.shape == (world, 8)
+        g, t, tot, allc, digest = out[r]
+        assert g.shape == (world, 15)
         assert torch.equal(g.sum(0), ref)
         assert t == float(world)              # max over ranks
         assert tot["frames"] == 450 * n_clips
         assert tot["window_hash"] == int(ref[4]) & ((1 << 64) - 1)
-    # same totals from a single process
-    single = odist.combine(ref.view(1, -1))
-    assert single == out[0][2]
+        assert torch.equal(allc, ref_rows)    # per-clip counters in clip order, every rank
+        assert digest == single               # per-clip hashes + totals independent of the sharding
+    assert odist.combine(ref.view(1, -1)) == out[0][2]

@@ -88,51 +88,6 @@ def test_proxy_parity(wl, n, blob):
         assert np.array_equal((got > np.float32(b))[far], (ref_bf16 > b)[far])
 
 
-# E1 fused into E2 (e12_umma_kernel: E1 activations computed on chip from a staged
-# image slab) vs the separate E1 + E2 kernels (OTIF_E12=0), on shapes that exercise odd
-# E1/E2 sizes (invalid parity-plane positions), rows that are not 16-B aligned (LSU slab
-# copies: 3*w % 16 != 0) and several strides.
-E12_CASES = [(67, 123, 3, 3), (64, 104, 3, 5), (45, 90, 2, 3), (33, 50, 5, 2), (135, 240, 3, 3), (90, 160, 4, 2)]
-
-
-@pytest.mark.parametrize("h,w,ns,n", E12_CASES, ids=[f"{c[0]}x{c[1]}s{c[2]}" for c in E12_CASES])
-def test_proxy_e1_fused_vs_separate(h, w, ns, n, blob, monkeypatch):
-    rng = np.random.default_rng(h * 1000 + w)
-    img = rng.integers(0, 256, (n, h, w, 3), dtype=np.uint8)
-    img[0, : h // 3] = 128                      # flat region (x = 0 after normalisation)
-    img[-1, :, : w // 4] = rng.integers(0, 2, (h, w // 4, 3)) * 255
-    fused = otif.Proxy(h, w, ns, blob)
-    monkeypatch.setenv("OTIF_E12", "0")
-    sep = otif.Proxy(h, w, ns, blob)
-    monkeypatch.delenv("OTIF_E12")
-    assert fused.workspace_bytes(n) < sep.workspace_bytes(n), "fused path not planned"
-    t = torch.from_numpy(img).cuda()
-    a = fused.score(t).cpu().numpy().astype(np.float64)
-    b = sep.score(t).cpu().numpy().astype(np.float64)
-    ref_none = oracle_scores(img, type("W", (), {"n_strided": ns})(), blob, oracle.QUANT_NONE)
-    assert np.abs(a - ref_none).max() <= 2e-2
-    assert np.abs(a - b).max() <= 1e-2
-    # the two paths differ only in the fp32 accumulation order of E1 (the fused path adds
-    # E1's bias inside the MMA), so bf16 roundings of E1 rarely differ
-    assert np.median(np.abs(a - b)) <= 1e-4
-
-
-@pytest.mark.parametrize("h,w,ns,n", [(135, 240, 3, 3), (67, 123, 3, 3), (45, 90, 2, 3)])
-def test_proxy_e12_ts_mode_matches_ss(h, w, ns, n, blob, monkeypatch):
-    """OTIF_E12_TS=1 (E1's im2col rows in TMEM, A-from-TMEM MMA) computes the same E1
-    sums (exact fp16 products, fp32 accumulation in the same K order) as the default
-    shared-memory operand path, so the scores are identical."""
-    rng = np.random.default_rng(h * 7 + w)
-    img = torch.from_numpy(rng.integers(0, 256, (n, h, w, 3), dtype=np.uint8)).cuda()
-    ss = otif.Proxy(h, w, ns, blob)
-    monkeypatch.setenv("OTIF_E12_TS", "1")
-    ts = otif.Proxy(h, w, ns, blob)
-    monkeypatch.delenv("OTIF_E12_TS")
-    a = ss.score(img).cpu().numpy()
-    b = ts.score(img).cpu().numpy()
-    assert np.array_equal(a, b)
-
-
 def test_proxy_repeat_calls_reuse_workspace(blob):
     wl = configs.C1
     img = torch.from_numpy(oracle.resize(_frames(wl, 8).numpy(), wl.proxy_h, wl.proxy_w)).cuda()
@@ -362,33 +317,6 @@ def test_pipeline_host_vs_stages(wl, blob):
     assert np.array_equal(win, r["windows"][:t].cpu().numpy())
     ref = windows_np(r["windows"], t)
     assert list(sc) == [int((ref["size_idx"] == s).sum()) for s in range(len(wl.sizes))]
-
-
-@pytest.mark.parametrize("green", [0, 32], ids=["coresident", "green32"])
-@pytest.mark.parametrize("wl,chunks", [(configs.C2, 3), (configs.C1, 4), (configs.C3, 2)], ids=["C2", "C1", "C3"])
-def test_pipeline_overlap_matches_serial(wl, chunks, green, blob, monkeypatch):
-    """Overlap mode (resize / select / pack of neighbouring chunks on a second stream while
-    the proxy scores a chunk) returns exactly the serial schedule's windows, per-frame counts,
-    per-size counts and device counters (incl. the order-independent window hash), over
-    several device batches with a ragged last chunk."""
-    b = threshold(wl.name, 0.7)
-    n = 75
-    src = video.frames(wl, n).contiguous()
-    ser = otif.Pipeline(wl, blob, b, max_batch=40)
-    if green:   # SM partition through two green contexts (read at create)
-        monkeypatch.setenv("OTIF_OVL_GREEN", str(green))
-    ovl = otif.Pipeline(wl, blob, b, max_batch=40, overlap_chunks=chunks)
-    monkeypatch.delenv("OTIF_OVL_GREEN", raising=False)
-    w0, c0, s0, t0 = ser.run_host(src)
-    w1, c1, s1, t1 = ovl.run_host(src)
-    assert t0 == t1 and np.array_equal(c0, c1) and list(s0) == list(s1)
-    assert np.array_equal(w0, w1)
-    src_d = src.cuda()
-    for pipe in (ser, ovl):
-        pipe.reset_counters()
-        pipe.run_device(src_d)
-    torch.cuda.synchronize()
-    assert torch.equal(ser.counters().cpu(), ovl.counters().cpu())
 
 
 def test_edge_cases():

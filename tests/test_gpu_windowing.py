@@ -180,7 +180,7 @@ def test_pack_subframe_hand_built():
     for f in range(4):
         rows += [(f, 0, 0, 128, 128, 0), (f, 16 * (f + 1), 200, 128, 128, 0), (f, 5 + f, 7, 128, 128, 0),
                  (f, 960 - 128, 540 - 128, 128, 128, 0), (f, 960 - 256, 100 + f, 256, 256, 1),
-                 (f, 333, 284, 256, 256, 1), (f, 848, 476, 112, 64, 3), (f, 17, 480, 112, 64, 3),
+                 (f, 333, 284, 256, 256, 1), (f, 848, 476, 112, 64, 3), (f, 17, 476, 112, 64, 3),
                  (f, 860, 480, 100, 60, 4), (f, 3, 1, 100, 60, 4)]
     rows.append((2, 0, 0, 960, 540, 2))
     win = _win_array(rows)
