@@ -9,13 +9,15 @@
 //       bf16-rounded D1 activations read back from TMEM).
 //
 // Activation layout in HBM ("padded linear, chunk-planar").  A stride-1 3x3 conv over
-// an H x W map reads, for output pixel q, the input pixels q + kh*(W+2) + kw of the
-// zero-padded map flattened row-major with pitch W+2 — a pure linear shift per tap.
-// So every GEMM layer's input is stored zero-padded and flattened, frames stacked
-// (each frame owns H+1 rows of pitch W+2; the bottom pad of frame f is the top pad
-// of frame f+1), and channel-chunk planar: [plane][C/8][pixels][8 bf16].  Then the
+// an H x W map reads, for output pixel q, the input pixels q + kh*(W+1) + kw of the
+// zero-padded map flattened row-major with pitch W+1 — a pure linear shift per tap.
+// ONE pad column per row suffices: data sits in columns 1..W, and the right neighbour
+// of column W is column 0 (the pad) of the next row.  So every GEMM layer's input is
+// stored zero-padded and flattened, frames stacked (each frame owns H+1 rows of pitch
+// W+1; the bottom pad of frame f is the top pad of frame f+1), and channel-chunk
+// planar: [plane][C/8][pixels][8 bf16].  Then the
 // A operand of one M tile (128 consecutive output positions) for ALL 9 taps is one
-// contiguous halo of 128 + 2(W+2) + 2 pixels per 8-channel chunk, loaded once with
+// contiguous halo of 128 + 2(W+1) + 2 pixels per 8-channel chunk, loaded once with
 // 1-D bulk async copies and reused by 9 MMAs through shifted smem descriptors (the
 // no-swizzle K-major layout puts consecutive rows 16 B apart, so a shift of s pixels
 // is a +16*s start address).  Stride-2 layers read a parity-split input (4 planes:
@@ -990,7 +992,7 @@ static void build_layer(GemmLayer &g, int cin, int cout, int stride, int in_h, i
     for (int i = 0; i < 4; i++) g.group_ntaps[i] = 0;
     if (stride == 1) {
         g.kind = 1;
-        g.pitch = in_w + 2;
+        g.pitch = in_w + 1;     // one shared pad column per row (see the layout note)
         g.fstride_unit = (int64_t)(in_h + 1) * g.pitch;
         g.max_shift = 2 * g.pitch + 2;
         g.ngroups = 1;

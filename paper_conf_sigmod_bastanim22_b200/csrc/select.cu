@@ -22,6 +22,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <vector>
 
 #include "common.cuh"
 
@@ -31,6 +32,15 @@ constexpr int kSelWarpsMax = 16;
 constexpr int kMatMax = 128;  // fit-matrix capacity (components per frame); larger n -> rescan path
 constexpr int kSmallClusters = 64;  // components per frame in the first (high-occupancy) pass
 constexpr int kMaxSizes = 8;
+
+// One window-size set W' (sorted by (cost, w*h, w, h)) for the multi-candidate launch
+// of NEXT-1 (blockIdx.y selects the table).
+struct WTable {
+    int k, full;
+    int sw[8], sh[8], orig[8];
+    long long cost[8];
+};
+static_assert(sizeof(WTable) <= 192, "tuning.cu sizes the W' table scratch at 192 B per entry");
 
 struct SelectParams {
     const float *scores;
@@ -59,6 +69,9 @@ struct SelectParams {
     int *defer_list;
     int *defer_count;
     int from_list;
+    // NEXT-1 multi-candidate mode (select_kernel<true>): W' per blockIdx.y, est_sum[blockIdx.y],
+    // no window / count outputs
+    const WTable *wtab;
 };
 
 struct Rect16 { short x0, y0, x1, y1; };  // cell units, half-open
@@ -384,8 +397,24 @@ __device__ bool greedy_rescan(const SelectParams &p, Frame &F, int n, int lane) 
 
 }
 
-__global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_constant__ SelectParams p) {
+// (MULTI returns after the est sum: the emission code below is unreachable there by design)
+#pragma nv_diag_suppress 128
+template <bool MULTI>
+__global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_constant__ SelectParams pin) {
     extern __shared__ __align__(16) uint8_t smem[];
+    // MULTI (NEXT-1): this CTA row groups its frames with the W' of candidate set blockIdx.y
+    SelectParams loc;
+    if constexpr (MULTI) {
+        loc = pin;
+        const WTable &t = pin.wtab[blockIdx.y];
+        loc.k = t.k;
+        loc.full = t.full;
+        for (int s = 0; s < kMaxSizes; s++) {
+            loc.sw[s] = t.sw[s]; loc.sh[s] = t.sh[s]; loc.orig[s] = t.orig[s]; loc.cost[s] = t.cost[s];
+        }
+        loc.est_sum = pin.est_sum + blockIdx.y;
+    }
+    const SelectParams &p = MULTI ? loc : pin;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     int f = blockIdx.x * (blockDim.x >> 5) + wid;
     if (p.from_list) {
@@ -474,7 +503,7 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
         return;
     }
     if (n == 0) {
-        if (lane == 0) {
+        if (lane == 0 && !MULTI) {
             p.counts[f] = 0;
             if (p.ctr) atomicAdd(&p.ctr[0], 1ull);
         }
@@ -540,6 +569,10 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
     }
     unsigned long long hsh = 0, pix = 0;
     if (full_hit || est > p.cost[p.full]) {
+        if (MULTI) {
+            if (lane == 0) atomicAdd(p.est_sum, (unsigned long long)p.cost[p.full]);
+            return;
+        }
         if (lane == 0) {
             otif_window w;
             w.frame = f; w.x = 0; w.y = 0; w.w = p.fw; w.h = p.fh; w.size_idx = p.orig[p.full];
@@ -557,6 +590,10 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
                 atomicAdd(&p.ctr[5 + w.size_idx], 1ull);
             }
         }
+        return;
+    }
+    if constexpr (MULTI) {
+        if (lane == 0) atomicAdd(p.est_sum, (unsigned long long)est);
         return;
     }
     // rank each alive cluster's placed window by (y, x); placements recomputed per lane
@@ -602,6 +639,8 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
         }
     }
 }
+
+#pragma nv_diag_default 128
 
 // K6: scan of per-frame counts + compaction into (frame, y, x) order
 __global__ void __launch_bounds__(1024) compact_kernel(const otif_window *__restrict__ tmp, int cap_f,
@@ -664,6 +703,28 @@ static int sel_frame_bytes(int gh, int gw, int ccap, int nmat, int *gmat_offset)
     return body + (int)round_up((int64_t)nmat * nmat, 16);
 }
 
+// W' = W sorted by (cost, w*h, w, h); full = first entry holding the whole frame
+static void sort_sizes(const otif_wsize *sizes, int k, int fw, int fh, WTable &t) {
+    int order[kMaxSizes];
+    for (int i = 0; i < k; i++) order[i] = i;
+    std::stable_sort(order, order + k, [&](int a, int b) {
+        const otif_wsize &x = sizes[a], &y = sizes[b];
+        if (x.cost != y.cost) return x.cost < y.cost;
+        long long ax = (long long)x.w * x.h, ay = (long long)y.w * y.h;
+        if (ax != ay) return ax < ay;
+        if (x.w != y.w) return x.w < y.w;
+        return x.h < y.h;
+    });
+    memset(&t, 0, sizeof(t));
+    t.k = k;
+    t.full = -1;
+    for (int s = 0; s < k; s++) {
+        const otif_wsize &z = sizes[order[s]];
+        t.sw[s] = z.w; t.sh[s] = z.h; t.cost[s] = z.cost; t.orig[s] = order[s];
+        if (t.full < 0 && z.w >= fw && z.h >= fh) t.full = s;
+    }
+}
+
 // internal entry: counters and global frame base for the pipeline (NULL / 0 from the ABI)
 otif_status launch_select(const float *scores, const uint8_t *mask_in, float threshold, int32_t n, int32_t gh,
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
@@ -676,21 +737,11 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
     p.n = n; p.gh = gh; p.gw = gw; p.cell = g->cell; p.fw = g->frame_w; p.fh = g->frame_h;
     p.conn = g->connectivity; p.k = k;
     // W' = W sorted by (cost, w*h, w, h)
-    int order[kMaxSizes];
-    for (int i = 0; i < k; i++) order[i] = i;
-    std::stable_sort(order, order + k, [&](int a, int b) {
-        const otif_wsize &x = sizes[a], &y = sizes[b];
-        if (x.cost != y.cost) return x.cost < y.cost;
-        long long ax = (long long)x.w * x.h, ay = (long long)y.w * y.h;
-        if (ax != ay) return ax < ay;
-        if (x.w != y.w) return x.w < y.w;
-        return x.h < y.h;
-    });
-    p.full = -1;
-    for (int s = 0; s < k; s++) {
-        const otif_wsize &z = sizes[order[s]];
-        p.sw[s] = z.w; p.sh[s] = z.h; p.cost[s] = z.cost; p.orig[s] = order[s];
-        if (p.full < 0 && z.w >= g->frame_w && z.h >= g->frame_h) p.full = s;
+    {
+        WTable t;
+        sort_sizes(sizes, k, g->frame_w, g->frame_h, t);
+        p.full = t.full;
+        for (int s = 0; s < k; s++) { p.sw[s] = t.sw[s]; p.sh[s] = t.sh[s]; p.cost[s] = t.cost[s]; p.orig[s] = t.orig[s]; }
     }
     p.mask_out = mask_out;
     p.cap_f = sel_cap(gh, gw);
@@ -727,12 +778,54 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
         }
         if (warps > n) warps = n;
         const size_t smem = (size_t)warps * p.frame_bytes;
-        OTIF_CUDA(cudaFuncSetAttribute(select_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        select_kernel<<<(unsigned)cdiv(n, warps), warps * 32, smem, stream>>>(p);
+        OTIF_CUDA(cudaFuncSetAttribute(select_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+        select_kernel<false><<<(unsigned)cdiv(n, warps), warps * 32, smem, stream>>>(p);
         OTIF_LAUNCH_CHECK();
     }
     compact_kernel<<<(unsigned)cdiv(n, 1024), 1024, 0, stream>>>(p.tmp, p.cap_f, p.counts, n, windows, capacity,
                                                                  frame_count, frame_offset, total);
+    OTIF_LAUNCH_CHECK();
+    return OTIF_OK;
+}
+
+// NEXT-1: Σ_t est(R(I_t; W_c)) for m window-size sets W_c (k_c <= 8 sizes each, host) over
+// n masks in ONE launch (grid.y = m; full-size slices, no deferred pass) -> est_sums[m]
+// (device, zeroed here).  wtab_dev: device scratch of m WTable entries.
+otif_status launch_select_multi(const uint8_t *masks, int32_t n, int32_t gh, int32_t gw, const otif_grid_desc *g,
+                                const otif_wsize *const *sets, const int32_t *set_k, int32_t m, void *wtab_dev,
+                                unsigned long long *est_sums, cudaStream_t stream) {
+    if (m <= 0) return OTIF_OK;
+    OTIF_CUDA(cudaMemsetAsync(est_sums, 0, (size_t)m * 8, stream));
+    if (n <= 0) return OTIF_OK;
+    std::vector<WTable> tabs(m);
+    long long max_cost = 0;
+    bool nonneg = true;
+    for (int c = 0; c < m; c++) {
+        sort_sizes(sets[c], set_k[c], g->frame_w, g->frame_h, tabs[c]);
+        for (int s = 0; s < set_k[c]; s++) {
+            max_cost = sets[c][s].cost > max_cost ? sets[c][s].cost : max_cost;
+            nonneg = nonneg && sets[c][s].cost >= 0;
+        }
+    }
+    OTIF_CUDA(cudaMemcpyAsync(wtab_dev, tabs.data(), (size_t)m * sizeof(WTable), cudaMemcpyHostToDevice, stream));
+    SelectParams p;
+    memset(&p, 0, sizeof(p));
+    p.mask_in = masks;
+    p.n = n; p.gh = gh; p.gw = gw; p.cell = g->cell; p.fw = g->frame_w; p.fh = g->frame_h;
+    p.conn = g->connectivity;
+    p.cap_f = sel_cap(gh, gw);
+    p.ccap = p.cap_f;
+    p.nmat = (max_cost < (1ll << 30) && nonneg) ? (int)round_up(p.ccap < kMatMax ? p.ccap : kMatMax, 8) : 0;
+    p.frame_bytes = sel_frame_bytes(gh, gw, p.ccap, p.nmat, &p.gmat_offset);
+    p.wtab = reinterpret_cast<const WTable *>(wtab_dev);
+    p.est_sum = est_sums;
+    int warps = (int)((size_t)200 * 1024 / p.frame_bytes);
+    warps = warps < 1 ? 1 : (warps > kSelWarpsMax ? kSelWarpsMax : warps);
+    if (warps > n) warps = n;
+    const size_t smem = (size_t)warps * p.frame_bytes;
+    OTIF_REQUIRE(smem <= 227 * 1024, "otif_choose_window_sizes: grid of %d cells too large", gh * gw);
+    OTIF_CUDA(cudaFuncSetAttribute(select_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    select_kernel<true><<<dim3((unsigned)cdiv(n, warps), (unsigned)m), warps * 32, smem, stream>>>(p);
     OTIF_LAUNCH_CHECK();
     return OTIF_OK;
 }

@@ -1,9 +1,10 @@
 // tuning.cu — §8(f) NEXT rows built on the stage-4 kernels.
 //
 // NEXT-1 otif_choose_window_sizes: greedy choice of the fixed window-size
-//   set W over perfect-proxy masks.  Every candidate of a round is scored by one launch of
-//   the select kernel over all frames accumulating Σ_t est(R_t) on the device; one
-//   device->host copy per round picks the greatest decrease.
+//   set W over perfect-proxy masks.  Each round scores EVERY remaining candidate in one
+//   launch of the grouping kernel (grid.y = candidate: warp per (frame, candidate),
+//   Σ_t est(R_t) accumulated per candidate on the device); one device->host copy per
+//   round picks the greatest decrease.
 // NEXT-2 otif_window_recall: the recall numerator of the proxy-tuning sweep —
 //   one thread per detection box tests containment in the windows of its frame.
 #include <string.h>
@@ -14,14 +15,12 @@
 
 namespace otif {
 
-otif_status launch_select(const float *scores, const uint8_t *mask_in, float threshold, int32_t n, int32_t gh,
-                          int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
-                          otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
-                          int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum);
 otif_status validate_select(const float *scores, const uint8_t *mask_in, int32_t n, int32_t gh, int32_t gw,
                             const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, int32_t capacity);
-size_t select_workspace_bytes(int32_t n, int32_t gh, int32_t gw);
+otif_status launch_select_multi(const uint8_t *masks, int32_t n, int32_t gh, int32_t gw, const otif_grid_desc *g,
+                                const otif_wsize *const *sets, const int32_t *set_k, int32_t m, void *wtab_dev,
+                                unsigned long long *est_sums, cudaStream_t stream);
+constexpr size_t kWTableBytes = 192;   // >= sizeof(WTable) (static_assert in select.cu)
 
 __global__ void covered_kernel(const int32_t *__restrict__ boxes, int64_t nb, const otif_window *__restrict__ win,
                                const int32_t *__restrict__ frame_offset, const int32_t *__restrict__ frame_count,
@@ -47,9 +46,8 @@ using namespace otif;
 
 extern "C" size_t otif_choose_workspace_bytes(int32_t n, int32_t gh, int32_t gw, int32_t m) {
     if (n < 0 || gh <= 0 || gw <= 0 || m < 0) return 0;
-    const size_t cap = (size_t)n * ((gh * gw + 1) / 2 > 1 ? (gh * gw + 1) / 2 : 1);
-    return select_workspace_bytes(n, gh, gw) + round_up((int64_t)(m + 1) * 8, 256) +
-           round_up((int64_t)cap * sizeof(otif_window), 256) + 3 * round_up((int64_t)n * 4 + 4, 256);
+    // [W' tables (m + 1)][est sums (m + 1) int64]
+    return round_up((int64_t)(m + 1) * kWTableBytes, 256) + round_up((int64_t)(m + 1) * 8, 256);
 }
 
 extern "C" otif_status otif_choose_window_sizes(const uint8_t *masks, int32_t n, int32_t gh, int32_t gw,
@@ -71,48 +69,50 @@ extern "C" otif_status otif_choose_window_sizes(const uint8_t *masks, int32_t n,
                      candidates[c].h);
     st = check_device(nullptr);
     if (st != OTIF_OK) return st;
-    // workspace: [select ws][est sums (m+1) int64][windows][counts][offsets][total]
     uint8_t *ws = (uint8_t *)workspace;
-    const size_t sel_bytes = select_workspace_bytes(n, gh, gw);
-    unsigned long long *sums = (unsigned long long *)(ws + sel_bytes);
-    const size_t cap = (size_t)n * ((gh * gw + 1) / 2 > 1 ? (gh * gw + 1) / 2 : 1);
-    otif_window *win = (otif_window *)(ws + sel_bytes + round_up((int64_t)(m + 1) * 8, 256));
-    int32_t *cnt = (int32_t *)((uint8_t *)win + round_up((int64_t)cap * sizeof(otif_window), 256));
-    int32_t *off = (int32_t *)((uint8_t *)cnt + round_up((int64_t)n * 4 + 4, 256));
-    int32_t *tot = (int32_t *)((uint8_t *)off + round_up((int64_t)n * 4 + 4, 256));
+    void *wtab = ws;
+    unsigned long long *sums = (unsigned long long *)(ws + round_up((int64_t)(m + 1) * kWTableBytes, 256));
 
-    std::vector<unsigned long long> h(m + 1);
+    std::vector<unsigned long long> h(m + 1, 0);
     std::vector<char> used(m > 0 ? m : 1, 0);
+    // candidate sets of a round: W + candidate c, one row of W' tables per active candidate
+    std::vector<otif_wsize> sets_mem((size_t)(m + 1) * 8);
+    std::vector<const otif_wsize *> sets(m + 1);
+    std::vector<int32_t> set_k(m + 1);
+    std::vector<int> active;
     int nw = 1;
     // Σ est with W = {full frame}
-    OTIF_CUDA(cudaMemsetAsync(sums, 0, (m + 1) * 8, stream));
-    if (n > 0) {
-        st = launch_select(nullptr, masks, 0.0f, n, gh, gw, g, W, 1, nullptr, win, 0, cnt, off, tot, ws, sel_bytes,
-                           stream, nullptr, 0, sums + m);
-        if (st != OTIF_OK) return st;
-    }
-    OTIF_CUDA(cudaMemcpyAsync(&h[m], sums + m, 8, cudaMemcpyDeviceToHost, stream));
+    sets[0] = W;
+    set_k[0] = 1;
+    st = launch_select_multi(masks, n, gh, gw, g, sets.data(), set_k.data(), 1, wtab, sums, stream);
+    if (st != OTIF_OK) return st;
+    OTIF_CUDA(cudaMemcpyAsync(h.data(), sums, 8, cudaMemcpyDeviceToHost, stream));
     OTIF_CUDA(cudaStreamSynchronize(stream));
     chosen_idx[0] = -1;
-    est[0] = (int64_t)h[m];
+    est[0] = n > 0 ? (int64_t)h[0] : 0;
     int64_t cur = est[0];
     while (nw < k) {
-        OTIF_CUDA(cudaMemsetAsync(sums, 0, m * 8, stream));
-        for (int c = 0; c < m && n > 0; c++) {
+        active.clear();
+        for (int c = 0; c < m; c++) {
             if (used[c]) continue;
-            W[nw] = candidates[c];
-            st = launch_select(nullptr, masks, 0.0f, n, gh, gw, g, W, nw + 1, nullptr, win, 0, cnt, off, tot, ws,
-                               sel_bytes, stream, nullptr, 0, sums + c);
-            if (st != OTIF_OK) return st;
+            otif_wsize *set = &sets_mem[(size_t)active.size() * 8];
+            for (int i = 0; i < nw; i++) set[i] = W[i];
+            set[nw] = candidates[c];
+            sets[active.size()] = set;
+            set_k[active.size()] = nw + 1;
+            active.push_back(c);
         }
-        if (m > 0) OTIF_CUDA(cudaMemcpyAsync(h.data(), sums, m * 8, cudaMemcpyDeviceToHost, stream));
+        if (active.empty()) break;
+        st = launch_select_multi(masks, n, gh, gw, g, sets.data(), set_k.data(), (int)active.size(), wtab, sums,
+                                 stream);
+        if (st != OTIF_OK) return st;
+        OTIF_CUDA(cudaMemcpyAsync(h.data(), sums, active.size() * 8, cudaMemcpyDeviceToHost, stream));
         OTIF_CUDA(cudaStreamSynchronize(stream));
         int best = -1;
         int64_t best_sum = cur;
-        for (int c = 0; c < m; c++) {
-            if (used[c]) continue;
-            const int64_t s = n > 0 ? (int64_t)h[c] : 0;
-            if (s < best_sum) { best_sum = s; best = c; }  // greatest decrease; ties: earliest candidate
+        for (size_t a = 0; a < active.size(); a++) {
+            const int64_t s = n > 0 ? (int64_t)h[a] : 0;
+            if (s < best_sum) { best_sum = s; best = active[a]; }  // greatest decrease; ties: earliest candidate
         }
         if (best < 0) break;  // no candidate decreases the sum (reading R19)
         used[best] = 1;
