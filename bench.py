@@ -309,16 +309,85 @@ def caps_for(wl, sizes, n, per_frame=8):
     return out
 
 
-def choose_wstar(otif_tuning, wl, clip, n, k, dev):
-    """NEXT-1 on the GPU: W* from the perfect-proxy masks of n frames of `clip`."""
+def choose_wstar(otif_tuning, wl, clip, start, n, k, dev):
+    """NEXT-1 on the GPU: W* from the perfect-proxy masks of frames
+    [start, start + n) of `clip` (the same camera, earlier/later than the measured frames)."""
     import torch
     from synth import video
     sc = video.make_scene(wl, clip=clip)
     masks = torch.from_numpy(np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell)
-                                       for t in range(n)])).to(dev)
+                                       for t in range(start, start + n)])).to(dev)
     cands = otif_tuning.candidate_sizes(wl.src_w, wl.src_h, wl.cell)
     chosen, sums, idx = otif_tuning.choose_window_sizes(masks, wl.src_w, wl.src_h, wl.cell, cands, k=k)
     return [tuple(int(v) for v in c[:2]) for c in chosen], sums
+
+
+def windowing_scenario(otif, otif_tuning, wl, src, rank, dev, peaks, peak_src, args):
+    """The path with the windowing active: the proxy trained by NEXT-3 and the
+    window set W* chosen by NEXT-1, both from frames [n, n + 1024) of the
+    same camera (the training split, later in time than the measured frames [0, n)),
+    through the whole pipeline; and stages 3–5 on the perfect proxy."""
+    import torch
+    from scripts import train_proxy
+    from synth import video
+    n = src.shape[0]
+    t0 = time.time()
+    tw, tinfo = train_proxy.train_weights(wl, steps=args.train_steps, batch=32, clip=rank, start=n)
+    wstar = {k: choose_wstar(otif_tuning, wl, rank, n, 600, k, dev) for k in (3, 5)}
+    out = {"what": f"{wl.name}: {n} frames of one camera through the whole path with the trained proxy (B = 0.5) "
+                   f"and W*; training and W* from frames [{n}, {n + 1024}) of the same camera",
+           "objects_mean": wl.objects,
+           "train": {k: tinfo[k] for k in ("steps", "batch", "ms_per_step", "loss", "train_frames")},
+           "prep_s": None}
+    for k, (W, sums) in wstar.items():
+        out[f"W*_k{k}"] = [list(x) for x in W]
+    out["prep_s"] = time.time() - t0
+    for k, (W, _) in wstar.items():
+        caps = caps_for(wl, W, n)
+        mw = measure_pipeline(otif, wl, tw, 0.5, src, args.steps, args.warmup, sizes=W, caps=caps)
+        out[f"trained_k{k}"] = {"frames_per_s": mw["frames"] / (mw["ms_total"] / 1e3),
+                                "ms_per_step": mw["ms_total"] / args.steps, "windows": window_stats(mw, wl, W),
+                                "roofline": rooflines(wl, mw, peaks, peak_src), "batch_cap": caps}
+        mw["pipe"].close()
+        torch.cuda.empty_cache()
+    # perfect proxy (P:L153): stages 3-5 on the ground-truth cell masks of the measured frames
+    sc = video.make_scene(wl, clip=rank)
+    masks = torch.from_numpy(np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell)
+                                       for t in range(n)])).to(dev)
+    pp = {}
+    for tag, W in [("default_W", list(wl.sizes))] + [(f"W*_k{k}", W) for k, (W, _) in wstar.items()]:
+        caps = caps_for(wl, W, n)
+        r = otif.otif_select_windows(None, masks, 0.0, wl.src_w, wl.src_h, wl.cell, W)
+        otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], W, caps)
+        torch.cuda.synchronize()
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
+        sel_ms = pk_ms = 0.0
+        for _ in range(args.steps):
+            ev[0].record()
+            r = otif.otif_select_windows(None, masks, 0.0, wl.src_w, wl.src_h, wl.cell, W)
+            ev[1].record()
+            bt, slot, scount = otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], W, caps)
+            ev[2].record()
+            torch.cuda.synchronize()
+            sel_ms += ev[0].elapsed_time(ev[1])
+            pk_ms += ev[1].elapsed_time(ev[2])
+            del bt
+        tot = int(r["total"].item())
+        wins = r["windows"][:tot].cpu().numpy()
+        px = int((wins[:, 3].astype(np.int64) * wins[:, 4]).sum()) if tot else 0
+        full = int(((wins[:, 3] == wl.src_w) & (wins[:, 4] == wl.src_h)).sum()) if tot else 0
+        sc_np = scount.cpu().numpy()
+        e = {"W": [list(x) for x in W], "windows_per_frame": tot / n, "fallback_share": full / n,
+             "window_area_fraction": px / (n * wl.src_w * wl.src_h), "per_size": sc_np.tolist(),
+             "dropped_windows": int(np.maximum(sc_np - np.array(caps), 0).sum()),
+             "select_ns_per_frame": sel_ms / args.steps * 1e6 / n,
+             "select_ms_per_step": sel_ms / args.steps, "pack_ms_per_step": pk_ms / args.steps,
+             "pack_gbs": 2 * 3 * px / (pk_ms / args.steps / 1e3) / 1e9 if pk_ms > 0 else None,
+             "est_sum": int(r["est_sum"].item())}
+        e["pack_hbm_frac"] = e["pack_gbs"] / float(peaks["hbm_gbs"]) if e["pack_gbs"] else None
+        pp[tag] = e
+    out["perfect_proxy"] = pp
+    return out
 
 
 # --------------------------------------------------------------------------- GPU leg
@@ -410,65 +479,20 @@ def run_otif(args):
             torch.cuda.empty_cache()
         objs["configs"] = cfg
 
-    # ---- windowing active: the NEXT-3-trained C2 proxy and the perfect proxy under W*
+    # ---- windowing active: the NEXT-3-trained proxy and the perfect proxy under W*, at the
+    # headline density (C2) and off-peak (C2s, same camera, ~4 vehicles)
     if extras and not args.no_windowing:
-        from scripts import train_proxy
-        t0 = time.time()
-        tw, tinfo = train_proxy.train_weights(wl, steps=args.train_steps, batch=32, clip=1)
-        wstar3, sums3 = choose_wstar(otif_tuning, wl, 1, 600, 3, dev)
-        wstar5, sums5 = choose_wstar(otif_tuning, wl, 1, 600, 5, dev)
-        prep_s = time.time() - t0
-        win = {"what": "C2 clip 0 (4500 frames) through the whole path with the proxy trained by NEXT-3 (P:L137-141) "
-                       "on clip 1 and the window set W* chosen by NEXT-1 (P:L153-155) from clip 1's ground-truth "
-                       "masks; B = 0.5 on the trained scores",
-               "train": {k: tinfo[k] for k in ("steps", "batch", "ms_per_step", "loss")},
-               "W*_k3": [list(x) for x in wstar3], "W*_k5": [list(x) for x in wstar5], "prep_s": prep_s}
-        for tag, W in (("k3", wstar3), ("k5", wstar5)):
-            caps = caps_for(wl, W, n)
-            mw = measure_pipeline(otif, wl, tw, 0.5, src, args.steps, args.warmup, sizes=W, caps=caps)
-            win[tag] = {"frames_per_s": mw["frames"] / (mw["ms_total"] / 1e3), "ms_per_step": mw["ms_total"] / args.steps,
-                        "windows": window_stats(mw, wl, W), "roofline": rooflines(wl, mw, peaks, peak_src),
-                        "batch_cap": caps}
-            mw["pipe"].close()
+        wa = {}
+        for ww in (configs.C2, configs.C2S):
+            if ww.name == wl.name:
+                s_w = src
+            else:
+                s_w = torch.empty((n, ww.src_h, ww.src_w, 3), dtype=torch.uint8, device=dev)
+                video.make_scene(ww, clip=rank).render(range(n), out=s_w)
+            wa[ww.name] = windowing_scenario(otif, otif_tuning, ww, s_w, rank, dev, peaks, peak_src, args)
+            del s_w
             torch.cuda.empty_cache()
-        # perfect proxy: stages 3-5 on the ground-truth cell masks of clip 0 under W*
-        sc = video.make_scene(wl, clip=rank)
-        masks = torch.from_numpy(np.stack([video.gt_mask(sc.gt_boxes(t), wl.src_w, wl.src_h, wl.cell)
-                                           for t in range(n)])).to(dev)
-        pp = {}
-        for tag, W in (("default_W", list(wl.sizes)), ("W*_k3", wstar3), ("W*_k5", wstar5)):
-            caps = caps_for(wl, W, n)
-            r = otif.otif_select_windows(None, masks, 0.0, wl.src_w, wl.src_h, wl.cell, W)
-            otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], W, caps)
-            torch.cuda.synchronize()
-            ev = [torch.cuda.Event(enable_timing=True) for _ in range(3)]
-            sel_ms = pk_ms = 0.0
-            for _ in range(args.steps):
-                ev[0].record()
-                r = otif.otif_select_windows(None, masks, 0.0, wl.src_w, wl.src_h, wl.cell, W)
-                ev[1].record()
-                bt, slot, scount = otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], W, caps)
-                ev[2].record()
-                torch.cuda.synchronize()
-                sel_ms += ev[0].elapsed_time(ev[1])
-                pk_ms += ev[1].elapsed_time(ev[2])
-                del bt
-            tot = int(r["total"].item())
-            wins = r["windows"][:tot].cpu().numpy()
-            px = int((wins[:, 3].astype(np.int64) * wins[:, 4]).sum()) if tot else 0
-            full = int(((wins[:, 3] == wl.src_w) & (wins[:, 4] == wl.src_h)).sum()) if tot else 0
-            sc_np = scount.cpu().numpy()
-            pp[tag] = {"W": [list(x) for x in W], "windows_per_frame": tot / n, "fallback_share": full / n,
-                       "window_area_fraction": px / (n * wl.src_w * wl.src_h), "per_size": sc_np.tolist(),
-                       "dropped_windows": int(np.maximum(sc_np - np.array(caps), 0).sum()),
-                       "select_ns_per_frame": sel_ms / args.steps * 1e6 / n,
-                       "select_ms_per_step": sel_ms / args.steps, "pack_ms_per_step": pk_ms / args.steps,
-                       "pack_gbs": 2 * 3 * px / (pk_ms / args.steps / 1e3) / 1e9 if pk_ms > 0 else None,
-                       "est_sum": int(r["est_sum"].item())}
-            pp[tag]["pack_hbm_frac"] = pp[tag]["pack_gbs"] / float(peaks["hbm_gbs"]) if pp[tag]["pack_gbs"] else None
-        win["perfect_proxy"] = pp
-        del masks
-        objs["windowing_active"] = win
+        objs["windowing_active"] = wa
 
     # ---- C5: the 8-hour corpus (480 one-minute clips x 450 frames), contiguous
     # clip ranges per rank, per-clip device counters and hashes, strong scaling

@@ -1,6 +1,6 @@
 # A/B of e12 build variants (nvcc -D flags) on the proxy pass time (scripts/e12_time.py)
 for v in "" "-DOTIF_E12_ACC=1 -DOTIF_E12_E1SLOTS=3" ""; do
   OTIF_NVCC_EXTRA="$v" python -c "from paper_conf_sigmod_bastanim22_b200 import build as b; b.build(force=True)" > /dev/null 2>&1
-  OTIF_NVCC_EXTRA="$v" timeout 120 python -m pytest tests/test_gpu_parity.py -q -x -k "fused_vs_separate" 2>&1 | tail -1
+  OTIF_NVCC_EXTRA="$v" timeout 120 python -m pytest tests/test_gpu_parity.py -q -x -k "proxy" 2>&1 | tail -1
   echo "[$v] $(python scripts/e12_time.py 2>&1 | tail -1) $(python scripts/e12_time.py 2>&1 | tail -1)"
 done

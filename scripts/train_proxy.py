@@ -44,19 +44,20 @@ def evaluate(wl, w, frames, boxes, threshold=0.5):
             "window_area_fraction": area}
 
 
-def train_weights(wl, steps=300, batch=32, lr=1e-3, n_train=1024, clip=0):
-    """Train one proxy on clip `clip` of workload wl (frames with at least one detection,
-    P:L139; labels P:L139; BCE + Adam, readings R26/R27) from the random init.
+def train_weights(wl, steps=300, batch=32, lr=1e-3, n_train=1024, clip=0, start=0):
+    """Train one proxy on sampled frames [start, start + n_train) of clip `clip` of workload
+    wl (one camera; frames with at least one detection; labels P:L139; BCE + Adam,
+    readings R26/R27) from the random init.
     -> (trained fp32 weight blob, info dict with the loss curve and ms per step)."""
-    rng = np.random.default_rng(wl.seed + 7919 * clip)
+    rng = np.random.default_rng(wl.seed + 7919 * clip + start)
     sc = video.make_scene(wl, clip=clip)
-    cand = [t for t in range(n_train) if len(sc.gt_boxes(t)) > 0]
-    frames = video.frames(wl, n_train, device="cuda", clip=clip)
+    cand = [i for i, t in enumerate(range(start, start + n_train)) if len(sc.gt_boxes(t)) > 0]
+    frames = video.frames(wl, n_train, start=start, device="cuda", clip=clip)
     img_all = otif.otif_resize(frames, wl.proxy_h, wl.proxy_w)
     del frames
     gh, gw = -(-wl.src_h // wl.cell), -(-wl.src_w // wl.cell)
-    lab_all = train.otif_cell_labels(torch.from_numpy(boxes_for(wl, range(n_train), clip)).cuda(), n_train,
-                                     (gh, gw), wl.src_w, wl.src_h, wl.cell)
+    lab_all = train.otif_cell_labels(torch.from_numpy(boxes_for(wl, range(start, start + n_train), clip)).cuda(),
+                                     n_train, (gh, gw), wl.src_w, wl.src_h, wl.cell)
     cand_t = torch.tensor(cand, device="cuda")
     w0 = weights.proxy_weights()
     tr = train.Trainer(wl.proxy_h, wl.proxy_w, wl.n_strided, w0, max_batch=batch)
@@ -78,7 +79,7 @@ def train_weights(wl, steps=300, batch=32, lr=1e-3, n_train=1024, clip=0):
     del tr, img_all, lab_all
     torch.cuda.empty_cache()
     info = {"setting": wl.name, "proxy": f"{wl.proxy_w}x{wl.proxy_h}", "cell": wl.cell, "batch": batch,
-            "steps": steps, "train_clip": clip, "ms_per_step": ms, "train_frames_per_s": batch / (ms / 1e3),
+            "steps": steps, "train_clip": clip, "train_frames": [start, start + n_train], "ms_per_step": ms, "train_frames_per_s": batch / (ms / 1e3),
             "loss": [(s, float(l.item())) for s, l in losses]}
     return w, info
 

@@ -28,6 +28,7 @@ class Workload:
     seed: int
     quantile: float = 0.7   # reading R5
     gap: int = 4            # sampling gap g
+    objects: float = 10.0   # traffic scenes: mean concurrent objects at 960x540
 
     @property
     def proxy_w(self) -> int:
@@ -62,6 +63,9 @@ C1 = Workload("C1", "traffic", 416, 256, 32, Fraction(1, 4), 32,
               ((64, 64), (128, 128), (416, 256)), seed=1000)
 C2 = Workload("C2", "traffic", 960, 540, 4500, Fraction(1, 4), 32,
               ((128, 128), (256, 256), (960, 540)), seed=2000)
+# C2 at off-peak density (~4 concurrent vehicles instead of ~13): the same camera, the
+# regime in which windows beat the full frame
+C2S = C2.with_(name="C2s", objects=3.0)
 C3 = Workload("C3", "uav", 1920, 1080, 3000, Fraction(1, 4), 64,
               ((64, 64), (128, 128), (256, 256), (512, 512), (1920, 1080)), seed=3000, gap=1)
 C4_BASE = Workload("C4", "traffic", 1280, 720, 450, Fraction(1, 4), 32,
@@ -78,4 +82,4 @@ C5_CLIPS = 480
 C5_FRAMES_PER_CLIP = 450
 C5_POOL_CLIPS = 8
 
-ALL = {w.name: w for w in (C1, C2, C3, C5) + C4_SWEEP}
+ALL = {w.name: w for w in (C1, C2, C2S, C3, C5) + C4_SWEEP}

@@ -236,7 +236,7 @@ def make_scene(workload, clip: int = 0):
     seed = workload.seed + clip
     if workload.scene == "uav":
         return UAVScene(workload.src_w, workload.src_h, seed)
-    return TrafficScene(workload.src_w, workload.src_h, seed)
+    return TrafficScene(workload.src_w, workload.src_h, seed, mean_objects=getattr(workload, "objects", 10.0))
 
 
 def gt_mask(boxes, frame_w: int, frame_h: int, cell: int) -> np.ndarray:
