@@ -210,16 +210,19 @@ def run_reference(args):
 
 
 # --------------------------------------------------------------------------- GPU measurement helpers
-def measure_pipeline(otif, wl, blob, thr, src, steps, warmup, sizes=None, caps=None, batch=None):
+def measure_pipeline(otif, wl, blob, thr, src, steps, warmup, sizes=None, caps=None, batch=None, overlap=2):
     """Whole path (otif_pipeline_run_device) over the device-resident frames `src`: warm-up,
     then `steps` timed passes bracketed by CUDA events on the launching stream; per-stage
-    event times, kernel launches and device counters."""
+    event times, kernel launches and device counters.  overlap = the pipeline's pack_overlap:
+    2 = the pack of step s is copied under step s+1's proxy; the last one is flushed INSIDE
+    the timed region, so every step's work is timed."""
     import torch
     n = src.shape[0]
-    pipe = otif.Pipeline(wl, blob, thr, max_batch=batch or n, sizes=sizes, batch_cap=caps)
+    pipe = otif.Pipeline(wl, blob, thr, max_batch=batch or n, sizes=sizes, batch_cap=caps, pack_overlap=overlap)
     stream = torch.cuda.current_stream()
     for _ in range(warmup):
         pipe.run_device(src)
+    pipe.flush()
     torch.cuda.synchronize()
     pipe.reset_counters()
     pipe.set_timing(True)
@@ -228,6 +231,7 @@ def measure_pipeline(otif, wl, blob, thr, src, steps, warmup, sizes=None, caps=N
     e0.record(stream)
     for _ in range(steps):
         pipe.run_device(src)
+    pipe.flush()
     e1.record(stream)
     torch.cuda.synchronize()
     ms_total = e0.elapsed_time(e1)
@@ -344,7 +348,8 @@ def windowing_scenario(otif, otif_tuning, wl, src, rank, dev, peaks, peak_src, a
     out["prep_s"] = time.time() - t0
     for k, (W, _) in wstar.items():
         caps = caps_for(wl, W, n)
-        mw = measure_pipeline(otif, wl, tw, 0.5, src, args.steps, args.warmup, sizes=W, caps=caps)
+        mw = measure_pipeline(otif, wl, tw, 0.5, src, args.steps, args.warmup, sizes=W, caps=caps,
+                              overlap=args.pack_overlap)
         out[f"trained_k{k}"] = {"frames_per_s": mw["frames"] / (mw["ms_total"] / 1e3),
                                 "ms_per_step": mw["ms_total"] / args.steps, "windows": window_stats(mw, wl, W),
                                 "roofline": rooflines(wl, mw, peaks, peak_src), "batch_cap": caps}
@@ -436,7 +441,8 @@ def run_otif(args):
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    m = measure_pipeline(otif, wl, blob, b, src, args.steps, args.warmup, batch=args.batch or None)
+    m = measure_pipeline(otif, wl, blob, b, src, args.steps, args.warmup, batch=args.batch or None,
+                         overlap=args.pack_overlap)
     if world > 1:
         dist.barrier()
     clocks = sampler.stop()
@@ -465,7 +471,7 @@ def run_otif(args):
             video.make_scene(cw).render(range(nn), out=s2)
             thr = threshold_for(cw.name)
             steps_c = max(args.steps, int(np.ceil(2000.0 / nn)) if nn < 1000 else args.steps)
-            mc = measure_pipeline(otif, cw, blob, thr, s2, steps_c, args.warmup)
+            mc = measure_pipeline(otif, cw, blob, thr, s2, steps_c, args.warmup, overlap=args.pack_overlap)
             r = rooflines(cw, mc, peaks, peak_src)
             cfg[cw.name] = {"workload": f"{cw.src_w}x{cw.src_h} {cw.scene}, {nn} frames, proxy {cw.proxy_w}x{cw.proxy_h} "
                                         f"(S={cw.stride}), {cw.cell}-px cells, W={[list(x) for x in cw.sizes]}",
@@ -672,6 +678,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["otif", "reference"], default="otif")
     ap.add_argument("--batch", type=int, default=0, help="device batch (0 = whole clip)")
+    ap.add_argument("--pack-overlap", type=int, default=2, choices=[0, 1, 2],
+                    help="pipeline pack_overlap (0 = serial pack; 2 = pack of step s under step s+1's proxy)")
     ap.add_argument("--host-batch", type=int, default=512, help="device batch of the host (e2e) path")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--oracle-frames", type=int, default=64)

@@ -288,6 +288,18 @@ typedef struct {
     int32_t max_batch;          /* frames per device batch (one select / pack launch each) */
     int32_t batch_cap[8];       /* detector batch capacity per size, per device batch */
     int32_t proxy_batch;        /* frames per resize + proxy launch within a batch (0 = max_batch) */
+    int32_t pack_overlap;       /* stage 5 scheduling on device runs (identity crops, sizes with
+                                   w*3 % 16 == 0; otherwise ignored):
+                                   0 = pack each batch right after its selection;
+                                   1 = the pack of batch b is copied by spare warps of batch b+1's
+                                       tensor-bound proxy kernels (E4..D1, whose HBM is mostly idle),
+                                       the remainder by a drain kernel; the last batch of a call is
+                                       drained before the call returns;
+                                   2 = as 1, and the last batch's pack also rides in the NEXT
+                                       run_device call (or otif_pipeline_flush): its frames must stay
+                                       valid until then.  Windows, counts and counters are final when
+                                       the selection of a batch is; only the detector-batch bytes are
+                                       deferred.  Host runs always use 0. */
 } otif_pipeline_desc;
 
 typedef struct otif_pipeline otif_pipeline;
@@ -312,6 +324,11 @@ otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t *src_dev, i
  * of (global frame, x, y, w, h, s)), [5 + s] windows of size s (8 slots), [13] windows
  * dropped because their slot exceeded batch_cap[s], [14] pixels of the windows packed. */
 const int64_t *otif_pipeline_counters(const otif_pipeline *p);
+/* Device pointer to the detector batch of size s ([batch_cap[s], h_s, w_s, 3] u8, the
+ * last packed device batch), or NULL. */
+uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s);
+/* Complete a pack left pending by pack_overlap = 2 (enqueued on `stream`). */
+otif_status otif_pipeline_flush(otif_pipeline *p, cudaStream_t stream);
 otif_status otif_pipeline_reset_counters(otif_pipeline *p, cudaStream_t stream);
 /* Per-stage device timing (CUDA events recorded between the stage launches on the
  * compute stream).  enable != 0 starts recording (and clears previous records). */

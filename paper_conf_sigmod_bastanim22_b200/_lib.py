@@ -41,7 +41,8 @@ class PipelineDesc(ctypes.Structure):
     _fields_ = [("proxy", ProxyDesc), ("src_h", ctypes.c_int32), ("src_w", ctypes.c_int32),
                 ("det_h", ctypes.c_int32), ("det_w", ctypes.c_int32), ("grid", GridDesc),
                 ("threshold", ctypes.c_float), ("k", ctypes.c_int32), ("sizes", WSize * 8),
-                ("max_batch", ctypes.c_int32), ("batch_cap", ctypes.c_int32 * 8), ("proxy_batch", ctypes.c_int32)]
+                ("max_batch", ctypes.c_int32), ("batch_cap", ctypes.c_int32 * 8), ("proxy_batch", ctypes.c_int32),
+                ("pack_overlap", ctypes.c_int32)]
 
 
 _lib = None
@@ -123,6 +124,10 @@ def lib() -> ctypes.CDLL:
         L.otif_pipeline_run_host.restype = st
         L.otif_pipeline_run_device.argtypes = [P, P, i32, ctypes.c_int64, P]
         L.otif_pipeline_run_device.restype = st
+        L.otif_pipeline_detector_batch.argtypes = [P, i32]
+        L.otif_pipeline_detector_batch.restype = P
+        L.otif_pipeline_flush.argtypes = [P, P]
+        L.otif_pipeline_flush.restype = st
         L.otif_pipeline_counters.argtypes = [P]
         L.otif_pipeline_counters.restype = P
         L.otif_pipeline_reset_counters.argtypes = [P, P]
@@ -145,7 +150,7 @@ EXPORTED = ("otif_status_str", "otif_last_error", "otif_version", "otif_resize",
             "otif_proxy_destroy", "otif_proxy_grid", "otif_proxy_workspace_bytes", "otif_proxy_score",
             "otif_select_workspace_bytes", "otif_select_windows", "otif_pack_windows",
             "otif_pipeline_create", "otif_pipeline_destroy", "otif_pipeline_run_host",
-            "otif_pipeline_run_device", "otif_pipeline_counters", "otif_pipeline_reset_counters",
+            "otif_pipeline_run_device", "otif_pipeline_flush", "otif_pipeline_detector_batch", "otif_pipeline_counters", "otif_pipeline_reset_counters",
             "otif_pipeline_set_timing", "otif_pipeline_stage_ms", "otif_choose_workspace_bytes",
             "otif_choose_window_sizes", "otif_window_recall", "otif_track_resample", "otif_dbscan_workspace_bytes",
             "otif_track_dbscan", "otif_centers_workspace_bytes", "otif_track_centers", "otif_track_refine",

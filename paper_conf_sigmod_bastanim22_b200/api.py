@@ -176,10 +176,12 @@ class Pipeline:
 
     def __init__(self, workload, weights: np.ndarray, threshold: float, max_batch: int = 256,
                  batch_cap: Sequence[int] | None = None, connectivity: int = 4,
-                 enc=(32, 64, 128, 256, 256), dec=128, proxy_batch: int = 0, sizes=None):
-        """sizes: W as [(w, h)] or [(w, h, cost)] (default: the workload's own W)."""
+                 enc=(32, 64, 128, 256, 256), dec=128, proxy_batch: int = 0, sizes=None, pack_overlap: int = 0):
+        """sizes: W as [(w, h)] or [(w, h, cost)] (default: the workload's own W).
+        pack_overlap: 0 / 1 / 2 (otif.h: pack of batch b copied under batch b+1's proxy)."""
         d = PipelineDesc()
         d.proxy_batch = int(proxy_batch)
+        d.pack_overlap = int(pack_overlap)
         sizes = list(workload.sizes) if sizes is None else list(sizes)
         d.proxy.in_h, d.proxy.in_w, d.proxy.n_strided = workload.proxy_h, workload.proxy_w, workload.n_strided
         for i, e in enumerate(enc):
@@ -236,6 +238,22 @@ class Pipeline:
         _require_cuda(frames)
         check(lib().otif_pipeline_run_device(self.handle, _ptr(frames), frames.shape[0], int(frame_base),
                                              _stream(stream)), "otif_pipeline_run_device")
+
+    def detector_batch(self, s: int) -> torch.Tensor:
+        """Copy of the detector batch of size s ([batch_cap[s], h_s, w_s, 3] u8) as last packed."""
+        ptr = lib().otif_pipeline_detector_batch(self.handle, s)
+        w, h = int(self.sizes[s][0]), int(self.sizes[s][1])
+        shape = (self.batch_cap[s], h, w, 3)
+        out = torch.empty(shape, dtype=torch.uint8, device="cuda")
+        if ptr and out.numel():
+            class _CAI:
+                __cuda_array_interface__ = {"shape": shape, "typestr": "|u1", "data": (ptr, False), "version": 3}
+            out.copy_(torch.as_tensor(_CAI(), device="cuda"))
+        return out
+
+    def flush(self, stream=None):
+        """Complete a pack left pending by pack_overlap = 2."""
+        check(lib().otif_pipeline_flush(self.handle, _stream(stream)), "otif_pipeline_flush")
 
     def counters(self) -> torch.Tensor:
         """int64 [15] device counters: frames, positive cells, windows, window pixels, window hash,

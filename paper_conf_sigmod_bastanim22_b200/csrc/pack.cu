@@ -10,9 +10,11 @@
 //   every size in W with w*3 % 16 == 0) from two aligned 16-B source loads and a
 //   funnel shift, since a window's x offset makes the source row arbitrarily aligned.
 //   Resampling case: per output pixel bilinear blend (same arithmetic as resize.cu).
+#include <stddef.h>
 #include <string.h>
 
 #include "common.cuh"
+#include "packjob.cuh"
 
 namespace otif {
 
@@ -33,6 +35,7 @@ struct PackParams {
     int *size_count;
     unsigned long long *ctr_pack;  // internal (pipeline): [0] windows dropped for batch_cap, [1] packed pixels
     int stage_bytes;  // bulk ring stage size (<= kBulkStage)
+    PackJob *job;     // internal (pipeline): build the copy-unit queue (packjob.cuh) instead of copying here
 };
 
 __global__ void __launch_bounds__(1024) slot_kernel(const __grid_constant__ PackParams p) {
@@ -57,8 +60,12 @@ __global__ void __launch_bounds__(1024) slot_kernel(const __grid_constant__ Pack
             int pre = s_carry[s];
             for (int w = 0; w < warp; w++) pre += s_warp_cnt[w][s];
             p.slot[g] = pre + rank;
-            if (pre + rank < p.cap[s]) packed_px += (unsigned long long)p.win[g].w * p.win[g].h;
-            else dropped++;
+            if (pre + rank < p.cap[s]) {
+                packed_px += (unsigned long long)p.win[g].w * p.win[g].h;
+                if (p.job) p.job->inv[p.job->inv_off[s] + pre + rank] = g;
+            } else {
+                dropped++;
+            }
         }
         __syncthreads();
         if (threadIdx.x < p.k) {
@@ -70,6 +77,18 @@ __global__ void __launch_bounds__(1024) slot_kernel(const __grid_constant__ Pack
     }
     // size_count counts every listed window, including those dropped for batch_cap
     if (threadIdx.x < p.k) p.size_count[threadIdx.x] = s_carry[threadIdx.x];
+    if (p.job && threadIdx.x == 0) {
+        // unit queue: per size min(count, cap) windows x ceil(h / rows_per_unit) units
+        unsigned long long base = 0;
+        for (int z = 0; z < p.k; z++) {
+            p.job->units_base[z] = base;
+            const int kept = min(s_carry[z], p.cap[z]);
+            const int rpu = p.job->rows_per_unit[z];
+            base += (unsigned long long)kept * ((p.bh[z] + rpu - 1) / rpu);
+        }
+        for (int z = p.k; z <= kPackJobMaxK; z++) p.job->units_base[z] = base;
+        p.job->next = 0;
+    }
     if (p.ctr_pack) {
         for (int o = 16; o > 0; o >>= 1) {
             dropped += __shfl_xor_sync(0xffffffffu, dropped, o);
@@ -263,11 +282,70 @@ __global__ void __launch_bounds__(kThreads) pack_kernel(const __grid_constant__ 
     }
 }
 
+// Drains a pack job's remaining copy units (those the fused copy warps of the proxy did
+// not take): 4 warps per CTA, several CTAs per SM.
+__global__ void __launch_bounds__(128) pack_units_kernel(PackJob *job) {
+    pj_drain_warp<8>(job, nullptr, threadIdx.x & 31);
+}
+
 }  // namespace otif
 
 using namespace otif;
 
 namespace otif {
+
+// A pack job applies when the detector resolution is the source's (identity crop) and every
+// size's rows are whole 16-B pieces (w * 3 % 16 == 0) in 16-B aligned batch buffers.
+bool pack_job_applies(int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w, const otif_wsize *sizes, int32_t k,
+                      uint8_t *const *batches) {
+    if (src_h != det_h || src_w != det_w || k > kPackJobMaxK) return false;
+    for (int s = 0; s < k; s++)
+        if ((sizes[s].w * 3) % 16 != 0 || (((uintptr_t)batches[s]) & 15) != 0) return false;
+    return true;
+}
+
+// Stage-5 slot assignment that also builds the copy-unit queue `job_dev` (device) for
+// later draining (fused copy warps, pack_units_kernel).  inv: >= sum(batch_cap) ints.
+otif_status launch_pack_prepare(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w,
+                                const otif_window *windows, const int32_t *total, int32_t capacity,
+                                const otif_wsize *sizes, int32_t k, uint8_t *const *batches, const int32_t *batch_cap,
+                                int32_t *slot, int32_t *size_count, cudaStream_t stream, unsigned long long *ctr_pack,
+                                PackJob *job_dev, int *inv) {
+    PackJob h;
+    memset(&h, 0, sizeof(h));
+    h.src = src; h.src_bytes = (size_t)n * src_h * src_w * 3; h.sh = src_h; h.sw = src_w; h.k = k;
+    h.win = windows; h.inv = inv;
+    int off = 0;
+    for (int s = 0; s < k; s++) {
+        h.batch[s] = batches[s]; h.bw[s] = sizes[s].w; h.bh[s] = sizes[s].h;
+        const int rb = sizes[s].w * 3;
+        int rpu = (int)(kUnitBytes / (uint32_t)rb);
+        h.rows_per_unit[s] = rpu < 1 ? 1 : (rpu > sizes[s].h ? sizes[s].h : rpu);
+        h.inv_off[s] = off;
+        off += batch_cap[s];
+    }
+    // static part; the slot kernel fills units_base / next (stream order)
+    OTIF_CUDA(cudaMemcpyAsync(job_dev, &h, offsetof(PackJob, units_base), cudaMemcpyHostToDevice, stream));
+    PackParams p;
+    memset(&p, 0, sizeof(p));
+    p.src = src; p.n = n; p.sh = src_h; p.sw = src_w; p.dh = src_h; p.dw = src_w;
+    p.win = windows; p.total = total; p.capacity = capacity; p.k = k;
+    for (int s = 0; s < k; s++) {
+        p.batch[s] = batches[s]; p.cap[s] = batch_cap[s]; p.bw[s] = sizes[s].w; p.bh[s] = sizes[s].h;
+    }
+    p.slot = slot; p.size_count = size_count; p.ctr_pack = ctr_pack; p.job = job_dev;
+    slot_kernel<<<1, 1024, 0, stream>>>(p);
+    OTIF_LAUNCH_CHECK();
+    return OTIF_OK;
+}
+
+otif_status launch_pack_units(PackJob *job_dev, cudaStream_t stream) {
+    int num_sms = 148;
+    check_device(&num_sms);
+    pack_units_kernel<<<num_sms * 8, 128, 0, stream>>>(job_dev);
+    OTIF_LAUNCH_CHECK();
+    return OTIF_OK;
+}
 
 // internal entry; ctr_pack (pipeline, may be NULL): device counters of dropped windows
 // and packed pixels, accumulated

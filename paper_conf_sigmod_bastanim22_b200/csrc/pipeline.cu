@@ -17,11 +17,20 @@
 #include <vector>
 
 #include "common.cuh"
+#include "packjob.cuh"
 
 namespace otif {
 
 otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws, size_t ws_bytes,
-                         cudaStream_t stream, cudaEvent_t *evs);
+                         cudaStream_t stream, cudaEvent_t *evs, PackJob *pj);
+bool pack_job_applies(int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w, const otif_wsize *sizes, int32_t k,
+                      uint8_t *const *batches);
+otif_status launch_pack_prepare(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w,
+                                const otif_window *windows, const int32_t *total, int32_t capacity,
+                                const otif_wsize *sizes, int32_t k, uint8_t *const *batches, const int32_t *batch_cap,
+                                int32_t *slot, int32_t *size_count, cudaStream_t stream, unsigned long long *ctr_pack,
+                                PackJob *job_dev, int *inv);
+otif_status launch_pack_units(PackJob *job_dev, cudaStream_t stream);
 otif_status launch_select(const float *scores, const uint8_t *mask_in, float threshold, int32_t n, int32_t gh,
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
@@ -94,7 +103,20 @@ struct otif_pipeline {
     std::vector<int> ev_stage, ev_from;
     size_t ev_used = 0;
     int64_t launches = 0;
+    // pack overlap (desc.pack_overlap): the copy-unit queue of the last selected batch,
+    // drained by the next batch's proxy kernels and pack_units_kernel
+    PackJob *job = nullptr;
+    int *inv = nullptr;
+    int job_pending = 0;
+    cudaEvent_t ev_pending = nullptr;       // recorded where the pending job was built
+    cudaStream_t pending_stream = nullptr;
 };
+
+// a pending job built on another stream: order this stream after it
+static otif_status wait_pending(otif_pipeline *p, cudaStream_t st) {
+    if (p->job_pending && st != p->pending_stream) OTIF_CUDA(cudaStreamWaitEvent(st, p->ev_pending, 0));
+    return OTIF_OK;
+}
 
 // reserve a log entry (stage, from); its event is returned for the caller to record
 static int treserve(otif_pipeline *p, int stage, int from, cudaEvent_t *ev) {
@@ -142,21 +164,39 @@ struct NvtxRange {
     ~NvtxRange() { nvtxRangePop(); }
 };
 
-static otif_status run_proxy(otif_pipeline *p, const uint8_t *img, int mb, float *scores, cudaStream_t st) {
+static otif_status run_proxy(otif_pipeline *p, const uint8_t *img, int mb, float *scores, cudaStream_t st,
+                             PackJob *pj) {
     NvtxRange r("otif.proxy");
     // six spans for the proxy (prep/E1, then each GEMM layer); launch_proxy records their
     // end events at the actual points in the stream
     cudaEvent_t evs[6];
     int from = tmark(p, st);
     for (int i = 0; i < 6 && p->timing; i++) from = treserve(p, ST_PREP + i, from, &evs[i]);
-    RC(launch_proxy(p->proxy, img, mb, scores, p->proxy_ws, p->proxy_ws_bytes, st, p->timing ? evs : nullptr));
+    RC(launch_proxy(p->proxy, img, mb, scores, p->proxy_ws, p->proxy_ws_bytes, st, p->timing ? evs : nullptr, pj));
     p->launches += proxy_launches(p->proxy);
     return OTIF_OK;
 }
 
-static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int frame_base, cudaStream_t st) {
+// drain the pending pack job (whatever the fused copy warps did not take)
+static otif_status drain_pack(otif_pipeline *p, cudaStream_t st) {
+    if (!p->job_pending) return OTIF_OK;
+    RC(wait_pending(p, st));
+    NvtxRange r("otif.pack_drain");
+    int t0 = tmark(p, st);
+    RC(launch_pack_units(p->job, st));
+    tspan(p, ST_PACK, st, t0);
+    p->launches += 1;
+    p->job_pending = 0;
+    return OTIF_OK;
+}
+
+// overlap: 0 = pack right after select; 1 = leave the pack pending for the next batch's
+// proxy (the caller drains it at the end of the call or keeps it for the next call)
+static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int frame_base, cudaStream_t st,
+                             int overlap) {
     const otif_pipeline_desc &d = p->d;
     const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
+    RC(wait_pending(p, st));
     for (int m0 = 0; m0 < nb; m0 += p->pb) {
         const int mb = nb - m0 < p->pb ? nb - m0 : p->pb;
         {
@@ -167,8 +207,10 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
             tspan(p, ST_RESIZE, st, t0);
             p->launches += 1;
         }
-        RC(run_proxy(p, p->img, mb, p->scores + (size_t)m0 * p->cells, st));
+        // the pending pack (previous batch) rides in this proxy pass's tensor-bound layers
+        RC(run_proxy(p, p->img, mb, p->scores + (size_t)m0 * p->cells, st, p->job_pending ? p->job : nullptr));
     }
+    RC(drain_pack(p, st));
     {
         NvtxRange r("otif.select");
         int t0 = tmark(p, st);
@@ -180,10 +222,19 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
     }
     NvtxRange r("otif.pack");
     int t0 = tmark(p, st);
-    RC(launch_pack(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
-                   p->batches, d.batch_cap, p->slot, p->size_count, st, p->ctr + kCtrPack));
+    if (overlap && p->job) {
+        RC(launch_pack_prepare(src, nb, d.src_h, d.src_w, p->windows, p->total, p->cap_w, d.sizes, d.k, p->batches,
+                               d.batch_cap, p->slot, p->size_count, st, p->ctr + kCtrPack, p->job, p->inv));
+        p->job_pending = 1;
+        p->pending_stream = st;
+        OTIF_CUDA(cudaEventRecord(p->ev_pending, st));
+        p->launches += 1;
+    } else {
+        RC(launch_pack(src, nb, d.src_h, d.src_w, d.det_h, d.det_w, p->windows, p->total, p->cap_w, d.sizes, d.k,
+                       p->batches, d.batch_cap, p->slot, p->size_count, st, p->ctr + kCtrPack));
+        p->launches += 2;
+    }
     t0 = tspan(p, ST_PACK, st, t0);
-    p->launches += 2;
     if (p->out_win) {
         append_kernel<<<1, 1024, 0, st>>>(p->windows, p->total, p->cap_w, p->counts, nb, frame_base, p->out_win,
                                           p->out_win_cap, p->out_counts, p->out_total);
@@ -214,6 +265,7 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     OTIF_REQUIRE(d->grid.frame_w == d->det_w && d->grid.frame_h == d->det_h,
                  "otif_pipeline_create: grid frame must be the detector resolution");
     for (int s = 0; s < d->k; s++) OTIF_REQUIRE(d->batch_cap[s] >= 0, "otif_pipeline_create: batch_cap[%d] < 0", s);
+    OTIF_REQUIRE(d->pack_overlap >= 0 && d->pack_overlap <= 2, "otif_pipeline_create: pack_overlap %d", d->pack_overlap);
     otif_pipeline *p = new (std::nothrow) otif_pipeline();
     if (!p) return OTIF_ENOMEM;
     p->d = *d;
@@ -247,6 +299,13 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     for (int s = 0; s < d->k; s++)
         if (d->batch_cap[s] > 0)
             PCUDA(cudaMalloc(&p->batches[s], (size_t)d->batch_cap[s] * d->sizes[s].w * d->sizes[s].h * 3));
+    if (d->pack_overlap && pack_job_applies(d->src_h, d->src_w, d->det_h, d->det_w, d->sizes, d->k, p->batches)) {
+        int64_t inv_n = 0;
+        for (int s = 0; s < d->k; s++) inv_n += d->batch_cap[s];
+        PCUDA(cudaMalloc(&p->job, sizeof(PackJob)));
+        PCUDA(cudaEventCreateWithFlags(&p->ev_pending, cudaEventDisableTiming));
+        PCUDA(cudaMalloc(&p->inv, (size_t)(inv_n > 0 ? inv_n : 1) * 4));
+    }
     PCUDA(cudaMalloc(&p->ctr, kCtrTotal * 8));
     PCUDA(cudaMemset(p->ctr, 0, kCtrTotal * 8));
     PCUDA(cudaMalloc(&p->out_total, 4));
@@ -263,15 +322,18 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
 
 extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     if (!p) return;
+    if (p->job_pending && p->pending_stream) cudaStreamSynchronize(p->pending_stream);
     if (p->s_compute) cudaStreamSynchronize(p->s_compute);
     if (p->s_copy) cudaStreamSynchronize(p->s_copy);
     void *bufs[] = {p->src[0], p->src[1], p->img, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
-                    p->offsets, p->total, p->slot, p->size_count, p->ctr, p->out_win, p->out_counts, p->out_total};
+                    p->offsets, p->total, p->slot, p->size_count, p->ctr, p->out_win, p->out_counts, p->out_total,
+                    p->job, p->inv};
     for (void *b : bufs)
         if (b) cudaFree(b);
     for (int s = 0; s < 8; s++)
         if (p->batches[s]) cudaFree(p->batches[s]);
     for (cudaEvent_t e : p->ev_pool) cudaEventDestroy(e);
+    if (p->ev_pending) cudaEventDestroy(p->ev_pending);
     for (int i = 0; i < 2; i++) {
         if (p->ev_h2d[i]) cudaEventDestroy(p->ev_h2d[i]);
         if (p->ev_free[i]) cudaEventDestroy(p->ev_free[i]);
@@ -312,6 +374,7 @@ extern "C" otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *s
     RC(ensure_outputs(p, n > 0 ? n : 1, cap_windows > 0 ? cap_windows : 1));
     const otif_pipeline_desc &d = p->d;
     const size_t frame_bytes = (size_t)d.src_h * d.src_w * 3;
+    RC(drain_pack(p, p->s_compute));   // a pack left pending by a device run (same frames lifetime rule)
     OTIF_CUDA(cudaMemsetAsync(p->out_total, 0, 4, p->s_compute));
     OTIF_CUDA(cudaMemsetAsync(p->ctr, 0, kCtrTotal * 8, p->s_compute));
     // the copy stream must not overwrite a src buffer before the compute stream is done with it
@@ -328,7 +391,7 @@ extern "C" otif_status otif_pipeline_run_host(otif_pipeline *p, const uint8_t *s
                                   cudaMemcpyHostToDevice, p->s_copy));
         OTIF_CUDA(cudaEventRecord(p->ev_h2d[buf], p->s_copy));
         OTIF_CUDA(cudaStreamWaitEvent(p->s_compute, p->ev_h2d[buf], 0));
-        rc = run_batch(p, p->src[buf], nb, f0, p->s_compute);
+        rc = run_batch(p, p->src[buf], nb, f0, p->s_compute, 0);   // host runs are PCIe-bound: no pack overlap
         if (rc == OTIF_OK) OTIF_CUDA(cudaEventRecord(p->ev_free[buf], p->s_compute));
     }
     p->out_win_cap = cap_saved;
@@ -363,11 +426,24 @@ extern "C" otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t 
     otif_status rc = OTIF_OK;
     for (int f0 = 0; f0 < n && rc == OTIF_OK; f0 += p->d.max_batch) {
         const int nb = n - f0 < p->d.max_batch ? n - f0 : p->d.max_batch;
-        rc = run_batch(p, src_dev + (size_t)f0 * frame_bytes, nb, (int)(frame_base + f0), stream);
+        rc = run_batch(p, src_dev + (size_t)f0 * frame_bytes, nb, (int)(frame_base + f0), stream,
+                       p->d.pack_overlap != 0);
     }
+    // pack_overlap 1: the last batch's pack completes within this call; 2: it stays pending
+    // for the next call's proxy (or otif_pipeline_flush)
+    if (rc == OTIF_OK && p->d.pack_overlap == 1) rc = drain_pack(p, stream);
     p->out_win = ow;
     p->out_counts = oc;
     return rc;
+}
+
+extern "C" uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s) {
+    return (p && s >= 0 && s < p->d.k) ? p->batches[s] : nullptr;
+}
+
+extern "C" otif_status otif_pipeline_flush(otif_pipeline *p, cudaStream_t stream) {
+    OTIF_REQUIRE(p, "otif_pipeline_flush: NULL");
+    return drain_pack(p, stream);
 }
 
 extern "C" const int64_t *otif_pipeline_counters(const otif_pipeline *p) {

@@ -34,10 +34,21 @@
 #include <vector>
 
 #include "common.cuh"
+#include "packjob.cuh"
 
 namespace otif {
 
-constexpr int kConvThreads = 256;   // warp0 producer, warp1 MMA, warp2 TMEM alloc, warps4-7 epilogue
+// warp0 producer, warp1 MMA, warp2 TMEM alloc, warps4-7 epilogue, warps 8.. fused pack copy
+#ifndef OTIF_PJ_WARPS
+#define OTIF_PJ_WARPS 8          // fused copy warps per conv CTA (A/B builds)
+#endif
+#ifndef OTIF_PJ_UNROLL
+#define OTIF_PJ_UNROLL 8         // 16-B pieces in flight per copy lane
+#endif
+#ifndef OTIF_PJ_LAYERS
+#define OTIF_PJ_LAYERS 0x1C      // GEMM layers (bit li: 0 = E2 .. 4 = D1) whose CTAs copy; E4, E5, D1
+#endif
+constexpr int kConvThreads = 256 + 32 * OTIF_PJ_WARPS;
 constexpr int kTileM = 128;
 constexpr int kMaxStagesA = 4;
 constexpr int kMaxStagesB = 8;
@@ -96,6 +107,9 @@ struct ConvParams {
     float *scores;
     const float *w2;            // [N] bf16-rounded head weights (fp32 storage)
     float b2;
+    // fused stage 5 of the PREVIOUS device batch (packjob.cuh): warps 8-15 drain its copy
+    // units while this layer's MMAs run (the layer is tensor-bound, its HBM mostly idle)
+    PackJob *pj;
 };
 
 // ---------------------------------------------------------------------------
@@ -258,8 +272,10 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
 
     const uint32_t acc_cols = 2 * MT * p.N;  // two accumulator stages of MT sub-tiles x N columns
     const uint32_t tmem_cols = acc_cols <= 32 ? 32 : (acc_cols <= 64 ? 64 : (acc_cols <= 128 ? 128 : (acc_cols <= 256 ? 256 : 512)));
+    int &s_conv_done = *reinterpret_cast<int *>(s_red + 4 * 256);   // set when the epilogue drained its last tile
 
     if (threadIdx.x == 0) {
+        s_conv_done = 0;
         for (int i = 0; i < p.stages_a; i++) { mbar_init(&a_full[i], 1); mbar_init(&a_empty[i], 1); }
         for (int i = 0; i < p.stages_b; i++) { mbar_init(&b_full[i], 1); mbar_init(&b_empty[i], 1); }
         for (int i = 0; i < 2; i++) { mbar_init(&t_full[i], 1); mbar_init(&t_empty[i], 128); }
@@ -355,7 +371,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                 if (++acc == 2) { acc = 0; accp ^= 1; }
             }
         }
-    } else if (SWAP && warp >= 4) {
+    } else if (SWAP && warp >= 4 && warp < 8) {
         // ===== head epilogue, transposed accumulator: lane = D1 channel, column = pixel =====
         const int quarter = warp & 3;
         const int ch = quarter * 32 + lane;
@@ -407,7 +423,8 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
             asm volatile("bar.sync 1, 128;" ::: "memory");
             if (++acc == 2) { acc = 0; accp ^= 1; }
         }
-    } else if (warp >= 4) {
+        if (threadIdx.x == 128) *(volatile int *)&s_conv_done = 1;
+    } else if (warp >= 4 && warp < 8) {
         // ===== epilogue: TMEM -> regs -> bias, ReLU, bf16 -> next layer's layout =====
         const int row = threadIdx.x - 128;          // TMEM lane == tile row
         const int quarter = warp & 3;               // lanes 32*quarter .. +31
@@ -460,6 +477,11 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
             mbar_arrive(&t_empty[acc]);
             if (++acc == 2) { acc = 0; accp ^= 1; }
         }
+        if (threadIdx.x == 128) *(volatile int *)&s_conv_done = 1;
+    } else if (warp >= 8 && p.pj) {
+        // ===== fused pack of the previous batch: drain copy units until this CTA's conv
+        // work is done (the rest continues in the next layer / pack_units_kernel) =====
+        pj_drain_warp<OTIF_PJ_UNROLL>(p.pj, &s_conv_done, lane);
     }
     __syncwarp();
     tc_fence_before();
@@ -1199,7 +1221,7 @@ static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
 
 // evs (optional): 6 events recorded after E1 (prep) and after each of the 5 GEMM layers
 otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws,
-                         size_t ws_bytes, cudaStream_t stream, cudaEvent_t *evs) {
+                         size_t ws_bytes, cudaStream_t stream, cudaEvent_t *evs, PackJob *pj) {
     Layout lay[5];
     size_t need = plan_workspace(p, n, lay);
     if (ws_bytes < need) {
@@ -1295,6 +1317,8 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
             for (int t = 0; t < 9; t++) c.group_shift[i][t] = g.group_shift[i][t];
         }
         c.wpk = g.wpk_dev; c.bias = g.bias_dev; c.N = g.cout;
+        // fused copy warps only in the tensor-bound layers past E3 (E3 is HBM-bound)
+        c.pj = ((OTIF_PJ_LAYERS >> li) & 1) ? pj : nullptr;
         c.mtot = (int64_t)n * g.fstride_unit;
         c.ntiles = (int)cdiv(c.mtot, (int64_t)kTileM * g.mt);
         c.pitch = g.pitch; c.fstride = g.fstride_unit; c.out_h = g.out_h; c.out_w = g.out_w;
@@ -1505,5 +1529,5 @@ extern "C" otif_status otif_proxy_score(const otif_proxy *p, const uint8_t *img,
     OTIF_REQUIRE((((uintptr_t)workspace) & 255) == 0, "otif_proxy_score: workspace must be 256-B aligned");
     otif_status st = check_device(nullptr);
     if (st != OTIF_OK) return st;
-    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream, nullptr);
+    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream, nullptr, nullptr);
 }

@@ -1,0 +1,83 @@
+#!/usr/bin/env python
+"""One isolated launch of each HBM / latency-bound stage for `ncu --set full`:
+resize_even_kernel (C2, 4500 frames, 1/4), select_kernel on random-init proxy scores
+(C2, every frame falls back) and on the trained proxy's scores (C2, windowing active),
+pack_kernel with full-frame windows and with the trained proxy's multi-size windows
+under W* (C2s: ~8% fallback).  Prints the algorithmic bytes of each launch as JSON.
+
+    ncu --set full -k regex:"resize_even|select_kernel|pack_kernel" -o gpurun_out/r02_stages \
+        python scripts/prof_stages.py
+"""
+import json
+import os
+import sys
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import paper_conf_sigmod_bastanim22_b200 as otif  # noqa: E402
+from scripts import train_proxy  # noqa: E402
+from synth import configs, video, weights  # noqa: E402
+
+
+# W* (k = 5) that NEXT-1 chose from frames [4500, 5100) of clip 0 in the r02c bench run
+# (bench.py windowing_active); fixed here so that the capture holds no choose launches
+WSTAR = {"C2": [(960, 540), (960, 192), (160, 128), (960, 288), (256, 224)],
+         "C2s": [(960, 540), (224, 160), (320, 512), (128, 128), (256, 224)]}
+
+
+def thr(name, q=0.7):
+    d = json.load(open(os.path.join(ROOT, "tests", "golden", "thresholds.json")))
+    return d["workloads"][name][str(q)]["B"]
+
+
+def main():
+    out = {}
+    wl = configs.C2
+    n = wl.n_frames
+    src = torch.empty((n, wl.src_h, wl.src_w, 3), dtype=torch.uint8, device="cuda")
+    video.make_scene(wl).render(range(n), out=src)
+    torch.cuda.nvtx.range_push("prof")
+    img = otif.otif_resize(src, wl.proxy_h, wl.proxy_w)                                  # resize
+    torch.cuda.nvtx.range_pop()
+    out["resize"] = {"algorithmic_bytes": n * (2 * 135 * 960 * 3 + 135 * 240 * 3)}
+    sc = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, weights.proxy_weights()).score(img)
+    torch.cuda.nvtx.range_push("prof")
+    r = otif.otif_select_windows(sc, None, thr("C2"), wl.src_w, wl.src_h, wl.cell, wl.sizes)  # select (random)
+    torch.cuda.nvtx.range_pop()
+    out["select_random"] = {"algorithmic_bytes": n * (510 * 4) + 24 * int(r["total"].item())}
+    caps = [n, n, n]
+    torch.cuda.nvtx.range_push("prof")
+    otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], wl.sizes, caps)  # pack (full frame)
+    torch.cuda.nvtx.range_pop()
+    w = r["windows"][:int(r["total"].item())].cpu().numpy()
+    out["pack_full"] = {"algorithmic_bytes": int(2 * 3 * (w[:, 3].astype(np.int64) * w[:, 4]).sum())}
+    for name, ww in (("C2", configs.C2), ("C2s", configs.C2S)):
+        if name == "C2s":
+            video.make_scene(ww).render(range(n), out=src)
+        tw, _ = train_proxy.train_weights(ww, steps=400, batch=32, clip=0, start=n)
+        W = WSTAR[name]
+        im = otif.otif_resize(src, ww.proxy_h, ww.proxy_w)
+        s2 = otif.Proxy(ww.proxy_h, ww.proxy_w, ww.n_strided, tw).score(im)
+        torch.cuda.nvtx.range_push("prof")
+        r2 = otif.otif_select_windows(s2, None, 0.5, ww.src_w, ww.src_h, ww.cell, W)      # select (trained)
+        torch.cuda.nvtx.range_pop()
+        t2 = int(r2["total"].item())
+        out[f"select_trained_{name}"] = {"algorithmic_bytes": n * 510 * 4 + 24 * t2, "W": W, "windows": t2}
+        if name == "C2s":
+            cap2 = [n * 8] * len(W)
+            torch.cuda.nvtx.range_push("prof")
+            otif.otif_pack_windows(src, ww.src_h, ww.src_w, r2["windows"], r2["total"], W, cap2)  # pack (multi)
+            torch.cuda.nvtx.range_pop()
+            w2 = r2["windows"][:t2].cpu().numpy()
+            out["pack_multi_C2s"] = {"algorithmic_bytes": int(2 * 3 * (w2[:, 3].astype(np.int64) * w2[:, 4]).sum()),
+                                     "windows": t2, "fallback_share": float(((w2[:, 3] == 960) & (w2[:, 4] == 540)).sum() / n)}
+    torch.cuda.synchronize()
+    print(json.dumps(out))
+
+
+if __name__ == "__main__":
+    main()
