@@ -46,8 +46,10 @@ namespace otif {
 #define OTIF_PJ_UNROLL 8         // 16-B pieces in flight per copy lane
 #endif
 #ifndef OTIF_PJ_LAYERS
-#define OTIF_PJ_LAYERS 0x1C      // GEMM layers (bit li: 0 = E2 .. 4 = D1) whose CTAs copy; E4, E5, D1
+#define OTIF_PJ_LAYERS 0x18      // GEMM layers (bit li: 0 = E2 .. 4 = D1) whose CTAs copy: E5, D1
 #endif
+// (measured, scripts/pj_ab.sh, profiles/r02_pack_overlap.md: hosting the copy in E4 or in
+// the latency-bound E1+E2 kernel costs about as much conv time as it saves)
 constexpr int kConvThreads = 256 + 32 * OTIF_PJ_WARPS;
 constexpr int kTileM = 128;
 constexpr int kMaxStagesA = 4;
@@ -519,7 +521,10 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
 // (#pragma unroll 1): 5720 -> 3950 SASS instructions, 1.66 -> 0.97 ms per C2 step.
 // TMEM: E2 accumulators 2 x 128 columns at 0, E1 accumulators 2 plane slots x 32 KT at 256.
 // ---------------------------------------------------------------------------
-constexpr int kE12Threads = 768;
+#ifndef OTIF_PJ_E12
+#define OTIF_PJ_E12 0            // fused pack copy warps in the E1+E2 kernel (A/B builds; 0 = none)
+#endif
+constexpr int kE12Threads = 768 + 32 * OTIF_PJ_E12;
 #ifndef OTIF_E12_ACC
 #define OTIF_E12_ACC 2        // E2 accumulator stages (A/B builds)
 #endif
@@ -552,6 +557,7 @@ struct E12Params {
     int64_t out_lcap;
     int out_c8, out_pitch;
     int64_t out_fstride;
+    PackJob *pj;                // fused stage 5 of the previous batch (warps 24..), or NULL
 };
 
 // Trace / knock-out bits (OTIF_E12_TRACE, read at launch) exist only in a trace build
@@ -668,6 +674,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acc_empty + 2);
     float *s_b1 = reinterpret_cast<float *>(tmem_slot + 4);
     float *s_b2 = s_b1 + 32;
+    int &s_e12_done = *reinterpret_cast<int *>(s_b2 + 64);   // E2 epilogue drained its last tile
 
     // ---- prologue: barriers, TMEM, resident weights, slab pads = 128 ----
     if (threadIdx.x == 0) {
@@ -688,6 +695,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
     for (uint32_t i = threadIdx.x; i < 2 * slab_bytes / 16; i += blockDim.x)
         reinterpret_cast<uint4 *>(slab_s)[i] = make_uint4(0x80808080u, 0x80808080u, 0x80808080u, 0x80808080u);
     if (threadIdx.x < N2) s_b2[threadIdx.x] = p.b2[threadIdx.x];
+    if (threadIdx.x == 0) s_e12_done = 0;
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // resident weights -> tensor core
     tc_fence_before();
     __syncthreads();
@@ -900,6 +908,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
             }
         }
         E12_TR_DUMP("E1EP a2empty e1full arrived", 3);
+    } else if (warp >= 24) {
+        // ===== fused pack of the previous batch (packjob.cuh) until the E2 epilogue is done =====
+        if (p.pj) pj_drain_warp<OTIF_PJ_UNROLL>(p.pj, &s_e12_done, lane);
     } else if (warp >= 20) {
         // ===== E2 epilogue: TMEM -> bias, ReLU, bf16 -> E3's input layout =====
         const int row = threadIdx.x - 640;
@@ -943,6 +954,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
             mbar_arrive(&acc_empty[acc]);
             if (++acc == kAccStages) { acc = 0; accp ^= 1; }
         }
+        if (threadIdx.x == 640) *(volatile int *)&s_e12_done = 1;
     }
     __syncwarp();
     tc_fence_before();
@@ -1280,6 +1292,7 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         e.wt2 = p->e12_w2_dev; e.b2 = g.bias_dev;
         e.out_kind = lay[1].kind; e.out = ws + lay[1].offset; e.out_lcap = lay[1].lcap;
         e.out_c8 = lay[1].c8; e.out_pitch = lay[1].pitch; e.out_fstride = lay[1].fstride;
+        e.pj = OTIF_PJ_E12 > 0 ? pj : nullptr;
         auto kern = e.P == 384 ? e12_umma_kernel<3> : e12_umma_kernel<4>;
         OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->e12_smem));
         const int grid = e.ntiles < p->num_sms ? e.ntiles : p->num_sms;
