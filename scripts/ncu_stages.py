@@ -38,9 +38,10 @@ def main():
     # launch order in prof_stages.py (select launches K5 once, or twice with a deferred pass)
     order = ["resize", "select_random", "pack_full", "select_trained_C2", "select_trained_C2s", "pack_multi_C2s"]
     out, recs = [], []
-    seen = {"resize_even": 0, "select": 0, "pack": 0}
+    seen = {"resize": 0, "select": 0, "pack": 0}
+    rs_names = ["resize", "resize_C3"]
     sel_names = ["select_random", "select_trained_C2", "select_trained_C2s"]
-    pack_names = ["pack_full", "pack_multi_C2s"]
+    pack_names = ["pack_full", "pack_multi_C2s", "pack_full_C3"]
     for r in data:
         name = r[col["Kernel Name"]]
 
@@ -50,14 +51,15 @@ def main():
             v = float(r[col[m]].replace(",", ""))
             return v * SCALE.get(units[col[m]], 1)
         if "resize_even" in name:
-            key = "resize"
+            key = rs_names[min(seen["resize"], 1)]
+            seen["resize"] += 1
         elif "select_kernel" in name:
             # each select call launches K5 twice (the small-slice pass and the deferred
             # full-slice pass, usually empty): pair them up, report the pass-0 launch
             key = sel_names[min(seen["select"] // 2, 2)] + ("" if seen["select"] % 2 == 0 else "_pass1")
             seen["select"] += 1
         elif "pack_kernel" in name:
-            key = pack_names[min(seen["pack"], 1)]
+            key = pack_names[min(seen["pack"], 2)]
             seen["pack"] += 1
         else:
             continue

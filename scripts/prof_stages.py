@@ -75,6 +75,22 @@ def main():
             w2 = r2["windows"][:t2].cpu().numpy()
             out["pack_multi_C2s"] = {"algorithmic_bytes": int(2 * 3 * (w2[:, 3].astype(np.int64) * w2[:, 4]).sum()),
                                      "windows": t2, "fallback_share": float(((w2[:, 3] == 960) & (w2[:, 4] == 540)).sum() / n)}
+    # C3 (3000 1920x1080 UAV frames, BASELINE configs[2]): resize 1/4 and full-frame pack
+    del src
+    c3 = configs.C3
+    s3 = torch.empty((c3.n_frames, c3.src_h, c3.src_w, 3), dtype=torch.uint8, device="cuda")
+    video.make_scene(c3).render(range(c3.n_frames), out=s3)
+    torch.cuda.nvtx.range_push("prof")
+    otif.otif_resize(s3, c3.proxy_h, c3.proxy_w)
+    torch.cuda.nvtx.range_pop()
+    out["resize_C3"] = {"algorithmic_bytes": c3.n_frames * (2 * c3.proxy_h * c3.src_w * 3 + c3.proxy_h * c3.proxy_w * 3)}
+    full = torch.tensor([[f, 0, 0, c3.src_w, c3.src_h, 4] for f in range(c3.n_frames)], dtype=torch.int32,
+                        device="cuda")
+    tot = torch.tensor([c3.n_frames], dtype=torch.int32, device="cuda")
+    torch.cuda.nvtx.range_push("prof")
+    otif.otif_pack_windows(s3, c3.src_h, c3.src_w, full, tot, c3.sizes, [1, 1, 1, 1, c3.n_frames])
+    torch.cuda.nvtx.range_pop()
+    out["pack_full_C3"] = {"algorithmic_bytes": 2 * c3.n_frames * c3.src_h * c3.src_w * 3}
     torch.cuda.synchronize()
     print(json.dumps(out))
 
