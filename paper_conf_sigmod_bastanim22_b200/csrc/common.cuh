@@ -265,6 +265,28 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
 
+// ---- clusters: TMA multicast of a shared operand + multicast MMA-completion arrivals ----
+// 1-D bulk copy global -> the same shared offset in every CTA of cta_mask; each
+// destination's mbarrier (same offset) receives complete_tx for the bytes.
+__device__ __forceinline__ void bulk_g2s_mc(void *dst_smem, const void *src_gmem, uint32_t bytes, uint64_t *bar,
+                                            uint16_t cta_mask) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], %4;" ::"r"(
+            smem_u32(dst_smem)),
+        "l"(src_gmem), "r"(bytes), "r"(smem_u32(bar)), "h"(cta_mask)
+        : "memory");
+}
+// arrive (once) on the mbarrier at this shared offset in every CTA of cta_mask when this
+// thread's previously issued tcgen05.mma (cta_group::1) complete; elected lane of the warp
+__device__ __forceinline__ void umma_commit_mc_warp(uint64_t *bar, uint16_t cta_mask) {
+    asm volatile(
+        "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;\n\t}" ::"r"(
+            smem_u32(bar)),
+        "h"(cta_mask)
+        : "memory");
+}
+
 // ---- clusters and tcgen05 cta_group::2 (CTA pair sharing one M=256 MMA) ----
 __device__ __forceinline__ uint32_t cluster_ctarank() {
     uint32_t r;

@@ -51,6 +51,9 @@ namespace otif {
 // (measured, scripts/pj_ab.sh, profiles/r02_pack_overlap.md: hosting the copy in E4 or in
 // the latency-bound E1+E2 kernel costs about as much conv time as it saves)
 constexpr int kConvThreads = 256 + 32 * OTIF_PJ_WARPS;
+#ifndef OTIF_CONV_CL_LAYERS
+#define OTIF_CONV_CL_LAYERS 0     // GEMM layers (bit li: 0 = E2 .. 4 = D1) run as weight-sharing CTA pairs:
+#endif                            // parity-exact, no faster (profiles/r02i_cta_pairs.md), so off by default
 constexpr int kTileM = 128;
 constexpr int kMaxStagesA = 4;
 constexpr int kMaxStagesB = 8;
@@ -249,11 +252,23 @@ __global__ void __launch_bounds__(128) e1_umma_kernel(const __grid_constant__ E1
 // (N = 128 layers are shared-memory-bandwidth bound).  The accumulator is transposed
 // (TMEM lane = output channel, column = pixel); the head epilogue reduces the D2 dot
 // product across lanes (reduce-scatter shuffles) and across the 4 epilogue warps.
-template <int MT, bool SWAP = false>
+//
+// CL = 2 (cluster of two CTAs, each with its own M tiles and its own cta_group::1 MMAs):
+// the weights (B stages) are shared — each CTA bulk-copies HALF of every B stage with
+// .multicast::cluster into both CTAs' shared memory, and each MMA warp's "stage consumed"
+// commit is multicast to both CTAs' b_empty barriers (count 2), so a stage is refilled
+// only when both CTAs are done with it.  Per-SM L2 weight traffic halves (E4 / E5 stream
+// 0.6-1.2 MB of weights per 128-row tile: 11-18 TB/s of L2 reads per step).  The two CTAs
+// walk the same (cb, group, tap) sequence; an odd tile count gives the second CTA of the
+// last pair a dummy tile (A re-read from the last tile, no stores: q >= mtot).
+template <int MT, bool SWAP = false, int CL = 1>
 __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid_constant__ ConvParams p) {
     extern __shared__ __align__(1024) uint8_t smem[];
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
+    const int rank = CL == 2 ? (int)cluster_ctarank() : 0;
+    const int pair0 = blockIdx.x / CL, npairs = gridDim.x / CL;
+    const int ntp = (p.ntiles + CL - 1) / CL;   // tile pairs (tile = tp * CL + rank)
 
     const uint32_t chunks = p.kb >> 3;
     const uint32_t a_bytes = chunks * p.P * 16;
@@ -279,7 +294,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
     if (threadIdx.x == 0) {
         s_conv_done = 0;
         for (int i = 0; i < p.stages_a; i++) { mbar_init(&a_full[i], 1); mbar_init(&a_empty[i], 1); }
-        for (int i = 0; i < p.stages_b; i++) { mbar_init(&b_full[i], 1); mbar_init(&b_empty[i], 1); }
+        for (int i = 0; i < p.stages_b; i++) { mbar_init(&b_full[i], 1); mbar_init(&b_empty[i], CL); }
         for (int i = 0; i < 2; i++) { mbar_init(&t_full[i], 1); mbar_init(&t_empty[i], 128); }
         fence_barrier_init();
     }
@@ -290,6 +305,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
     }
     tc_fence_before();
     __syncthreads();
+    if (CL == 2) cluster_sync();   // the peer's barriers exist before any multicast reaches them
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
@@ -297,8 +313,10 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
         // ===== producer: halo (A) and weight (B) bulk copies =====
         if (lane == 0) {
             uint32_t as = 0, ap = 0, bs = 0, bp = 0;
-            for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
-                const int64_t q0 = (int64_t)tile * kTileM * MT;
+            const uint32_t b_half = b_bytes / CL;
+            for (int tp = pair0; tp < ntp; tp += npairs) {
+                const int tile = tp * CL + rank;
+                const int64_t q0 = (int64_t)(tile < p.ntiles ? tile : p.ntiles - 1) * kTileM * MT;
                 int tap_pos = 0;
                 for (int cb = 0; cb < p.ncb; cb++) {
                     tap_pos = 0;
@@ -316,8 +334,14 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                                                 for (int t = 0; t < p.group_ntaps[g]; t++, tap_pos++) {
                             mbar_wait(&b_empty[bs], bp ^ 1);
                             mbar_arrive_expect_tx(&b_full[bs], b_bytes);
-                            bulk_g2s(b_buf + (size_t)bs * b_bytes, p.wpk + ((size_t)cb * 9 + tap_pos) * b_bytes, b_bytes,
-                                     &b_full[bs]);
+                            if (CL == 2) {   // this CTA's half of the stage, into both CTAs
+                                bulk_g2s_mc(b_buf + (size_t)bs * b_bytes + rank * b_half,
+                                            p.wpk + ((size_t)cb * 9 + tap_pos) * b_bytes + rank * b_half, b_half,
+                                            &b_full[bs], 0x3);
+                            } else {
+                                bulk_g2s(b_buf + (size_t)bs * b_bytes, p.wpk + ((size_t)cb * 9 + tap_pos) * b_bytes,
+                                         b_bytes, &b_full[bs]);
+                            }
                             if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
                         }
                     }
@@ -331,7 +355,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
             uint32_t as = 0, ap = 0, bs = 0, bp = 0, acc = 0, accp = 0;
             const uint32_t a_base = smem_u32(a_buf), b_base = smem_u32(b_buf);
             const uint32_t lbo_a = p.P * 16, lbo_b = p.N * 16;
-            for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+            for (int tp = pair0; tp < ntp; tp += npairs) {
                 mbar_wait(&t_empty[acc], accp ^ 1);
                 tc_fence_after();
                 const uint32_t d = tmem_base + acc * MT * p.N;
@@ -362,7 +386,8 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
                                 }
                                 accumulate = 1;
                             }
-                            umma_commit_warp(&b_empty[bs]);
+                            if (CL == 2) umma_commit_mc_warp(&b_empty[bs], 0x3);   // both CTAs' stage
+                            else umma_commit_warp(&b_empty[bs]);
                             if (++bs == (uint32_t)p.stages_b) { bs = 0; bp ^= 1; }
                         }
                         umma_commit_warp(&a_empty[as]);
@@ -380,7 +405,8 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
         const float bias_c = s_bias[ch], w2_c = s_w2[ch];
         const int r = threadIdx.x - 128;
         uint32_t acc = 0, accp = 0;
-        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+        for (int tp = pair0; tp < ntp; tp += npairs) {
+            const int tile = tp * CL + rank;   // >= ntiles: dummy tile, q >= mtot, nothing stored
             mbar_wait(&t_full[acc], accp);
             tc_fence_after();
             const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * (kTileM * MT);
@@ -431,7 +457,8 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
         const int row = threadIdx.x - 128;          // TMEM lane == tile row
         const int quarter = warp & 3;               // lanes 32*quarter .. +31
         uint32_t acc = 0, accp = 0;
-        for (int tile = blockIdx.x; tile < p.ntiles; tile += gridDim.x) {
+        for (int tp = pair0; tp < ntp; tp += npairs) {
+            const int tile = tp * CL + rank;   // >= ntiles: dummy tile, q >= mtot, nothing stored
             mbar_wait(&t_full[acc], accp);
             tc_fence_after();
           for (int m = 0; m < MT; m++) {
@@ -488,6 +515,7 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
     __syncwarp();
     tc_fence_before();
     __syncthreads();
+    if (CL == 2) cluster_sync();   // no CTA leaves while its peer may still multicast into it
     if (warp == 2) {
         tc_fence_after();
         tmem_dealloc(tmem_base, tmem_cols);
@@ -1350,14 +1378,45 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         }
         size_t smem;
         conv_smem(g, c.stages_a, c.stages_b, smem);
-        int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
-        if (grid < 1) grid = 1;
         // head layer with N = 128: swapped operands (see conv_umma_kernel)
         const bool swap = c.out_kind == 3 && g.mt == 2 && g.cout == 128;
-        auto kern = swap ? conv_umma_kernel<2, true>
-                         : (g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>));
-        OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-        kern<<<grid, kConvThreads, smem, stream>>>(c);
+        // weight-sharing CTA pairs (CL = 2) for the layers in OTIF_CONV_CL_LAYERS
+#if OTIF_CONV_CL_LAYERS
+        const bool pair = ((OTIF_CONV_CL_LAYERS >> li) & 1) && c.ntiles >= 2 && p->num_sms >= 2;
+#else
+        constexpr bool pair = false;
+#endif
+        if (pair) {
+#if OTIF_CONV_CL_LAYERS
+            const int pairs_max = p->num_sms / 2;
+            const int ntp = (c.ntiles + 1) / 2;
+            const int pairs = ntp < pairs_max ? ntp : pairs_max;
+            auto kern = swap ? conv_umma_kernel<2, true, 2>
+                             : (g.mt == 4 ? conv_umma_kernel<4, false, 2>
+                                          : (g.mt == 2 ? conv_umma_kernel<2, false, 2> : conv_umma_kernel<1, false, 2>));
+            OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(2 * pairs);
+            cfg.blockDim = dim3(kConvThreads);
+            cfg.dynamicSmemBytes = smem;
+            cfg.stream = stream;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeClusterDimension;
+            attr[0].val.clusterDim.x = 2;
+            attr[0].val.clusterDim.y = 1;
+            attr[0].val.clusterDim.z = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            OTIF_CUDA(cudaLaunchKernelEx(&cfg, kern, c));
+#endif
+        } else {
+            int grid = c.ntiles < p->num_sms ? c.ntiles : p->num_sms;
+            if (grid < 1) grid = 1;
+            auto kern = swap ? conv_umma_kernel<2, true>
+                             : (g.mt == 4 ? conv_umma_kernel<4> : (g.mt == 2 ? conv_umma_kernel<2> : conv_umma_kernel<1>));
+            OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            kern<<<grid, kConvThreads, smem, stream>>>(c);
+        }
         OTIF_LAUNCH_CHECK();
         if (evs) OTIF_CUDA(cudaEventRecord(evs[1 + li], stream));
     }
