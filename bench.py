@@ -238,14 +238,14 @@ def measure_pipeline(otif, wl, blob, thr, src, steps, warmup, sizes=None, caps=N
     stage_ms, launches = pipe.stage_ms()
     ctr = pipe.counters()
     out = {"pipe": pipe, "ms_total": ms_total, "stage_ms": stage_ms, "launches": launches, "ctr": ctr,
-           "frames": n * steps, "steps": steps}
+           "frames": n * steps, "steps": steps, "overlap": overlap}
     return out
 
 
 CONV_STAGES = ["proxy_prep_e1", "conv_e2", "conv_e3", "conv_e4", "conv_e5", "conv_d1_head"]
 
 
-def rooflines(wl, m, peaks, peak_src, traffic=None):
+def rooflines(wl, m, peaks, peak_src, traffic=None, fused_pack=False):
     """Per-kernel rooflines of one measured pipeline: the proxy convolutions (tensor) against
     the measured bf16 burst peak (the timed regions are well under a second, at the
     maximum SM clock) with the sustained peak beside it; resize and pack (HBM) against
@@ -280,6 +280,13 @@ def rooflines(wl, m, peaks, peak_src, traffic=None):
     out = {"conv": conv}
     for k, byts in (("resize", rs_bytes), ("pack", pk_bytes)):
         ms = sm[k]
+        if k == "pack" and fused_pack:
+            # the copy runs inside the E5 / D1 kernels of the next step; "pack" holds only the
+            # slot kernel and the drain of what the fused warps left
+            out[k] = {"bound": "hbm", "fused_into": "conv_e5, conv_d1_head (next step)", "bytes_per_step": byts / steps,
+                      "slot_and_drain_ms_per_step": ms / steps,
+                      "hbm_frac_of_step": byts / steps / (float(m["ms_total"]) / steps / 1e3) / 1e9 / hbm}
+            continue
         gbs = byts / (ms / 1e3) / 1e9 if ms > 0 else None
         out[k] = {"bound": "hbm", "achieved": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm if gbs else None,
                   "frac_spec_8tbs": gbs / 8000.0 if gbs else None, "bytes_per_step": byts / steps,
@@ -352,7 +359,8 @@ def windowing_scenario(otif, otif_tuning, wl, src, rank, dev, peaks, peak_src, a
                               overlap=args.pack_overlap)
         out[f"trained_k{k}"] = {"frames_per_s": mw["frames"] / (mw["ms_total"] / 1e3),
                                 "ms_per_step": mw["ms_total"] / args.steps, "windows": window_stats(mw, wl, W),
-                                "roofline": rooflines(wl, mw, peaks, peak_src), "batch_cap": caps}
+                                "roofline": rooflines(wl, mw, peaks, peak_src, fused_pack=args.pack_overlap > 0),
+                                "batch_cap": caps}
         mw["pipe"].close()
         torch.cuda.empty_cache()
     # perfect proxy: stages 3-5 on the ground-truth cell masks of the measured frames
@@ -457,9 +465,18 @@ def run_otif(args):
             traffic = json.load(open(prof)).get("conv_dram_bytes_per_batch")
         except Exception:
             traffic = None
-    rl = rooflines(wl, m, peaks, peak_src, traffic)
+    rl = rooflines(wl, m, peaks, peak_src, traffic, fused_pack=args.pack_overlap > 0)
     launches = m["launches"]
     m["pipe"].close()
+    # the same pipeline with the serial stage-5 schedule (pack_overlap 0, 10 steps): every
+    # kernel alone on the GPU, so resize / pack / conv rooflines without the fused copy
+    serial = None
+    if extras and args.pack_overlap > 0:
+        ms_ = measure_pipeline(otif, wl, blob, b, src, 10, args.warmup, batch=args.batch or None, overlap=0)
+        rs_ = rooflines(wl, ms_, peaks, peak_src, traffic)
+        serial = {"frames_per_s": ms_["frames"] / (ms_["ms_total"] / 1e3), "ms_per_step": ms_["ms_total"] / 10,
+                  "rooflines": rs_, "note": "pack_overlap 0: stage 5 as its own kernel after the selection"}
+        ms_["pipe"].close()
 
     objs = {}
     # ---- the other BASELINE configs, each with its own rooflines and oracle sample
@@ -472,7 +489,7 @@ def run_otif(args):
             thr = threshold_for(cw.name)
             steps_c = max(args.steps, int(np.ceil(2000.0 / nn)) if nn < 1000 else args.steps)
             mc = measure_pipeline(otif, cw, blob, thr, s2, steps_c, args.warmup, overlap=args.pack_overlap)
-            r = rooflines(cw, mc, peaks, peak_src)
+            r = rooflines(cw, mc, peaks, peak_src, fused_pack=args.pack_overlap > 0)
             cfg[cw.name] = {"workload": f"{cw.src_w}x{cw.src_h} {cw.scene}, {nn} frames, proxy {cw.proxy_w}x{cw.proxy_h} "
                                         f"(S={cw.stride}), {cw.cell}-px cells, W={[list(x) for x in cw.sizes]}",
                             "frames_per_s": mc["frames"] / (mc["ms_total"] / 1e3),
@@ -597,6 +614,7 @@ def run_otif(args):
                              per_launch="5 launches per batch of 4500 frames; achieved = algorithmic FLOPs of "
                                         "E1..D1 / CUDA-event time of those launches on the pipeline stream"),
             "stages": {k: v for k, v in rl.items() if k != "conv"},
+            "serial_schedule": serial,
             **objs,
             "cpu_baseline": cpu_baseline,
             "e2e": e2e,
@@ -625,7 +643,7 @@ def run_c5(otif, odist, configs, video, blob, b, dev, world, rank, args):
     pool = torch.empty((configs.C5_POOL_CLIPS * fpc, wl.src_h, wl.src_w, 3), dtype=torch.uint8, device=dev)
     for j in range(configs.C5_POOL_CLIPS):
         video.make_scene(wl, clip=j).render(range(fpc), out=pool[j * fpc:(j + 1) * fpc])
-    pipe = otif.Pipeline(wl, blob, b, max_batch=fpc)
+    pipe = otif.Pipeline(wl, blob, b, max_batch=fpc, pack_overlap=args.pack_overlap)
     clips = odist.shard_clips(n_clips, world, rank)
 
     def run_clip(k):
@@ -637,6 +655,7 @@ def run_c5(otif, odist, configs, video, blob, b, dev, world, rank, args):
 
     for k in list(clips)[:2]:     # warm-up
         run_clip(k)
+    pipe.flush()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -646,6 +665,7 @@ def run_c5(otif, odist, configs, video, blob, b, dev, world, rank, args):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         per_clip = odist.run_corpus(clips, run_clip)
+        pipe.flush()              # the last clip's pack (pack_overlap 2) inside the timed pass
         e1.record()
         torch.cuda.synchronize()
         times.append(e0.elapsed_time(e1))
@@ -658,7 +678,8 @@ def run_c5(otif, odist, configs, video, blob, b, dev, world, rank, args):
     del pool
     torch.cuda.empty_cache()
     return {"what": f"{n_clips} one-minute 960x540 clips x {fpc} sampled frames (P:L99, P:L244), 8-clip pool, "
-                    f"contiguous clip ranges per rank; one pipeline call per clip",
+                    f"contiguous clip ranges per rank; one pipeline call per clip (pack of clip k under "
+                    f"clip k+1's proxy, pack_overlap {args.pack_overlap})",
             "frames_per_s": n_clips * fpc / (ms / 1e3), "ms_per_pass": ms, "passes": args.c5_passes,
             "scaling": "strong (fixed corpus)", "clips_per_rank": len(clips), "corpus": digest}
 

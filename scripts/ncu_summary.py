@@ -61,12 +61,17 @@ METRICS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.
 
 
 def to_bytes(v, unit):
-    f = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9}.get(unit, 1)
+    f = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "KB": 1e3, "MB": 1e6, "GB": 1e9,
+         "Tbyte": 1e12}.get(unit, 1)
     return float(v.replace(",", "")) * f
 
 
 def full(path, tag, names):
-    out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    if path.endswith(".csv"):     # raw page exported on the GPU box (the .ncu-rep stays there)
+        out = open(path).read()
+        out = out[out.index('"ID"'):]
+    else:
+        out = subprocess.run(["ncu", "-i", path, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     r = list(csv.reader(io.StringIO(out)))
     hdr, units, rows = r[0], r[1], r[2:]
     col = {h: i for i, h in enumerate(hdr)}
@@ -89,7 +94,15 @@ def full(path, tag, names):
              f"Source: `{os.path.basename(path)}` (one 4500-frame C2 batch, layers in capture order).", "",
              "| layer | time (us) | DRAM read (MB) | DRAM write (MB) | L2 bytes (MB) | tensor pipe % (mem_tensor) | "
              "tensor realtime % | DRAM % | regs |", "|---|---|---|---|---|---|---|---|---|"]
+    def num(v):
+        try:
+            return float(str(v).replace(",", ""))
+        except ValueError:
+            return 0.0
     for d in res:
+        for m in METRICS:
+            if m in d:
+                d[m] = num(d[m])
         t = d.get("gpu__time_duration.sum", 0)
         tu = d.get("gpu__time_duration.sum.unit", "")
         t_us = t / 1000 if tu in ("nsecond", "ns") else (t * 1000 if tu in ("msecond", "ms") else t)
@@ -108,7 +121,8 @@ def main():
     ap.add_argument("--launches")
     ap.add_argument("--full")
     ap.add_argument("--tag", required=True)
-    ap.add_argument("--layers", default="E2,E3,E4,E5,D1")
+    ap.add_argument("--layers", default="E1+E2,E3,E4,E5,D1")
+    ap.add_argument("--no-traffic", action="store_true", help="do not update conv_dram_bytes_per_batch")
     args = ap.parse_args()
     os.makedirs(PROF, exist_ok=True)
     summ_path = os.path.join(PROF, "ncu_summary.json")
@@ -118,8 +132,9 @@ def main():
         summ["launch_shares"] = launches(args.launches, args.tag)
     if args.full:
         res = full(args.full, args.tag, args.layers.split(","))
-        summ["conv_full"] = res
-        summ["conv_dram_bytes_per_batch"] = sum(d.get("dram__bytes_read.sum", 0) + d.get("dram__bytes_write.sum", 0)
+        summ["conv_full" if not args.no_traffic else f"conv_full_{args.tag}"] = res
+        if not args.no_traffic:
+            summ["conv_dram_bytes_per_batch"] = sum(d.get("dram__bytes_read.sum", 0) + d.get("dram__bytes_write.sum", 0)
                                                 for d in res)
     json.dump(summ, open(summ_path, "w"), indent=1)
     print(json.dumps({k: v for k, v in summ.items() if k != "conv_full"}, indent=1)[:3000])
