@@ -51,6 +51,10 @@ namespace otif {
 // (measured, scripts/pj_ab.sh, profiles/r02_pack_overlap.md: hosting the copy in E4 or in
 // the latency-bound E1+E2 kernel costs about as much conv time as it saves)
 constexpr int kConvThreads = 256 + 32 * OTIF_PJ_WARPS;
+#ifndef OTIF_E12B
+#define OTIF_E12B 0   // band variant of the fused E1+E2 kernel (A/B builds: 1 = band where it fits);
+#endif            // parity-exact but 1.07 vs 0.88 ms per C2 step (profiles/r02l_e12_band.md)
+#define OTIF_E12B_BUILD OTIF_E12B
 #ifndef OTIF_CONV_CL_LAYERS
 #define OTIF_CONV_CL_LAYERS 0     // GEMM layers (bit li: 0 = E2 .. 4 = D1) run as weight-sharing CTA pairs:
 #endif                            // parity-exact, no faster (profiles/r02i_cta_pairs.md), so off by default
@@ -993,6 +997,409 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
     }
 }
 
+#if OTIF_E12B_BUILD
+// ---------------------------------------------------------------------------
+// E1 fused into E2, "band" variant (e12b).  Same arithmetic as e12_umma_kernel (exact fp16
+// im2col rows u - 128 against w * 2^s, bias folded into K, E2 weights * 2^-(s+7)), but the
+// unit of work is a BAND: R consecutive E2 output rows of one frame (M = 256 positions,
+// R * pitch <= 256 valid) with ALL FOUR parity planes of its E1 input computed at once
+// (4 x PB plane-buffer rows, PB >= 256 + pitch + 1).  Per band there are four hand-offs
+// (gather -> E1 MMA -> E1 epilogue -> E2 MMA) instead of sixteen per 256-position tile,
+// and consecutive bands of a frame share image rows through a ring (only 4R new image
+// rows per band are loaded).  Buffers are single-stage (A1 im2col 256 PB B, planes
+// 256 PB B, E1 accumulators PB TMEM columns, E2 accumulators 128 columns); E2's weights
+// stream through a 3-stage ring of per-tap stages.  Roles (768 threads): warp 0 image-row
+// loader, warp 1 E1 MMA, warp 2 TMEM allocator then weight-stage loader, warp 3 E2 MMA,
+// warps 4-11 gather (5 im2col rows per thread), 12-19 E1 epilogue (alternate 128-row
+// sub-tiles), 20-23 E2 epilogue.
+// ---------------------------------------------------------------------------
+struct E12bParams {
+    const uint8_t *img;         // u8 [n, hp, wp, 3]
+    int n, hp, wp, row_bytes;
+    int h1, w1, h2, w2, pitch;  // E1 / E2 output sizes; pitch = w2 + 1 (E2-input plane layout)
+    int R;                      // E2 output rows per band
+    int nbpf;                   // bands per frame = ceil(h2 / R)
+    int njobs;                  // n * nbpf
+    int PB;                     // plane-buffer rows (multiple of 32)
+    int D;                      // (PB - 1) / pitch: plane rows spanned beyond the band's first
+    int NR;                     // image rows per band = 4 D + 5
+    int RC;                     // image-row ring capacity (rows) = 2 NR
+    int ring_pitch;             // bytes per ring row (16-B left pad, row, right pad)
+    int bulk;                   // rows may be bulk-copied (16-B aligned)
+    FastDiv div_pitch, div_PB, div_RC;
+    const uint16_t *wt1;        // fp16 [4 chunks][32 n][8] (as e12)
+    const uint16_t *wt2;        // bf16 [9 taps in loop order][4 chunks][64 n][8] (as e12)
+    const float *b2;
+    int group_ntaps[4], group_shift[4][9];
+    int out_kind;
+    uint8_t *out;
+    int64_t out_lcap;
+    int out_c8, out_pitch;
+    int64_t out_fstride;
+};
+
+constexpr int kE12bThreads = 768;
+constexpr int kE12bW2Stages = 3;
+
+// job index -> (frame, band) and whether it continues the previous job's frame band
+__device__ __forceinline__ void e12b_job(const E12bParams &p, int j, int &f, int &b) {
+    f = j / p.nbpf;
+    b = j - f * p.nbpf;
+}
+
+// One E1 im2col row (fp16, K = 32 with the bias slots), as e12_im2col_row, from three
+// ring rows (image rows 2y-1, 2y, 2y+1) at byte offset `off` (column 2x-1, can be the pad)
+__device__ __forceinline__ void e12b_im2col_row(const uint8_t *r0, const uint8_t *r1, const uint8_t *r2, uint32_t off,
+                                                uint32_t (&wv)[16]) {
+    const uint32_t sh = (off & 3) * 8;
+    const uint8_t *rows[3] = {r0, r1, r2};
+#pragma unroll
+    for (int kh = 0; kh < 3; kh++) {
+        const uint32_t *wp = reinterpret_cast<const uint32_t *>(rows[kh] + (off & ~3u));
+        const uint32_t w0 = wp[0], w1 = wp[1], w2 = wp[2];
+        const uint32_t a0 = __funnelshift_r(w0, w1, sh), a1 = __funnelshift_r(w1, w2, sh);
+        wv[5 * kh + 0] = sub_f16x2(__byte_perm(a0, 0x64646464u, 0x4140), 0x64806480u);
+        wv[5 * kh + 1] = sub_f16x2(__byte_perm(a0, 0x64646464u, 0x4342), 0x64806480u);
+        wv[5 * kh + 2] = sub_f16x2(__byte_perm(a1, 0x64646464u, 0x4140), 0x64806480u);
+        wv[5 * kh + 3] = sub_f16x2(__byte_perm(a1, 0x64646464u, 0x4342), 0x64806480u);
+        wv[5 * kh + 4] = sub_f16x2(0x64006400u | ((w2 >> sh) & 0xFFu), 0x63006480u);
+    }
+    wv[15] = 0;
+}
+
+#ifdef OTIF_E12_TRACE_BUILD   // timeline of CTA 0, bands 20..35 (debug builds only)
+#define E12B_TR_DECL const bool trb = blockIdx.x == 0 && (threadIdx.x & 31) == 0; long long tb[3][16]; const long long tb0 = clock64();
+#define E12B_TR(slot) do { if (trb && k >= 20 && k < 36) tb[slot][k - 20] = clock64() - tb0; } while (0)
+#define E12B_TR_DUMP(name) do { if (trb && (threadIdx.x == 0 || threadIdx.x == 32 || threadIdx.x == 96 || threadIdx.x == 128 || threadIdx.x == 384 || threadIdx.x == 640)) \
+    for (int q_ = 0; q_ < 16 && q_ + 20 < (j1 - j0); q_++) printf("%s k=%2d %8lld %8lld %8lld\n", name, q_ + 20, tb[0][q_], tb[1][q_], tb[2][q_]); } while (0)
+#else
+#define E12B_TR_DECL
+#define E12B_TR(slot) do {} while (0)
+#define E12B_TR_DUMP(name) do {} while (0)
+#endif
+__global__ void __launch_bounds__(kE12bThreads, 1) e12b_umma_kernel(const __grid_constant__ E12bParams p) {
+    extern __shared__ __align__(1024) uint8_t smem[];
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    constexpr int N2 = 64;
+    constexpr uint32_t kW2Stage = 4 * N2 * 16;         // one tap: [4 chunks][64 n][8] bf16 = 4 KB
+    constexpr uint32_t kW1Bytes = 4 * 32 * 16;
+    const int PB = p.PB;
+    const int nsub = 4 * PB / 128;                     // E1 M sub-tiles per band
+    const uint32_t a1_bytes = (uint32_t)nsub * 8192;   // [sub][chunk][128 rows][16 B]
+    const uint32_t pl_bytes = (uint32_t)PB * 64;       // one plane: [chunk][PB rows][16 B]
+    const uint32_t ring_bytes = (uint32_t)p.RC * p.ring_pitch;
+
+    uint8_t *a1_s = smem;
+    uint8_t *pl_s = a1_s + a1_bytes;
+    uint8_t *w2_s = pl_s + 4 * pl_bytes;
+    uint8_t *w1_s = w2_s + kE12bW2Stages * kW2Stage;
+    uint8_t *ring_s = w1_s + kW1Bytes;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(ring_s + ring_bytes);
+    uint64_t *ring_full = bars, *ring_empty = bars + 2;
+    uint64_t *w2_full = bars + 4, *w2_empty = w2_full + kE12bW2Stages;
+    uint64_t *a1_full = w2_empty + kE12bW2Stages, *a1_empty = a1_full + 1;
+    uint64_t *e1_full = a1_empty + 1, *e1_empty = e1_full + 1;
+    uint64_t *pl_full = e1_empty + 1, *pl_empty = pl_full + 1;
+    uint64_t *acc_full = pl_empty + 1, *acc_empty = acc_full + 1;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acc_empty + 1);
+    float *s_b2 = reinterpret_cast<float *>(tmem_slot + 4);
+
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < 2; i++) { mbar_init(&ring_full[i], 1); mbar_init(&ring_empty[i], 256); }
+        for (int i = 0; i < kE12bW2Stages; i++) { mbar_init(&w2_full[i], 1); mbar_init(&w2_empty[i], 1); }
+        mbar_init(a1_full, 256); mbar_init(a1_empty, 1);
+        mbar_init(e1_full, 1); mbar_init(e1_empty, 256);
+        mbar_init(pl_full, 256); mbar_init(pl_empty, 1);
+        mbar_init(acc_full, 1); mbar_init(acc_empty, 128);
+        fence_barrier_init();
+    }
+    if (warp == 2) tmem_alloc(tmem_slot, 512);
+    for (uint32_t i = threadIdx.x; i < kW1Bytes / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(w1_s)[i] = reinterpret_cast<const uint4 *>(p.wt1)[i];
+    // ring: every byte 128 (x = 0): the pads around each row are never written again
+    for (uint32_t i = threadIdx.x; i < ring_bytes / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(ring_s)[i] = make_uint4(0x80808080u, 0x80808080u, 0x80808080u, 0x80808080u);
+    if (threadIdx.x < N2) s_b2[threadIdx.x] = p.b2[threadIdx.x];
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    constexpr uint32_t kE1Col = 128;                  // E2 accumulators: columns [0, 128)
+
+    // contiguous job range of this CTA (consecutive bands of a frame share image rows)
+    const int j0 = (int)((int64_t)blockIdx.x * p.njobs / gridDim.x);
+    const int j1 = (int)((int64_t)(blockIdx.x + 1) * p.njobs / gridDim.x);
+    E12B_TR_DECL
+
+    if (warp == 0) {
+        // ===== loader: image rows of each band into the ring =====
+        int seq_base = -p.NR, pf = -1, pb = -1;
+        for (int j = j0, k = 0; j < j1; j++, k++) {
+            int f, b;
+            e12b_job(p, j, f, b);
+            const bool cont = (f == pf && b == pb + 1);
+            const int fresh0 = cont ? p.NR - 4 * p.R : 0;   // first band-relative row to load
+            seq_base = cont ? seq_base + 4 * p.R : seq_base + p.NR;
+            pf = f; pb = b;
+            const int Y0 = 4 * b * p.R - 5;
+            E12B_TR(0);
+            // band k-2's rows are free once its gather is done
+            mbar_wait(&ring_empty[k & 1], ((k >> 1) & 1) ^ 1);
+            E12B_TR(1);
+            uint32_t my_bytes = 0;
+            for (int i = fresh0 + lane; i < p.NR; i += 32) {
+                const int y = Y0 + i;
+                if (y >= 0 && y < p.hp) my_bytes += p.row_bytes;
+            }
+            if (p.bulk) {
+#pragma unroll
+                for (int o = 16; o >= 1; o >>= 1) my_bytes += __shfl_xor_sync(0xffffffffu, my_bytes, o);
+                if (lane == 0 && my_bytes) mbar_expect_tx(&ring_full[k & 1], my_bytes);
+                __syncwarp();
+            }
+            for (int i = fresh0 + lane; i < p.NR; i += 32) {
+                const int y = Y0 + i;
+                const uint32_t slot = (uint32_t)(seq_base + i) - fdiv((uint32_t)(seq_base + i), p.div_RC) * p.RC;
+                uint8_t *dst = ring_s + (size_t)slot * p.ring_pitch + 16;
+                if (y >= 0 && y < p.hp) {
+                    const uint8_t *src = p.img + ((size_t)f * p.hp + y) * p.row_bytes;
+                    if (p.bulk) {
+                        bulk_g2s(dst, src, p.row_bytes, &ring_full[k & 1]);
+                    } else {
+#pragma unroll 1
+                        for (int q = 0; q < p.row_bytes; q++) dst[q] = __ldg(src + q);
+                    }
+                } else {
+#pragma unroll 1
+                    for (int q = 0; q < p.row_bytes; q += 4)
+                        *reinterpret_cast<uint32_t *>(dst + q) = 0x80808080u;
+                }
+            }
+            __threadfence_block();
+            __syncwarp();
+            if (lane == 0) mbar_arrive(&ring_full[k & 1]);
+            E12B_TR(2);
+        }
+        E12B_TR_DUMP("LOAD");
+    } else if (warp == 2) {
+        // ===== weight loader (after the TMEM allocation): the nine E2 tap stages per band =====
+        if (lane == 0) {
+            uint32_t ws = 0, wph = 0;
+            for (int j = j0; j < j1; j++) {
+#pragma unroll 1
+                for (int t = 0; t < 9; t++) {
+                    mbar_wait(&w2_empty[ws], wph ^ 1);
+                    mbar_arrive_expect_tx(&w2_full[ws], kW2Stage);
+                    bulk_g2s(w2_s + ws * kW2Stage, reinterpret_cast<const uint8_t *>(p.wt2) + t * kW2Stage, kW2Stage,
+                             &w2_full[ws]);
+                    if (++ws == kE12bW2Stages) { ws = 0; wph ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ===== E1 MMA issuer (whole warp, elected lane): nsub x 2 MMAs per band =====
+        const uint32_t idesc1 = umma_idesc_f16(128, 32);
+        const uint64_t a1d = umma_desc(smem_u32(a1_s), 2048, 128);
+        const uint64_t w1d = umma_desc(smem_u32(w1_s), 512, 128);
+        for (int j = j0, k = 0; j < j1; j++, k++) {
+            mbar_wait(a1_full, k & 1);
+            E12B_TR(0);
+            mbar_wait(e1_empty, (k & 1) ^ 1);
+            E12B_TR(1);
+            tc_fence_after();
+#pragma unroll 1
+            for (int m = 0; m < nsub; m++)
+#pragma unroll
+                for (int s = 0; s < 2; s++)
+                    umma_bf16_warp(tmem_base + kE1Col + m * 32, a1d + ((m * 8192 + 2 * s * 2048) >> 4),
+                                   w1d + ((2 * s * 512) >> 4), idesc1, s);
+            umma_commit_warp(a1_empty);
+            umma_commit_warp(e1_full);
+            E12B_TR(2);
+        }
+        E12B_TR_DUMP("E1MMA");
+    } else if (warp == 3) {
+        // ===== E2 MMA issuer: 9 taps x 2 K halves x 2 M sub-tiles per band =====
+        const uint32_t idesc2 = umma_idesc_bf16(128, N2);
+        const uint64_t pld = umma_desc(smem_u32(pl_s), PB * 16, 128);
+        const uint64_t w2d = umma_desc(smem_u32(w2_s), N2 * 16, 128);
+        uint32_t ws = 0, wph = 0;
+        for (int j = j0, k = 0; j < j1; j++, k++) {
+            mbar_wait(pl_full, k & 1);
+            E12B_TR(0);
+            mbar_wait(acc_empty, (k & 1) ^ 1);
+            E12B_TR(1);
+            tc_fence_after();
+            int pos = 0;
+#pragma unroll 1
+            for (int g = 0; g < 4; g++) {
+                const uint64_t a = pld + ((g * pl_bytes) >> 4);
+#pragma unroll 1
+                for (int t = 0; t < p.group_ntaps[g]; t++, pos++) {
+                    mbar_wait(&w2_full[ws], wph);
+                    tc_fence_after();
+                    const uint64_t at = a + p.group_shift[g][t];          // +16 B per position
+                    const uint64_t bt = w2d + ((ws * kW2Stage) >> 4);
+#pragma unroll
+                    for (int s = 0; s < 2; s++)
+#pragma unroll
+                        for (int mm = 0; mm < 2; mm++)
+                            umma_bf16_warp(tmem_base + mm * N2, at + ((2 * s * PB * 16 + mm * 2048) >> 4),
+                                           bt + ((2 * s * N2 * 16) >> 4), idesc2, (pos == 0 && s == 0) ? 0u : 1u);
+                    umma_commit_warp(&w2_empty[ws]);
+                    if (++ws == kE12bW2Stages) { ws = 0; wph ^= 1; }
+                }
+            }
+            umma_commit_warp(pl_empty);
+            umma_commit_warp(acc_full);
+            E12B_TR(2);
+        }
+        E12B_TR_DUMP("E2MMA");
+    } else if (warp >= 4 && warp < 12) {
+        // ===== gather: the band's 4 x PB im2col rows (plane g = r / PB, row j = r % PB) =====
+        const int gt = threadIdx.x - 128;            // 0..255
+        int seq_base = -p.NR, pf = -1, pb = -1;
+        for (int j = j0, k = 0; j < j1; j++, k++) {
+            int f, b;
+            e12b_job(p, j, f, b);
+            const bool cont = (f == pf && b == pb + 1);
+            seq_base = cont ? seq_base + 4 * p.R : seq_base + p.NR;
+            pf = f; pb = b;
+            const int oy0 = b * p.R;
+            const int Y0 = 4 * oy0 - 5;
+            mbar_wait(&ring_full[k & 1], (k >> 1) & 1);
+            E12B_TR(0);
+            mbar_wait(a1_empty, (k & 1) ^ 1);
+            E12B_TR(1);
+#pragma unroll 1
+            for (int r = gt; r < 4 * PB; r += 256) {
+                const uint32_t g = fdiv((uint32_t)r, p.div_PB);
+                const uint32_t jj = (uint32_t)r - g * (uint32_t)PB;
+                const uint32_t pp = (uint32_t)(oy0 * p.pitch) + jj;
+                const uint32_t pr = fdiv(pp, p.div_pitch);
+                const uint32_t pc = pp - pr * (uint32_t)p.pitch;
+                const int rp = (int)(g >> 1), cp = (int)(g & 1);
+                const int y = 2 * ((int)pr - 1) + rp, x = 2 * ((int)pc - 1) + cp;
+                const bool valid = pr >= 1 && (int)pr <= p.h2 && pc >= 1 && (int)pc <= p.w2 && y < p.h1 && x < p.w1;
+                uint32_t wv[16];
+                if (valid) {
+                    const uint8_t *rr[3];
+#pragma unroll
+                    for (int kh = 0; kh < 3; kh++) {
+                        const uint32_t s = (uint32_t)(seq_base + (2 * y - 1 + kh - Y0));
+                        const uint32_t slot = s - fdiv(s, p.div_RC) * p.RC;
+                        rr[kh] = ring_s + (size_t)slot * p.ring_pitch;
+                    }
+                    e12b_im2col_row(rr[0], rr[1], rr[2], (uint32_t)(6 * x + 13), wv);
+                } else {
+#pragma unroll
+                    for (int q = 0; q < 16; q++) wv[q] = 0;
+                }
+                uint8_t *dst = a1_s + (size_t)(r >> 7) * 8192 + (r & 127) * 16;
+#pragma unroll
+                for (int c = 0; c < 4; c++)
+                    *reinterpret_cast<uint4 *>(dst + c * 2048) = make_uint4(wv[4 * c], wv[4 * c + 1], wv[4 * c + 2], wv[4 * c + 3]);
+            }
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive(a1_full);
+            mbar_arrive(&ring_empty[k & 1]);
+            E12B_TR(2);
+        }
+        E12B_TR_DUMP("GATH");
+    } else if (warp >= 12 && warp < 20) {
+        // ===== E1 epilogue: TMEM -> ReLU, bf16 -> plane buffers (E2's A operand) =====
+        const int wg = (warp - 12) >> 2;
+        const int quarter = warp & 3;
+        const int lrow = quarter * 32 + lane;
+        for (int j = j0, k = 0; j < j1; j++, k++) {
+            mbar_wait(e1_full, k & 1);
+            E12B_TR(0);
+            mbar_wait(pl_empty, (k & 1) ^ 1);
+            E12B_TR(1);
+            tc_fence_after();
+#pragma unroll 1
+            for (int m = wg; m < nsub; m += 2) {
+                uint32_t v[32];
+                tmem_ld32(tmem_base + ((uint32_t)(quarter * 32) << 16) + kE1Col + m * 32, v);
+                uint32_t pk[16];
+#pragma unroll
+                for (int q = 0; q < 16; q++) pk[q] = pack_bf16x2_relu(__uint_as_float(v[2 * q]), __uint_as_float(v[2 * q + 1]));
+                const uint32_t r = (uint32_t)(m * 128 + lrow);
+                const uint32_t g = fdiv(r, p.div_PB);
+                const uint32_t jj = r - g * (uint32_t)PB;
+                uint8_t *dst = pl_s + (size_t)g * pl_bytes + (size_t)jj * 16;
+#pragma unroll
+                for (int c = 0; c < 4; c++)
+                    *reinterpret_cast<uint4 *>(dst + (size_t)c * PB * 16) =
+                        make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+            }
+            tc_fence_before();
+            mbar_arrive(e1_empty);
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive(pl_full);
+            E12B_TR(2);
+        }
+        E12B_TR_DUMP("E1EP");
+    } else if (warp >= 20) {
+        // ===== E2 epilogue: TMEM -> bias, ReLU, bf16 -> E3's input layout =====
+        const int row = threadIdx.x - 640;
+        const int quarter = warp & 3;
+        for (int j = j0, k = 0; j < j1; j++, k++) {
+            int f, b;
+            e12b_job(p, j, f, b);
+            const int oy0 = b * p.R;
+            const int oy_end = min(oy0 + p.R, p.h2);
+            E12B_TR(0);
+            mbar_wait(acc_full, k & 1);
+            E12B_TR(1);
+            tc_fence_after();
+#pragma unroll 1
+            for (int mm = 0; mm < 2; mm++) {
+                const uint32_t qr = (uint32_t)(oy0 * p.pitch + mm * 128 + row);
+                const uint32_t oy = fdiv(qr, p.div_pitch);
+                const int ox = (int)(qr - oy * (uint32_t)p.pitch);
+                const bool valid = (int)oy < oy_end && ox < p.w2;
+                int plane = 0;
+                const int64_t L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, f, (int)oy, ox, plane);
+                const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + mm * N2;
+                uint8_t *const row_out = p.out + ((int64_t)plane * p.out_c8 * p.out_lcap + L) * 16;
+                const int64_t chunk_stride = p.out_lcap * 16;
+#pragma unroll
+                for (int cc = 0; cc < N2 / 32; cc++) {
+                    uint32_t v[32];
+                    tmem_ld32(taddr + cc * 32, v);
+                    if (valid) {
+                        uint32_t pk[16];
+#pragma unroll
+                        for (int q = 0; q < 16; q++)
+                            pk[q] = pack_bf16x2_relu(__uint_as_float(v[2 * q]) + s_b2[cc * 32 + 2 * q],
+                                                     __uint_as_float(v[2 * q + 1]) + s_b2[cc * 32 + 2 * q + 1]);
+#pragma unroll
+                        for (int c = 0; c < 4; c++)
+                            *reinterpret_cast<uint4 *>(row_out + (cc * 4 + c) * chunk_stride) =
+                                make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+                    }
+                }
+            }
+            tc_fence_before();
+            mbar_arrive(acc_empty);
+            E12B_TR(2);
+        }
+        E12B_TR_DUMP("E2EP");
+    }
+    __syncwarp();
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        tmem_dealloc(tmem_base, 512);
+    }
+}
+
+#endif  // OTIF_E12B_BUILD
+
 // ---------------------------------------------------------------------------
 // host side: plan, weight packing, launch
 // ---------------------------------------------------------------------------
@@ -1038,6 +1445,9 @@ struct otif_proxy {
     int e12;
     int e12_P, e12_np, e12_na1, e12_slab_rows, e12_slab_pitch;
     size_t e12_smem, e12_fixed, e12_unit;
+    // band variant of the fused E1+E2 kernel (e12b_umma_kernel); 0 = tile variant
+    int e12b, e12b_R, e12b_PB, e12b_D, e12b_NR, e12b_RC, e12b_ring_pitch;
+    size_t e12b_smem;
     uint16_t *e12_w1_dev;         // fp16 [4][32][8] = bf16(w1) * 2^s, K = kh*10 + kw*3 + c; bias parts at K = 9, 19, 29
     uint16_t *e12_w2_dev;         // E2's packed bf16 weights * 2^-(s+7)
     uint64_t plan_hash;
@@ -1242,6 +1652,30 @@ static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const f
     return true;
 }
 
+// Plan the band variant (needs the tile variant's scaled weights): R E2 rows per band with
+// R * pitch <= 256, plane buffers of PB >= 256 + pitch + 1 rows; fits TMEM (128 + PB
+// columns) and shared memory.
+static bool plan_e12b(otif_proxy *p) {
+    if (!OTIF_E12B || !p->e12) return false;
+    const GemmLayer &g = p->L[0];
+    const int pitch = g.pitch;
+    const int R = 256 / pitch;
+    if (R < 1) return false;
+    const int PB = (int)round_up(256 + pitch + 1, 32);
+    if (128 + PB > 512) return false;
+    const int D = (PB - 1) / pitch;
+    const int NR = 4 * D + 5;
+    const int RC = 2 * NR;
+    const int ring_pitch = (int)round_up(16 + 3 * p->d.in_w + 32, 16);
+    const size_t smem = (size_t)(4 * PB / 128) * 8192 + (size_t)4 * PB * 64 + 3 * 4096 + 2048 +
+                        (size_t)RC * ring_pitch + 32 * 8 + 16 + 64 * 4 + 1024;
+    if (smem > 227 * 1024) return false;
+    p->e12b_R = R; p->e12b_PB = PB; p->e12b_D = D; p->e12b_NR = NR; p->e12b_RC = RC;
+    p->e12b_ring_pitch = ring_pitch;
+    p->e12b_smem = smem;
+    return true;
+}
+
 // kernel launches of one launch_proxy call (workspace zero + tag, E1+E2 fused or E1 and E2, E3..D1)
 int proxy_launches(const otif_proxy *p) { return p->e12 ? 7 : 8; }
 
@@ -1292,6 +1726,39 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
     OTIF_LAUNCH_CHECK();
 
     const bool e12 = p->e12 && (int64_t)n * p->L[0].fstride_unit + 4096 < (1ll << 31);
+#if OTIF_E12B_BUILD
+    if (e12 && p->e12b) {
+        // E1 fused into E2, band variant: one kernel writes E3's input
+        if (evs) OTIF_CUDA(cudaEventRecord(evs[0], stream));
+        const GemmLayer &g = p->L[0];
+        E12bParams e;
+        memset(&e, 0, sizeof(e));
+        e.img = img; e.n = n; e.hp = p->d.in_h; e.wp = p->d.in_w; e.row_bytes = 3 * p->d.in_w;
+        e.h1 = p->e1_oh; e.w1 = p->e1_ow; e.h2 = g.out_h; e.w2 = g.out_w; e.pitch = g.pitch;
+        e.R = p->e12b_R;
+        e.nbpf = (e.h2 + e.R - 1) / e.R;
+        e.njobs = n * e.nbpf;
+        e.PB = p->e12b_PB; e.D = p->e12b_D; e.NR = p->e12b_NR; e.RC = p->e12b_RC;
+        e.ring_pitch = p->e12b_ring_pitch;
+        e.bulk = (e.row_bytes % 16 == 0) && (((uintptr_t)img & 15) == 0);
+        e.div_pitch = make_fastdiv((uint32_t)g.pitch);
+        e.div_PB = make_fastdiv((uint32_t)e.PB);
+        e.div_RC = make_fastdiv((uint32_t)e.RC);
+        e.wt1 = p->e12_w1_dev; e.wt2 = p->e12_w2_dev; e.b2 = g.bias_dev;
+        for (int i = 0; i < 4; i++) {
+            e.group_ntaps[i] = g.group_ntaps[i];
+            for (int t = 0; t < 9; t++) e.group_shift[i][t] = g.group_shift[i][t];
+        }
+        e.out_kind = lay[1].kind; e.out = ws + lay[1].offset; e.out_lcap = lay[1].lcap;
+        e.out_c8 = lay[1].c8; e.out_pitch = lay[1].pitch; e.out_fstride = lay[1].fstride;
+        OTIF_CUDA(cudaFuncSetAttribute(e12b_umma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)p->e12b_smem));
+        const int grid = e.njobs < p->num_sms ? e.njobs : p->num_sms;
+        e12b_umma_kernel<<<grid, kE12bThreads, p->e12b_smem, stream>>>(e);
+        OTIF_LAUNCH_CHECK();
+        if (evs) OTIF_CUDA(cudaEventRecord(evs[1], stream));
+    } else
+#endif
     if (e12) {
         // E1 fused into E2: one kernel writes E3's input
         if (evs) OTIF_CUDA(cudaEventRecord(evs[0], stream));
@@ -1549,6 +2016,7 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
         }
     }
     if (rc == OTIF_OK) p->e12 = plan_e12(p, weights + offs[0], weights + offs[0] + 32 * 27) ? 1 : 0;
+    if (rc == OTIF_OK) p->e12b = plan_e12b(p) ? 1 : 0;
     if (cudaGetLastError() != cudaSuccess && rc == OTIF_OK) rc = OTIF_ECUDA;
     if (rc != OTIF_OK) {
         otif_proxy_destroy(p);
@@ -1560,6 +2028,7 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
     for (int i = 0; i < 5; i++) mix(d->enc[i]);
     mix(d->dec);
     mix(p->e12);
+    mix(p->e12b);
     p->plan_hash = hsh | 1;
     *out = p;
     return OTIF_OK;
