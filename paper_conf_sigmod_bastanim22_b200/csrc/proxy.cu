@@ -557,13 +557,16 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
 #define OTIF_PJ_E12 0            // fused pack copy warps in the E1+E2 kernel (A/B builds; 0 = none)
 #endif
 constexpr int kE12Threads = 768 + 32 * OTIF_PJ_E12;
+#ifndef OTIF_E12_TS
+#define OTIF_E12_TS 0         // 1: E1's im2col rows in TMEM (two buffers, tcgen05.st by the gather,
+#endif                        //    A-from-TMEM MMAs): 194 KB less shared-memory traffic per tile
 #ifndef OTIF_E12_ACC
-#define OTIF_E12_ACC 2        // E2 accumulator stages (A/B builds)
+#define OTIF_E12_ACC (OTIF_E12_TS ? 1 : 2)   // E2 accumulator stages (A/B builds; TS needs the TMEM of one)
 #endif
 #ifndef OTIF_E12_E1SLOTS
 #define OTIF_E12_E1SLOTS 2    // E1 accumulator slots (A/B builds; 3 needs OTIF_E12_ACC=1)
 #endif
-constexpr int kE12MaxPlaneBufs = 3;
+constexpr int kE12MaxPlaneBufs = 4;
 
 struct E12Params {
     const uint8_t *img;         // u8 [n, hp, wp, 3]
@@ -679,7 +682,9 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
     // TMEM: E2 accumulators kAccStages x (MT x 64) at 0, E1 accumulators kE1Slots x 32 KT
     constexpr int kAccStages = OTIF_E12_ACC, kE1Slots = OTIF_E12_E1SLOTS;
     constexpr uint32_t kE1Col = kAccStages * 2 * 64;
-    static_assert(kE1Col + kE1Slots * 32 * KT <= 512, "TMEM budget");
+    // TS: two im2col buffers of KT x 16 columns (K = 32 fp16 per row) after the E1 slots
+    constexpr uint32_t kA1Col = kE1Col + kE1Slots * 32 * KT;
+    static_assert(kA1Col + (OTIF_E12_TS ? 2 * 16 * KT : 0) <= 512, "TMEM budget");
     extern __shared__ __align__(1024) uint8_t smem[];
     const int warp = threadIdx.x >> 5;
     const int lane = threadIdx.x & 31;
@@ -695,7 +700,7 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
     uint8_t *w2_s = smem;
     uint8_t *w1_s = w2_s + kW2Bytes;
     uint8_t *a1_s = w1_s + kW1Bytes;
-    uint8_t *a2_s = a1_s + (size_t)p.na1 * kA1Bytes;
+    uint8_t *a2_s = a1_s + (OTIF_E12_TS ? (size_t)0 : (size_t)p.na1 * kA1Bytes);
     uint8_t *slab_s = a2_s + (size_t)p.np * kPlaneBytes;
     uint64_t *bars = reinterpret_cast<uint64_t *>(slab_s + 2 * (size_t)slab_bytes);
     uint64_t *slab_full = bars, *slab_empty = bars + 2;
@@ -806,8 +811,13 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 for (int k = 0; k < KT; k++)
 #pragma unroll
                     for (int s = 0; s < 2; s++) {
+#if OTIF_E12_TS
+                        umma_ts_warp(d + k * 32, tmem_base + kA1Col + s1 * 16 * KT + k * 16 + s * 8,
+                                     w1d + ((2 * s * 512) >> 4), idesc1, s);
+#else
                         umma_bf16_warp(d + k * 32, a1d + ((s1 * kA1Bytes + k * 8192 + 2 * s * 2048) >> 4),
                                            w1d + ((2 * s * 512) >> 4), idesc1, s);
+#endif
                     }
                 umma_commit_warp(&a1_empty[s1]);
                 umma_commit_warp(&e1_full[J % kE1Slots]);
@@ -884,13 +894,23 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                             if (k == i) { vmk = vm[i]; ofk = of[i]; }
                         uint32_t wv[16];
                         e12_im2col_row(p, slab, (vmk >> g) & 1, ofk, rp, cp, wv);
+#if OTIF_E12_TS
+                        // this warp's 32 TMEM lanes = its 32 rows of sub-tile k (lane = row)
+                        tmem_st16(tmem_base + ((uint32_t)(row & ~31) << 16) + kA1Col + s1 * 16 * KT + k * 16, wv);
+#else
                         uint8_t *dst = a1_s + s1 * kA1Bytes + k * 8192 + row * 16;
 #pragma unroll
                         for (int c = 0; c < 4; c++)
                             *reinterpret_cast<uint4 *>(dst + c * 2048) = make_uint4(wv[4 * c], wv[4 * c + 1], wv[4 * c + 2], wv[4 * c + 3]);
+#endif
                     }
                 }
+#if OTIF_E12_TS
+                tmem_wait_st();
+                tc_fence_before();
+#else
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+#endif
                 mbar_arrive(&a1_full[s1]);
                 E12_TR(2, 0);
             }
@@ -1579,6 +1599,11 @@ static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes);
 // deepest (im2col stages, plane buffers) of the E1+E2 kernel within `budget` bytes
 static bool e12_stages(size_t fixed, size_t unit, size_t budget, int &np, int &na1) {
     np = 0; na1 = 0;
+    if (OTIF_E12_TS) {   // the im2col buffers live in TMEM: only plane buffers in shared memory
+        for (int cand = kE12MaxPlaneBufs; cand >= 2 && !np; cand--)
+            if (fixed + (size_t)cand * unit <= budget) { np = cand; na1 = 2; }
+        return np != 0;
+    }
     for (int cand_a1 = 2; cand_a1 >= 1 && !np; cand_a1--)
         for (int cand = kE12MaxPlaneBufs; cand >= 2 && !np; cand--)
             if (fixed + (size_t)(cand_a1 + cand) * unit <= budget) { np = cand; na1 = cand_a1; }
@@ -1646,7 +1671,7 @@ static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const f
     p->e12_slab_rows = slab_rows;
     p->e12_slab_pitch = slab_pitch;
     p->e12_na1 = na1;
-    p->e12_smem = fixed + (size_t)na1 * a1 + (size_t)np * plane;
+    p->e12_smem = fixed + (OTIF_E12_TS ? 0 : (size_t)na1 * a1) + (size_t)np * plane;
     p->e12_fixed = fixed;
     p->e12_unit = a1;
     return true;
