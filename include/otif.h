@@ -324,6 +324,12 @@ otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t *src_dev, i
  * of (global frame, x, y, w, h, s)), [5 + s] windows of size s (8 slots), [13] windows
  * dropped because their slot exceeded batch_cap[s], [14] pixels of the windows packed. */
 const int64_t *otif_pipeline_counters(const otif_pipeline *p);
+/* Device pointers, valid after the last device batch's selection (stream order): per
+ * frame of that batch (index = frame - batch start) the window-hash term (the sum of the
+ * 64-bit mixes counter [4] accumulates; so a clip's hash is the wrapping sum over its
+ * frames) and the window count. */
+const int64_t *otif_pipeline_frame_hashes(const otif_pipeline *p);
+const int32_t *otif_pipeline_frame_counts(const otif_pipeline *p);
 /* Device pointer to the detector batch of size s ([batch_cap[s], h_s, w_s, 3] u8, the
  * last packed device batch), or NULL. */
 uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s);

@@ -251,6 +251,20 @@ class Pipeline:
             out.copy_(torch.as_tensor(_CAI(), device="cuda"))
         return out
 
+    def frame_results(self, n: int):
+        """(window-hash terms int64 [n], window counts int32 [n]) of the first n frames of the
+        last device batch (copies; the per-clip hash is the wrapping sum over a clip's frames)."""
+        hp = lib().otif_pipeline_frame_hashes(self.handle)
+        cp = lib().otif_pipeline_frame_counts(self.handle)
+
+        def view(ptr, typestr, dtype):
+            class _CAI:
+                __cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3}
+            out = torch.empty(n, dtype=dtype, device="cuda")
+            out.copy_(torch.as_tensor(_CAI(), device="cuda"))
+            return out
+        return view(hp, "<i8", torch.int64), view(cp, "<i4", torch.int32)
+
     def flush(self, stream=None):
         """Complete a pack left pending by pack_overlap = 2."""
         check(lib().otif_pipeline_flush(self.handle, _stream(stream)), "otif_pipeline_flush")

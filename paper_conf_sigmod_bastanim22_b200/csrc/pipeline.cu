@@ -35,7 +35,8 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum);
+                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum,
+                          unsigned long long *frame_hash);
 otif_status launch_pack(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w,
                         const otif_window *windows, const int32_t *total, int32_t capacity, const otif_wsize *sizes,
                         int32_t k, uint8_t *const *batches, const int32_t *batch_cap, int32_t *slot,
@@ -86,6 +87,7 @@ struct otif_pipeline {
     float *scores = nullptr;
     otif_window *windows = nullptr;
     int *counts = nullptr, *offsets = nullptr, *total = nullptr, *slot = nullptr, *size_count = nullptr;
+    unsigned long long *frame_hash = nullptr;   // per-frame window hash of the last device batch
     uint8_t *batches[8] = {};
     unsigned long long *ctr = nullptr;
     // run outputs of host calls (grown on demand)
@@ -216,7 +218,7 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
         int t0 = tmark(p, st);
         RC(launch_select(p->scores, nullptr, d.threshold, nb, p->gh, p->gw, &d.grid, d.sizes, d.k, p->mask, p->windows,
                          p->cap_w, p->counts, p->offsets, p->total, p->sel_ws, p->sel_ws_bytes, st, p->ctr, frame_base,
-                         nullptr));
+                         nullptr, p->frame_hash));
         tspan(p, ST_SELECT, st, t0);
         p->launches += 2;
     }
@@ -292,6 +294,7 @@ extern "C" otif_status otif_pipeline_create(const otif_pipeline_desc *d, const f
     PCUDA(cudaMalloc(&p->mask, (size_t)B * p->cells));
     PCUDA(cudaMalloc(&p->windows, (size_t)p->cap_w * sizeof(otif_window)));
     PCUDA(cudaMalloc(&p->counts, B * 4));
+    PCUDA(cudaMalloc(&p->frame_hash, (size_t)B * 8));
     PCUDA(cudaMalloc(&p->offsets, B * 4));
     PCUDA(cudaMalloc(&p->total, 4));
     PCUDA(cudaMalloc(&p->slot, (size_t)p->cap_w * 4));
@@ -327,7 +330,7 @@ extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     if (p->s_copy) cudaStreamSynchronize(p->s_copy);
     void *bufs[] = {p->src[0], p->src[1], p->img, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
                     p->offsets, p->total, p->slot, p->size_count, p->ctr, p->out_win, p->out_counts, p->out_total,
-                    p->job, p->inv};
+                    p->job, p->inv, p->frame_hash};
     for (void *b : bufs)
         if (b) cudaFree(b);
     for (int s = 0; s < 8; s++)
@@ -435,6 +438,14 @@ extern "C" otif_status otif_pipeline_run_device(otif_pipeline *p, const uint8_t 
     p->out_win = ow;
     p->out_counts = oc;
     return rc;
+}
+
+extern "C" const int64_t *otif_pipeline_frame_hashes(const otif_pipeline *p) {
+    return p ? reinterpret_cast<const int64_t *>(p->frame_hash) : nullptr;
+}
+
+extern "C" const int32_t *otif_pipeline_frame_counts(const otif_pipeline *p) {
+    return p ? p->counts : nullptr;
 }
 
 extern "C" uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s) {

@@ -63,6 +63,7 @@ struct SelectParams {
     unsigned long long *ctr;
     int frame_base;
     unsigned long long *est_sum;  // internal: Σ est(R_t) over frames (window-size selection)
+    unsigned long long *frame_hash;  // internal (pipeline): per-frame window hash [n] (the ctr[4] terms)
     // two-pass scheduling: pass 1 gives every frame a small slice (ccap clusters) and
     // defers frames with more components to pass 2 (full-size slices, frames from the list)
     int ccap;                   // cluster capacity of a slice
@@ -506,6 +507,7 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
         if (lane == 0 && !MULTI) {
             p.counts[f] = 0;
             if (p.ctr) atomicAdd(&p.ctr[0], 1ull);
+            if (p.frame_hash) p.frame_hash[f] = 0ull;
         }
         return;
     }
@@ -579,15 +581,19 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
             out[0] = w;
             p.counts[f] = 1;
             if (p.est_sum) atomicAdd(p.est_sum, (unsigned long long)p.cost[p.full]);
-            if (p.ctr) {
+            if (p.ctr || p.frame_hash) {
                 unsigned long long gf = (unsigned long long)(unsigned)(f + p.frame_base);
-                atomicAdd(&p.ctr[0], 1ull);
-                atomicAdd(&p.ctr[1], (unsigned long long)npos);
-                atomicAdd(&p.ctr[2], 1ull);
-                atomicAdd(&p.ctr[3], (unsigned long long)p.fw * p.fh);
-                atomicAdd(&p.ctr[4], mix64((gf << 32) ^ mix64(((unsigned long long)p.fw << 20) ^
-                                                               ((unsigned long long)p.fh << 4) ^ (unsigned)w.size_idx)));
-                atomicAdd(&p.ctr[5 + w.size_idx], 1ull);
+                const unsigned long long h = mix64((gf << 32) ^ mix64(((unsigned long long)p.fw << 20) ^
+                                                                      ((unsigned long long)p.fh << 4) ^ (unsigned)w.size_idx));
+                if (p.frame_hash) p.frame_hash[f] = h;
+                if (p.ctr) {
+                    atomicAdd(&p.ctr[0], 1ull);
+                    atomicAdd(&p.ctr[1], (unsigned long long)npos);
+                    atomicAdd(&p.ctr[2], 1ull);
+                    atomicAdd(&p.ctr[3], (unsigned long long)p.fw * p.fh);
+                    atomicAdd(&p.ctr[4], h);
+                    atomicAdd(&p.ctr[5 + w.size_idx], 1ull);
+                }
             }
         }
         return;
@@ -611,16 +617,16 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
         otif_window w;
         w.frame = f; w.x = xc; w.y = yc; w.w = p.sw[sc]; w.h = p.sh[sc]; w.size_idx = p.orig[sc];
         out[rank] = w;
-        if (p.ctr) {
+        if (p.ctr || p.frame_hash) {
             unsigned long long gf = (unsigned long long)(unsigned)(f + p.frame_base);
             unsigned long long key = (gf << 32) ^ ((unsigned long long)(unsigned)xc << 16) ^ (unsigned)yc;
             hsh += mix64(key ^ mix64(((unsigned long long)w.w << 20) ^ ((unsigned long long)w.h << 4) ^
                                      (unsigned)w.size_idx));
             pix += (unsigned long long)w.w * w.h;
-            atomicAdd(&p.ctr[5 + w.size_idx], 1ull);
+            if (p.ctr) atomicAdd(&p.ctr[5 + w.size_idx], 1ull);
         }
     }
-    if (p.ctr) {
+    if (p.ctr || p.frame_hash) {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) {
             hsh += __shfl_xor_sync(0xffffffffu, hsh, o);
@@ -629,6 +635,7 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
     }
     if (lane == 0) {
         p.counts[f] = m;
+        if (p.frame_hash) p.frame_hash[f] = hsh;
         if (p.est_sum) atomicAdd(p.est_sum, (unsigned long long)est);
         if (p.ctr) {
             atomicAdd(&p.ctr[0], 1ull);
@@ -730,7 +737,8 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
                           int32_t gw, const otif_grid_desc *g, const otif_wsize *sizes, int32_t k, uint8_t *mask_out,
                           otif_window *windows, int32_t capacity, int32_t *frame_count, int32_t *frame_offset,
                           int32_t *total, void *workspace, size_t ws_bytes, cudaStream_t stream,
-                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum) {
+                          unsigned long long *ctr, int frame_base, unsigned long long *est_sum,
+                          unsigned long long *frame_hash) {
     SelectParams p;
     memset(&p, 0, sizeof(p));
     p.scores = scores; p.mask_in = mask_in; p.thr = threshold;
@@ -756,6 +764,7 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
     p.ctr = ctr;
     p.frame_base = frame_base;
     p.est_sum = est_sum;
+    p.frame_hash = frame_hash;
     p.defer_list = p.counts + round_up(n, 64);
     p.defer_count = p.defer_list + round_up(n, 64);
     OTIF_CUDA(cudaMemsetAsync(p.defer_count, 0, 4, stream));
@@ -892,5 +901,5 @@ extern "C" otif_status otif_select_windows(const float *scores, const uint8_t *m
     if (st != OTIF_OK) return st;
     return launch_select(scores, mask_in, threshold, n, gh, gw, g, sizes, k, mask_out, windows, capacity, frame_count,
                          frame_offset, total, workspace, ws_bytes, stream, nullptr, 0,
-                         reinterpret_cast<unsigned long long *>(est_sum));
+                         reinterpret_cast<unsigned long long *>(est_sum), nullptr);
 }

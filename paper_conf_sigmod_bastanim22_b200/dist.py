@@ -62,6 +62,29 @@ def run_corpus(clips: range, run_clip: Callable[[int], torch.Tensor]) -> torch.T
     return torch.stack(rows)
 
 
+def clip_groups(clips: range, pool: int) -> list:
+    """Split a contiguous clip range into runs whose frames are contiguous in the frame pool
+    (clip k reads pool slot k mod pool): each run is one pipeline call."""
+    out, start = [], clips.start
+    for k in clips:
+        if k != start and k % pool == 0:
+            out.append(range(start, k))
+            start = k
+    if len(clips):
+        out.append(range(start, clips.stop))
+    return out
+
+
+def run_corpus_grouped(clips: range, pool: int, run_group: Callable[[range], torch.Tensor]) -> torch.Tensor:
+    """The shard loop with one call per pool-contiguous run of clips: run_group(r) -> per-clip
+    counters [len(r), C] (exact frames, windows and window hash per clip; the group's other
+    totals attributed to its first clip, so column sums stay exact)."""
+    rows = [run_group(r) for r in clip_groups(clips, pool)]
+    if not rows:
+        return torch.zeros((0, 0), dtype=torch.int64)
+    return torch.cat(rows)
+
+
 def gather_clip_counters(per_clip: torch.Tensor, n_clips: int, width: int, group=None) -> torch.Tensor:
     """Per-clip counters of every rank -> [n_clips, width] on every rank, in clip order.
     Ranks hold contiguous clip ranges (shard_clips), so the gathered blocks concatenate

@@ -75,3 +75,14 @@ def test_gloo_gather_and_sharding_invariance(world, n_clips):
         assert torch.equal(allc, ref_rows)    # per-clip counters in clip order, every rank
         assert digest == single               # per-clip hashes + totals independent of the sharding
     assert odist.combine(ref.view(1, -1)) == out[0][2]
+
+
+def test_clip_groups_follow_the_pool():
+    for n, pool in ((480, 8), (10, 4), (7, 8), (0, 8)):
+        for world in (1, 2, 3, 4, 8):
+            for r in range(world):
+                clips = odist.shard_clips(n, world, r)
+                groups = odist.clip_groups(clips, pool)
+                assert [k for g in groups for k in g] == list(clips)
+                for g in groups:
+                    assert len(g) <= pool and g.start // pool == (g.stop - 1) // pool

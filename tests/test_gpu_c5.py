@@ -46,3 +46,30 @@ def test_c5_shard_loop_invariant_over_world_sizes():
         c, d = results[world]
         assert torch.equal(c, ref_c), world
         assert d == ref_d, world
+    # the bench's grouped loop: one call per pool-contiguous run of clips (max_batch = pool x
+    # clip), per-clip hashes / windows from the per-frame results: same per-clip hashes,
+    # windows and frames, same column totals, same digest
+    big = otif.Pipeline(wl, weights.proxy_weights(), threshold("C2", 0.7), max_batch=pool_clips * fpc,
+                        pack_overlap=2)
+
+    def run_group(r):
+        j = r.start % pool_clips
+        big.run_device(pool[j * fpc:(j + len(r)) * fpc], frame_base=r.start * fpc)
+        tot = big.counters()
+        big.reset_counters()
+        fh, fc = big.frame_results(len(r) * fpc)
+        rows = torch.zeros((len(r), tot.numel()), dtype=torch.int64, device=tot.device)
+        rows[0] = tot
+        rows[:, 0] = fpc
+        rows[:, 2] = fc.view(len(r), fpc).sum(1)
+        rows[:, 4] = fh.view(len(r), fpc).sum(1)
+        return rows
+
+    for world in (1, 2, 4):
+        rows = [odist.run_corpus_grouped(odist.shard_clips(n_clips, world, r), pool_clips, run_group)
+                for r in range(world)]
+        big.flush()
+        g = torch.cat([r for r in rows if r.numel()]).cpu()
+        assert torch.equal(g[:, [0, 2, 4]], ref_c[:, [0, 2, 4]]), world
+        assert torch.equal(g.sum(0), ref_c.sum(0)), world
+        assert odist.corpus_digest(g) == ref_d, world
