@@ -557,6 +557,9 @@ __global__ void __launch_bounds__(kConvThreads, 1) conv_umma_kernel(const __grid
 #define OTIF_PJ_E12 0            // fused pack copy warps in the E1+E2 kernel (A/B builds; 0 = none)
 #endif
 constexpr int kE12Threads = 768 + 32 * OTIF_PJ_E12;
+#ifndef OTIF_E12_GATHER2
+#define OTIF_E12_GATHER2 0    // 1: a thread's two im2col rows per job built together (measured neutral, r02q)
+#endif
 #ifndef OTIF_E12_TS
 #define OTIF_E12_TS 0         // 1: E1's im2col rows in TMEM (two buffers, tcgen05.st by the gather,
 #endif                        //    A-from-TMEM MMAs): 194 KB less shared-memory traffic per tile
@@ -884,6 +887,34 @@ __global__ void __launch_bounds__(kE12Threads, 1) e12_umma_kernel(const __grid_c
                 E12_WAIT_CHAIN(&a1_empty[s1], ph1 ^ 1);
                 E12_TR(1, 0);
                 {
+#if OTIF_E12_GATHER2 && !OTIF_E12_TS
+                    // both of this thread's rows (sub-tiles k0 and k0 + 2) built together: their
+                    // slab loads and conversions interleave (the gather is the critical role,
+                    // profiles/r02p_e12_source.md)
+                    const int k0 = (int)((wg - J * KT) & 1);
+                    const bool two = k0 + 2 < KT;
+                    uint32_t va = vm[0], oa = of[0], vb = vm[KT - 1], ob = of[KT - 1];
+#pragma unroll
+                    for (int i = 1; i < KT; i++)
+                        if (k0 == i) { va = vm[i]; oa = of[i]; }
+                    if (KT == 4 && k0 == 0) { vb = vm[2]; ob = of[2]; }
+                    uint32_t wa[16], wb[16];
+                    e12_im2col_row(p, slab, (va >> g) & 1, oa, rp, cp, wa);
+                    e12_im2col_row(p, slab, two ? ((vb >> g) & 1) : 0u, ob, rp, cp, wb);
+                    {
+                        uint8_t *dst = a1_s + s1 * kA1Bytes + k0 * 8192 + row * 16;
+#pragma unroll
+                        for (int c = 0; c < 4; c++)
+                            *reinterpret_cast<uint4 *>(dst + c * 2048) = make_uint4(wa[4 * c], wa[4 * c + 1], wa[4 * c + 2], wa[4 * c + 3]);
+                        if (two) {
+#pragma unroll
+                            for (int c = 0; c < 4; c++)
+                                *reinterpret_cast<uint4 *>(dst + 2 * 8192 + c * 2048) =
+                                    make_uint4(wb[4 * c], wb[4 * c + 1], wb[4 * c + 2], wb[4 * c + 3]);
+                        }
+                    }
+                    if (false)
+#endif
                     // rolled loop over this warpgroup's k sub-tiles (code size: the kernel is
                     // instruction-cache bound, see the header)
 #pragma unroll 1
