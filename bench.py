@@ -612,7 +612,12 @@ def run_otif(args):
             "roofline": dict(rl["conv"], kernel="proxy convs on tcgen05: e12_umma_kernel (E1 fused into E2) + "
                                                 "conv_umma_kernel (E3..E5, D1+D2 head)",
                              per_launch="5 launches per batch of 4500 frames; achieved = algorithmic FLOPs of "
-                                        "E1..D1 / CUDA-event time of those launches on the pipeline stream"),
+                                        "E1..D1 / CUDA-event time of those launches on the pipeline stream",
+                             fused_work=("the E5 and D1 launches also copy the previous step's detector batches "
+                                         f"({rl['pack']['bytes_per_step'] / 1e9:.1f} GB per step through HBM; "
+                                         "pack_overlap 2), which the tensor FLOP count does not credit"
+                                         if args.pack_overlap > 0 else None),
+                             frac_serial_schedule=(serial["rooflines"]["conv"]["frac"] if serial else None)),
             "stages": {k: v for k, v in rl.items() if k != "conv"},
             "serial_schedule": serial,
             **objs,
