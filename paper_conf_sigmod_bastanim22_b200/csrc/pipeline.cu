@@ -22,7 +22,9 @@
 namespace otif {
 
 otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws, size_t ws_bytes,
-                         cudaStream_t stream, cudaEvent_t *evs, PackJob *pj);
+                         cudaStream_t stream, cudaEvent_t *evs, PackJob *pj, const uint8_t *frames, int sh,
+                         int sw);
+bool proxy_fuses_resize(const otif_proxy *p, int n, const uint8_t *src, int sh, int sw);
 bool pack_job_applies(int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w, const otif_wsize *sizes, int32_t k,
                       uint8_t *const *batches);
 otif_status launch_pack_prepare(const uint8_t *src, int32_t n, int32_t src_h, int32_t src_w,
@@ -167,14 +169,15 @@ struct NvtxRange {
 };
 
 static otif_status run_proxy(otif_pipeline *p, const uint8_t *img, int mb, float *scores, cudaStream_t st,
-                             PackJob *pj) {
+                             PackJob *pj, const uint8_t *frames) {
     NvtxRange r("otif.proxy");
     // six spans for the proxy (prep/E1, then each GEMM layer); launch_proxy records their
     // end events at the actual points in the stream
     cudaEvent_t evs[6];
     int from = tmark(p, st);
     for (int i = 0; i < 6 && p->timing; i++) from = treserve(p, ST_PREP + i, from, &evs[i]);
-    RC(launch_proxy(p->proxy, img, mb, scores, p->proxy_ws, p->proxy_ws_bytes, st, p->timing ? evs : nullptr, pj));
+    RC(launch_proxy(p->proxy, img, mb, scores, p->proxy_ws, p->proxy_ws_bytes, st, p->timing ? evs : nullptr, pj,
+                    frames, p->d.src_h, p->d.src_w));
     p->launches += proxy_launches(p->proxy);
     return OTIF_OK;
 }
@@ -201,16 +204,22 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
     RC(wait_pending(p, st));
     for (int m0 = 0; m0 < nb; m0 += p->pb) {
         const int mb = nb - m0 < p->pb ? nb - m0 : p->pb;
+        const uint8_t *frames = src + (size_t)m0 * frame_bytes;
+        // even integer downscale: the fused E1+E2 kernel reads the frames itself (stage 1
+        // fused into the proxy's first kernel, no proxy image in HBM)
+        const bool fused = proxy_fuses_resize(p->proxy, mb, frames, d.src_h, d.src_w);
         {
             NvtxRange r("otif.resize");
             int t0 = tmark(p, st);
-            RC(otif_resize(src + (size_t)m0 * frame_bytes, mb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w,
-                           st));
+            if (!fused) {
+                RC(otif_resize(frames, mb, d.src_h, d.src_w, p->img, d.proxy.in_h, d.proxy.in_w, st));
+                p->launches += 1;
+            }
             tspan(p, ST_RESIZE, st, t0);
-            p->launches += 1;
         }
         // the pending pack (previous batch) rides in this proxy pass's tensor-bound layers
-        RC(run_proxy(p, p->img, mb, p->scores + (size_t)m0 * p->cells, st, p->job_pending ? p->job : nullptr));
+        RC(run_proxy(p, p->img, mb, p->scores + (size_t)m0 * p->cells, st, p->job_pending ? p->job : nullptr,
+                     fused ? frames : nullptr));
     }
     RC(drain_pack(p, st));
     {

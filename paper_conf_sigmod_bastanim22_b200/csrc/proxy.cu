@@ -33,6 +33,8 @@
 
 #include <vector>
 
+#include <cuda_fp16.h>
+
 #include "common.cuh"
 #include "packjob.cuh"
 
@@ -1452,6 +1454,581 @@ __global__ void __launch_bounds__(kE12bThreads, 1) e12b_umma_kernel(const __grid
 #endif  // OTIF_E12B_BUILD
 
 // ---------------------------------------------------------------------------
+// E1 fused into E2, space-to-depth variant (e12s), with the resize fused in.  E1 (3x3,
+// stride 2, 3 -> 32) is the stride-1 2x2 convolution over the space-to-depth image (one
+// s2d pixel = the 2x2 proxy pixels (2Y + sy, 2X + sx) x 3 channels: 12 of 16 fp16
+// channels (sy * 2 + sx) * 3 + c holding u - 128, exact), and for each of E2's four parity
+// planes its four taps are LINEAR SHIFTS (0, -1, -pitch, -pitch - 1) within one of four
+// s2d parity planes laid out with E2's plane pitch.  So E1's A operand is read straight
+// from a staged halo ("slab") of the s2d planes through shifted descriptors — no per-row
+// im2col gather (the critical role of the tile kernel, profiles/r02p_e12_source.md) — at
+// 2.25x E1's MMA work (K = 4 taps x 16 instead of 32), which the tensor pipe has spare.
+//
+// The slab is built in shared memory by converter warps straight from the u8 source
+// frames: with an even integer downscale FX x fy (every workload of SURVEY.md §8(d)) a
+// proxy pixel is (sum of the 2x2 central source pixels + 2) >> 2 — exactly resize.cu's
+// value — so stage 1 and E1's input conversion are one pass over the frames and the proxy
+// image never exists in HBM (FX == 1: the input is the u8 proxy image itself).  Each CTA
+// runs a contiguous range of tiles and the slab of tile t + 1 overlaps tile t's by
+// 2 (pitch + 1) positions, which are copied on chip, so every s2d pixel is converted once.
+//
+// Roles (768 threads): warp 1 E1 MMA (KT x 4 per plane job), warp 2 TMEM allocator, warp 3
+// E2 MMA, warps 4-11 E1 epilogue (+ bias, ReLU, zero padding -> E2's A operand), 12-15 E2
+// epilogue, 16-23 converters.
+// ---------------------------------------------------------------------------
+constexpr int kE12sThreads = 768;
+constexpr int kE12sConv = 256;   // converter threads
+// s2d channels 12 and 13 of every pixel inside the image hold 128.0 (fp16 0x5800): with
+// tap (1, 1) weights (b_hi, b_lo) = E1's bias * 2^s split into two fp16 terms, the MMA adds
+// E1's bias (x 2^(s+7), the accumulator scale) exactly as far as fp32 goes
+constexpr uint32_t kE12sBiasCh = 0x58005800u;
+#ifndef OTIF_E12S_PREFETCH
+#define OTIF_E12S_PREFETCH 0      // tiles of source rows prefetched to L2 ahead of the converters (measured slower: off)
+#endif
+#ifndef OTIF_E12S_NOLOAD
+#define OTIF_E12S_NOLOAD 0
+#endif
+constexpr int kE12sPrefetch = OTIF_E12S_PREFETCH;
+
+struct E12sParams {
+    const uint8_t *src;         // u8 NHWC frames [n, sh, sw, 3] (FX >= 2) or proxy image [n, hp, wp, 3] (FX == 1)
+    int sh, sw, hp, wp, fy;
+    int prefetch;               // source rows are 16-B aligned: L2 bulk prefetch usable
+    int h1, w1, h2, w2, pitch;
+    uint32_t fstride, mtot;
+    FastDiv div_pitch, div_rpf, div_fstride;
+    int PS;                     // slab positions per s2d plane = 256 + 2 (pitch + 1), rounded to 16
+    int nslab;                  // slab buffers (1 or 2)
+    int np;                     // plane buffers
+    int ntiles;
+    int group_ntaps[4], group_shift[4][9];
+    const uint16_t *w1s;        // fp16 [4 taps][2 chunks][32 n][8] = w * 2^s (+ the bias terms, kE12sBiasCh)
+    const uint16_t *wt2;        // as e12
+    const float *b2;
+    int out_kind;
+    uint8_t *out;
+    int64_t out_lcap;
+    int out_c8, out_pitch;
+    int64_t out_fstride;
+};
+
+// s2d parity plane and shift (positions) of E1 tap t = (ty, tx) for E2 plane g = (rp, cp)
+__device__ __forceinline__ void e12s_tap(int g, int t, int pitch, int &h, int &shift) {
+    const int rp = g >> 1, cp = g & 1, ty = t >> 1, tx = t & 1;
+    h = (((rp + 1 + ty) & 1) << 1) | ((cp + 1 + tx) & 1);
+    const int ry = (rp == 0 && ty == 0) ? -1 : 0, rx = (cp == 0 && tx == 0) ? -1 : 0;
+    shift = ry * pitch + rx;
+}
+
+// bytes I and J of the little-endian byte string w[] as two zero-extended 16-bit lanes
+template <int I, int J>
+__device__ __forceinline__ uint32_t s2d_pair(const uint32_t *w) {
+    if constexpr (I / 4 == J / 4) {
+        return __byte_perm(w[I / 4], 0u, (I % 4) | (4 << 4) | ((J % 4) << 8) | (4 << 12));
+    } else if constexpr (J / 4 == I / 4 + 1) {
+        return __byte_perm(w[I / 4], w[J / 4], (I % 4) | ((J % 4 + 4) << 8)) & 0x00FF00FFu;
+    } else {
+        return __byte_perm(w[I / 4], 0u, (I % 4) | 0x4440) | __byte_perm(w[J / 4], 0u, 0x4044 | ((J % 4) << 8));
+    }
+}
+
+// 16-bit lanes holding 0..255 -> fp16x2 of (v - 128), exact (0x6400 | v is 1024 + v)
+__device__ __forceinline__ uint32_t s2d_f16(uint32_t v) { return sub_f16x2(0x64006400u | v, 0x64806480u); }
+// 16-bit lanes holding sums of four bytes -> fp16x2 of ((s + 2) >> 2) - 128
+__device__ __forceinline__ uint32_t s2d_avg_f16(uint32_t s) {
+    return s2d_f16(((s + 0x00020002u) >> 2) & 0x00FF00FFu);
+}
+
+#ifndef OTIF_E12S_LD
+#define OTIF_E12S_LD 0   // converter source loads: 0 ld.global.nc, 1 .cs, 2 ld.global, 3 .cg (L2 only)
+#endif
+template <typename T>
+__device__ __forceinline__ T s2d_ld(const T *p) {
+#if OTIF_E12S_LD == 1
+    return __ldcs(p);
+#elif OTIF_E12S_LD == 2
+    return *p;
+#elif OTIF_E12S_LD == 3
+    return __ldcg(p);
+#else
+    return __ldg(p);
+#endif
+}
+
+// Source bytes of two adjacent s2d columns X = 2xx, 2xx + 1 (proxy columns 4xx .. 4xx + 3)
+// in one source row: w[] gets a little-endian byte string; O(xp, sx) is the offset of the
+// first source pixel of proxy column 2X + sx (FX >= 2: the second one follows at + 3).
+template <int FX> struct S2dRow;
+template <> struct S2dRow<1> {      // proxy image: bytes 12xx .. 12xx + 11
+    static constexpr int NW = 3;
+    static constexpr int O(int xp, int sx) { return 6 * xp + 3 * sx; }
+    __device__ __forceinline__ static void load(const uint8_t *row, int xx, uint32_t *w) {
+        const uint32_t *s = reinterpret_cast<const uint32_t *>(row + 12 * xx);
+        w[0] = s2d_ld(s); w[1] = s2d_ld(s + 1); w[2] = s2d_ld(s + 2);
+    }
+};
+template <> struct S2dRow<2> {      // source columns 8xx .. 8xx + 7: bytes 24xx .. 24xx + 23
+    static constexpr int NW = 6;
+    static constexpr int O(int xp, int sx) { return 12 * xp + 6 * sx; }
+    __device__ __forceinline__ static void load(const uint8_t *row, int xx, uint32_t *w) {
+        const uint2 *s = reinterpret_cast<const uint2 *>(row + 24 * xx);
+        const uint2 a = s2d_ld(s), b = s2d_ld(s + 1), c = s2d_ld(s + 2);
+        w[0] = a.x; w[1] = a.y; w[2] = b.x; w[3] = b.y; w[4] = c.x; w[5] = c.y;
+    }
+};
+template <> struct S2dRow<4> {      // source columns 16xx + {1, 2, 5, 6, 9, 10, 13, 14}: bytes 48xx + [0, 48)
+    static constexpr int NW = 12;
+    static constexpr int O(int xp, int sx) { return 24 * xp + 12 * sx + 3; }
+    __device__ __forceinline__ static void load(const uint8_t *row, int xx, uint32_t *w) {
+        const uint4 *s = reinterpret_cast<const uint4 *>(row + 48 * xx);
+        const uint4 a = s2d_ld(s), b = s2d_ld(s + 1), c = s2d_ld(s + 2);
+        w[0] = a.x; w[1] = a.y; w[2] = a.z; w[3] = a.w; w[4] = b.x; w[5] = b.y;
+        w[6] = b.z; w[7] = b.w; w[8] = c.x; w[9] = c.y; w[10] = c.z; w[11] = c.w;
+    }
+};
+template <> struct S2dRow<8> {      // source columns 32xx + {3, 4, 11, 12, 19, 20, 27, 28}: bytes 96xx + 8 + [0, 8), +24, +48, +72
+    static constexpr int NW = 8;
+    static constexpr int O(int xp, int sx) { return 16 * xp + 8 * sx + 1; }
+    __device__ __forceinline__ static void load(const uint8_t *row, int xx, uint32_t *w) {
+        const uint8_t *s = row + 96 * xx + 8;
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint2 v = s2d_ld(reinterpret_cast<const uint2 *>(s + 24 * k));
+            w[2 * k] = v.x; w[2 * k + 1] = v.y;
+        }
+    }
+};
+
+// one proxy pixel value (generic, byte loads): the right edge of odd proxy widths
+template <int FX>
+__device__ __forceinline__ uint32_t s2d_px_slow(const E12sParams &p, int f, int py, int px, int c) {
+    if (py >= p.hp || px >= p.wp) return 128u;
+    if (FX == 1) return __ldg(p.src + (((size_t)f * p.hp + py) * p.wp + px) * 3 + c);
+    const int r0 = p.fy * py + p.fy / 2 - 1, c0 = FX * px + FX / 2 - 1;
+    const uint8_t *a = p.src + (((size_t)f * p.sh + r0) * p.sw + c0) * 3 + c;
+    const uint8_t *b = a + (size_t)p.sw * 3;
+    return ((uint32_t)__ldg(a) + __ldg(a + 3) + __ldg(b) + __ldg(b + 3) + 2) >> 2;
+}
+
+// channel sums of one source row for s2d column parity XP into s0..s2 (16-bit lanes:
+// channel pairs (0,1), (2,3), (4,5) of the proxy columns 2X, 2X + 1)
+template <int FX, int XP>
+__device__ __forceinline__ void s2d_row_sums(const uint32_t *w, uint32_t &s0, uint32_t &s1, uint32_t &s2) {
+    using R = S2dRow<FX>;
+    constexpr int A = R::O(XP, 0), B = R::O(XP, 1);
+    if constexpr (FX == 1) {
+        s0 += s2d_pair<A, A + 1>(w);
+        s1 += s2d_pair<A + 2, B>(w);
+        s2 += s2d_pair<B + 1, B + 2>(w);
+    } else {
+        s0 += s2d_pair<A, A + 1>(w) + s2d_pair<A + 3, A + 4>(w);
+        s1 += s2d_pair<A + 2, B>(w) + s2d_pair<A + 5, B + 3>(w);
+        s2 += s2d_pair<B + 1, B + 2>(w) + s2d_pair<B + 4, B + 5>(w);
+    }
+}
+
+// the 12 channels of s2d pixels (Y, 2xx) and (Y, 2xx + 1) of frame f as 6 fp16x2 words
+// each; all source loads are issued before any is used (one memory latency per call)
+template <int FX>
+__device__ __forceinline__ void s2d_pixels(const E12sParams &p, int f, int Y, int xx, uint32_t (&o)[2][6]) {
+    using R = S2dRow<FX>;
+    if (4 * xx + 3 >= p.wp) {      // right edge of an odd proxy width: byte loads
+#pragma unroll
+        for (int xp = 0; xp < 2; xp++)
+#pragma unroll
+            for (int k = 0; k < 6; k++) {
+                const int k0 = 2 * k, k1 = 2 * k + 1, X = 2 * xx + xp;
+                const uint32_t lo = s2d_px_slow<FX>(p, f, 2 * Y + k0 / 6, 2 * X + (k0 / 3) % 2, k0 % 3);
+                const uint32_t hi = s2d_px_slow<FX>(p, f, 2 * Y + k1 / 6, 2 * X + (k1 / 3) % 2, k1 % 3);
+                o[xp][k] = s2d_f16(lo | (hi << 16));
+            }
+        return;
+    }
+    const bool row1 = 2 * Y + 1 < p.hp;   // else the bottom edge of an odd proxy height
+    constexpr int NR = FX == 1 ? 1 : 2;   // source rows per proxy row
+    uint32_t w[2][NR][R::NW];
+#pragma unroll
+    for (int sy = 0; sy < 2; sy++) {
+        const int py = 2 * Y + sy;
+        const size_t r0 = FX == 1 ? (size_t)f * p.hp + py : (size_t)f * p.sh + p.fy * py + p.fy / 2 - 1;
+        const uint8_t *row = p.src + r0 * (size_t)p.sw * 3;
+#pragma unroll
+        for (int d = 0; d < NR; d++) {
+            if (sy == 0 || row1) {
+                R::load(row + (size_t)d * p.sw * 3, xx, w[sy][d]);
+            } else {
+#pragma unroll
+                for (int k = 0; k < R::NW; k++) w[sy][d][k] = 0u;
+            }
+        }
+    }
+#pragma unroll
+    for (int sy = 0; sy < 2; sy++) {
+        uint32_t a0 = 0, a1 = 0, a2 = 0, b0 = 0, b1 = 0, b2 = 0;
+#pragma unroll
+        for (int d = 0; d < NR; d++) {
+            s2d_row_sums<FX, 0>(w[sy][d], a0, a1, a2);
+            s2d_row_sums<FX, 1>(w[sy][d], b0, b1, b2);
+        }
+        if (FX == 1) {
+            o[0][3 * sy] = s2d_f16(a0); o[0][3 * sy + 1] = s2d_f16(a1); o[0][3 * sy + 2] = s2d_f16(a2);
+            o[1][3 * sy] = s2d_f16(b0); o[1][3 * sy + 1] = s2d_f16(b1); o[1][3 * sy + 2] = s2d_f16(b2);
+        } else {
+            o[0][3 * sy] = s2d_avg_f16(a0); o[0][3 * sy + 1] = s2d_avg_f16(a1); o[0][3 * sy + 2] = s2d_avg_f16(a2);
+            o[1][3 * sy] = s2d_avg_f16(b0); o[1][3 * sy + 1] = s2d_avg_f16(b1); o[1][3 * sy + 2] = s2d_avg_f16(b2);
+        }
+        if (sy == 1 && !row1) {
+#pragma unroll
+            for (int k = 3; k < 6; k++) o[0][k] = o[1][k] = 0u;
+        }
+    }
+}
+
+// L2 prefetch of the source rows behind E2-layout rows [r0, r1) (row id = q / pitch)
+template <int FX>
+__device__ __forceinline__ void s2d_prefetch_rows(const E12sParams &p, int r0, int r1) {
+    const size_t rb = (size_t)p.sw * 3;
+    for (int rid = r0; rid < r1; rid++) {
+        const int f = rid / (p.h2 + 1), gr = rid - f * (p.h2 + 1);
+        if (gr == 0 || (uint32_t)f * p.fstride >= p.mtot) continue;   // top pad row / past the batch
+        const int yy = gr - 1;
+        if (FX == 1) {                 // proxy rows 4yy .. 4yy + 3 (as far as the image goes)
+            const int py0 = 4 * yy, npy = min(4, p.hp - py0);
+            if (npy > 0) bulk_prefetch_l2(p.src + ((size_t)f * p.hp + py0) * rb, (uint32_t)(npy * rb));
+        } else {
+            for (int py = 4 * yy; py < 4 * yy + 4 && py < p.hp; py++)
+                bulk_prefetch_l2(p.src + ((size_t)f * p.sh + p.fy * py + p.fy / 2 - 1) * rb, (uint32_t)(2 * rb));
+        }
+    }
+}
+
+template <int KT, int FX>
+__global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid_constant__ E12sParams p) {
+    constexpr int kAccStages = 2, kE1Slots = 2;
+    constexpr uint32_t kE1Col = kAccStages * 2 * 64;
+    static_assert(kE1Col + kE1Slots * 32 * KT <= 512, "TMEM budget");
+    extern __shared__ __align__(1024) uint8_t smem[];
+    const int warp = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
+    constexpr int N2 = 64;
+    constexpr int MT = 2;
+    constexpr int P = 128 * KT;
+    constexpr uint32_t kW2Bytes = 9 * 4 * N2 * 16;
+    constexpr uint32_t kW1Bytes = 4 * 2 * 32 * 16;    // 4 taps x K16 x N32 fp16
+    constexpr uint32_t kPlaneBytes = P * 64;
+    const uint32_t slab_bytes = 8u * p.PS * 16;        // 4 planes x 2 chunks
+
+    // the E1 MMAs of the last rows (P - 1 + pitch + 1 >= PS) read past a slab chunk into the
+    // next one / the plane buffers: garbage for E1 rows that E2 never reads
+    uint8_t *w2_s = smem;
+    uint8_t *w1_s = w2_s + kW2Bytes;
+    uint8_t *slab_s = w1_s + kW1Bytes;
+    uint8_t *a2_s = slab_s + (size_t)p.nslab * slab_bytes;
+    uint64_t *bars = reinterpret_cast<uint64_t *>(a2_s + (size_t)p.np * kPlaneBytes);
+    uint64_t *slab_full = bars, *slab_empty = bars + 2;
+    uint64_t *e1_full = bars + 4, *e1_empty = bars + 6;
+    uint64_t *a2_full = bars + 8, *a2_empty = a2_full + kE12MaxPlaneBufs;
+    uint64_t *acc_full = a2_empty + kE12MaxPlaneBufs, *acc_empty = acc_full + 2;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(acc_empty + 2);
+    float *s_b2 = reinterpret_cast<float *>(tmem_slot + 4);
+
+    // a contiguous range of tiles per CTA (consecutive slabs overlap)
+    const int t_begin = (int)((int64_t)blockIdx.x * p.ntiles / gridDim.x);
+    const int t_end = (int)((int64_t)(blockIdx.x + 1) * p.ntiles / gridDim.x);
+
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < 2; i++) {
+            mbar_init(&slab_full[i], kE12sConv); mbar_init(&slab_empty[i], 1);
+            mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 128);
+        }
+        for (int i = 0; i < kE1Slots; i++) { mbar_init(&e1_full[i], 1); mbar_init(&e1_empty[i], 256); }
+        for (int i = 0; i < kE12MaxPlaneBufs; i++) { mbar_init(&a2_full[i], 256); mbar_init(&a2_empty[i], 1); }
+        fence_barrier_init();
+    }
+    if (warp == 2) tmem_alloc(tmem_slot, 512);
+    for (uint32_t i = threadIdx.x; i < kW2Bytes / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(w2_s)[i] = reinterpret_cast<const uint4 *>(p.wt2)[i];
+    for (uint32_t i = threadIdx.x; i < kW1Bytes / 16; i += blockDim.x)
+        reinterpret_cast<uint4 *>(w1_s)[i] = reinterpret_cast<const uint4 *>(p.w1s)[i];
+    if (threadIdx.x < N2) s_b2[threadIdx.x] = p.b2[threadIdx.x];
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp >= 16) {
+        // ===== converters: slab positions j <-> E2-layout position q = q0 - pitch - 1 + j
+        // of the 4 s2d parity planes, 2 chunks each; items (j, plane) with the plane's
+        // column parity fastest, so lane pairs read adjacent source spans =====
+        const int ct = threadIdx.x - (kE12sThreads - kE12sConv);
+        const int PS = p.PS, nov = PS - 128 * MT;
+        uint32_t sb = 0, sp = 0;
+        for (int tile = t_begin; tile < t_end; tile++) {
+            mbar_wait_sleep(&slab_empty[sb], sp ^ 1);
+            uint8_t *slab = slab_s + (size_t)sb * slab_bytes;
+            int j0 = 0;
+            if (tile != t_begin) {
+                // positions [256, PS) of the previous slab are [0, PS - 256) of this one: each
+                // thread moves the ones it converted itself (no converter-wide barrier; with
+                // one slab, in place: sources >= 256 > destinations, then one barrier before
+                // the new positions [PS - 256, PS) overwrite sources)
+                const uint8_t *prev = slab_s + (size_t)(p.nslab == 2 ? sb ^ 1 : sb) * slab_bytes;
+                const int j0p = tile - 1 == t_begin ? 0 : nov;
+#pragma unroll 1
+                for (int it = ct; it < 2 * (PS - j0p); it += kE12sConv) {
+                    const int j = j0p + ((it >> 5) << 4) + (it & 15), rh = (it >> 4) & 1;
+                    if (j < 128 * MT) continue;
+#pragma unroll
+                    for (int c = 0; c < 4; c++) {
+                        const size_t ch = 4 * rh + c;
+                        *reinterpret_cast<uint4 *>(slab + (ch * PS + j - 128 * MT) * 16) =
+                            *reinterpret_cast<const uint4 *>(prev + (ch * PS + j) * 16);
+                    }
+                }
+                if (p.nslab == 1) asm volatile("bar.sync 1, %0;" ::"n"(kE12sConv) : "memory");
+                j0 = nov;
+            }
+            const int q0 = tile * (128 * MT) - (p.pitch + 1);
+            // items (j, s2d row parity rh), both column parities per item; half-warps run
+            // 16 consecutive positions of one rh (adjacent source spans)
+            const int items = 2 * (PS - j0);
+#pragma unroll 1
+            for (int it = ct; it < items; it += kE12sConv) {
+                const int j = j0 + ((it >> 5) << 4) + (it & 15), rh = (it >> 4) & 1;
+                const int q = q0 + j;
+                uint32_t o[2][6] = {{0, 0, 0, 0, 0, 0}, {0, 0, 0, 0, 0, 0}};
+                uint32_t bias[2] = {0u, 0u};    // channels 12, 13 of the pixels inside the image
+                if (q >= 0 && (uint32_t)q < p.mtot) {
+                    const uint32_t f = fdiv((uint32_t)q, p.div_fstride);
+                    const uint32_t r = (uint32_t)q - f * p.fstride;
+                    const uint32_t gr = fdiv(r, p.div_pitch);
+                    const int yy = (int)gr - 1, xx = (int)(r - gr * (uint32_t)p.pitch) - 1;
+                    const int Y = 2 * yy + rh;
+                    if (yy >= 0 && xx >= 0 && Y < p.h1 && 2 * xx < p.w1) {
+#if OTIF_E12S_NOLOAD    // timing experiment only: no source loads (wrong results)
+                        o[0][0] = (uint32_t)(Y + xx);
+#else
+                        s2d_pixels<FX>(p, (int)f, Y, xx, o);
+#endif
+                        bias[0] = kE12sBiasCh;
+                        if (2 * xx + 1 < p.w1) {
+                            bias[1] = kE12sBiasCh;
+                        } else {
+#pragma unroll
+                            for (int k = 0; k < 6; k++) o[1][k] = 0u;
+                        }
+                    }
+                }
+#pragma unroll
+                for (int xp = 0; xp < 2; xp++) {
+                    const int h = 2 * rh + xp;
+                    *reinterpret_cast<uint4 *>(slab + ((size_t)(2 * h) * PS + j) * 16) =
+                        make_uint4(o[xp][0], o[xp][1], o[xp][2], o[xp][3]);
+                    *reinterpret_cast<uint4 *>(slab + ((size_t)(2 * h + 1) * PS + j) * 16) =
+                        make_uint4(o[xp][4], o[xp][5], bias[xp], 0u);
+                }
+            }
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_arrive(&slab_full[sb]);
+            if (++sb == (uint32_t)p.nslab) { sb = 0; sp ^= 1; }
+        }
+    } else if (warp == 0) {
+        // ===== prefetcher: keeps the source rows of the tiles kE12sPrefetch ahead of the
+        // converters on their way to L2 (their loads then wait for L2, not DRAM) =====
+        if (lane == 0 && kE12sPrefetch > 0 && p.prefetch) {
+            const uint32_t rows_q = (uint32_t)p.pitch;
+            int pf_next = (int)(max(t_begin * (128 * MT) - (p.pitch + 1), 0) / rows_q);
+            uint32_t sb = 0, sp = 0;
+            for (int tile = t_begin; tile < t_end; tile++) {
+                const int tl = min(tile + kE12sPrefetch, t_end - 1);
+                const int pf_end = (int)(((uint32_t)(tl + 1) * (128 * MT) + p.pitch + 1) / rows_q) + 1;
+                if (pf_end > pf_next) {
+                    s2d_prefetch_rows<FX>(p, pf_next, pf_end);
+                    pf_next = pf_end;
+                }
+                mbar_wait_sleep(&slab_full[sb], sp);     // the converters finished this tile
+                if (++sb == (uint32_t)p.nslab) { sb = 0; sp ^= 1; }
+            }
+        }
+    } else if (warp == 1) {
+        // ===== E1 MMA issuer: per plane job KT sub-tiles x 4 shifted taps (K16 each) =====
+        const uint32_t idesc1 = umma_idesc_f16(128, 32);
+        const uint64_t w1d = umma_desc(smem_u32(w1_s), 512, 128);
+        uint32_t J = 0, sb = 0, sp = 0;
+        for (int tile = t_begin; tile < t_end; tile++) {
+            mbar_wait(&slab_full[sb], sp);
+            tc_fence_after();
+            const uint32_t slab = smem_u32(slab_s + (size_t)sb * slab_bytes);
+#pragma unroll 1
+            for (int g = 0; g < 4; g++, J++) {
+                mbar_wait(&e1_empty[J % kE1Slots], ((J / kE1Slots) & 1) ^ 1);
+                tc_fence_after();
+                const uint32_t d = tmem_base + kE1Col + (J % kE1Slots) * (32 * KT);
+#pragma unroll 1
+                for (int t = 0; t < 4; t++) {
+                    int h, shift;
+                    e12s_tap(g, t, p.pitch, h, shift);
+                    // rows of plane h, chunk 0; chunk 1 is PS rows further (LBO)
+                    const uint32_t a0 = slab + (uint32_t)(2 * h * p.PS + (p.pitch + 1) + shift) * 16;
+                    const uint64_t ad = umma_desc(a0, p.PS * 16, 128);
+                    const uint64_t bd = w1d + ((t * 1024) >> 4);
+#pragma unroll
+                    for (int k = 0; k < KT; k++) umma_bf16_warp(d + k * 32, ad + ((k * 2048) >> 4), bd, idesc1, t);
+                }
+                umma_commit_warp(&e1_full[J % kE1Slots]);
+            }
+            umma_commit_warp(&slab_empty[sb]);   // the slab is free once this tile's E1 MMAs read it
+            if (++sb == (uint32_t)p.nslab) { sb = 0; sp ^= 1; }
+        }
+    } else if (warp == 3) {
+        // ===== E2 MMA issuer (as e12) =====
+        const uint32_t idesc2 = umma_idesc_bf16(128, N2);
+        const uint64_t a2d = umma_desc(smem_u32(a2_s), P * 16, 128);
+        const uint64_t w2d = umma_desc(smem_u32(w2_s), N2 * 16, 128);
+        uint32_t pb = 0, pp = 0, acc = 0, accp = 0;
+        for (int tile = t_begin; tile < t_end; tile++) {
+            mbar_wait(&acc_empty[acc], accp ^ 1);
+            tc_fence_after();
+            const uint32_t d = tmem_base + acc * (MT * N2);
+            int pos = 0;
+            for (int g = 0; g < 4; g++) {
+                mbar_wait(&a2_full[pb], pp);
+                tc_fence_after();
+                const uint64_t a = a2d + ((pb * kPlaneBytes) >> 4);
+#pragma unroll 1
+                for (int t = 0; t < p.group_ntaps[g]; t++, pos++) {
+                    const uint64_t at = a + p.group_shift[g][t];
+                    const uint64_t bt = w2d + ((pos * (4 * N2 * 16)) >> 4);
+#pragma unroll
+                    for (int s = 0; s < 2; s++)
+#pragma unroll
+                        for (int mm = 0; mm < MT; mm++)
+                            umma_bf16_warp(d + mm * N2, at + ((2 * s * P * 16 + mm * 2048) >> 4), bt + ((2 * s * N2 * 16) >> 4),
+                                           idesc2, (g == 0 && t == 0 && s == 0) ? 0u : 1u);
+                }
+                umma_commit_warp(&a2_empty[pb]);
+                if (++pb == (uint32_t)p.np) { pb = 0; pp ^= 1; }
+            }
+            umma_commit_warp(&acc_full[acc]);
+            if (++acc == kAccStages) { acc = 0; accp ^= 1; }
+        }
+    } else if (warp >= 4 && warp < 12) {
+        // ===== E1 epilogue (2 warpgroups, alternate sub-tiles): acc + b, ReLU, zero padding,
+        // bf16 -> plane buffer (E2's A operand, scaled by 2^(s+7) like the tile kernel) =====
+        const int wg = (warp - 4) >> 2;
+        const int row = (threadIdx.x - 128) & 127;
+        const int quarter = warp & 3;
+        uint32_t J = 0, pb = 0, pp = 0;
+        for (int tile = t_begin; tile < t_end; tile++) {
+            const uint32_t q0 = (uint32_t)tile * (128 * MT);
+            uint32_t vm[KT];
+#pragma unroll
+            for (int k = 0; k < KT; k++) {
+                // which parity planes hold an E1 pixel at E2-layout position q (e12_decode)
+                const uint32_t q = q0 + k * 128 + row;
+                const uint32_t gr = fdiv(q, p.div_pitch);
+                const int jc = (int)(q - gr * (uint32_t)p.pitch);
+                const int i = (int)(gr - fdiv(gr, p.div_rpf) * (uint32_t)(p.h2 + 1));
+                const bool in = q < p.mtot && i >= 1 && jc >= 1;
+                const uint32_t r1 = 2 * i - 1 < p.h1, c1 = 2 * jc - 1 < p.w1;
+                vm[k] = in ? (1u | (c1 << 1) | (r1 << 2) | ((r1 & c1) << 3)) : 0u;
+            }
+#pragma unroll 1
+            for (int g = 0; g < 4; g++, J++) {
+                mbar_wait(&a2_empty[pb], pp ^ 1);
+                mbar_wait(&e1_full[J % kE1Slots], (J / kE1Slots) & 1);
+                tc_fence_after();
+                uint8_t *plane = a2_s + pb * kPlaneBytes;
+                const uint32_t tacc = tmem_base + ((uint32_t)(quarter * 32) << 16) + kE1Col + (J % kE1Slots) * (32 * KT);
+#pragma unroll 1
+                for (int k = (int)((wg - J * KT) & 1); k < KT; k += 2) {
+                    // E2 reads plane rows < 256 + pitch + 1: the rows of this warp's quarter
+                    // past that (M = 128 granularity) are never read
+                    if (k * 128 + quarter * 32 >= 128 * MT + p.pitch + 1) continue;
+                    uint32_t vmk = vm[0];
+#pragma unroll
+                    for (int i = 1; i < KT; i++)
+                        if (k == i) vmk = vm[i];
+                    const bool valid = (vmk >> g) & 1;
+                    uint32_t v[32];
+                    tmem_ld32(tacc + k * 32, v);
+                    uint32_t pk[16];
+#pragma unroll
+                    for (int j = 0; j < 16; j++)
+                        pk[j] = valid ? pack_bf16x2_relu(__uint_as_float(v[2 * j]), __uint_as_float(v[2 * j + 1])) : 0u;
+                    uint8_t *dst = plane + (size_t)(k * 128 + row) * 16;
+#pragma unroll
+                    for (int c = 0; c < 4; c++)
+                        *reinterpret_cast<uint4 *>(dst + (size_t)c * P * 16) =
+                            make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+                }
+                tc_fence_before();
+                mbar_arrive(&e1_empty[J % kE1Slots]);
+                asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+                mbar_arrive(&a2_full[pb]);
+                if (++pb == (uint32_t)p.np) { pb = 0; pp ^= 1; }
+            }
+        }
+    } else if (warp >= 12) {
+        // ===== E2 epilogue (as e12) =====
+        const int row = threadIdx.x - 384;
+        const int quarter = warp & 3;
+        uint32_t acc = 0, accp = 0;
+        for (int tile = t_begin; tile < t_end; tile++) {
+            mbar_wait_sleep(&acc_full[acc], accp);
+            tc_fence_after();
+#pragma unroll 1
+            for (int mm = 0; mm < MT; mm++) {
+                const uint32_t q = (uint32_t)tile * (128 * MT) + mm * 128 + row;
+                const uint32_t f = fdiv(q, p.div_fstride);
+                const uint32_t r = q - f * p.fstride;
+                const uint32_t oy = fdiv(r, p.div_pitch);
+                const int ox = (int)(r - oy * (uint32_t)p.pitch);
+                const bool valid = q < p.mtot && (int)oy < p.h2 && ox < p.w2;
+                int plane = 0;
+                const int64_t L = layout_pixel(p.out_kind, p.out_pitch, p.out_fstride, (int)f, (int)oy, ox, plane);
+                const uint32_t taddr = tmem_base + ((uint32_t)(quarter * 32) << 16) + acc * (MT * N2) + mm * N2;
+                uint8_t *const row_out = p.out + ((int64_t)plane * p.out_c8 * p.out_lcap + L) * 16;
+                const int64_t chunk_stride = p.out_lcap * 16;
+#pragma unroll
+                for (int cc = 0; cc < N2 / 32; cc++) {
+                    uint32_t v[32];
+                    tmem_ld32(taddr + cc * 32, v);
+                    if (valid) {
+                        uint32_t pk[16];
+#pragma unroll
+                        for (int j = 0; j < 16; j++)
+                            pk[j] = pack_bf16x2_relu(__uint_as_float(v[2 * j]) + s_b2[cc * 32 + 2 * j],
+                                                     __uint_as_float(v[2 * j + 1]) + s_b2[cc * 32 + 2 * j + 1]);
+#pragma unroll
+                        for (int c = 0; c < 4; c++)
+                            *reinterpret_cast<uint4 *>(row_out + (cc * 4 + c) * chunk_stride) =
+                                make_uint4(pk[4 * c], pk[4 * c + 1], pk[4 * c + 2], pk[4 * c + 3]);
+                    }
+                }
+            }
+            tc_fence_before();
+            mbar_arrive(&acc_empty[acc]);
+            if (++acc == kAccStages) { acc = 0; accp ^= 1; }
+        }
+    }
+    __syncwarp();
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 2) {
+        tc_fence_after();
+        tmem_dealloc(tmem_base, 512);
+    }
+}
+
+#define RC_PROXY(x)                     \
+    do {                                \
+        otif_status rc_ = (x);          \
+        if (rc_ != OTIF_OK) return rc_; \
+    } while (0)
+
+// ---------------------------------------------------------------------------
 // host side: plan, weight packing, launch
 // ---------------------------------------------------------------------------
 static uint16_t f32_to_bf16_rne(float f) {
@@ -1496,6 +2073,11 @@ struct otif_proxy {
     int e12;
     int e12_P, e12_np, e12_na1, e12_slab_rows, e12_slab_pitch;
     size_t e12_smem, e12_fixed, e12_unit;
+    int e12_scale;                // s: E1 weights are scaled by 2^s (plan_e12)
+    // space-to-depth variant of the fused E1+E2 kernel (e12s_umma_kernel)
+    int e12s, e12s_PS, e12s_nslab, e12s_np;
+    size_t e12s_smem;
+    uint16_t *e12s_w1_dev;        // fp16 [4 taps][2 chunks][32][8] = bf16(w1) * 2^s
     // band variant of the fused E1+E2 kernel (e12b_umma_kernel); 0 = tile variant
     int e12b, e12b_R, e12b_PB, e12b_D, e12b_NR, e12b_RC, e12b_ring_pitch;
     size_t e12b_smem;
@@ -1705,6 +2287,67 @@ static bool plan_e12(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const f
     p->e12_smem = fixed + (OTIF_E12_TS ? 0 : (size_t)na1 * a1) + (size_t)np * plane;
     p->e12_fixed = fixed;
     p->e12_unit = a1;
+    p->e12_scale = s;
+    return true;
+}
+
+#ifndef OTIF_E12S
+#define OTIF_E12S 1   // space-to-depth variant of the fused E1+E2 kernel where it applies (A/B: 0 = tile)
+#endif
+// Plan the s2d variant (needs plan_e12's scale s and scaled E2 weights): E1's weights as
+// four 2x2-tap K16 blocks over the s2d channels (sy * 2 + sx) * 3 + c, bias * 2^(s+7).
+static bool plan_e12s(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const float *b1) {
+    if (!OTIF_E12S || !p->e12) return false;
+    const GemmLayer &g = p->L[0];
+    const int KT = p->e12_P / 128;
+    const int pitch = g.pitch;
+    const int PS = (int)round_up(128 * 2 + 2 * (pitch + 1), 16);
+    const int s = p->e12_scale;
+    std::vector<uint16_t> w((size_t)4 * 2 * 32 * 8, 0);
+    for (int t = 0; t < 4; t++) {
+        const int ty = t >> 1, tx = t & 1;
+        for (int o = 0; o < 32; o++)
+            for (int sy = 0; sy < 2; sy++)
+                for (int sx = 0; sx < 2; sx++) {
+                    // tap (ty, tx) reads s2d row y - 1 + ty: image row 2(y - 1 + ty) + sy = 2y - 1 + kh
+                    const int kh = 2 * ty + sy - 1, kw = 2 * tx + sx - 1;
+                    if (kh < 0 || kh > 2 || kw < 0 || kw > 2) continue;
+                    for (int c = 0; c < 3; c++) {
+                        const int k = (sy * 2 + sx) * 3 + c;
+                        const float v = ldexpf(bf16_to_f32(f32_to_bf16_rne(w1[((o * 3 + kh) * 3 + kw) * 3 + c])), s);
+                        uint16_t h;
+                        if (!f16_exact(v, &h)) return false;
+                        w[(((size_t)t * 2 + k / 8) * 32 + o) * 8 + (k % 8)] = h;
+                    }
+                }
+    }
+    // E1's bias on s2d channels 12, 13 (128.0 inside the image) of tap (1, 1), chunk 1:
+    // b * 2^s = hi + lo in two fp16 terms (hi * 128 + lo * 128 is exact in the fp32 accumulator)
+    for (int o = 0; o < 32; o++) {
+        const float v = ldexpf(b1[o], s);
+        const __half hi = __float2half_rn(v);
+        const __half lo = __float2half_rn(v - __half2float(hi));
+        if (!isfinite(__half2float(hi))) return false;
+        w[(((size_t)3 * 2 + 1) * 32 + o) * 8 + 4] = __half_as_ushort(hi);
+        w[(((size_t)3 * 2 + 1) * 32 + o) * 8 + 5] = __half_as_ushort(lo);
+    }
+    const size_t fixed = 9 * 4 * 64 * 16 + 4 * 2 * 32 * 16 + 64 * 8 + 16 + 96 * 4 + 1024;
+    const size_t slab = (size_t)8 * PS * 16, plane = (size_t)p->e12_P * 64;
+    int nslab = 0, np = 0;
+#ifndef OTIF_E12S_NSLAB
+#define OTIF_E12S_NSLAB 2
+#endif
+#ifndef OTIF_E12S_NP
+#define OTIF_E12S_NP 2      // 2 plane buffers: the smaller carve-out leaves L1 to the converters (1.18 vs 1.33 ms)
+#endif
+    for (int cs = OTIF_E12S_NSLAB; cs >= 1 && !np; cs--)
+        for (int cp = OTIF_E12S_NP; cp >= 2 && !np; cp--)
+            if (fixed + cs * slab + cp * plane <= 227 * 1024) { nslab = cs; np = cp; }
+    if (!np || KT < 3 || KT > 4 || PS - 256 > 256) return false;
+    if (cudaMalloc(&p->e12s_w1_dev, w.size() * 2) != cudaSuccess) return false;
+    cudaMemcpy(p->e12s_w1_dev, w.data(), w.size() * 2, cudaMemcpyHostToDevice);
+    p->e12s_PS = PS; p->e12s_nslab = nslab; p->e12s_np = np;
+    p->e12s_smem = fixed + nslab * slab + np * plane;
     return true;
 }
 
@@ -1749,18 +2392,16 @@ static void conv_smem(const GemmLayer &g, int &sa, int &sb, size_t &bytes) {
     bytes = sa * a + sb * b + fixed;
 }
 
-// evs (optional): 6 events recorded after E1 (prep) and after each of the 5 GEMM layers
-otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws,
-                         size_t ws_bytes, cudaStream_t stream, cudaEvent_t *evs, PackJob *pj) {
-    Layout lay[5];
+// Lay the workspace out for the largest batch it can hold (so every batch size up to it
+// shares one layout and one zero-initialisation: a smaller final batch does not re-zero)
+// and enqueue the one-time zeroing (a no-op while the header tag matches).
+static otif_status prepare_ws(const otif_proxy *p, int n, uint8_t *ws, size_t ws_bytes, cudaStream_t stream,
+                              Layout lay[5]) {
     size_t need = plan_workspace(p, n, lay);
     if (ws_bytes < need) {
         set_error("otif_proxy_score: workspace %zu B < required %zu B", ws_bytes, need);
         return OTIF_ENOMEM;
     }
-    // Lay the buffers out for the largest batch this workspace can hold, so that every
-    // batch size up to it shares one layout (and one zero-initialisation): a smaller
-    // final batch then does not re-zero the workspace.
     int n_plan = n;
     {
         int64_t lo = n, hi = n;
@@ -1780,6 +2421,40 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
     OTIF_LAUNCH_CHECK();
     ws_tag_kernel<<<1, 1, 0, stream>>>(ws, tag);
     OTIF_LAUNCH_CHECK();
+    return OTIF_OK;
+}
+
+// Source of the s2d variant's converters: FX = 1 (the u8 proxy image) or the frames with
+// an even integer downscale FX x fy, FX in {2, 4, 8} (0: the s2d variant does not apply).
+static int e12s_fx(const otif_proxy *p, int n, const uint8_t *src, int sh, int sw, int *fy) {
+    if (!p->e12s || n <= 0 || !(p->e12 && (int64_t)n * p->L[0].fstride_unit + 4096 < (1ll << 31))) return 0;
+    const int hp = p->d.in_h, wp = p->d.in_w;
+    if (sh == hp && sw == wp) {
+        *fy = 1;
+        return ((uintptr_t)src & 3) == 0 && (wp * 3) % 4 == 0 ? 1 : 0;
+    }
+    if (sw % wp || sh % hp) return 0;
+    const int fx = sw / wp;
+    *fy = sh / hp;
+    if (!(fx == 2 || fx == 4 || fx == 8) || *fy < 2 || *fy % 2) return 0;
+    return ((uintptr_t)src & 15) == 0 && (sw * 3) % 16 == 0 ? fx : 0;
+}
+
+// The pipeline skips stage 1 when the proxy reads its frames directly (e12s_umma_kernel).
+bool proxy_fuses_resize(const otif_proxy *p, int n, const uint8_t *src, int sh, int sw) {
+    int fy;
+    return e12s_fx(p, n, src, sh, sw, &fy) >= 2;
+}
+
+// evs (optional): 6 events recorded after E1 (prep) and after each of the 5 GEMM layers;
+// frames (optional, proxy_fuses_resize true): the source frames [n, sh, sw, 3], read by
+// the fused E1+E2 kernel in place of the proxy image (img unused)
+otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws,
+                         size_t ws_bytes, cudaStream_t stream, cudaEvent_t *evs, PackJob *pj,
+                         const uint8_t *frames, int sh, int sw) {
+    Layout lay[5];
+    otif_status pst = prepare_ws(p, n, ws, ws_bytes, stream, lay);
+    if (pst != OTIF_OK) return pst;
 
     const bool e12 = p->e12 && (int64_t)n * p->L[0].fstride_unit + 4096 < (1ll << 31);
 #if OTIF_E12B_BUILD
@@ -1815,7 +2490,51 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         if (evs) OTIF_CUDA(cudaEventRecord(evs[1], stream));
     } else
 #endif
-    if (e12) {
+    int s_fy = 1;
+    const int s_fx = frames ? e12s_fx(p, n, frames, sh, sw, &s_fy) : e12s_fx(p, n, img, p->d.in_h, p->d.in_w, &s_fy);
+    if (frames && s_fx < 2) {
+        set_error("launch_proxy: frames %dx%d are not an even downscale read by the fused kernel", sw, sh);
+        return OTIF_EINVAL;
+    }
+    if (e12 && s_fx) {
+        // E1 fused into E2, s2d variant, reading the frames (or the proxy image) directly
+        if (evs) OTIF_CUDA(cudaEventRecord(evs[0], stream));
+        const GemmLayer &g = p->L[0];
+        E12sParams e;
+        memset(&e, 0, sizeof(e));
+        e.src = frames ? frames : img;
+        e.sh = frames ? sh : p->d.in_h; e.sw = frames ? sw : p->d.in_w;
+        e.hp = p->d.in_h; e.wp = p->d.in_w; e.fy = s_fy;
+        e.prefetch = kE12sPrefetch > 0 && ((uintptr_t)e.src & 15) == 0 && ((size_t)e.sw * 3) % 16 == 0;
+        e.h1 = p->e1_oh; e.w1 = p->e1_ow; e.h2 = g.out_h; e.w2 = g.out_w; e.pitch = g.pitch;
+        e.fstride = (uint32_t)g.fstride_unit; e.mtot = (uint32_t)((int64_t)n * g.fstride_unit);
+        e.div_pitch = make_fastdiv((uint32_t)g.pitch);
+        e.div_rpf = make_fastdiv((uint32_t)g.out_h + 1);
+        e.div_fstride = make_fastdiv((uint32_t)g.fstride_unit);
+        e.PS = p->e12s_PS; e.nslab = p->e12s_nslab; e.np = p->e12s_np;
+        e.ntiles = (int)cdiv(e.mtot, 256);
+        for (int i = 0; i < 4; i++) {
+            e.group_ntaps[i] = g.group_ntaps[i];
+            for (int t = 0; t < 9; t++) e.group_shift[i][t] = g.group_shift[i][t];
+        }
+        e.w1s = p->e12s_w1_dev;
+        e.wt2 = p->e12_w2_dev; e.b2 = g.bias_dev;
+        e.out_kind = lay[1].kind; e.out = ws + lay[1].offset; e.out_lcap = lay[1].lcap;
+        e.out_c8 = lay[1].c8; e.out_pitch = lay[1].pitch; e.out_fstride = lay[1].fstride;
+        void (*kern)(E12sParams) = nullptr;
+        const bool k3 = p->e12_P == 384;
+        switch (s_fx) {
+            case 1: kern = k3 ? e12s_umma_kernel<3, 1> : e12s_umma_kernel<4, 1>; break;
+            case 2: kern = k3 ? e12s_umma_kernel<3, 2> : e12s_umma_kernel<4, 2>; break;
+            case 4: kern = k3 ? e12s_umma_kernel<3, 4> : e12s_umma_kernel<4, 4>; break;
+            default: kern = k3 ? e12s_umma_kernel<3, 8> : e12s_umma_kernel<4, 8>; break;
+        }
+        OTIF_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)p->e12s_smem));
+        const int grid = e.ntiles < p->num_sms ? e.ntiles : p->num_sms;
+        kern<<<grid, kE12sThreads, p->e12s_smem, stream>>>(e);
+        OTIF_LAUNCH_CHECK();
+        if (evs) OTIF_CUDA(cudaEventRecord(evs[1], stream));
+    } else if (e12) {
         // E1 fused into E2: one kernel writes E3's input
         if (evs) OTIF_CUDA(cudaEventRecord(evs[0], stream));
         const GemmLayer &g = p->L[0];
@@ -2073,6 +2792,7 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
     }
     if (rc == OTIF_OK) p->e12 = plan_e12(p, weights + offs[0], weights + offs[0] + 32 * 27) ? 1 : 0;
     if (rc == OTIF_OK) p->e12b = plan_e12b(p) ? 1 : 0;
+    if (rc == OTIF_OK && !p->e12b) p->e12s = plan_e12s(p, weights + offs[0], weights + offs[0] + 32 * 27) ? 1 : 0;
     if (cudaGetLastError() != cudaSuccess && rc == OTIF_OK) rc = OTIF_ECUDA;
     if (rc != OTIF_OK) {
         otif_proxy_destroy(p);
@@ -2085,6 +2805,7 @@ extern "C" otif_status otif_proxy_create(const otif_proxy_desc *d, const float *
     mix(d->dec);
     mix(p->e12);
     mix(p->e12b);
+    mix(p->e12s);
     p->plan_hash = hsh | 1;
     *out = p;
     return OTIF_OK;
@@ -2101,6 +2822,7 @@ extern "C" void otif_proxy_destroy(otif_proxy *p) {
     if (p->w2_dev) cudaFree(p->w2_dev);
     if (p->e12_w1_dev) cudaFree(p->e12_w1_dev);
     if (p->e12_w2_dev) cudaFree(p->e12_w2_dev);
+    if (p->e12s_w1_dev) cudaFree(p->e12s_w1_dev);
     delete p;
 }
 
@@ -2126,5 +2848,5 @@ extern "C" otif_status otif_proxy_score(const otif_proxy *p, const uint8_t *img,
     OTIF_REQUIRE((((uintptr_t)workspace) & 255) == 0, "otif_proxy_score: workspace must be 256-B aligned");
     otif_status st = check_device(nullptr);
     if (st != OTIF_OK) return st;
-    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream, nullptr, nullptr);
+    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream, nullptr, nullptr, nullptr, 0, 0);
 }

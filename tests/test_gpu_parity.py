@@ -298,11 +298,18 @@ def test_full_size_sampled(wl, blob):
             assert np.array_equal(batches[w["size_idx"]][slot_np[gi]].cpu().numpy(), crop)
 
 
-@pytest.mark.parametrize("wl", [configs.C3, configs.C4_SWEEP[3], configs.C1], ids=lambda w: w.name)
+# C1o: an odd proxy width (105) — the right-edge path of the fused resize
+C1_ODD = configs.C1.with_(name="C1o", src_w=420, sizes=((64, 64), (128, 128), (420, 256)))
+
+
+@pytest.mark.parametrize("wl", [configs.C3, configs.C4_SWEEP[3], configs.C1, configs.C4_SWEEP[2], C1_ODD],
+                         ids=lambda w: w.name)
 def test_pipeline_host_vs_stages(wl, blob):
     """The native runtime (otif_pipeline_run_host, several device batches) returns exactly
-    the windows of the stage-by-stage path (whose parity with the oracle is tested above)."""
-    b = threshold(wl.name, 0.7)
+    the windows of the stage-by-stage path (whose parity with the oracle is tested above).
+    The runtime's proxy reads the frames itself (resize fused into E1's input, downscale
+    factors 4 (C3, C1), 2 (C4d), 8 (C4c)); the stages path reads the resized image."""
+    b = threshold({"C1o": "C1"}.get(wl.name, wl.name), 0.7)
     n = 70
     src = video.frames(wl, n)
     pipe = otif.Pipeline(wl, blob, b, max_batch=32)
