@@ -1477,10 +1477,19 @@ __global__ void __launch_bounds__(kE12bThreads, 1) e12b_umma_kernel(const __grid
 // epilogue, 16-23 converters.
 // ---------------------------------------------------------------------------
 constexpr int kE12sThreads = 768;
-constexpr int kE12sConv = 256;   // converter threads
-// s2d channels 12 and 13 of every pixel inside the image hold 128.0 (fp16 0x5800): with
-// tap (1, 1) weights (b_hi, b_lo) = E1's bias * 2^s split into two fp16 terms, the MMA adds
-// E1's bias (x 2^(s+7), the accumulator scale) exactly as far as fp32 goes
+#ifndef OTIF_E12S_EPI1
+#define OTIF_E12S_EPI1 4          // E1 epilogue warps (4 or 8); the rest after E2's 4 convert
+#endif
+constexpr int kE12sEpi1 = OTIF_E12S_EPI1 * 32;                  // E1 epilogue threads
+constexpr int kE12sEpi2Warp = 4 + OTIF_E12S_EPI1;               // first E2 epilogue warp
+constexpr int kE12sConvWarp = kE12sEpi2Warp + 4;                // first converter warp
+constexpr int kE12sConv = kE12sThreads - kE12sConvWarp * 32;    // converter threads
+// Channel slots of an s2d pixel (the s2d slot order): chunk A (K 0-7) = proxy row 2Y + 1: (sx 1,
+// c 0-2), (sx 0, c 0-2), two bias slots; chunk B (K 8-15) = proxy row 2Y, same order, two
+// zero slots.  The bias slots of every pixel inside the image hold 128.0 (fp16 0x5800):
+// with tap (1, 1) weights (b_hi, b_lo) = E1's bias * 2^s split into two fp16 terms, the MMA
+// adds E1's bias (x 2^(s+7), the accumulator scale) exactly as far as fp32 goes.  Taps
+// (0, 0) and (0, 1) use only chunk A, so they share one K16 MMA (3 MMAs per E1 row, not 4).
 constexpr uint32_t kE12sBiasCh = 0x58005800u;
 #ifndef OTIF_E12S_PREFETCH
 #define OTIF_E12S_PREFETCH 0      // tiles of source rows prefetched to L2 ahead of the converters (measured slower: off)
@@ -1610,25 +1619,26 @@ __device__ __forceinline__ uint32_t s2d_px_slow(const E12sParams &p, int f, int 
     return ((uint32_t)__ldg(a) + __ldg(a + 3) + __ldg(b) + __ldg(b + 3) + 2) >> 2;
 }
 
-// channel sums of one source row for s2d column parity XP into s0..s2 (16-bit lanes:
-// channel pairs (0,1), (2,3), (4,5) of the proxy columns 2X, 2X + 1)
+// channel sums of one source row for s2d column parity XP into s0..s2 (16-bit lanes, the
+// s2d slot order: (sx1 c0, sx1 c1), (sx1 c2, sx0 c0), (sx0 c1, sx0 c2))
 template <int FX, int XP>
 __device__ __forceinline__ void s2d_row_sums(const uint32_t *w, uint32_t &s0, uint32_t &s1, uint32_t &s2) {
     using R = S2dRow<FX>;
     constexpr int A = R::O(XP, 0), B = R::O(XP, 1);
     if constexpr (FX == 1) {
-        s0 += s2d_pair<A, A + 1>(w);
-        s1 += s2d_pair<A + 2, B>(w);
-        s2 += s2d_pair<B + 1, B + 2>(w);
+        s0 += s2d_pair<B, B + 1>(w);
+        s1 += s2d_pair<B + 2, A>(w);
+        s2 += s2d_pair<A + 1, A + 2>(w);
     } else {
-        s0 += s2d_pair<A, A + 1>(w) + s2d_pair<A + 3, A + 4>(w);
-        s1 += s2d_pair<A + 2, B>(w) + s2d_pair<A + 5, B + 3>(w);
-        s2 += s2d_pair<B + 1, B + 2>(w) + s2d_pair<B + 4, B + 5>(w);
+        s0 += s2d_pair<B, B + 1>(w) + s2d_pair<B + 3, B + 4>(w);
+        s1 += s2d_pair<B + 2, A>(w) + s2d_pair<B + 5, A + 3>(w);
+        s2 += s2d_pair<A + 1, A + 2>(w) + s2d_pair<A + 4, A + 5>(w);
     }
 }
 
 // the 12 channels of s2d pixels (Y, 2xx) and (Y, 2xx + 1) of frame f as 6 fp16x2 words
-// each; all source loads are issued before any is used (one memory latency per call)
+// each, words 3 sy .. 3 sy + 2 = proxy row 2Y + sy in the s2d slot order; all source loads
+// are issued before any is used (one memory latency per call)
 template <int FX>
 __device__ __forceinline__ void s2d_pixels(const E12sParams &p, int f, int Y, int xx, uint32_t (&o)[2][6]) {
     using R = S2dRow<FX>;
@@ -1637,9 +1647,10 @@ __device__ __forceinline__ void s2d_pixels(const E12sParams &p, int f, int Y, in
         for (int xp = 0; xp < 2; xp++)
 #pragma unroll
             for (int k = 0; k < 6; k++) {
-                const int k0 = 2 * k, k1 = 2 * k + 1, X = 2 * xx + xp;
-                const uint32_t lo = s2d_px_slow<FX>(p, f, 2 * Y + k0 / 6, 2 * X + (k0 / 3) % 2, k0 % 3);
-                const uint32_t hi = s2d_px_slow<FX>(p, f, 2 * Y + k1 / 6, 2 * X + (k1 / 3) % 2, k1 % 3);
+                // slot s of proxy row sy: s < 3 -> (sx 1, c s), else (sx 0, c s - 3)
+                const int sy = k / 3, s0 = 2 * (k % 3), s1 = s0 + 1, X = 2 * xx + xp;
+                const uint32_t lo = s2d_px_slow<FX>(p, f, 2 * Y + sy, 2 * X + (s0 < 3), s0 % 3);
+                const uint32_t hi = s2d_px_slow<FX>(p, f, 2 * Y + sy, 2 * X + (s1 < 3), s1 % 3);
                 o[xp][k] = s2d_f16(lo | (hi << 16));
             }
         return;
@@ -1741,8 +1752,8 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
             mbar_init(&slab_full[i], kE12sConv); mbar_init(&slab_empty[i], 1);
             mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 128);
         }
-        for (int i = 0; i < kE1Slots; i++) { mbar_init(&e1_full[i], 1); mbar_init(&e1_empty[i], 256); }
-        for (int i = 0; i < kE12MaxPlaneBufs; i++) { mbar_init(&a2_full[i], 256); mbar_init(&a2_empty[i], 1); }
+        for (int i = 0; i < kE1Slots; i++) { mbar_init(&e1_full[i], 1); mbar_init(&e1_empty[i], kE12sEpi1); }
+        for (int i = 0; i < kE12MaxPlaneBufs; i++) { mbar_init(&a2_full[i], kE12sEpi1); mbar_init(&a2_empty[i], 1); }
         fence_barrier_init();
     }
     if (warp == 2) tmem_alloc(tmem_slot, 512);
@@ -1757,7 +1768,7 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
-    if (warp >= 16) {
+    if (warp >= kE12sConvWarp) {
         // ===== converters: slab positions j <-> E2-layout position q = q0 - pitch - 1 + j
         // of the 4 s2d parity planes, 2 chunks each; items (j, plane) with the plane's
         // column parity fastest, so lane pairs read adjacent source spans =====
@@ -1824,9 +1835,9 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
                 for (int xp = 0; xp < 2; xp++) {
                     const int h = 2 * rh + xp;
                     *reinterpret_cast<uint4 *>(slab + ((size_t)(2 * h) * PS + j) * 16) =
-                        make_uint4(o[xp][0], o[xp][1], o[xp][2], o[xp][3]);
+                        make_uint4(o[xp][3], o[xp][4], o[xp][5], bias[xp]);
                     *reinterpret_cast<uint4 *>(slab + ((size_t)(2 * h + 1) * PS + j) * 16) =
-                        make_uint4(o[xp][4], o[xp][5], bias[xp], 0u);
+                        make_uint4(o[xp][0], o[xp][1], o[xp][2], 0u);
                 }
             }
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -1865,16 +1876,28 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
                 mbar_wait(&e1_empty[J % kE1Slots], ((J / kE1Slots) & 1) ^ 1);
                 tc_fence_after();
                 const uint32_t d = tmem_base + kE1Col + (J % kE1Slots) * (32 * KT);
+                // taps (0, 0) and (0, 1) read only chunk A: one K16 MMA takes both (its two
+                // K halves LBO apart, in address order; weight block 0 or 1 to match);
+                // taps (1, 0) and (1, 1) read chunks A and B of their plane (LBO = PS)
+                int h0, s0, h1, s1;
+                e12s_tap(g, 0, p.pitch, h0, s0);
+                e12s_tap(g, 1, p.pitch, h1, s1);
+                const uint32_t a00 = slab + (uint32_t)(2 * h0 * p.PS + (p.pitch + 1) + s0) * 16;
+                const uint32_t a01 = slab + (uint32_t)(2 * h1 * p.PS + (p.pitch + 1) + s1) * 16;
+                const bool fwd = a01 > a00;
+                const uint64_t ad0 = umma_desc(fwd ? a00 : a01, fwd ? a01 - a00 : a00 - a01, 128);
+                const uint64_t bd0 = w1d + ((fwd ? 0 : 1024) >> 4);
+#pragma unroll
+                for (int k = 0; k < KT; k++) umma_bf16_warp(d + k * 32, ad0 + ((k * 2048) >> 4), bd0, idesc1, 0u);
 #pragma unroll 1
-                for (int t = 0; t < 4; t++) {
+                for (int t = 2; t < 4; t++) {
                     int h, shift;
                     e12s_tap(g, t, p.pitch, h, shift);
-                    // rows of plane h, chunk 0; chunk 1 is PS rows further (LBO)
                     const uint32_t a0 = slab + (uint32_t)(2 * h * p.PS + (p.pitch + 1) + shift) * 16;
                     const uint64_t ad = umma_desc(a0, p.PS * 16, 128);
                     const uint64_t bd = w1d + ((t * 1024) >> 4);
 #pragma unroll
-                    for (int k = 0; k < KT; k++) umma_bf16_warp(d + k * 32, ad + ((k * 2048) >> 4), bd, idesc1, t);
+                    for (int k = 0; k < KT; k++) umma_bf16_warp(d + k * 32, ad + ((k * 2048) >> 4), bd, idesc1, 1u);
                 }
                 umma_commit_warp(&e1_full[J % kE1Slots]);
             }
@@ -1913,9 +1936,10 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
             umma_commit_warp(&acc_full[acc]);
             if (++acc == kAccStages) { acc = 0; accp ^= 1; }
         }
-    } else if (warp >= 4 && warp < 12) {
-        // ===== E1 epilogue (2 warpgroups, alternate sub-tiles): acc + b, ReLU, zero padding,
-        // bf16 -> plane buffer (E2's A operand, scaled by 2^(s+7) like the tile kernel) =====
+    } else if (warp >= 4 && warp < kE12sEpi2Warp) {
+        // ===== E1 epilogue (1 or 2 warpgroups, alternate sub-tiles): ReLU (the bias is in
+        // the accumulator), zero padding, bf16 -> plane buffer (E2's A operand) =====
+        constexpr int nwg = kE12sEpi1 / 128;
         const int wg = (warp - 4) >> 2;
         const int row = (threadIdx.x - 128) & 127;
         const int quarter = warp & 3;
@@ -1942,7 +1966,7 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
                 uint8_t *plane = a2_s + pb * kPlaneBytes;
                 const uint32_t tacc = tmem_base + ((uint32_t)(quarter * 32) << 16) + kE1Col + (J % kE1Slots) * (32 * KT);
 #pragma unroll 1
-                for (int k = (int)((wg - J * KT) & 1); k < KT; k += 2) {
+                for (int k = (int)(((uint32_t)wg + nwg * KT * 4 - J * KT % nwg) % nwg); k < KT; k += nwg) {
                     // E2 reads plane rows < 256 + pitch + 1: the rows of this warp's quarter
                     // past that (M = 128 granularity) are never read
                     if (k * 128 + quarter * 32 >= 128 * MT + p.pitch + 1) continue;
@@ -1970,9 +1994,9 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
                 if (++pb == (uint32_t)p.np) { pb = 0; pp ^= 1; }
             }
         }
-    } else if (warp >= 12) {
+    } else if (warp >= kE12sEpi2Warp) {
         // ===== E2 epilogue (as e12) =====
-        const int row = threadIdx.x - 384;
+        const int row = threadIdx.x - kE12sEpi2Warp * 32;
         const int quarter = warp & 3;
         uint32_t acc = 0, accp = 0;
         for (int tile = t_begin; tile < t_end; tile++) {
@@ -2303,33 +2327,38 @@ static bool plan_e12s(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const 
     const int pitch = g.pitch;
     const int PS = (int)round_up(128 * 2 + 2 * (pitch + 1), 16);
     const int s = p->e12_scale;
+    // s2d channel slots (the s2d slot order): chunk A = (sy 1: sx 1 c0-2, sx 0 c0-2, bias, bias),
+    // chunk B = (sy 0: sx 1 c0-2, sx 0 c0-2, 0, 0).  Weight blocks [K half][32 n][8]:
+    // 0 = (tap (0,0) A | tap (0,1) A), 1 = (tap (0,1) A | tap (0,0) A),
+    // 2 = (tap (1,0) A | tap (1,0) B), 3 = (tap (1,1) A | tap (1,1) B)
     std::vector<uint16_t> w((size_t)4 * 2 * 32 * 8, 0);
-    for (int t = 0; t < 4; t++) {
-        const int ty = t >> 1, tx = t & 1;
+    auto put = [&](int blk, int half, int t, int chunk) -> bool {
+        const int ty = t >> 1, tx = t & 1, sy = chunk == 0 ? 1 : 0;
         for (int o = 0; o < 32; o++)
-            for (int sy = 0; sy < 2; sy++)
-                for (int sx = 0; sx < 2; sx++) {
-                    // tap (ty, tx) reads s2d row y - 1 + ty: image row 2(y - 1 + ty) + sy = 2y - 1 + kh
-                    const int kh = 2 * ty + sy - 1, kw = 2 * tx + sx - 1;
-                    if (kh < 0 || kh > 2 || kw < 0 || kw > 2) continue;
-                    for (int c = 0; c < 3; c++) {
-                        const int k = (sy * 2 + sx) * 3 + c;
-                        const float v = ldexpf(bf16_to_f32(f32_to_bf16_rne(w1[((o * 3 + kh) * 3 + kw) * 3 + c])), s);
-                        uint16_t h;
-                        if (!f16_exact(v, &h)) return false;
-                        w[(((size_t)t * 2 + k / 8) * 32 + o) * 8 + (k % 8)] = h;
-                    }
-                }
-    }
-    // E1's bias on s2d channels 12, 13 (128.0 inside the image) of tap (1, 1), chunk 1:
+            for (int slot = 0; slot < 6; slot++) {
+                const int sx = slot < 3 ? 1 : 0, c = slot % 3;
+                // tap (ty, tx) reads s2d row y - 1 + ty: image row 2(y - 1 + ty) + sy = 2y - 1 + kh
+                const int kh = 2 * ty + sy - 1, kw = 2 * tx + sx - 1;
+                if (kh < 0 || kh > 2 || kw < 0 || kw > 2) continue;
+                const float v = ldexpf(bf16_to_f32(f32_to_bf16_rne(w1[((o * 3 + kh) * 3 + kw) * 3 + c])), s);
+                uint16_t h;
+                if (!f16_exact(v, &h)) return false;
+                w[(((size_t)blk * 2 + half) * 32 + o) * 8 + slot] = h;
+            }
+        return true;
+    };
+    if (!(put(0, 0, 0, 0) && put(0, 1, 1, 0) && put(1, 0, 1, 0) && put(1, 1, 0, 0) && put(2, 0, 2, 0) &&
+          put(2, 1, 2, 1) && put(3, 0, 3, 0) && put(3, 1, 3, 1)))
+        return false;
+    // E1's bias on chunk A slots 6, 7 (128.0 inside the image) of tap (1, 1):
     // b * 2^s = hi + lo in two fp16 terms (hi * 128 + lo * 128 is exact in the fp32 accumulator)
     for (int o = 0; o < 32; o++) {
         const float v = ldexpf(b1[o], s);
         const __half hi = __float2half_rn(v);
         const __half lo = __float2half_rn(v - __half2float(hi));
         if (!isfinite(__half2float(hi))) return false;
-        w[(((size_t)3 * 2 + 1) * 32 + o) * 8 + 4] = __half_as_ushort(hi);
-        w[(((size_t)3 * 2 + 1) * 32 + o) * 8 + 5] = __half_as_ushort(lo);
+        w[(((size_t)3 * 2 + 0) * 32 + o) * 8 + 6] = __half_as_ushort(hi);
+        w[(((size_t)3 * 2 + 0) * 32 + o) * 8 + 7] = __half_as_ushort(lo);
     }
     const size_t fixed = 9 * 4 * 64 * 16 + 4 * 2 * 32 * 16 + 64 * 8 + 16 + 96 * 4 + 1024;
     const size_t slab = (size_t)8 * PS * 16, plane = (size_t)p->e12_P * 64;
