@@ -238,7 +238,7 @@ def measure_pipeline(otif, wl, blob, thr, src, steps, warmup, sizes=None, caps=N
     stage_ms, launches = pipe.stage_ms()
     ctr = pipe.counters()
     out = {"pipe": pipe, "ms_total": ms_total, "stage_ms": stage_ms, "launches": launches, "ctr": ctr,
-           "frames": n * steps, "steps": steps, "overlap": overlap}
+           "frames": n * steps, "steps": steps, "overlap": overlap, "resize_fused": pipe.resize_fused()}
     return out
 
 
@@ -280,6 +280,16 @@ def rooflines(wl, m, peaks, peak_src, traffic=None, fused_pack=False):
     out = {"conv": conv}
     for k, byts in (("resize", rs_bytes), ("pack", pk_bytes)):
         ms = sm[k]
+        if k == "resize" and m.get("resize_fused"):
+            # stage 1 runs inside the E1+E2 kernel (its converter warps read the frames; the
+            # proxy image is never written): the source-row bytes against that kernel's time
+            src_b = byts - wl.proxy_h * wl.proxy_w * 3 * frames
+            e12_ms = sm["proxy_prep_e1"] + sm["conv_e2"]
+            gbs = src_b / (e12_ms / 1e3) / 1e9 if e12_ms > 0 else None
+            out[k] = {"bound": "hbm", "fused_into": "conv_e1_e2 (e12s_umma_kernel: converter warps read the frames)",
+                      "bytes_per_step": src_b / steps, "e1_e2_ms_per_step": e12_ms / steps,
+                      "achieved_in_e1_e2": gbs, "peak": hbm, "unit": "GB/s", "frac": gbs / hbm if gbs else None}
+            continue
         if k == "pack" and fused_pack:
             # the copy runs inside the E5 / D1 kernels of the next step; "pack" holds only the
             # slot kernel and the drain of what the fused warps left
@@ -609,8 +619,11 @@ def run_otif(args):
                        "threshold": b, "threshold_q": 0.7, "proxy": "E1-E5 (32,64,128,256,256) + D1 128 + D2 1, "
                        "random init PCG64(20220612)", "l2": "inputs (7.0 GB/GPU) exceed the 126 MB L2; no flush",
                        "parallelism": f"dp{world} (clip-sharded)"},
-            "roofline": dict(rl["conv"], kernel="proxy convs on tcgen05: e12_umma_kernel (E1 fused into E2) + "
-                                                "conv_umma_kernel (E3..E5, D1+D2 head)",
+            "roofline": dict(rl["conv"], kernel=("proxy convs on tcgen05: e12s_umma_kernel (resize + E1 fused into "
+                                                 "E2: reads the u8 frames) + conv_umma_kernel (E3..E5, D1+D2 head)"
+                                                 if m.get("resize_fused") else
+                                                 "proxy convs on tcgen05: e12_umma_kernel (E1 fused into E2) + "
+                                                 "conv_umma_kernel (E3..E5, D1+D2 head)"),
                              per_launch="5 launches per batch of 4500 frames; achieved = algorithmic FLOPs of "
                                         "E1..D1 / CUDA-event time of those launches on the pipeline stream",
                              fused_work=("the E5 and D1 launches also copy the previous step's detector batches "

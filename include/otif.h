@@ -333,6 +333,9 @@ const int32_t *otif_pipeline_frame_counts(const otif_pipeline *p);
 /* Device pointer to the detector batch of size s ([batch_cap[s], h_s, w_s, 3] u8, the
  * last packed device batch), or NULL. */
 uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s);
+/* 1 if the last device batch skipped stage 1: the proxy's first kernel read the frames
+ * itself (even integer downscale, the space-to-depth E1 variant), else 0. */
+int32_t otif_pipeline_resize_fused(const otif_pipeline *p);
 /* Complete a pack left pending by pack_overlap = 2 (enqueued on `stream`). */
 otif_status otif_pipeline_flush(otif_pipeline *p, cudaStream_t stream);
 otif_status otif_pipeline_reset_counters(otif_pipeline *p, cudaStream_t stream);

@@ -128,6 +128,8 @@ def lib() -> ctypes.CDLL:
         L.otif_pipeline_frame_hashes.restype = P
         L.otif_pipeline_frame_counts.argtypes = [P]
         L.otif_pipeline_frame_counts.restype = P
+        L.otif_pipeline_resize_fused.argtypes = [P]
+        L.otif_pipeline_resize_fused.restype = i32
         L.otif_pipeline_detector_batch.argtypes = [P, i32]
         L.otif_pipeline_detector_batch.restype = P
         L.otif_pipeline_flush.argtypes = [P, P]
@@ -154,7 +156,7 @@ EXPORTED = ("otif_status_str", "otif_last_error", "otif_version", "otif_resize",
             "otif_proxy_destroy", "otif_proxy_grid", "otif_proxy_workspace_bytes", "otif_proxy_score",
             "otif_select_workspace_bytes", "otif_select_windows", "otif_pack_windows",
             "otif_pipeline_create", "otif_pipeline_destroy", "otif_pipeline_run_host",
-            "otif_pipeline_run_device", "otif_pipeline_flush", "otif_pipeline_detector_batch", "otif_pipeline_frame_hashes",
+            "otif_pipeline_run_device", "otif_pipeline_flush", "otif_pipeline_resize_fused", "otif_pipeline_detector_batch", "otif_pipeline_frame_hashes",
             "otif_pipeline_frame_counts", "otif_pipeline_counters", "otif_pipeline_reset_counters",
             "otif_pipeline_set_timing", "otif_pipeline_stage_ms", "otif_choose_workspace_bytes",
             "otif_choose_window_sizes", "otif_window_recall", "otif_track_resample", "otif_dbscan_workspace_bytes",

@@ -239,6 +239,10 @@ class Pipeline:
         check(lib().otif_pipeline_run_device(self.handle, _ptr(frames), frames.shape[0], int(frame_base),
                                              _stream(stream)), "otif_pipeline_run_device")
 
+    def resize_fused(self) -> bool:
+        """True if the last device batch's proxy read the frames itself (no stage-1 launch)."""
+        return bool(lib().otif_pipeline_resize_fused(self.handle))
+
     def detector_batch(self, s: int) -> torch.Tensor:
         """Copy of the detector batch of size s ([batch_cap[s], h_s, w_s, 3] u8) as last packed."""
         ptr = lib().otif_pipeline_detector_batch(self.handle, s)

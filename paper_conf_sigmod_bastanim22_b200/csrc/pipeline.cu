@@ -112,6 +112,7 @@ struct otif_pipeline {
     PackJob *job = nullptr;
     int *inv = nullptr;
     int job_pending = 0;
+    int resize_fused = 0;          // the last device batch read its frames in the proxy (no stage 1)
     cudaEvent_t ev_pending = nullptr;       // recorded where the pending job was built
     cudaStream_t pending_stream = nullptr;
 };
@@ -208,6 +209,7 @@ static otif_status run_batch(otif_pipeline *p, const uint8_t *src, int nb, int f
         // even integer downscale: the fused E1+E2 kernel reads the frames itself (stage 1
         // fused into the proxy's first kernel, no proxy image in HBM)
         const bool fused = proxy_fuses_resize(p->proxy, mb, frames, d.src_h, d.src_w);
+        p->resize_fused = fused ? 1 : 0;
         {
             NvtxRange r("otif.resize");
             int t0 = tmark(p, st);
@@ -460,6 +462,8 @@ extern "C" const int32_t *otif_pipeline_frame_counts(const otif_pipeline *p) {
 extern "C" uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s) {
     return (p && s >= 0 && s < p->d.k) ? p->batches[s] : nullptr;
 }
+
+extern "C" int32_t otif_pipeline_resize_fused(const otif_pipeline *p) { return p ? p->resize_fused : 0; }
 
 extern "C" otif_status otif_pipeline_flush(otif_pipeline *p, cudaStream_t stream) {
     OTIF_REQUIRE(p, "otif_pipeline_flush: NULL");

@@ -90,7 +90,7 @@ def full(path, tag, names):
                         d[m] = v
                 d[m + ".unit"] = units[col[m]]
         res.append(d)
-    lines = [f"# ncu --set full: proxy conv kernels (e12_umma_kernel = E1+E2, conv_umma_kernel = E3..D1) ({tag})", "",
+    lines = [f"# ncu --set full: proxy conv kernels (e12s_umma_kernel = resize + E1 + E2, conv_umma_kernel = E3..D1) ({tag})", "",
              f"Source: `{os.path.basename(path)}` (one 4500-frame C2 batch, layers in capture order).", "",
              "| layer | time (us) | DRAM read (MB) | DRAM write (MB) | L2 bytes (MB) | tensor pipe % (mem_tensor) | "
              "tensor realtime % | DRAM % | regs |", "|---|---|---|---|---|---|---|---|---|"]

@@ -2,7 +2,7 @@
 """Two C2 pipeline steps (4500 frames each) for ncu captures of the proxy kernels of the
 second step, with the fused pack of the first step riding in them (pack_overlap 2) or not.
 
-    ncu --set full -k regex:"conv_umma|e12_umma" -s 5 -c 5 python scripts/prof_conv.py [--overlap 2]
+    ncu --set full -k regex:"conv_umma|e12s?_umma" -s 5 -c 5 python scripts/prof_conv.py [--overlap 2]
 """
 import argparse
 import json

@@ -1,6 +1,7 @@
 #!/usr/bin/env python
 """Small C1 run of every hot-path kernel for compute-sanitizer (memcheck / racecheck /
-synccheck / initcheck): resize (even-factor and general), proxy (E1+E2 fused, E3..D1 and
+synccheck / initcheck): resize (even-factor and general), proxy (E1+E2 fused reading the
+proxy image or the frames, several tiles per CTA, E3..D1 and
 the S = 2 separate-E1 path), select (scores and mask input, 4- and 8-connectivity, the
 deferred pass and the rescan path), pack (bulk, funnel and byte branches), the native
 pipeline, NEXT-1 choose (multi-candidate launch) and the recall kernel.
@@ -46,6 +47,12 @@ otif.otif_pack_windows(src, wl.src_h, wl.src_w, wt, torch.tensor([len(rows)], dt
 otif.otif_pack_windows(src, wl.src_h, wl.src_w, r["windows"], r["total"], wl.sizes, [8, 8, 4])
 pipe = otif.Pipeline(wl, blob, 0.5, max_batch=3)
 pipe.run_host(src.cpu().contiguous())
+# resize fused into E1+E2 with several tiles per CTA (the slab overlap carried between tiles)
+src_many = video.frames(wl, 170).cuda()
+pipe_many = otif.Pipeline(wl, blob, 0.5, max_batch=170, pack_overlap=2)
+pipe_many.run_device(src_many)
+pipe_many.flush()
+assert pipe_many.resize_fused()
 gm = torch.from_numpy(np.stack([video.gt_mask(video.make_scene(wl).gt_boxes(t), wl.src_w, wl.src_h, wl.cell)
                                 for t in range(4)])).cuda()
 tuning.choose_window_sizes(gm, wl.src_w, wl.src_h, wl.cell, tuning.candidate_sizes(wl.src_w, wl.src_h, wl.cell)[:6], k=3)
