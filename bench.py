@@ -267,6 +267,16 @@ def rooflines(wl, m, peaks, peak_src, traffic=None, fused_pack=False):
         name = "conv_e1_e2" if i == 0 else s
         per_layer[name] = {"ms_per_step": ms / steps, "tflops": fl / (ms / 1e3) / 1e12 if ms > 0 else None,
                            "frac_burst": fl / (ms / 1e3) / 1e12 / burst if ms > 0 else None}
+        if i == 0 and m.get("resize_fused") and ms > 0:
+            # the launch also streams the frames (stage 1 fused in): its own roofline is the
+            # larger of the HBM time of those bytes and the tensor time of E1 + E2
+            src_b = (resize_bytes_per_frame(wl) - wl.proxy_h * wl.proxy_w * 3) * frames
+            t_hbm = src_b / (float(peaks.get("hbm_gbs")) * 1e9) * 1e3
+            t_tc = fl / (burst * 1e12) * 1e3
+            per_layer[name].update({"reads_frames_bytes_per_step": src_b / steps,
+                                    "roofline_ms_per_step": max(t_hbm, t_tc) / steps,
+                                    "roofline_bound": "hbm" if t_hbm >= t_tc else "tensor",
+                                    "frac_of_roofline": max(t_hbm, t_tc) / ms})
     hbm = float(peaks.get("hbm_gbs"))
     rs_bytes = resize_bytes_per_frame(wl) * frames
     pk_bytes = 2.0 * 3 * int(m["ctr"][14].item())
@@ -626,10 +636,14 @@ def run_otif(args):
                                                  "conv_umma_kernel (E3..E5, D1+D2 head)"),
                              per_launch="5 launches per batch of 4500 frames; achieved = algorithmic FLOPs of "
                                         "E1..D1 / CUDA-event time of those launches on the pipeline stream",
-                             fused_work=("the E5 and D1 launches also copy the previous step's detector batches "
-                                         f"({rl['pack']['bytes_per_step'] / 1e9:.1f} GB per step through HBM; "
-                                         "pack_overlap 2), which the tensor FLOP count does not credit"
-                                         if args.pack_overlap > 0 else None),
+                             fused_work=("; ".join(x for x in (
+                                 ("the E5 and D1 launches also copy the previous step's detector batches "
+                                  f"({rl['pack']['bytes_per_step'] / 1e9:.1f} GB per step through HBM; pack_overlap 2)"
+                                  if args.pack_overlap > 0 else None),
+                                 (f"the E1+E2 launch also reads the frames ({rl['resize']['bytes_per_step'] / 1e9:.1f} GB "
+                                  "per step: stage 1 fused in)" if m.get("resize_fused") else None)) if x)
+                                 + ", which the tensor FLOP count does not credit") if (args.pack_overlap > 0 or
+                                                                                      m.get("resize_fused")) else None,
                              frac_serial_schedule=(serial["rooflines"]["conv"]["frac"] if serial else None)),
             "stages": {k: v for k, v in rl.items() if k != "conv"},
             "serial_schedule": serial,
