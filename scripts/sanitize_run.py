@@ -28,6 +28,11 @@ img = otif.otif_resize(src, wl.proxy_h, wl.proxy_w)
 otif.otif_resize(src, 187, 333)
 px = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, blob)
 sc = px.score(img)
+# a 640-wide proxy (E2 pitch 161 > 127): the tile E1+E2 kernel (e12_umma_kernel) instead of e12s
+c4d = configs.C4_SWEEP[3]
+src_w = video.frames(c4d, 2).cuda()
+img_w = otif.otif_resize(src_w, c4d.proxy_h, c4d.proxy_w)
+otif.Proxy(c4d.proxy_h, c4d.proxy_w, c4d.n_strided, blob).score(img_w)
 s2 = wl.with_(name="C1s2", cell=8)
 otif.Proxy(s2.proxy_h, s2.proxy_w, s2.n_strided, blob).score(img[:2])
 r = otif.otif_select_windows(sc, None, 0.5, wl.src_w, wl.src_h, wl.cell, wl.sizes, want_mask=True)
