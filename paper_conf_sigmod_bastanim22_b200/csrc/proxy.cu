@@ -1817,8 +1817,10 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
                     const int yy = (int)gr - 1, xx = (int)(r - gr * (uint32_t)p.pitch) - 1;
                     const int Y = 2 * yy + rh;
                     if (yy >= 0 && xx >= 0 && Y < p.h1 && 2 * xx < p.w1) {
-#if OTIF_E12S_NOLOAD    // timing experiment only: no source loads (wrong results)
+#if OTIF_E12S_NOLOAD == 1    // timing experiment only: no source loads (wrong results)
                         o[0][0] = (uint32_t)(Y + xx);
+#elif OTIF_E12S_NOLOAD == 2  // timing experiment only: loads from a cache-resident corner
+                        s2d_pixels<FX>(p, 0, Y & 7, xx & 15, o);
 #else
                         s2d_pixels<FX>(p, (int)f, Y, xx, o);
 #endif
