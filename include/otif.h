@@ -330,6 +330,10 @@ const int64_t *otif_pipeline_counters(const otif_pipeline *p);
  * frames) and the window count. */
 const int64_t *otif_pipeline_frame_hashes(const otif_pipeline *p);
 const int32_t *otif_pipeline_frame_counts(const otif_pipeline *p);
+/* Device pointer, valid after the last device batch's proxy (stream order): its cell
+ * scores fp32 [n, gh, gw] (the proxy's score of every cell), index = frame -
+ * batch start. */
+const float *otif_pipeline_scores(const otif_pipeline *p);
 /* Device pointer to the detector batch of size s ([batch_cap[s], h_s, w_s, 3] u8, the
  * last packed device batch), or NULL. */
 uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s);

@@ -206,6 +206,7 @@ class Pipeline:
             d.batch_cap[i] = int(caps[i])
         self.k = d.k
         self.sizes = sizes
+        self.grid = (-(-workload.src_h // workload.cell), -(-workload.src_w // workload.cell))
         self.batch_cap = [int(c) for c in caps]
         self.desc = d
         w = np.ascontiguousarray(weights, np.float32)
@@ -268,6 +269,17 @@ class Pipeline:
             out.copy_(torch.as_tensor(_CAI(), device="cuda"))
             return out
         return view(hp, "<i8", torch.int64), view(cp, "<i4", torch.int32)
+
+    def scores(self, n: int) -> torch.Tensor:
+        """Copy of the cell scores fp32 [n, gh, gw] of the first n frames of the last device batch."""
+        ptr = lib().otif_pipeline_scores(self.handle)
+        shape = (n, self.grid[0], self.grid[1])
+
+        class _CAI:
+            __cuda_array_interface__ = {"shape": shape, "typestr": "<f4", "data": (ptr, False), "version": 3}
+        out = torch.empty(shape, dtype=torch.float32, device="cuda")
+        out.copy_(torch.as_tensor(_CAI(), device="cuda"))
+        return out
 
     def flush(self, stream=None):
         """Complete a pack left pending by pack_overlap = 2."""

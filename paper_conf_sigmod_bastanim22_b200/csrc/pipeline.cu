@@ -459,6 +459,10 @@ extern "C" const int32_t *otif_pipeline_frame_counts(const otif_pipeline *p) {
     return p ? p->counts : nullptr;
 }
 
+extern "C" const float *otif_pipeline_scores(const otif_pipeline *p) {
+    return p ? p->scores : nullptr;
+}
+
 extern "C" uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s) {
     return (p && s >= 0 && s < p->d.k) ? p->batches[s] : nullptr;
 }

@@ -302,6 +302,26 @@ def test_full_size_sampled(wl, blob):
 C1_ODD = configs.C1.with_(name="C1o", src_w=420, sizes=((64, 64), (128, 128), (420, 256)))
 
 
+@pytest.mark.parametrize("wl,n", [(configs.C2, 300), (configs.C3, 60), (configs.C1, 32), (C1_ODD, 32),
+                                  (configs.C4_SWEEP[1], 64), (configs.C4_SWEEP[3], 16), (configs.C4_SWEEP[2], 16)],
+                         ids=lambda v: getattr(v, "name", str(v)))
+def test_pipeline_fused_scores_bit_identical(wl, n, blob):
+    """The runtime's proxy reading the frames itself (stage 1 inside the E1+E2 kernel for
+    the even downscales 4 (C2, C3, C1, C4b) and 8 (C4c), incl. the odd width's right edge
+    (C1o); C4d's 640-wide proxy takes the separate resize and the tile kernel) gives the
+    SAME fp32 scores as the stage-by-stage path (otif_resize, then the proxy on the resized
+    image), whose parity with the oracle is tested above; the bottom edge of an odd proxy
+    height (C2: 135) is in every frame."""
+    src = video.frames(wl, n).cuda()
+    pipe = otif.Pipeline(wl, blob, 0.5, max_batch=n)     # (the threshold does not touch the scores)
+    pipe.run_device(src)
+    torch.cuda.synchronize()
+    got = pipe.scores(n)
+    img = otif.otif_resize(src, wl.proxy_h, wl.proxy_w)
+    ref = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, blob).score(img)
+    assert torch.equal(got, ref), (wl.name, (got - ref).abs().max().item())
+
+
 @pytest.mark.parametrize("wl", [configs.C3, configs.C4_SWEEP[3], configs.C1, configs.C4_SWEEP[2], C1_ODD],
                          ids=lambda w: w.name)
 def test_pipeline_host_vs_stages(wl, blob):
