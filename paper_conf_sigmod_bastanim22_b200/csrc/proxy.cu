@@ -2371,8 +2371,21 @@ static bool plan_e12s(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const 
 #ifndef OTIF_E12S_NP
 #define OTIF_E12S_NP 2      // 2 plane buffers: the smaller carve-out leaves L1 to the converters (1.18 vs 1.33 ms)
 #endif
+    // Plane buffers: two (the E1 epilogue writes one while E2 reads the other) when the
+    // whole carve-out still fits 196 KB, so that >= 60 KB of L1 are left to the converters'
+    // source loads (in-flight lines, profiles/r02s_e12s.md); else ONE plane buffer, which
+    // brings wide frames under that carve-out (C3 3.71 -> 3.35 ms per 3000 frames; C2,
+    // which fits with two, would lose 1.6% with one: profiles/r02y_e12s_smem_ab.log)
+#ifndef OTIF_E12S_L1_CARVE
+#define OTIF_E12S_L1_CARVE (196 * 1024)
+#endif
+    // (one slab instead of two is far slower: the converters could not run ahead of E1)
+    for (int cp = OTIF_E12S_NP; cp >= 1 && !np; cp--)
+        if (fixed + OTIF_E12S_NSLAB * slab + cp * plane + 1024 /* static */ <= OTIF_E12S_L1_CARVE) {
+            nslab = OTIF_E12S_NSLAB; np = cp;
+        }
     for (int cs = OTIF_E12S_NSLAB; cs >= 1 && !np; cs--)
-        for (int cp = OTIF_E12S_NP; cp >= 2 && !np; cp--)
+        for (int cp = OTIF_E12S_NP; cp >= 1 && !np; cp--)
             if (fixed + cs * slab + cp * plane <= 227 * 1024) { nslab = cs; np = cp; }
     if (!np || KT < 3 || KT > 4 || PS - 256 > 256) return false;
     if (cudaMalloc(&p->e12s_w1_dev, w.size() * 2) != cudaSuccess) return false;
