@@ -28,6 +28,12 @@
 
 namespace otif {
 
+#ifdef OTIF_SEL_PROF     // profiling build: keep the grouping phases out of line (per-line ncu attribution)
+#define OTIF_SEL_NOINLINE __noinline__
+#else
+#define OTIF_SEL_NOINLINE
+#endif
+
 constexpr int kSelWarpsMax = 16;
 constexpr int kMatMax = 128;  // fit-matrix capacity (components per frame); larger n -> rescan path
 constexpr int kSmallClusters = 64;  // components per frame in the first (high-occupancy) pass
@@ -152,7 +158,44 @@ struct Frame {  // one warp's shared-memory slice
     short *bj;         // [cap] best partner
     signed char *sidx; // [cap]
     signed char *alive;// [cap]
+    Rect16 *pw;        // [cap] placed windows (pixels) during a phase-B search; aliases par
 };
+
+// Phase B (reading R10): the lexicographically first pair (i < j) of alive clusters whose
+// placed windows overlap.  The placements are computed once per search into F.pw (the
+// union-find array, dead after the bounding boxes), then the warp tests 32 partners j of
+// one i per step (ballot: the smallest j of the first i with an overlap).
+__device__ __forceinline__ bool first_overlap(const SelectParams &p, Frame &F, int n, int lane, int &mi, int &mj) {
+    for (int i = lane; i < n; i += 32) {
+        if (!F.alive[i]) continue;
+        int x, y;
+        const int s = F.sidx[i];
+        place(p, F.cl[i], s, x, y);
+        Rect16 r;
+        r.x0 = (short)x; r.y0 = (short)y; r.x1 = (short)(x + p.sw[s]); r.y1 = (short)(y + p.sh[s]);
+        F.pw[i] = r;
+    }
+    __syncwarp();
+    for (int i = 0; i + 1 < n; i++) {
+        if (!F.alive[i]) continue;
+        const Rect16 a = F.pw[i];
+        for (int j0 = i + 1; j0 < n; j0 += 32) {
+            const int j = j0 + lane;
+            bool ov = false;
+            if (j < n && F.alive[j]) {
+                const Rect16 b = F.pw[j];
+                ov = a.x0 < b.x1 && b.x0 < a.x1 && a.y0 < b.y1 && b.y0 < a.y1;
+            }
+            const unsigned m = __ballot_sync(0xffffffffu, ov);
+            if (m) {
+                mi = i;
+                mj = j0 + __ffs(m) - 1;
+                return true;
+            }
+        }
+    }
+    return false;
+}
 
 // best partner of row i over alive j > i (max gain, smallest j)
 __device__ __forceinline__ void rescan_row(const SelectParams &p, Frame &F, int n, int i) {
@@ -207,7 +250,7 @@ __device__ __forceinline__ void row_best_warp(const SelectParams &p, Frame &F, c
     }
 }
 
-__device__ void merge_update_mat(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U, int I, int J) {
+__device__ OTIF_SEL_NOINLINE void merge_update_mat(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U, int I, int J) {
     const int S = p.nmat;
     __syncwarp();
     if (lane == 0) {
@@ -262,7 +305,7 @@ __device__ void merge_update_mat(const SelectParams &p, Frame &F, int n, int lan
     __syncwarp();
 }
 
-__device__ bool greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U) {
+__device__ OTIF_SEL_NOINLINE bool greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U) {
     const int S = p.nmat;
     for (int q = lane; q < n * n; q += 32) {
         const int i = q / n, j = q - i * n;
@@ -288,29 +331,8 @@ __device__ bool greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, 
             if (F.sidx[I] == p.full) return true;  // exact full-frame exit (see select_kernel)
         }
         // phase B: lexicographically first pair of alive clusters whose placed windows overlap
-        int mi = 0x7FFF, mj = 0x7FFF;
-        for (int i = lane; i < n; i += 32) {
-            if (!F.alive[i]) continue;
-            int xi, yi, si = F.sidx[i];
-            place(p, F.cl[i], si, xi, yi);
-            for (int j = i + 1; j < n; j++) {
-                if (!F.alive[j]) continue;
-                int xj, yj, sj = F.sidx[j];
-                place(p, F.cl[j], sj, xj, yj);
-                if (xi < xj + p.sw[sj] && xj < xi + p.sw[si] && yi < yj + p.sh[sj] && yj < yi + p.sh[si]) {
-                    if (i < mi) { mi = i; mj = j; }
-                    break;
-                }
-            }
-            if (mi != 0x7FFF) break;
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            int oi = __shfl_xor_sync(0xffffffffu, mi, o);
-            int oj = __shfl_xor_sync(0xffffffffu, mj, o);
-            if (oi < mi) { mi = oi; mj = oj; }
-        }
-        if (mi == 0x7FFF) break;
+        int mi, mj;
+        if (!first_overlap(p, F, n, lane, mi, mj)) break;
         merge_update_mat(p, F, n, lane, U, mi, mj);
         if (F.sidx[mi] == p.full) return true;
     }
@@ -360,29 +382,8 @@ __device__ bool greedy_rescan(const SelectParams &p, Frame &F, int n, int lane) 
             __syncwarp();
         }
         // phase B: merge the lexicographically first pair whose placed windows overlap
-        int mi = 0x7FFF, mj = 0x7FFF;
-        for (int i = lane; i < n; i += 32) {
-            if (!F.alive[i]) continue;
-            int xi, yi, si = F.sidx[i];
-            place(p, F.cl[i], si, xi, yi);
-            for (int j = i + 1; j < n; j++) {
-                if (!F.alive[j]) continue;
-                int xj, yj, sj = F.sidx[j];
-                place(p, F.cl[j], sj, xj, yj);
-                if (xi < xj + p.sw[sj] && xj < xi + p.sw[si] && yi < yj + p.sh[sj] && yj < yi + p.sh[si]) {
-                    if (i < mi) { mi = i; mj = j; }
-                    break;
-                }
-            }
-            if (mi != 0x7FFF) break;  // later i of this lane are larger
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            int oi = __shfl_xor_sync(0xffffffffu, mi, o);
-            int oj = __shfl_xor_sync(0xffffffffu, mj, o);
-            if (oi < mi) { mi = oi; mj = oj; }
-        }
-        if (mi == 0x7FFF) break;
+        int mi, mj;
+        if (!first_overlap(p, F, n, lane, mi, mj)) break;
         __syncwarp();
         if (lane == 0) {
             F.cl[mi] = runion(F.cl[mi], F.cl[mj]);
@@ -437,6 +438,7 @@ __global__ void __launch_bounds__(kSelWarpsMax * 32) select_kernel(const __grid_
     F.bj = reinterpret_cast<short *>(F.bg + cap);
     F.sidx = reinterpret_cast<signed char *>(F.bj + cap);
     F.alive = F.sidx + cap;
+    F.pw = reinterpret_cast<Rect16 *>(base);   // par / cid are dead once the boxes are built
 
     // --- stage 3: threshold (strict ">") ---
     int npos = 0;
