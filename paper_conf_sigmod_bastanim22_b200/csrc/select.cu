@@ -307,12 +307,30 @@ __device__ OTIF_SEL_NOINLINE void merge_update_mat(const SelectParams &p, Frame 
 
 __device__ OTIF_SEL_NOINLINE bool greedy_matrix(const SelectParams &p, Frame &F, int n, int lane, uint8_t *U) {
     const int S = p.nmat;
-    for (int q = lane; q < n * n; q += 32) {
-        const int i = q / n, j = q - i * n;
-        if (j > i) U[(size_t)i * S + j] = (uint8_t)fit_rect(p, runion(F.cl[i], F.cl[j]));
+    // fit matrix and row bests in one pass: row i's entries are computed by the lanes that
+    // reduce them (all clusters alive; same max / smallest-j rule as row_best_warp)
+    for (int i = 0; i < n; i++) {
+        const Rect16 ri = F.cl[i];
+        const long long ci = F.cost[i];
+        long long best = kNoGain;
+        int arg = 0x7FFF;
+        for (int j = i + 1 + lane; j < n; j += 32) {
+            const uint8_t u = (uint8_t)fit_rect(p, runion(ri, F.cl[j]));
+            U[(size_t)i * S + j] = u;
+            const long long g = ci + F.cost[j] - p.cost[u];
+            if (g > best) { best = g; arg = j; }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            long long ob = __shfl_xor_sync(0xffffffffu, best, o);
+            int oa = __shfl_xor_sync(0xffffffffu, arg, o);
+            if (ob > best || (ob == best && oa < arg)) { best = ob; arg = oa; }
+        }
+        if (lane == 0) {
+            F.bg[i] = arg == 0x7FFF ? kNoGain : best;
+            F.bj[i] = (short)(arg == 0x7FFF ? -1 : arg);
+        }
     }
-    __syncwarp();
-    for (int i = 0; i < n; i++) row_best_warp(p, F, U, S, n, i, lane);
     __syncwarp();
     while (true) {
         while (true) {  // phase A
@@ -772,16 +790,25 @@ otif_status launch_select(const float *scores, const uint8_t *mask_in, float thr
     OTIF_CUDA(cudaMemsetAsync(p.defer_count, 0, 4, stream));
     int num_sms = 148;
     check_device(&num_sms);
+    const size_t cap_bytes = 200 * 1024;
+    // a batch that fits ONE wave with full-size slices takes a single pass with them (the
+    // small-slice pass only buys occupancy, and a deferred frame redoes its components)
+    int small_cap = p.cap_f < kSmallClusters ? p.cap_f : kSmallClusters;
+    {
+        int gm;
+        const int fb = sel_frame_bytes(gh, gw, p.cap_f, small_costs ? (int)round_up(p.cap_f < kMatMax ? p.cap_f : kMatMax, 8) : 0, &gm);
+        const int64_t full_warps = std::max<int64_t>(1, std::min<int64_t>(kSelWarpsMax, (int64_t)cap_bytes / fb));
+        if ((int64_t)n <= full_warps * num_sms) small_cap = p.cap_f;
+    }
     for (int pass = 0; pass < 2; pass++) {
         // pass 0: small slices (<= kSmallClusters components, many frames per SM);
         // pass 1: the deferred frames with full-size slices
-        const int ccap = pass == 0 ? (p.cap_f < kSmallClusters ? p.cap_f : kSmallClusters) : p.cap_f;
-        if (pass == 1 && ccap == (p.cap_f < kSmallClusters ? p.cap_f : kSmallClusters)) break;  // nothing deferred
+        const int ccap = pass == 0 ? small_cap : p.cap_f;
+        if (pass == 1 && ccap == small_cap) break;  // nothing deferred
         p.ccap = ccap;
         p.from_list = pass;
         p.nmat = small_costs ? (int)round_up(ccap < kMatMax ? ccap : kMatMax, 8) : 0;
         p.frame_bytes = sel_frame_bytes(gh, gw, ccap, p.nmat, &p.gmat_offset);
-        const size_t cap_bytes = 200 * 1024;
         int warps = (int)(cap_bytes / p.frame_bytes);
         warps = warps < 1 ? 1 : (warps > kSelWarpsMax ? kSelWarpsMax : warps);
         if (pass == 0) {  // spread small batches over the SMs rather than packing frames into few CTAs
