@@ -1779,7 +1779,19 @@ __global__ void __launch_bounds__(kE12sThreads, 1) e12s_umma_kernel(const __grid
             mbar_wait_sleep(&slab_empty[sb], sp ^ 1);
             uint8_t *slab = slab_s + (size_t)sb * slab_bytes;
             int j0 = 0;
-            if (tile != t_begin) {
+            if (tile != t_begin && nov > 128 * MT) {
+                // wide frames (overlap longer than a tile; two slabs): positions [256, nov) of
+                // the previous slab were moved in, not converted, so after a converter-wide
+                // barrier any thread moves any position
+                const uint8_t *prev = slab_s + (size_t)(sb ^ 1) * slab_bytes;
+                asm volatile("bar.sync 1, %0;" ::"n"(kE12sConv) : "memory");
+#pragma unroll 1
+                for (int ch = 0; ch < 8; ch++)
+                    for (int j = ct; j < nov; j += kE12sConv)
+                        *reinterpret_cast<uint4 *>(slab + ((size_t)ch * PS + j) * 16) =
+                            *reinterpret_cast<const uint4 *>(prev + ((size_t)ch * PS + j + 128 * MT) * 16);
+                j0 = nov;
+            } else if (tile != t_begin) {
                 // positions [256, PS) of the previous slab are [0, PS - 256) of this one: each
                 // thread moves the ones it converted itself (no converter-wide barrier; with
                 // one slab, in place: sources >= 256 > destinations, then one barrier before
@@ -2362,7 +2374,10 @@ static bool plan_e12s(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const 
         w[(((size_t)3 * 2 + 0) * 32 + o) * 8 + 6] = __half_as_ushort(hi);
         w[(((size_t)3 * 2 + 0) * 32 + o) * 8 + 7] = __half_as_ushort(lo);
     }
-    const size_t fixed = 9 * 4 * 64 * 16 + 4 * 2 * 32 * 16 + 64 * 8 + 16 + 96 * 4 + 1024;
+    // weights, then (after the slabs and plane buffers) the barriers, TMEM slot and E2 bias
+    // (432 B, 1 KB reserved); the 1 KB static reservation of the kernel's aligned buffer is
+    // counted by the carve-out rule below
+    const size_t fixed = 9 * 4 * 64 * 16 + 4 * 2 * 32 * 16 + 1024;
     const size_t slab = (size_t)8 * PS * 16, plane = (size_t)p->e12_P * 64;
     int nslab = 0, np = 0;
 #ifndef OTIF_E12S_NSLAB
@@ -2386,8 +2401,9 @@ static bool plan_e12s(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const 
         }
     for (int cs = OTIF_E12S_NSLAB; cs >= 1 && !np; cs--)
         for (int cp = OTIF_E12S_NP; cp >= 1 && !np; cp--)
-            if (fixed + cs * slab + cp * plane <= 227 * 1024) { nslab = cs; np = cp; }
-    if (!np || KT < 3 || KT > 4 || PS - 256 > 256) return false;
+            if (fixed + cs * slab + cp * plane + 1024 <= 227 * 1024) { nslab = cs; np = cp; }
+    // an overlap longer than a tile (proxy width > 508) is moved between two slabs
+    if (!np || KT < 3 || KT > 4 || (PS - 256 > 256 && nslab < 2)) return false;
     if (cudaMalloc(&p->e12s_w1_dev, w.size() * 2) != cudaSuccess) return false;
     cudaMemcpy(p->e12s_w1_dev, w.data(), w.size() * 2, cudaMemcpyHostToDevice);
     p->e12s_PS = PS; p->e12s_nslab = nslab; p->e12s_np = np;
