@@ -28,11 +28,17 @@ img = otif.otif_resize(src, wl.proxy_h, wl.proxy_w)
 otif.otif_resize(src, 187, 333)
 px = otif.Proxy(wl.proxy_h, wl.proxy_w, wl.n_strided, blob)
 sc = px.score(img)
-# a 640-wide proxy (E2 pitch 161 > 127): the tile E1+E2 kernel (e12_umma_kernel) instead of e12s
+# a 640-wide proxy (E2 pitch 161: the slab overlap is longer than a tile and moved between
+# the two slabs after a converter barrier), 8 frames = several tiles per CTA
 c4d = configs.C4_SWEEP[3]
-src_w = video.frames(c4d, 2).cuda()
+src_w = video.frames(c4d, 8).cuda()
 img_w = otif.otif_resize(src_w, c4d.proxy_h, c4d.proxy_w)
 otif.Proxy(c4d.proxy_h, c4d.proxy_w, c4d.n_strided, blob).score(img_w)
+# an odd-width proxy image (105 px: 315-B rows, not 4-B aligned): the tile E1+E2 kernel
+# (e12_umma_kernel) instead of e12s
+c1o = wl.with_(name="C1o", src_w=420, sizes=((64, 64), (128, 128), (420, 256)))
+img_o = otif.otif_resize(video.frames(c1o, 4).cuda(), c1o.proxy_h, c1o.proxy_w)
+otif.Proxy(c1o.proxy_h, c1o.proxy_w, c1o.n_strided, blob).score(img_o)
 s2 = wl.with_(name="C1s2", cell=8)
 otif.Proxy(s2.proxy_h, s2.proxy_w, s2.n_strided, blob).score(img[:2])
 r = otif.otif_select_windows(sc, None, 0.5, wl.src_w, wl.src_h, wl.cell, wl.sizes, want_mask=True)

@@ -307,11 +307,12 @@ C1_ODD = configs.C1.with_(name="C1o", src_w=420, sizes=((64, 64), (128, 128), (4
                          ids=lambda v: getattr(v, "name", str(v)))
 def test_pipeline_fused_scores_bit_identical(wl, n, blob):
     """The runtime's proxy reading the frames itself (stage 1 inside the E1+E2 kernel for
-    the even downscales 4 (C2, C3, C1, C4b) and 8 (C4c), incl. the odd width's right edge
-    (C1o); C4d's 640-wide proxy takes the separate resize and the tile kernel) gives the
-    SAME fp32 scores as the stage-by-stage path (otif_resize, then the proxy on the resized
-    image), whose parity with the oracle is tested above; the bottom edge of an odd proxy
-    height (C2: 135) is in every frame."""
+    the even downscales 4 (C2, C3, C1, C4b), 2 (C4d: a 640-wide proxy, slab overlap longer
+    than a tile) and 8 (C4c)) gives the SAME fp32 scores as the stage-by-stage path
+    (otif_resize, then the proxy on the resized image), whose parity with the oracle is
+    tested above; C1o's 1260-B source rows are not 16-B aligned, so it takes the separate
+    resize and the tile E1+E2 kernel on its odd-width proxy.  The bottom edge of an odd
+    proxy height (C2: 135) is in every frame."""
     src = video.frames(wl, n).cuda()
     pipe = otif.Pipeline(wl, blob, 0.5, max_batch=n)     # (the threshold does not touch the scores)
     pipe.run_device(src)
