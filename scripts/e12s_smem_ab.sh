@@ -8,7 +8,7 @@ while read -r v; do
   echo "[$v] $t | C2 $(timeout 120 python scripts/e12_stage_time.py 2>&1 | tail -1) | C2 $(timeout 120 python scripts/e12_stage_time.py 2>&1 | tail -1) | C3 $(timeout 200 python scripts/e12_stage_time.py C3 2>&1 | tail -1)" >> $LOG
 done <<VARS
 ${VARIANTS:-
--DOTIF_E12S_NP=1 -DOTIF_E12S_NPMIN=1
+-DOTIF_E12S_NP=1
 -DOTIF_E12S_NSLAB=1
--DOTIF_E12S_NSLAB=1 -DOTIF_E12S_NP=1 -DOTIF_E12S_NPMIN=1}
+-DOTIF_E12S_NSLAB=1 -DOTIF_E12S_NP=1}
 VARS
