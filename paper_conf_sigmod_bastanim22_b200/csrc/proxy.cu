@@ -1492,7 +1492,7 @@ constexpr int kE12sConv = kE12sThreads - kE12sConvWarp * 32;    // converter thr
 // (0, 0) and (0, 1) use only chunk A, so they share one K16 MMA (3 MMAs per E1 row, not 4).
 constexpr uint32_t kE12sBiasCh = 0x58005800u;
 #ifndef OTIF_E12S_PREFETCH
-#define OTIF_E12S_PREFETCH 0      // tiles of source rows prefetched to L2 ahead of the converters (measured slower: off)
+#define OTIF_E12S_PREFETCH 1      // tiles of source rows prefetched to L2 ahead of the converters (1: C2 E1+E2 1.156 -> 1.000 ms; 2: 1.081; profiles/r02y_e12s_prefetch_ab.log)
 #endif
 #ifndef OTIF_E12S_NOLOAD
 #define OTIF_E12S_NOLOAD 0
