@@ -2386,22 +2386,15 @@ static bool plan_e12s(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const 
 #ifndef OTIF_E12S_NP
 #define OTIF_E12S_NP 2      // 2 plane buffers: the smaller carve-out leaves L1 to the converters (1.18 vs 1.33 ms)
 #endif
-    // Plane buffers: two (the E1 epilogue writes one while E2 reads the other) when the
-    // whole carve-out still fits 196 KB, so that >= 60 KB of L1 are left to the converters'
-    // source loads (in-flight lines, profiles/r02s_e12s.md); else ONE plane buffer, which
-    // brings wide frames under that carve-out (C3 3.71 -> 3.35 ms per 3000 frames; C2,
-    // which fits with two, would lose 1.6% with one: profiles/r02y_e12s_smem_ab.log)
-#ifndef OTIF_E12S_L1_CARVE
-#define OTIF_E12S_L1_CARVE (196 * 1024)
-#endif
-    // (one slab instead of two is far slower: the converters could not run ahead of E1)
-    for (int cp = OTIF_E12S_NP; cp >= 1 && !np; cp--)
-        if (fixed + OTIF_E12S_NSLAB * slab + cp * plane + 1024 /* static */ <= OTIF_E12S_L1_CARVE) {
-            nslab = OTIF_E12S_NSLAB; np = cp;
-        }
+    // Plane buffers: two (the E1 epilogue writes one while E2 reads the other) where they
+    // fit, else one (the 640-wide C4d).  Before the L2 prefetch of the source rows, one
+    // plane buffer paid on wide frames because it left more L1 to the converters' DRAM
+    // loads (C3 3.71 -> 3.35 ms, profiles/r02y_e12s_smem_ab.log); with the prefetch their
+    // loads hit L2 and two buffers are faster again (C4b 0.236 -> 0.213 ms, C3 3.23 -> 3.17,
+    // profiles/r02y_e12s_carve_ab.log).
     for (int cs = OTIF_E12S_NSLAB; cs >= 1 && !np; cs--)
         for (int cp = OTIF_E12S_NP; cp >= 1 && !np; cp--)
-            if (fixed + cs * slab + cp * plane + 1024 <= 227 * 1024) { nslab = cs; np = cp; }
+            if (fixed + cs * slab + cp * plane + 1024 /* static */ <= 227 * 1024) { nslab = cs; np = cp; }
     // an overlap longer than a tile (proxy width > 508) is moved between two slabs
     if (!np || KT < 3 || KT > 4 || (PS - 256 > 256 && nslab < 2)) return false;
     if (cudaMalloc(&p->e12s_w1_dev, w.size() * 2) != cudaSuccess) return false;
