@@ -19,16 +19,21 @@ from paper_conf_sigmod_bastanim22_b200 import refine  # noqa: E402
 from synth import tracks  # noqa: E402
 
 
-def timed(fn, reps):
+def timed(fn, reps, trials=3):
+    """Mean time of `reps` back-to-back calls (CUDA events), median over `trials` blocks
+    (the blocks differ by the SM clock the power controller settles on)."""
     fn()
     torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record()
-    for _ in range(reps):
-        r = fn()
-    e1.record()
-    torch.cuda.synchronize()
-    return e0.elapsed_time(e1) / reps, r
+    ts = []
+    for _ in range(trials):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        for _ in range(reps):
+            r = fn()
+        e1.record()
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1) / reps)
+    return float(np.median(ts)), r
 
 
 def run(wl, reps=5):
@@ -50,6 +55,7 @@ def run(wl, reps=5):
     pairs = wl.n_train * (wl.n_train + 1) / 2           # blocks on/above the diagonal ~ n^2/2
     return {"workload": f"{wl.name}: {wl.n_train} S* tracks (native rate), {wl.n_query} queries at g={wl.gap}, "
                         f"N={wl.n_points}, eps={wl.eps}, min_pts={wl.min_pts}, k={wl.k}, rho={wl.rho}",
+            "timing": f"per call: median over 3 blocks of {reps} back-to-back calls (CUDA events)",
             "resample_ms": t_res, "dbscan_ms": t_db, "centers_ms": t_c, "refine_ms": t_ref,
             "index_build_ms": t_res + t_db + t_c, "refine_tracks_per_s": wl.n_query / (t_ref / 1e3),
             "clusters": n_clusters, "noise_fraction": float((labels < 0).float().mean().item()),
