@@ -1472,11 +1472,14 @@ __global__ void __launch_bounds__(kE12bThreads, 1) e12b_umma_kernel(const __grid
 // runs a contiguous range of tiles and the slab of tile t + 1 overlaps tile t's by
 // 2 (pitch + 1) positions, which are copied on chip, so every s2d pixel is converted once.
 //
-// Roles (768 threads): warp 1 E1 MMA (KT x 4 per plane job), warp 2 TMEM allocator, warp 3
-// E2 MMA, warps 4-11 E1 epilogue (+ bias, ReLU, zero padding -> E2's A operand), 12-15 E2
-// epilogue, 16-23 converters.
+// Roles (OTIF_E12S_THREADS = 640): warp 0 L2 prefetch of the next tile's source rows,
+// warp 1 E1 MMA (KT x 4 per plane job), warp 2 TMEM allocator, warp 3 E2 MMA, warps 4-7 E1
+// epilogue (ReLU, zero padding -> E2's A operand), 8-11 E2 epilogue, 12-19 converters.
 // ---------------------------------------------------------------------------
-constexpr int kE12sThreads = 768;
+#ifndef OTIF_E12S_THREADS
+#define OTIF_E12S_THREADS 640   // 20 warps: 8 converter warps (with the L2 prefetch: C3 E1+E2 3.12 -> 2.87 ms, C2 -1%; 12 / 6 converter warps slower; profiles/r02y_e12s_threads_ab.log)
+#endif
+constexpr int kE12sThreads = OTIF_E12S_THREADS;
 #ifndef OTIF_E12S_EPI1
 #define OTIF_E12S_EPI1 4          // E1 epilogue warps (4 or 8); the rest after E2's 4 convert
 #endif
