@@ -1,5 +1,5 @@
 """Per-stage times (pipeline stage events) on a workload, 5 steps.
-usage: e12_stage_time.py [workload (default C2, the headline)] [pack_overlap (default 0)] [quantile q]
+usage: e12_stage_time.py [workload (default C2, the headline)] [pack_overlap (default 0)] [quantile q] [proxy_batch]
 With q the threshold is the frozen B_q of the workload (tests/golden/thresholds.json),
 else 0.5; "total" = the mean step time (CUDA events around each run_device)."""
 import json, os, sys
@@ -13,10 +13,11 @@ ov = int(sys.argv[2]) if len(sys.argv) > 2 else 0
 thr = 0.5
 if len(sys.argv) > 3:
     from tests.helpers import threshold
-    thr = threshold(wl.name, float(sys.argv[3]))
+    thr = threshold(wl.name, float(sys.argv[3])) if float(sys.argv[3]) > 0 else 0.5
 src = torch.empty((wl.n_frames, wl.src_h, wl.src_w, 3), dtype=torch.uint8, device="cuda")
 video.make_scene(wl).render(range(wl.n_frames), out=src)
-pipe = otif.Pipeline(wl, weights.proxy_weights(), thr, max_batch=wl.n_frames, pack_overlap=ov)
+pb = int(sys.argv[4]) if len(sys.argv) > 4 else 0
+pipe = otif.Pipeline(wl, weights.proxy_weights(), thr, max_batch=wl.n_frames, pack_overlap=ov, proxy_batch=pb)
 pipe.run_device(src)
 torch.cuda.synchronize()
 pipe.set_timing(True)
