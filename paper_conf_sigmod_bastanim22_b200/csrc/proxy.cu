@@ -2379,7 +2379,7 @@ static bool plan_e12s(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const 
     }
     // weights, then (after the slabs and plane buffers) the barriers, TMEM slot and E2 bias
     // (432 B, 1 KB reserved); the 1 KB static reservation of the kernel's aligned buffer is
-    // counted by the carve-out rule below
+    // added in the fit test below
     const size_t fixed = 9 * 4 * 64 * 16 + 4 * 2 * 32 * 16 + 1024;
     const size_t slab = (size_t)8 * PS * 16, plane = (size_t)p->e12_P * 64;
     int nslab = 0, np = 0;
@@ -2387,7 +2387,7 @@ static bool plan_e12s(otif_proxy *p, const float *w1 /* [32][3][3][3] */, const 
 #define OTIF_E12S_NSLAB 2
 #endif
 #ifndef OTIF_E12S_NP
-#define OTIF_E12S_NP 2      // 2 plane buffers: the smaller carve-out leaves L1 to the converters (1.18 vs 1.33 ms)
+#define OTIF_E12S_NP 2      // max plane buffers (3 measured slower: 1.33 vs 1.18 ms, less L1 for the converters)
 #endif
     // Plane buffers: two (the E1 epilogue writes one while E2 reads the other) where they
     // fit, else one (the 640-wide C4d).  Before the L2 prefetch of the source rows, one
