@@ -72,6 +72,22 @@ def conv_macs_per_frame(wl, enc, dec):
     return layers, head   # layers[0] = E1, [1..5] = E2..E5, D1
 
 
+def conv_act_bytes_per_frame(wl, enc, dec):
+    """Algorithmic activation bytes of E2..E5, D1 per frame (bf16 input + output; D1 writes the
+    fp32 scores): the HBM bytes a layer-by-layer schedule must move (weights are L2-resident)."""
+    h, w, c = wl.proxy_h, wl.proxy_w, 3
+    dims = []
+    for i in range(6):
+        cout = enc[i] if i < 5 else dec
+        s = 2 if (i < 5 and i < wl.n_strided) else 1
+        h2, w2 = -(-h // s), -(-w // s)
+        dims.append((h * w * c, h2 * w2 * cout))
+        h, w, c = h2, w2, cout
+    out = [2 * (dims[i][0] + dims[i][1]) for i in range(1, 5)]
+    out.append(2 * dims[5][0] + 4 * h * w)
+    return out   # [E2, E3, E4, E5, D1]
+
+
 def resize_bytes_per_frame(wl):
     """Algorithmic bytes of stage 1: the distinct source rows bilinear touches + the output."""
     rows = set()
@@ -236,9 +252,11 @@ def measure_pipeline(otif, wl, blob, thr, src, steps, warmup, sizes=None, caps=N
     torch.cuda.synchronize()
     ms_total = e0.elapsed_time(e1)
     stage_ms, launches = pipe.stage_ms()
+    pack_units = pipe.pack_units() if overlap else None   # which layer carried how much of the copy
     ctr = pipe.counters()
     out = {"pipe": pipe, "ms_total": ms_total, "stage_ms": stage_ms, "launches": launches, "ctr": ctr,
-           "frames": n * steps, "steps": steps, "overlap": overlap, "resize_fused": pipe.resize_fused()}
+           "frames": n * steps, "steps": steps, "overlap": overlap, "resize_fused": pipe.resize_fused(),
+           "pack_units": pack_units}
     return out
 
 
@@ -280,6 +298,27 @@ def rooflines(wl, m, peaks, peak_src, traffic=None, fused_pack=False):
     hbm = float(peaks.get("hbm_gbs"))
     rs_bytes = resize_bytes_per_frame(wl) * frames
     pk_bytes = 2.0 * 3 * int(m["ctr"][14].item())
+    pu = m.get("pack_units")
+    drain_share = None
+    if pu and pu["total"] > 0:
+        # fused pack: a layer that also copied detector-batch units has the combined roofline
+        # max(tensor time of its FLOPs, HBM time of its activation bytes + the pack bytes it
+        # copied); pack bytes per layer from the unit claim counter (average unit size)
+        act = conv_act_bytes_per_frame(wl, configs.ENC_WIDTHS, configs.DEC_WIDTH)
+        for i, (name, key) in enumerate(zip(["conv_e3", "conv_e4", "conv_e5", "conv_d1_head"],
+                                            ["E3", "E4", "E5", "D1"])):
+            if pu[key] == 0 or per_layer[name]["ms_per_step"] <= 0:
+                continue
+            share = pu[key] / pu["total"]
+            pb = share * pk_bytes / steps
+            ab = act[i + 1] * frames / steps
+            fl = 2.0 * macs[i + 2] * frames / steps
+            t_tc, t_hbm = fl / (burst * 1e12) * 1e3, (ab + pb) / (hbm * 1e9) * 1e3
+            per_layer[name].update({"pack_share": share, "pack_bytes_per_step": pb, "act_bytes_per_step": ab,
+                                    "combined_roofline_ms_per_step": max(t_tc, t_hbm),
+                                    "combined_bound": "hbm" if t_hbm >= t_tc else "tensor",
+                                    "frac_of_combined_roofline": max(t_tc, t_hbm) / per_layer[name]["ms_per_step"]})
+        drain_share = pu["drain"] / pu["total"]
     step_sum = sum(sm.values())
     conv = {"bound": "tensor", "achieved": tflops, "peak": burst, "unit": "TFLOP/s", "frac": tflops / burst,
             "frac_vs_sustained": tflops / sustained, "traffic": traffic,
@@ -287,6 +326,8 @@ def rooflines(wl, m, peaks, peak_src, traffic=None, fused_pack=False):
                                       "sustained (4 s loop under the power cap) beside it",
             "algorithmic": f"2 x {sum(macs) / 1e6:.1f} MMAC/frame (E1..D1) x {frames // steps} frames per launch set",
             "layers": per_layer, "ms_per_step": conv_ms / steps, "share_of_step": conv_ms / step_sum}
+    if drain_share is not None:
+        conv["pack_units_left_to_drain"] = drain_share
     out = {"conv": conv}
     for k, byts in (("resize", rs_bytes), ("pack", pk_bytes)):
         ms = sm[k]

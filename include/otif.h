@@ -334,6 +334,12 @@ const int32_t *otif_pipeline_frame_counts(const otif_pipeline *p);
  * scores fp32 [n, gh, gw] (the proxy's score of every cell), index = frame -
  * batch start. */
 const float *otif_pipeline_scores(const otif_pipeline *p);
+/* Timing aid (otif_pipeline_set_timing on, pack_overlap > 0): pack copy units (P:L133's
+ * crop/pack, in units of <= 32 KB of one window's rows) copied during each proxy GEMM layer
+ * since the last call: units[0..4] = E2 (when not fused into E1+E2), E3, E4, E5, D1 (the
+ * layers whose spare warps drain the previous batch's pack), units[5] = units left to the
+ * drain kernel, units[6] = all units.  Synchronises the device; resets the tally. */
+otif_status otif_pipeline_pack_units(otif_pipeline *p, uint64_t *units);
 /* Device pointer to the detector batch of size s ([batch_cap[s], h_s, w_s, 3] u8, the
  * last packed device batch), or NULL. */
 uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s);

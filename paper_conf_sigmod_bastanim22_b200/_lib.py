@@ -130,6 +130,8 @@ def lib() -> ctypes.CDLL:
         L.otif_pipeline_frame_counts.restype = P
         L.otif_pipeline_scores.argtypes = [P]
         L.otif_pipeline_scores.restype = P
+        L.otif_pipeline_pack_units.argtypes = [P, ctypes.POINTER(ctypes.c_uint64)]
+        L.otif_pipeline_pack_units.restype = ctypes.c_int
         L.otif_pipeline_resize_fused.argtypes = [P]
         L.otif_pipeline_resize_fused.restype = i32
         L.otif_pipeline_detector_batch.argtypes = [P, i32]
@@ -159,7 +161,7 @@ EXPORTED = ("otif_status_str", "otif_last_error", "otif_version", "otif_resize",
             "otif_select_workspace_bytes", "otif_select_windows", "otif_pack_windows",
             "otif_pipeline_create", "otif_pipeline_destroy", "otif_pipeline_run_host",
             "otif_pipeline_run_device", "otif_pipeline_flush", "otif_pipeline_resize_fused", "otif_pipeline_detector_batch", "otif_pipeline_frame_hashes",
-            "otif_pipeline_frame_counts", "otif_pipeline_scores", "otif_pipeline_counters", "otif_pipeline_reset_counters",
+            "otif_pipeline_frame_counts", "otif_pipeline_scores", "otif_pipeline_pack_units", "otif_pipeline_counters", "otif_pipeline_reset_counters",
             "otif_pipeline_set_timing", "otif_pipeline_stage_ms", "otif_choose_workspace_bytes",
             "otif_choose_window_sizes", "otif_window_recall", "otif_track_resample", "otif_dbscan_workspace_bytes",
             "otif_track_dbscan", "otif_centers_workspace_bytes", "otif_track_centers", "otif_track_refine",

@@ -281,6 +281,13 @@ class Pipeline:
         out.copy_(torch.as_tensor(_CAI(), device="cuda"))
         return out
 
+    def pack_units(self):
+        """Pack copy units per proxy GEMM layer since the last call (timing on, pack_overlap):
+        dict E2, E3, E4, E5, D1, drain, total."""
+        u = (ctypes.c_uint64 * 7)()
+        check(lib().otif_pipeline_pack_units(self.handle, u), "otif_pipeline_pack_units")
+        return dict(zip(("E2", "E3", "E4", "E5", "D1", "drain", "total"), [int(x) for x in u]))
+
     def flush(self, stream=None):
         """Complete a pack left pending by pack_overlap = 2."""
         check(lib().otif_pipeline_flush(self.handle, _stream(stream)), "otif_pipeline_flush")

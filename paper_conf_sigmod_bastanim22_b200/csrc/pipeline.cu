@@ -23,7 +23,7 @@ namespace otif {
 
 otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws, size_t ws_bytes,
                          cudaStream_t stream, cudaEvent_t *evs, PackJob *pj, const uint8_t *frames, int sh,
-                         int sw);
+                         int sw, unsigned long long *pj_snap);
 bool proxy_fuses_resize(const otif_proxy *p, int n, const uint8_t *src, int sh, int sw);
 bool pack_job_applies(int32_t src_h, int32_t src_w, int32_t det_h, int32_t det_w, const otif_wsize *sizes, int32_t k,
                       uint8_t *const *batches);
@@ -115,7 +115,13 @@ struct otif_pipeline {
     int resize_fused = 0;          // the last device batch read its frames in the proxy (no stage 1)
     cudaEvent_t ev_pending = nullptr;       // recorded where the pending job was built
     cudaStream_t pending_stream = nullptr;
+    // timing only: per proxy pass that carried a pending job, the claim counter after each
+    // GEMM layer [0..4] and the job's unit total [5] (device rows of 8, read by
+    // otif_pipeline_pack_units)
+    unsigned long long *pj_snaps = nullptr;
+    int n_snaps = 0;
 };
+constexpr int kMaxSnaps = 1024;
 
 // a pending job built on another stream: order this stream after it
 static otif_status wait_pending(otif_pipeline *p, cudaStream_t st) {
@@ -177,8 +183,15 @@ static otif_status run_proxy(otif_pipeline *p, const uint8_t *img, int mb, float
     cudaEvent_t evs[6];
     int from = tmark(p, st);
     for (int i = 0; i < 6 && p->timing; i++) from = treserve(p, ST_PREP + i, from, &evs[i]);
+    unsigned long long *snap = nullptr;
+    if (p->timing && pj && p->n_snaps < kMaxSnaps) {
+        if (!p->pj_snaps && cudaMalloc(&p->pj_snaps, (size_t)kMaxSnaps * 8 * 8) != cudaSuccess) return OTIF_ENOMEM;
+        snap = p->pj_snaps + (size_t)p->n_snaps++ * 8;
+        OTIF_CUDA(cudaMemsetAsync(snap, 0, 8 * 8, st));   // layers without a GEMM launch stay 0
+        OTIF_CUDA(cudaMemcpyAsync(snap + 5, &pj->units_base[p->d.k], 8, cudaMemcpyDeviceToDevice, st));
+    }
     RC(launch_proxy(p->proxy, img, mb, scores, p->proxy_ws, p->proxy_ws_bytes, st, p->timing ? evs : nullptr, pj,
-                    frames, p->d.src_h, p->d.src_w));
+                    frames, p->d.src_h, p->d.src_w, snap));
     p->launches += proxy_launches(p->proxy);
     return OTIF_OK;
 }
@@ -341,7 +354,7 @@ extern "C" void otif_pipeline_destroy(otif_pipeline *p) {
     if (p->s_copy) cudaStreamSynchronize(p->s_copy);
     void *bufs[] = {p->src[0], p->src[1], p->img, p->mask, p->proxy_ws, p->sel_ws, p->scores, p->windows, p->counts,
                     p->offsets, p->total, p->slot, p->size_count, p->ctr, p->out_win, p->out_counts, p->out_total,
-                    p->job, p->inv, p->frame_hash};
+                    p->job, p->inv, p->frame_hash, p->pj_snaps};
     for (void *b : bufs)
         if (b) cudaFree(b);
     for (int s = 0; s < 8; s++)
@@ -461,6 +474,29 @@ extern "C" const int32_t *otif_pipeline_frame_counts(const otif_pipeline *p) {
 
 extern "C" const float *otif_pipeline_scores(const otif_pipeline *p) {
     return p ? p->scores : nullptr;
+}
+
+extern "C" otif_status otif_pipeline_pack_units(otif_pipeline *p, uint64_t *units) {
+    OTIF_REQUIRE(p && units, "otif_pipeline_pack_units: NULL argument");
+    for (int i = 0; i < 7; i++) units[i] = 0;
+    if (p->n_snaps > 0) {
+        std::vector<unsigned long long> h((size_t)p->n_snaps * 8);
+        OTIF_CUDA(cudaMemcpy(h.data(), p->pj_snaps, h.size() * 8, cudaMemcpyDeviceToHost));
+        for (int c = 0; c < p->n_snaps; c++) {
+            const unsigned long long *r = &h[(size_t)c * 8];
+            const unsigned long long tot = r[5];
+            unsigned long long prev = 0;
+            for (int li = 0; li < 5; li++) {
+                // (a pass without an E2 GEMM layer never writes slot 0: it stays 0)
+                const unsigned long long cur = r[li] < tot ? r[li] : tot;
+                if (cur >= prev) { units[li] += cur - prev; prev = cur; }
+            }
+            units[5] += tot - prev;   // left to the drain kernel
+            units[6] += tot;
+        }
+    }
+    p->n_snaps = 0;
+    return OTIF_OK;
 }
 
 extern "C" uint8_t *otif_pipeline_detector_batch(const otif_pipeline *p, int32_t s) {

@@ -2507,7 +2507,7 @@ bool proxy_fuses_resize(const otif_proxy *p, int n, const uint8_t *src, int sh, 
 // the fused E1+E2 kernel in place of the proxy image (img unused)
 otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *scores, uint8_t *ws,
                          size_t ws_bytes, cudaStream_t stream, cudaEvent_t *evs, PackJob *pj,
-                         const uint8_t *frames, int sh, int sw) {
+                         const uint8_t *frames, int sh, int sw, unsigned long long *pj_snap) {
     Layout lay[5];
     otif_status pst = prepare_ws(p, n, ws, ws_bytes, stream, lay);
     if (pst != OTIF_OK) return pst;
@@ -2717,6 +2717,9 @@ otif_status launch_proxy(const otif_proxy *p, const uint8_t *img, int n, float *
         }
         OTIF_LAUNCH_CHECK();
         if (evs) OTIF_CUDA(cudaEventRecord(evs[1 + li], stream));
+        // timing only: the pack-unit claim counter after this layer (which layer carried how
+        // much of the fused copy)
+        if (pj && pj_snap) OTIF_CUDA(cudaMemcpyAsync(pj_snap + li, &pj->next, 8, cudaMemcpyDeviceToDevice, stream));
     }
     return OTIF_OK;
 }
@@ -2904,5 +2907,5 @@ extern "C" otif_status otif_proxy_score(const otif_proxy *p, const uint8_t *img,
     OTIF_REQUIRE((((uintptr_t)workspace) & 255) == 0, "otif_proxy_score: workspace must be 256-B aligned");
     otif_status st = check_device(nullptr);
     if (st != OTIF_OK) return st;
-    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream, nullptr, nullptr, nullptr, 0, 0);
+    return launch_proxy(p, img, n, scores, (uint8_t *)workspace, ws_bytes, stream, nullptr, nullptr, nullptr, 0, 0, nullptr);
 }
