@@ -525,6 +525,10 @@ extern "C" otif_status otif_pipeline_set_timing(otif_pipeline *p, int32_t enable
     p->timing = enable ? 1 : 0;
     p->ev_used = 0;
     p->launches = 0;
+    p->n_snaps = 0;
+    // the pack-unit snapshot rows are allocated here, not inside a timed run
+    if (p->timing && p->job && !p->pj_snaps && cudaMalloc(&p->pj_snaps, (size_t)kMaxSnaps * 8 * 8) != cudaSuccess)
+        return OTIF_ENOMEM;
     return OTIF_OK;
 }
 
